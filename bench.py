@@ -1,0 +1,340 @@
+"""Benchmark of the B200 phase-field step (BASELINE.json metric: MLUP/s per
+GPU, fp64, and % of roofline).
+
+    python bench.py [--gpus N --steps K --warmup W] [--impl reference]
+    torchrun --nproc-per-node N bench.py --gpus N ...
+
+One "step" = one full time step of the hot path (Algorithm 1: phi-sweep,
+phi ghosts, mu-sweep, mu ghosts, swap; plus the moving-window check every
+window_check steps) over the whole domain.  Workload (config 2 of
+BASELINE.json): 256^3 cells per GPU, ternary eutectic (4 phases, 2 mu),
+frozen-temperature directional solidification with moving window, IC-L,
+synthetic C.4 parameters.  For N > 1 the growth axis stays unsplit and the
+blocks tile x-y (weak scaling, 256^3 per GPU).  Prints one JSON line on
+rank 0.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "MLUP/s per GPU (fp64) at 1/2/4/8 B200 and % of roofline"
+UNIT = "MLUP/s"
+# Table 1, P1, split accounting: algorithmic fp64 ops per cell
+F_PHI = 66 + 124 + 202 + 282 + 9          # phi-split: adds + muls + divs = 683
+F_MU = 256 + 389 + 75 + 90 + 17 + 21 + 18  # mu-split: adds + muls + divs + sqrts + rsqrts = 866
+F_STEP = F_PHI + F_MU                      # 1549
+Q_STEP = 96                                # bytes/cell: read phi, mu; write phi, mu (fp64)
+# fp64 peak derived from unit counts and clocks: 148 SMs x 64
+# FP64 FMA lanes x 2 flop x 1.965 GHz (clocks.max.sm)
+SMS, FP64_LANES, SM_MAX_GHZ = 148, 64, 1.965
+
+
+def fp64_peak_tflops():
+    return SMS * FP64_LANES * 2 * SM_MAX_GHZ / 1e3
+
+
+def grid_for(n):
+    return {1: (1, 1, 1), 2: (2, 1, 1), 4: (2, 2, 1), 8: (4, 2, 1)}.get(n, (n, 1, 1))
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        return json.load(open(p))
+    except Exception:
+        return {}
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device):
+        self.device = device
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.t.join(timeout=2)
+        sm, smax, reasons, power = [], [], set(), []
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                smax.append(float(f[2]))
+                power.append(float(f[3]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(smax) if smax else None,
+                "reasons": sorted(reasons), "samples": len(sm),
+                "power_w_max": max(power) if power else None}
+
+
+def traffic_per_launch():
+    """dram read+write bytes per mu-sweep launch from the committed ncu --set
+    full summary (profiles/), or None."""
+    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        d = json.load(open(p))
+        return d["mu_sweep"]["dram_bytes_per_launch"]
+    except Exception:
+        return None
+
+
+def cpu_baseline(P, bc, seconds=12.0, shape=(64, 96, 96)):
+    """The oracle, as it stands, on the host cores (bounded sample)."""
+    from oracle import oracle as O
+    from paper_conf_sc_0003hehshhkwnr19_b200 import inputs as I
+    O.build()
+    cores = os.cpu_count() or 1
+    O.set_threads(cores)
+    phi, mu = I.ic_lamellar(shape, seed=20191117)
+    o = O.Oracle(shape, P, bc)
+    o.init(phi, mu)
+    n = 0
+    t0 = time.perf_counter()
+    while True:
+        o.step(1)
+        n += 1
+        el = time.perf_counter() - t0
+        if el >= seconds or n >= 200:
+            break
+    cells = shape[0] * shape[1] * shape[2]
+    O.set_threads(0)
+    return {"value": cells * n / el / 1e6, "unit": UNIT, "cores": cores, "kind": "oracle",
+            "sample": f"{n} step(s) of the config-2 workload on a {shape[2]}x{shape[1]}x{shape[0]} (x*y*z) "
+                      f"IC-L DS block, OpenMP over z on {cores} host threads, {el:.1f} s"}
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the oracle on the host cores, each step a bounded
+    sample (one oracle step on a 64x64x32 sub-block of the workload)."""
+    if rank != 0:
+        return
+    from oracle import oracle as O
+    from paper_conf_sc_0003hehshhkwnr19_b200 import inputs as I
+    O.build()
+    cores = os.cpu_count() or 1
+    O.set_threads(cores)
+    shape = (32, 64, 64)
+    P = I.params_c4("ds")
+    P["T0"] = I.ds_T0(8, P["G"])
+    phi, mu = I.ic_lamellar(shape, seed=20191117, z_front=8)
+    o = O.Oracle(shape, P, I.BC_DS)
+    o.init(phi, mu)
+    o.step(args.warmup)
+    t0 = time.perf_counter()
+    o.step(args.steps)
+    el = time.perf_counter() - t0
+    cells = shape[0] * shape[1] * shape[2]
+    val = cells * args.steps / el / 1e6
+    print(json.dumps({
+        "impl": "reference", "metric": METRIC, "value": val, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": el / args.steps * 1e3, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": "config 2 sample: 64x64x32 sub-block of the 256^3 DS moving-window run, IC-L, C.4",
+                   "global": [64, 64, 32]},
+        "cpu_baseline": {"value": val, "unit": UNIT, "cores": cores, "kind": "oracle",
+                         "sample": f"{args.steps} oracle steps on 64x64x32, OpenMP on {cores} threads"},
+        "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--n", type=int, default=256, help="block edge per GPU")
+    ap.add_argument("--variant", default="tuned", choices=["tuned", "naive"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    assert args.warmup >= 3 or args.impl == "reference" or os.environ.get("PF_BENCH_ALLOW_SHORT"), "W >= 3"
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", str(args.gpus)))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+
+    import numpy as np
+    import torch
+    from paper_conf_sc_0003hehshhkwnr19_b200 import inputs as I
+    from paper_conf_sc_0003hehshhkwnr19_b200 import pf
+
+    torch.cuda.set_device(local_rank)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    procs = grid_for(world)
+    n = args.n
+    gshape = (n, n * procs[1], n * procs[0])  # (nz, ny, nx): growth axis z unsplit
+    P = I.params_c4("ds", window_check=10, window_frac=0.5)
+    z_front = n // 4
+    P["T0"] = I.ds_T0(z_front, P["G"])
+    uid = None
+    if world > 1:
+        t = torch.zeros(128, dtype=torch.uint8, device="cuda")
+        if rank == 0:
+            t.copy_(torch.tensor(list(pf.nccl_unique_id()), dtype=torch.uint8))
+        dist.broadcast(t, 0)
+        uid = bytes(t.cpu().tolist())
+    g = pf.PhaseField(gshape, P, bc=I.BC_DS, procs=procs, rank=rank, world=world, device=local_rank, nccl_uid=uid)
+    g.set_variant(args.variant)
+    lshape = g.local
+    phi, mu = I.ic_lamellar(lshape, seed=20191117 + rank, z_front=z_front)
+    phi_pin = torch.from_numpy(phi).pin_memory()
+    mu_pin = torch.from_numpy(mu).pin_memory()
+    g.init_fields(phi_pin, mu_pin)
+    stream = g.stream
+    cells_local = lshape[0] * lshape[1] * lshape[2]
+
+    def barrier():
+        if dist is not None:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def max_over_ranks(x):
+        if dist is None:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    # ---- warm-up ----
+    g.step(args.warmup)
+    barrier()
+    # ---- timed region (device events on the library's stream) ----
+    g.profile(True)
+    clocks = ClockSampler(local_rank)
+    clocks.start()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    barrier()
+    e0.record(stream)
+    g.step(args.steps)
+    e1.record(stream)
+    e1.synchronize()
+    barrier()
+    ms = e0.elapsed_time(e1)
+    clk = clocks.stop()
+    prof = g.profile_read()
+    ms_max = max_over_ranks(ms)
+    launches = sum(v[1] for v in prof.values())
+    mon = g.monitor()
+    st = g.state()
+
+    total_cells = cells_local * world
+    value = total_cells * args.steps / (ms_max * 1e-3) / 1e6  # whole-job MLUP/s
+    # ---- roofline of the dominant kernel (mu-sweep) ----
+    mu_ms, mu_n = prof["mu_sweep"]
+    phi_ms, phi_n = prof["phi_sweep"]
+    peak_tf = fp64_peak_tflops()
+    mu_tf = F_MU * cells_local / (mu_ms / mu_n * 1e-3) / 1e12 if mu_n else None
+    phi_tf = F_PHI * cells_local / (phi_ms / phi_n * 1e-3) / 1e12 if phi_n else None
+    peaks = measured_peaks()
+    hbm = peaks.get("hbm_gbs", 6650.0)
+    R = min(peak_tf * 1e12 / F_STEP, hbm * 1e9 / Q_STEP) / 1e6  # MLUP/s per GPU
+    rec = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"config 2: {n}^3 block per GPU, ternary eutectic N=4/K-1=2, frozen-T directional "
+                               f"solidification, moving window (check every 10 steps), IC-L, C.4 parameters",
+                   "global_xyz": [gshape[2], gshape[1], gshape[0]], "procs_xyz": list(procs),
+                   "parallelism": f"domain decomposition {procs[0]}x{procs[1]}x{procs[2]}",
+                   "variant": args.variant,
+                   "l2": f"inputs larger than L2 ({(6 * 2) * cells_local * 8 / 1e9:.2f} GB of fields per GPU)"},
+        "per_gpu_mlups": value / world,
+        "step_roofline": {"R_mlups": R, "F_flop_per_cell": F_STEP, "Q_bytes_per_cell": Q_STEP,
+                          "frac": (value / world) / R, "peak_fp64_tflops": peak_tf, "hbm_gbs": hbm},
+        "roofline": {"bound": "alu", "kernel": "mu_sweep", "achieved": mu_tf, "peak": peak_tf, "unit": "TFLOP/s",
+                     "frac": (mu_tf / peak_tf) if mu_tf else None, "traffic": traffic_per_launch(),
+                     "flop_per_cell": F_MU, "cells_per_launch": cells_local,
+                     "avg_launch_ms": mu_ms / mu_n if mu_n else None,
+                     "peak_note": "derived: 148 SMs x 64 FP64 lanes x 2 x 1.965 GHz (DESIGN.md §6)"},
+        "kernels": {"phi_sweep_ms": phi_ms / max(phi_n, 1), "mu_sweep_ms": mu_ms / max(mu_n, 1),
+                    "phi_sweep_tflops": phi_tf, "share_mu": mu_ms / ms if ms else None,
+                    "share_phi": phi_ms / ms if ms else None,
+                    "ghost_ms_total": prof["ghost"][0], "window_ms_total": prof["window"][0]},
+        "gpu_launches": launches,
+        "clocks": clk,
+        "state": {"step": st["step"], "z_off": st["z_off"], "max_sum_err": mon[0], "min_phi": mon[1]},
+    }
+    # ---- end-to-end through the public API with host buffers ----
+    if not args.no_e2e:
+        g.profile(False)
+        out_phi = torch.empty_like(phi_pin).pin_memory()
+        out_mu = torch.empty_like(mu_pin).pin_memory()
+        barrier()
+        t0 = time.perf_counter()
+        f0 = torch.cuda.Event(enable_timing=True)
+        f1 = torch.cuda.Event(enable_timing=True)
+        f0.record(stream)
+        g.init_fields(phi_pin, mu_pin)
+        g.step(args.steps)
+        g.download(out=(out_phi, out_mu))
+        f1.record(stream)
+        f1.synchronize()
+        barrier()
+        ems = max_over_ranks(max(f0.elapsed_time(f1), (time.perf_counter() - t0) * 1e3))
+        bytes_state = (phi.nbytes + mu.nbytes)
+        rec["e2e"] = {"value": total_cells * args.steps / (ems * 1e-3) / 1e6, "unit": UNIT,
+                      "h2d_bytes_per_step": bytes_state / args.steps, "d2h_bytes_per_step": bytes_state / args.steps,
+                      "note": "one chunk = pf_init_fields from pinned host memory, K steps, pf_download to pinned "
+                              "host memory, all inside the timed region"}
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        rec["cpu_baseline"] = cpu_baseline(P, I.BC_DS)
+    if rank == 0:
+        print(json.dumps(rec), flush=True)
+    g.close()
+    if dist is not None:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

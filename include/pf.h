@@ -1,0 +1,195 @@
+/*
+ * pf.h -- C ABI of the B200-native grand-potential multiphase-field step.
+ *
+ * Implements the hot path of Bauer et al., "Code Generation for Massively
+ * Parallel Phase-Field Simulations" (SC'19): one explicit time step of the
+ * coupled phase-field (phi, N = 4 phases on the Gibbs simplex) and
+ * chemical-potential (mu, K-1 = 2 components, with anti-trapping current)
+ * equations on a 3-D Cartesian grid, as Algorithm 1 composes
+ * them.  Citations "P:Lx-y" are lines of the paper text; "A<n>" are the
+ * readings listed in DESIGN.md §3.
+ *
+ * Conventions for every entry point
+ *   - Pure C99, no exceptions cross the ABI, no exit/abort.  Every call
+ *     returns PF_OK (0) or a negative PF_E* status; pf_last_error() gives a
+ *     human-readable message for the last failure on that context.
+ *   - Field layout seen by callers: interior-only, structure of arrays,
+ *     phi[alpha][z][y][x] and mu[i][z][y][x], x fastest, fp64, block-local.
+ *   - Device buffers are OWNED BY THE CALLER (e.g. torch tensors) and sized
+ *     by pf_query_layout(); the library never frees caller memory.  It owns
+ *     only its NCCL communicator, streams, events and pinned scratch, released
+ *     by pf_destroy().
+ *   - All device work is enqueued on the caller's stream (pf_config.stream);
+ *     calls are asynchronous unless documented as synchronous.  Errors of
+ *     asynchronous work surface on a later call.
+ *   - Multi-GPU: one process per GPU; world > 1 decomposes the global domain
+ *     into procs[0] x procs[1] x procs[2] blocks, one per rank, with ghost
+ *     layers exchanged by NCCL send/recv.  Calls marked
+ *     "collective" must be made by every rank in the same order.
+ */
+#ifndef PF_H
+#define PF_H
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ---- status codes ------------------------------------------------------ */
+#define PF_OK 0
+#define PF_EINVAL (-1)   /* invalid argument / configuration / parameters   */
+#define PF_ENOMEM (-2)   /* buffer too small or allocation failed           */
+#define PF_ECUDA (-3)    /* CUDA runtime error (incl. earlier async errors) */
+#define PF_ENCCL (-4)    /* NCCL error or NCCL unavailable                  */
+#define PF_ESTATE (-5)   /* wrong call order (e.g. step before init)        */
+#define PF_ENUMERIC (-6) /* invariant monitor tripped (sum phi, phi >= 0)   */
+
+/* ---- boundary conditions per side (reading A15) ------------------------ */
+#define PF_BC_PERIODIC 0
+#define PF_BC_NEUMANN 1      /* phi and mu: ghost = adjacent interior value */
+#define PF_BC_DIRICHLET_MU 2 /* phi Neumann; mu ghost = mu_inf             */
+
+#define PF_HOST 0
+#define PF_DEVICE 1
+#define PF_PHI 1u
+#define PF_MU 2u
+
+#define PF_N 4 /* phases (P1: 3 solids + liquid)  */
+#define PF_M 2 /* chemical potentials K-1 (3 components)        */
+
+/* kernel schedule (pf_set_variant); results are identical to <= 1e-12 */
+#define PF_VARIANT_TUNED 0 /* default: z-marching, face fluxes computed once */
+#define PF_VARIANT_NAIVE 1 /* one thread per cell, every face computed twice */
+
+typedef struct pf_ctx pf_ctx;
+
+typedef struct {
+  int n_phases;     /* must be PF_N                                          */
+  int n_mu;         /* must be PF_M                                          */
+  int liquid;       /* index l of the liquid phase, 0..3 (eq. 10)            */
+  int global[3];    /* global interior extents nx, ny, nz                    */
+  int procs[3];     /* rank grid; product must equal world                   */
+  int bc_lo[3];     /* PF_BC_* of the low side of x, y, z                    */
+  int bc_hi[3];     /* PF_BC_* of the high side; periodic must match low     */
+  int rank, world;  /* this process' rank, number of ranks (= GPUs)          */
+  unsigned char nccl_uid[128]; /* ncclUniqueId bytes from rank 0 (world > 1) */
+  int device;       /* CUDA device ordinal                                   */
+  void* stream;     /* cudaStream_t borrowed from the caller (0 = legacy)     */
+  double* phi[2];   /* caller-owned device buffers, pf_layout.phi_bytes each */
+  double* mu[2];    /* caller-owned device buffers, pf_layout.mu_bytes each  */
+  void* workspace;  /* caller-owned device buffer, pf_layout.workspace_bytes */
+} pf_config;
+
+typedef struct {
+  int local[3];           /* this rank's interior extents nx, ny, nz          */
+  int offset[3];          /* global index of its first interior cell          */
+  int64_t pitch;          /* doubles per padded row (ghosts included)         */
+  int64_t plane;          /* doubles per z-plane = pitch * (ny + 2)           */
+  int64_t field;          /* doubles per component = plane * (nz + 2)         */
+  int64_t x_off;          /* row offset of interior x = 0 (128-B aligned)     */
+  size_t phi_bytes;       /* one time level of phi: PF_N * field * 8          */
+  size_t mu_bytes;        /* one time level of mu:  PF_M * field * 8          */
+  size_t workspace_bytes; /* tables, pack buffers, reduction scratch          */
+} pf_layout;
+
+/* Model parameters (eqs. 3-10 with A_ab = 1, P1).  Plain-old-data, fp64. */
+typedef struct {
+  double dx, dt, eps;                  /* grid spacing, time step, interface width */
+  double gamma[PF_N][PF_N];            /* gamma_ab, symmetric, eqs. 4-5            */
+  double gamma3[PF_N][PF_N][PF_N];     /* gamma_abd, symmetric, eq. 5              */
+  double tau[PF_N][PF_N];              /* tau_ab, symmetric            */
+  double A0[PF_N][PF_M][PF_M], A1[PF_N][PF_M][PF_M]; /* psi_a = mu.A mu + B.mu + C, */
+  double B0[PF_N][PF_M], B1[PF_N][PF_M];             /* A, B, C affine in T (eq. 6) */
+  double C0[PF_N], C1[PF_N];
+  double D[PF_N][PF_M][PF_M];          /* D_alpha of the mobility, eq. 9           */
+  double T0, G, v;                     /* T = T0 + G (z dx - v t)  [A13]           */
+  double mu_inf[PF_M];                 /* inflow / Dirichlet value of mu           */
+  double window_frac;                  /* moving window threshold fraction [A16]   */
+  int window_check;                    /* check every n steps; 0 = window off      */
+} pf_params;
+
+typedef struct {
+  int64_t step;  /* completed steps; t_n = step * dt         */
+  int64_t z_off; /* moving-window offset along z, in cells   */
+} pf_state;
+
+/* Sizes of the buffers a caller must provide for this configuration.
+ * Reads cfg->global/procs/rank only.  PF_EINVAL on a bad decomposition. */
+int pf_query_layout(const pf_config* cfg, pf_layout* out);
+
+/* Validate cfg, bind the caller's buffers, create streams/events and (world > 1)
+ * the NCCL communicator from cfg->nccl_uid.  Collective when world > 1.     */
+int pf_create(const pf_config* cfg, pf_ctx** out);
+int pf_destroy(pf_ctx* ctx);
+
+/* Copy the parameters (eqs. 3-10) after validation: positive dx, dt, eps,
+ * tau, gamma; symmetric gamma, gamma3, tau; negative-definite symmetric part
+ * of A_a(T) over the domain's T range (so dc/dmu is SPD, reading A6); finite
+ * values; dt below the explicit stability bound (PF_EINVAL otherwise).      */
+int pf_set_params(pf_ctx* ctx, const pf_params* p);
+
+/* Load block-local interior fields (layout above) from host (where = PF_HOST)
+ * or device (PF_DEVICE) memory.  Checks |sum phi - 1| <= 1e-12 and phi >= 0
+ * (PF_EINVAL otherwise), resets step = 0 and z_off = 0, fills ghost layers
+ * (collective halo exchange).  Synchronous.                                 */
+int pf_init_fields(pf_ctx* ctx, const double* phi, const double* mu, int where);
+
+/* Enqueue nsteps full time steps (Algorithm 1: phi-sweep, phi ghosts,
+ * mu-sweep, mu ghosts, swap) plus, every window_check steps,
+ * the moving-window check (front height max-reduction, shift if needed;
+ * this synchronises the stream once per check).  Collective.               */
+int pf_step(pf_ctx* ctx, int64_t nsteps);
+
+/* Debug entry (SURVEY C.7 split diagnosis): one phi-sweep + phi ghosts, mu
+ * copied unchanged, swap, step += 1.  Collective.                          */
+int pf_step_phi_only(pf_ctx* ctx);
+
+/* Refill ghost layers of the current fields: mask = PF_PHI | PF_MU.  Collective. */
+int pf_halo_exchange(pf_ctx* ctx, unsigned mask);
+
+/* Shift the current fields by k >= 0 planes along z (growth axis): new(z) =
+ * old(z + k), the top k planes become liquid (phi = e_l, mu = mu_inf);
+ * z_off += k (reading A16).  Requires procs[2] == 1.  Collective.          */
+int pf_shift_window(pf_ctx* ctx, int k);
+
+/* Front height H = max{z : exists (x,y) with phi_l < 1/2} over the global
+ * domain, -1 if there is no solid.  Collective, synchronous. */
+int pf_front_height(pf_ctx* ctx, int* H);
+
+/* Invariant monitors of the current phi: out[0] = max |sum_a phi_a - 1|,
+ * out[1] = min_a,cells phi_a (global over ranks).  Collective, synchronous. */
+int pf_monitor(pf_ctx* ctx, double out[2]);
+
+/* Copy the current interior fields to host (where = PF_HOST) or device
+ * (PF_DEVICE) memory in the layout above.  Synchronous.                     */
+int pf_download(pf_ctx* ctx, double* phi, double* mu, int where);
+
+int pf_get_state(const pf_ctx* ctx, pf_state* out);
+int pf_set_state(pf_ctx* ctx, const pf_state* s);
+
+/* Kernel schedule selection (PF_VARIANT_*), for ablations and parity. */
+int pf_set_variant(pf_ctx* ctx, int variant);
+
+/* Optional per-kernel timing with CUDA events on the compute stream:
+ * pf_profile(ctx, 1) resets the counters and enables event timing
+ * (pf_profile(ctx, 0) resets and disables it); pf_profile_read() returns the
+ * accumulated milliseconds (0 if timing is disabled) and the number of
+ * kernels launched since the reset, per category: phi-sweep (k = 0),
+ * mu-sweep (1), ghost / halo pack-unpack (2), tables + window (3).
+ * Synchronous read.                                                        */
+int pf_profile(pf_ctx* ctx, int enable);
+int pf_profile_read(pf_ctx* ctx, double ms[4], int64_t launches[4]);
+
+/* Rank 0 of a world > 1 job: create the NCCL unique id (128 bytes) that the
+ * caller broadcasts (e.g. with torch.distributed) into every rank's
+ * pf_config.nccl_uid before pf_create.  PF_ENCCL if NCCL cannot be loaded. */
+int pf_nccl_unique_id(unsigned char out[128]);
+
+const char* pf_last_error(const pf_ctx* ctx);
+const char* pf_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* PF_H */

@@ -1,0 +1,854 @@
+// pf_api.cu -- host runtime and C ABI of the B200 phase-field step.
+//
+// Context management, padded layout, parameter validation and explicit
+// stability bound, the per-step schedule of Algorithm 1 on
+// the caller's stream, ghost layers / NCCL halo exchange, the
+// moving window and the invariant monitors.  See include/pf.h for the ABI.
+#include <dlfcn.h>
+#include <math.h>
+#include <nccl.h>
+#include <stdarg.h>
+#include <stdio.h>
+#include <stdlib.h>
+#include <string.h>
+
+#include <algorithm>
+#include <string>
+#include <vector>
+
+#include "pf_model.cuh"
+
+using namespace pf;
+
+namespace pf {
+void launch_tuned_phi(const DevParams& P, const Geom& g, const Tables& T, const double* ps, const double* ms,
+                      double* pd, cudaStream_t s);
+void launch_tuned_mu(const DevParams& P, const Geom& g, const Tables& T, const double* ps, const double* pd,
+                     const double* ms, double* md, cudaStream_t s);
+void launch_ghost_stage(const Geom& g, int d, int klo, int khi, double* f, int ncomp, const double* dirichlet,
+                        cudaStream_t s);
+}  // namespace pf
+
+// ---------------------------------------------------------------------------
+// NCCL, loaded on demand (dlopen) so that the library loads and runs without
+// it for world == 1.  Prototypes from nccl.h.
+// ---------------------------------------------------------------------------
+namespace {
+struct NcclApi {
+  void* h = nullptr;
+  decltype(&ncclCommInitRank) CommInitRank = nullptr;
+  decltype(&ncclCommDestroy) CommDestroy = nullptr;
+  decltype(&ncclSend) Send = nullptr;
+  decltype(&ncclRecv) Recv = nullptr;
+  decltype(&ncclGroupStart) GroupStart = nullptr;
+  decltype(&ncclGroupEnd) GroupEnd = nullptr;
+  decltype(&ncclAllReduce) AllReduce = nullptr;
+  decltype(&ncclGetErrorString) GetErrorString = nullptr;
+  decltype(&ncclGetUniqueId) GetUniqueId = nullptr;
+  bool load(std::string* err) {
+    if (h) return true;
+    const char* names[] = {"libnccl.so.2", "libnccl.so"};
+    for (const char* n : names) {
+      h = dlopen(n, RTLD_NOW | RTLD_GLOBAL | RTLD_NOLOAD);
+      if (!h) h = dlopen(n, RTLD_NOW | RTLD_GLOBAL);
+      if (h) break;
+    }
+    if (!h) {
+      *err = std::string("cannot dlopen libnccl.so.2: ") + dlerror();
+      return false;
+    }
+#define PF_SYM(field, name)                                   \
+  field = reinterpret_cast<decltype(field)>(dlsym(h, name)); \
+  if (!field) { *err = std::string("NCCL symbol missing: ") + name; return false; }
+    PF_SYM(CommInitRank, "ncclCommInitRank");
+    PF_SYM(CommDestroy, "ncclCommDestroy");
+    PF_SYM(Send, "ncclSend");
+    PF_SYM(Recv, "ncclRecv");
+    PF_SYM(GroupStart, "ncclGroupStart");
+    PF_SYM(GroupEnd, "ncclGroupEnd");
+    PF_SYM(AllReduce, "ncclAllReduce");
+    PF_SYM(GetErrorString, "ncclGetErrorString");
+    PF_SYM(GetUniqueId, "ncclGetUniqueId");
+#undef PF_SYM
+    return true;
+  }
+};
+NcclApi g_nccl;
+}  // namespace
+
+// ---------------------------------------------------------------------------
+struct pf_ctx {
+  pf_config cfg;
+  pf_layout lay;
+  Geom g;
+  int coord[3];           // rank coordinates in the rank grid
+  int nb_lo[3], nb_hi[3];  // neighbour ranks (-1 = physical boundary)
+  BCSpec bc_all;          // local BC kinds, -1 where a halo exchange fills the side
+  bool exchange[3];       // dimension d is exchanged (procs[d] > 1 or forced)
+  bool force_exchange = false;
+  cudaStream_t stream = nullptr;
+  double* phi[2];
+  double* mu[2];
+  int cur = 0;
+  // workspace carve-up
+  double* tab = nullptr;
+  unsigned long long* red = nullptr;  // reduction scratch (4 x u64)
+  double* sendbuf[3][2] = {};
+  double* recvbuf[3][2] = {};
+  // host
+  unsigned long long* pinned = nullptr;
+  pf_params hp;
+  DevParams dp;
+  bool have_params = false, have_fields = false;
+  int64_t step = 0, z_off = 0;
+  int variant = PF_VARIANT_TUNED;
+  ncclComm_t comm = nullptr;
+  // profiling
+  bool prof = false;
+  std::vector<cudaEvent_t> ev_pool;
+  std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> ev_open;
+  double prof_ms[4] = {0, 0, 0, 0};
+  int64_t prof_n[4] = {0, 0, 0, 0};
+  int64_t nlaunch[4] = {0, 0, 0, 0};  // kernels launched per category since pf_profile()
+  std::string err;
+};
+
+namespace {
+
+int fail(pf_ctx* c, int code, const char* fmt, ...) {
+  if (c) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    c->err = buf;
+  }
+  return code;
+}
+
+#define CU(call)                                                                          \
+  do {                                                                                    \
+    cudaError_t e_ = (call);                                                              \
+    if (e_ != cudaSuccess) return fail(ctx, PF_ECUDA, "%s: %s", #call, cudaGetErrorString(e_)); \
+  } while (0)
+
+#define NC(call)                                                                                  \
+  do {                                                                                            \
+    ncclResult_t r_ = (call);                                                                     \
+    if (r_ != ncclSuccess) return fail(ctx, PF_ENCCL, "%s: %s", #call, g_nccl.GetErrorString(r_)); \
+  } while (0)
+
+int check_launch(pf_ctx* ctx, const char* what) {
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(ctx, PF_ECUDA, "%s launch: %s", what, cudaGetErrorString(e));
+  return PF_OK;
+}
+
+size_t align256(size_t b) { return (b + 255) & ~(size_t)255; }
+
+void split(int n, int p, int r, int* len, int* off) {
+  const int base = n / p, rem = n % p;
+  *len = base + (r < rem ? 1 : 0);
+  *off = r * base + std::min(r, rem);
+}
+
+int layout_of(const pf_config* cfg, pf_layout* L, int coord[3]) {
+  if (!cfg || !L) return PF_EINVAL;
+  const int world = cfg->world < 1 ? 1 : cfg->world;
+  int pr[3];
+  for (int d = 0; d < 3; ++d) {
+    pr[d] = cfg->procs[d] < 1 ? 1 : cfg->procs[d];
+    if (cfg->global[d] < 1) return PF_EINVAL;
+  }
+  if (pr[0] * pr[1] * pr[2] != world || cfg->rank < 0 || cfg->rank >= world) return PF_EINVAL;
+  int r = cfg->rank;
+  coord[0] = r % pr[0];
+  coord[1] = (r / pr[0]) % pr[1];
+  coord[2] = r / (pr[0] * pr[1]);
+  for (int d = 0; d < 3; ++d) {
+    split(cfg->global[d], pr[d], coord[d], &L->local[d], &L->offset[d]);
+    if (L->local[d] < 1) return PF_EINVAL;
+  }
+  const int nx = L->local[0], ny = L->local[1], nz = L->local[2];
+  L->x_off = 16;  // interior x = 0 at a 128-B boundary
+  L->pitch = ((L->x_off + nx + 1) + 15) / 16 * 16;
+  L->plane = L->pitch * (ny + 2);
+  L->field = L->plane * (nz + 2);
+  L->phi_bytes = (size_t)PF_N * L->field * sizeof(double) + 256;  // +256: tail slack for vector loads
+  L->mu_bytes = (size_t)PF_M * L->field * sizeof(double) + 256;
+  size_t ws = align256(table_doubles(nz) * sizeof(double)) + 256;  // tables + reduction scratch
+  Geom g{nx, ny, nz, L->offset[2], L->pitch, L->plane, L->field, L->x_off};
+  for (int d = 0; d < 3; ++d) ws += 4 * align256(halo_slab_elems(g, d) * PF_N * sizeof(double));
+  L->workspace_bytes = ws;
+  return PF_OK;
+}
+
+// Explicit (FTCS) stability bounds (SURVEY C.4 "dt"), in time units.
+//  phi: linearised diffusivity of the gradient flux 2 sum_b gamma_ab phi_b^2 / tau <= 2 gamma_max / tau_min
+//  mu:  D_eff = spectral radius of chi^{-1} M over sample points of the simplex
+double eig2_max_abs(const double a[2][2]) {
+  const double tr = a[0][0] + a[1][1], det = a[0][0] * a[1][1] - a[0][1] * a[1][0];
+  const double disc = tr * tr / 4 - det;
+  if (disc >= 0) return std::max(fabs(tr / 2 + sqrt(disc)), fabs(tr / 2 - sqrt(disc)));
+  return sqrt(det > 0 ? det : -det);  // complex pair: |lambda| = sqrt(det)
+}
+
+double deff_at(const pf_params& p, const double* ph, double T) {
+  double M[2][2] = {{0, 0}, {0, 0}}, X[2][2] = {{0, 0}, {0, 0}};
+  for (int a = 0; a < PF_N; ++a) {
+    double chi[2][2];
+    for (int i = 0; i < 2; ++i)
+      for (int j = 0; j < 2; ++j)
+        chi[i][j] = -((p.A0[a][i][j] + p.A1[a][i][j] * T) + (p.A0[a][j][i] + p.A1[a][j][i] * T));
+    const double x = ph[a], h = x * x * (3 - 2 * x);
+    for (int i = 0; i < 2; ++i)
+      for (int j = 0; j < 2; ++j) {
+        X[i][j] += h * chi[i][j];
+        M[i][j] += x * (p.D[a][i][0] * chi[0][j] + p.D[a][i][1] * chi[1][j]);
+      }
+  }
+  const double det = X[0][0] * X[1][1] - X[0][1] * X[1][0];
+  if (!(det > 0)) return INFINITY;
+  const double inv[2][2] = {{X[1][1] / det, -X[0][1] / det}, {-X[1][0] / det, X[0][0] / det}};
+  double K[2][2];
+  for (int i = 0; i < 2; ++i)
+    for (int j = 0; j < 2; ++j) K[i][j] = inv[i][0] * M[0][j] + inv[i][1] * M[1][j];
+  return eig2_max_abs(K);
+}
+
+}  // namespace
+
+// ===========================================================================
+extern "C" {
+
+const char* pf_version(void) { return "pf-b200 0.1 (sm_100a, fp64)"; }
+
+int pf_nccl_unique_id(unsigned char out[128]) {
+  if (!out) return PF_EINVAL;
+  std::string err;
+  if (!g_nccl.load(&err)) return PF_ENCCL;
+  ncclUniqueId id;
+  if (g_nccl.GetUniqueId(&id) != ncclSuccess) return PF_ENCCL;
+  memcpy(out, id.internal, 128);
+  return PF_OK;
+}
+
+const char* pf_last_error(const pf_ctx* ctx) { return ctx ? ctx->err.c_str() : "null context"; }
+
+int pf_query_layout(const pf_config* cfg, pf_layout* out) {
+  int coord[3];
+  return layout_of(cfg, out, coord);
+}
+
+int pf_create(const pf_config* cfg, pf_ctx** out) {
+  if (!cfg || !out) return PF_EINVAL;
+  *out = nullptr;
+  if (cfg->n_phases != PF_N || cfg->n_mu != PF_M || cfg->liquid < 0 || cfg->liquid >= PF_N) return PF_EINVAL;
+  pf_ctx* ctx = new (std::nothrow) pf_ctx();
+  if (!ctx) return PF_ENOMEM;
+  ctx->cfg = *cfg;
+  if (layout_of(cfg, &ctx->lay, ctx->coord) != PF_OK) {
+    delete ctx;
+    return PF_EINVAL;
+  }
+  const pf_layout& L = ctx->lay;
+  ctx->g = Geom{L.local[0], L.local[1], L.local[2], L.offset[2], L.pitch, L.plane, L.field, L.x_off};
+  for (int d = 0; d < 3; ++d) {
+    const int blo = cfg->bc_lo[d], bhi = cfg->bc_hi[d];
+    if (blo < 0 || blo > 2 || bhi < 0 || bhi > 2 || ((blo == PF_BC_PERIODIC) != (bhi == PF_BC_PERIODIC))) {
+      delete ctx;
+      return PF_EINVAL;
+    }
+  }
+  for (int i = 0; i < 2; ++i) {
+    ctx->phi[i] = cfg->phi[i];
+    ctx->mu[i] = cfg->mu[i];
+    if (!cfg->phi[i] || !cfg->mu[i]) {
+      delete ctx;
+      return PF_EINVAL;
+    }
+  }
+  if (!cfg->workspace) {
+    delete ctx;
+    return PF_EINVAL;
+  }
+  ctx->stream = (cudaStream_t)cfg->stream;
+  cudaError_t e = cudaSetDevice(cfg->device);
+  if (e != cudaSuccess) {
+    ctx->err = cudaGetErrorString(e);
+    *out = ctx;
+    return PF_ECUDA;
+  }
+  // workspace carve-up
+  char* w = (char*)cfg->workspace;
+  ctx->tab = (double*)w;
+  w += align256(table_doubles(ctx->g.nz) * sizeof(double));
+  ctx->red = (unsigned long long*)w;
+  w += 256;
+  for (int d = 0; d < 3; ++d) {
+    const size_t b = align256(halo_slab_elems(ctx->g, d) * PF_N * sizeof(double));
+    for (int s = 0; s < 2; ++s) {
+      ctx->sendbuf[d][s] = (double*)w;
+      w += b;
+      ctx->recvbuf[d][s] = (double*)w;
+      w += b;
+    }
+  }
+  // neighbours and BC kinds
+  const int world = cfg->world < 1 ? 1 : cfg->world;
+  int pr[3];
+  for (int d = 0; d < 3; ++d) pr[d] = cfg->procs[d] < 1 ? 1 : cfg->procs[d];
+  auto rank_of = [&](int cx, int cy, int cz) { return cx + pr[0] * (cy + pr[1] * cz); };
+  for (int d = 0; d < 3; ++d) {
+    const bool periodic = cfg->bc_lo[d] == PF_BC_PERIODIC;
+    int c[3] = {ctx->coord[0], ctx->coord[1], ctx->coord[2]};
+    int lo = c[d] - 1, hi = c[d] + 1;
+    if (periodic) {
+      lo = (lo + pr[d]) % pr[d];
+      hi = hi % pr[d];
+    }
+    int cl[3] = {c[0], c[1], c[2]}, ch[3] = {c[0], c[1], c[2]};
+    cl[d] = lo;
+    ch[d] = hi;
+    ctx->nb_lo[d] = (lo >= 0 && lo < pr[d]) ? rank_of(cl[0], cl[1], cl[2]) : -1;
+    ctx->nb_hi[d] = (hi >= 0 && hi < pr[d]) ? rank_of(ch[0], ch[1], ch[2]) : -1;
+    ctx->exchange[d] = pr[d] > 1;
+    ctx->bc_all.kind_lo[d] = (ctx->exchange[d] && ctx->nb_lo[d] >= 0) ? -1 : cfg->bc_lo[d];
+    ctx->bc_all.kind_hi[d] = (ctx->exchange[d] && ctx->nb_hi[d] >= 0) ? -1 : cfg->bc_hi[d];
+  }
+  if (world > 1) {
+    if (!g_nccl.load(&ctx->err)) {
+      *out = ctx;
+      return PF_ENCCL;
+    }
+    ncclUniqueId id;
+    static_assert(sizeof(id.internal) == 128, "ncclUniqueId size");
+    memcpy(id.internal, cfg->nccl_uid, 128);
+    ncclResult_t r = g_nccl.CommInitRank(&ctx->comm, world, id, cfg->rank);
+    if (r != ncclSuccess) {
+      ctx->err = std::string("ncclCommInitRank: ") + g_nccl.GetErrorString(r);
+      *out = ctx;
+      return PF_ENCCL;
+    }
+  }
+  {
+    const char* fe = getenv("PF_FORCE_EXCHANGE");  // debug: periodic self-exchange through pack/unpack
+    ctx->force_exchange = fe && fe[0] == '1';
+  }
+  e = cudaMallocHost(&ctx->pinned, 64);
+  if (e != cudaSuccess) {
+    ctx->err = cudaGetErrorString(e);
+    *out = ctx;
+    return PF_ECUDA;
+  }
+  *out = ctx;
+  return PF_OK;
+}
+
+int pf_destroy(pf_ctx* ctx) {
+  if (!ctx) return PF_OK;
+  if (ctx->stream || true) cudaStreamSynchronize(ctx->stream);
+  for (auto ev : ctx->ev_pool) cudaEventDestroy(ev);
+  for (auto& o : ctx->ev_open) {
+    cudaEventDestroy(o.second.first);
+    cudaEventDestroy(o.second.second);
+  }
+  if (ctx->comm) g_nccl.CommDestroy(ctx->comm);
+  if (ctx->pinned) cudaFreeHost(ctx->pinned);
+  delete ctx;
+  return PF_OK;
+}
+
+// ---------------------------------------------------------------------------
+int pf_set_params(pf_ctx* ctx, const pf_params* p) {
+  if (!ctx || !p) return PF_EINVAL;
+  const int L = ctx->cfg.liquid;
+  auto finite = [](double v) { return isfinite(v); };
+  const double* raw = (const double*)p;
+  for (size_t i = 0; i < offsetof(pf_params, window_check) / sizeof(double); ++i)
+    if (!finite(raw[i])) return fail(ctx, PF_EINVAL, "non-finite parameter at offset %zu", i);
+  if (!(p->dx > 0 && p->dt > 0 && p->eps > 0)) return fail(ctx, PF_EINVAL, "dx, dt, eps must be > 0");
+  double gmax = 0, tmin = INFINITY;
+  for (int a = 0; a < PF_N; ++a)
+    for (int b = 0; b < PF_N; ++b) {
+      if (p->gamma[a][b] != p->gamma[b][a] || p->tau[a][b] != p->tau[b][a])
+        return fail(ctx, PF_EINVAL, "gamma and tau must be symmetric");
+      if (a == b) continue;
+      if (!(p->gamma[a][b] > 0 && p->tau[a][b] > 0)) return fail(ctx, PF_EINVAL, "gamma_ab, tau_ab must be > 0");
+      gmax = std::max(gmax, p->gamma[a][b]);
+      tmin = std::min(tmin, p->tau[a][b]);
+    }
+  for (int a = 0; a < PF_N; ++a)
+    for (int b = 0; b < PF_N; ++b)
+      for (int d = 0; d < PF_N; ++d)
+        if (p->gamma3[a][b][d] != p->gamma3[b][a][d] || p->gamma3[a][b][d] != p->gamma3[a][d][b])
+          return fail(ctx, PF_EINVAL, "gamma3 must be symmetric");
+  if (p->window_check < 0 || (p->window_check > 0 && !(p->window_frac > 0 && p->window_frac < 1)))
+    return fail(ctx, PF_EINVAL, "window_check >= 0 and 0 < window_frac < 1");
+  // T range over the global domain at t = 0 (frozen gradient; window keeps it bounded)
+  const double zmax = (double)ctx->cfg.global[2];
+  const double Ts[2] = {p->T0 - fabs(p->G) * p->dx, p->T0 + fabs(p->G) * (zmax + 1) * p->dx};
+  for (double T : Ts)
+    for (int a = 0; a < PF_N; ++a) {
+      double c00 = -2 * (p->A0[a][0][0] + p->A1[a][0][0] * T), c11 = -2 * (p->A0[a][1][1] + p->A1[a][1][1] * T);
+      double c01 = -((p->A0[a][0][1] + p->A1[a][0][1] * T) + (p->A0[a][1][0] + p->A1[a][1][0] * T));
+      if (!(c00 > 0 && c00 * c11 - c01 * c01 > 0))
+        return fail(ctx, PF_EINVAL, "A_%d(T=%g) is not negative definite (dc/dmu must be SPD)", a, T);
+    }
+  // stability bounds
+  const double dt_phi = tmin * p->dx * p->dx / (12.0 * gmax);
+  double deff = 0;
+  {
+    std::vector<std::vector<double>> pts;
+    for (int a = 0; a < PF_N; ++a) {  // vertices, edge / face midpoints, barycentre
+      std::vector<double> v(PF_N, 0.0);
+      v[a] = 1;
+      pts.push_back(v);
+      for (int b = a + 1; b < PF_N; ++b) {
+        std::vector<double> e(PF_N, 0.0);
+        e[a] = e[b] = 0.5;
+        pts.push_back(e);
+        for (int c = b + 1; c < PF_N; ++c) {
+          std::vector<double> f(PF_N, 0.0);
+          f[a] = f[b] = f[c] = 1.0 / 3;
+          pts.push_back(f);
+        }
+      }
+    }
+    pts.push_back(std::vector<double>(PF_N, 0.25));
+    uint64_t s = 20191117ull;  // seeded random points on the simplex
+    for (int i = 0; i < 1000; ++i) {
+      std::vector<double> v(PF_N);
+      double sum = 0;
+      for (int a = 0; a < PF_N; ++a) {
+        s = s * 6364136223846793005ull + 1442695040888963407ull;
+        double u = ((s >> 11) + 0.5) * (1.0 / 9007199254740992.0);
+        v[a] = -log(u);
+        sum += v[a];
+      }
+      for (int a = 0; a < PF_N; ++a) v[a] /= sum;
+      pts.push_back(v);
+    }
+    for (auto& v : pts)
+      for (double T : Ts) deff = std::max(deff, deff_at(*p, v.data(), T));
+  }
+  const double dt_mu = deff > 0 ? p->dx * p->dx / (6.0 * deff) : INFINITY;
+  if (p->dt > dt_phi || p->dt > dt_mu)
+    return fail(ctx, PF_EINVAL, "dt = %g exceeds the explicit stability bound min(%g [phi], %g [mu])", p->dt, dt_phi,
+                dt_mu);
+  // device scalars
+  DevParams& D = ctx->dp;
+  memset(&D, 0, sizeof D);
+  D.dx = p->dx;
+  D.dt = p->dt;
+  D.eps = p->eps;
+  D.inv_dt = 1.0 / p->dt;
+  D.inv_dx2 = 1.0 / (p->dx * p->dx);
+  D.phi_grad_c = p->eps / (p->dx * p->dx);
+  D.inv_eps = 1.0 / p->eps;
+  D.dt_over_eps = p->dt / p->eps;
+  const double pi = 3.14159265358979323846;
+  for (int a = 0; a < PF_N; ++a)
+    for (int b = 0; b < PF_N; ++b) {
+      D.g[a][b] = a == b ? 0.0 : p->gamma[a][b];
+      D.og[a][b] = a == b ? 0.0 : 16.0 / (pi * pi) * p->gamma[a][b];
+    }
+  const int others[4][3] = {{1, 2, 3}, {0, 2, 3}, {0, 1, 3}, {0, 1, 2}};
+  for (int a = 0; a < PF_N; ++a) {
+    const int* o = others[a];
+    D.g3[a][0] = p->gamma3[a][o[0]][o[1]];
+    D.g3[a][1] = p->gamma3[a][o[0]][o[2]];
+    D.g3[a][2] = p->gamma3[a][o[1]][o[2]];
+  }
+  int k = 0;
+  double tm = 0;
+  for (int a = 0; a < PF_N; ++a)
+    for (int b = a + 1; b < PF_N; ++b) {
+      D.tau[k++] = p->tau[a][b];
+      tm += p->tau[a][b];
+    }
+  D.tau_mean = tm / 6.0;
+  for (int a = 0; a < PF_N; ++a) {
+    D.dcT[a][0] = -(p->A1[a][0][0] + p->A1[a][0][0]);
+    D.dcT[a][1] = -(p->A1[a][0][1] + p->A1[a][1][0]);
+    D.dcT[a][2] = -(p->A1[a][1][1] + p->A1[a][1][1]);
+    D.dcT[a][3] = -p->B1[a][0];
+    D.dcT[a][4] = -p->B1[a][1];
+  }
+  D.dTdt = -p->G * p->v;
+  D.at_c = p->dx * pi * p->eps / (8.0 * p->dt);
+  D.mu_inf[0] = p->mu_inf[0];
+  D.mu_inf[1] = p->mu_inf[1];
+  D.T0 = p->T0;
+  D.G = p->G;
+  D.v = p->v;
+  D.liquid = L;
+  ctx->hp = *p;
+  ctx->have_params = true;
+  return PF_OK;
+}
+
+// ---------------------------------------------------------------------------
+// ghost layers of one field set (Alg. 1 lines 2 / 4): local BCs + halo exchange
+// ---------------------------------------------------------------------------
+static int fill_ghosts(pf_ctx* ctx, double* f, int ncomp, bool is_mu) {
+  const double* dir = is_mu ? ctx->hp.mu_inf : nullptr;
+  const bool any_ex = ctx->exchange[0] || ctx->exchange[1] || ctx->exchange[2] || ctx->force_exchange;
+  if (!any_ex) {
+    launch_ghost_fill(ctx->g, ctx->bc_all, f, ncomp, dir, ctx->stream);
+    ctx->nlaunch[2] += 1;
+    return check_launch(ctx, "ghost_fill");
+  }
+  // ordered x -> y -> z stages so that edge ghosts travel with the slabs
+  for (int d = 0; d < 3; ++d) {
+    const bool ex = ctx->exchange[d] || (ctx->force_exchange && ctx->cfg.bc_lo[d] == PF_BC_PERIODIC);
+    if (!ex) {
+      launch_ghost_stage(ctx->g, d, ctx->cfg.bc_lo[d], ctx->cfg.bc_hi[d], f, ncomp, dir, ctx->stream);
+      ctx->nlaunch[2] += 1;
+      if (int r = check_launch(ctx, "ghost_stage")) return r;
+      continue;
+    }
+    const int n = d == 0 ? ctx->g.nx : (d == 1 ? ctx->g.ny : ctx->g.nz);
+    const size_t cnt = halo_slab_elems(ctx->g, d) * ncomp;
+    const int lo = ctx->nb_lo[d] >= 0 ? ctx->nb_lo[d] : -1;
+    const int hi = ctx->nb_hi[d] >= 0 ? ctx->nb_hi[d] : -1;
+    if (hi >= 0) launch_pack(ctx->g, d, n - 1, ncomp, f, ctx->sendbuf[d][1], ctx->stream);
+    if (lo >= 0) launch_pack(ctx->g, d, 0, ncomp, f, ctx->sendbuf[d][0], ctx->stream);
+    ctx->nlaunch[2] += (hi >= 0) + (lo >= 0);
+    if (int r = check_launch(ctx, "pack")) return r;
+    if (ctx->comm) {
+      // per peer pair the k-th send matches the k-th recv: send (hi, lo), recv (lo, hi)
+      NC(g_nccl.GroupStart());
+      if (hi >= 0) NC(g_nccl.Send(ctx->sendbuf[d][1], cnt, ncclDouble, hi, ctx->comm, ctx->stream));
+      if (lo >= 0) NC(g_nccl.Send(ctx->sendbuf[d][0], cnt, ncclDouble, lo, ctx->comm, ctx->stream));
+      if (lo >= 0) NC(g_nccl.Recv(ctx->recvbuf[d][0], cnt, ncclDouble, lo, ctx->comm, ctx->stream));
+      if (hi >= 0) NC(g_nccl.Recv(ctx->recvbuf[d][1], cnt, ncclDouble, hi, ctx->comm, ctx->stream));
+      NC(g_nccl.GroupEnd());
+    } else {
+      // world == 1, periodic self-exchange through the same pack/unpack path
+      CU(cudaMemcpyAsync(ctx->recvbuf[d][0], ctx->sendbuf[d][1], cnt * sizeof(double), cudaMemcpyDeviceToDevice,
+                         ctx->stream));
+      CU(cudaMemcpyAsync(ctx->recvbuf[d][1], ctx->sendbuf[d][0], cnt * sizeof(double), cudaMemcpyDeviceToDevice,
+                         ctx->stream));
+    }
+    if (lo >= 0) launch_unpack(ctx->g, d, -1, ncomp, f, ctx->recvbuf[d][0], ctx->stream);
+    if (hi >= 0) launch_unpack(ctx->g, d, n, ncomp, f, ctx->recvbuf[d][1], ctx->stream);
+    ctx->nlaunch[2] += (hi >= 0) + (lo >= 0);
+    if (int r = check_launch(ctx, "unpack")) return r;
+    if (lo < 0 || hi < 0) {  // physical boundary on one side of an exchanged dimension
+      launch_ghost_stage(ctx->g, d, lo < 0 ? ctx->cfg.bc_lo[d] : -1, hi < 0 ? ctx->cfg.bc_hi[d] : -1, f, ncomp, dir,
+                         ctx->stream);
+      ctx->nlaunch[2] += 1;
+      if (int r = check_launch(ctx, "ghost_stage")) return r;
+    }
+  }
+  return PF_OK;
+}
+
+// ---------------------------------------------------------------------------
+static cudaEvent_t ev_get(pf_ctx* ctx) {
+  if (!ctx->ev_pool.empty()) {
+    cudaEvent_t e = ctx->ev_pool.back();
+    ctx->ev_pool.pop_back();
+    return e;
+  }
+  cudaEvent_t e = nullptr;
+  cudaEventCreate(&e);
+  return e;
+}
+static void prof_begin(pf_ctx* ctx, int k, cudaEvent_t* a) {
+  if (!ctx->prof) return;
+  *a = ev_get(ctx);
+  cudaEventRecord(*a, ctx->stream);
+  (void)k;
+}
+static void prof_end(pf_ctx* ctx, int k, cudaEvent_t a) {
+  if (!ctx->prof) return;
+  cudaEvent_t b = ev_get(ctx);
+  cudaEventRecord(b, ctx->stream);
+  ctx->ev_open.push_back({k, {a, b}});
+  if (ctx->ev_open.size() > 4096) {  // drain to bound the pool
+    cudaEventSynchronize(b);
+    for (auto& o : ctx->ev_open) {
+      float ms = 0;
+      cudaEventElapsedTime(&ms, o.second.first, o.second.second);
+      ctx->prof_ms[o.first] += ms;
+      ctx->prof_n[o.first] += 1;
+      ctx->ev_pool.push_back(o.second.first);
+      ctx->ev_pool.push_back(o.second.second);
+    }
+    ctx->ev_open.clear();
+  }
+}
+
+static int window_maybe(pf_ctx* ctx);
+static int front_height_impl(pf_ctx* ctx, int* H);
+
+static int step_impl(pf_ctx* ctx, bool phi_only) {
+  const Geom& g = ctx->g;
+  double* ps = ctx->phi[ctx->cur];
+  double* pd = ctx->phi[1 - ctx->cur];
+  double* ms = ctx->mu[ctx->cur];
+  double* md = ctx->mu[1 - ctx->cur];
+  const double t = (double)ctx->step * ctx->hp.dt;
+  cudaEvent_t e0 = nullptr;
+  prof_begin(ctx, 3, &e0);
+  launch_tables(ctx->hp, ctx->cfg.liquid, g, t, ctx->z_off, ctx->tab, ctx->stream);
+  ctx->nlaunch[3] += 1;
+  prof_end(ctx, 3, e0);
+  if (int r = check_launch(ctx, "tables")) return r;
+  const Tables T = table_view(ctx->tab, g.nz);
+  // Algorithm 1, line 1: phi-sweep
+  prof_begin(ctx, 0, &e0);
+  if (ctx->variant == PF_VARIANT_NAIVE)
+    launch_phi_naive(ctx->dp, g, T, ps, ms, pd, ctx->stream);
+  else
+    launch_tuned_phi(ctx->dp, g, T, ps, ms, pd, ctx->stream);
+  ctx->nlaunch[0] += 1;
+  prof_end(ctx, 0, e0);
+  if (int r = check_launch(ctx, "phi_sweep")) return r;
+  // line 2: phi_dst communication and boundary handling
+  prof_begin(ctx, 2, &e0);
+  int r = fill_ghosts(ctx, pd, PF_N, false);
+  prof_end(ctx, 2, e0);
+  if (r) return r;
+  if (phi_only) {
+    CU(cudaMemcpyAsync(md, ms, ctx->lay.mu_bytes - 256, cudaMemcpyDeviceToDevice, ctx->stream));
+  } else {
+    // line 3: mu-sweep
+    prof_begin(ctx, 1, &e0);
+    if (ctx->variant == PF_VARIANT_NAIVE)
+      launch_mu_naive(ctx->dp, g, T, ps, pd, ms, md, ctx->stream);
+    else
+      launch_tuned_mu(ctx->dp, g, T, ps, pd, ms, md, ctx->stream);
+    ctx->nlaunch[1] += 1;
+    prof_end(ctx, 1, e0);
+    if (int r2 = check_launch(ctx, "mu_sweep")) return r2;
+    // line 4
+    prof_begin(ctx, 2, &e0);
+    r = fill_ghosts(ctx, md, PF_M, true);
+    prof_end(ctx, 2, e0);
+    if (r) return r;
+  }
+  // line 5: swap
+  ctx->cur = 1 - ctx->cur;
+  ctx->step += 1;
+  return PF_OK;
+}
+
+int pf_step(pf_ctx* ctx, int64_t nsteps) {
+  if (!ctx) return PF_EINVAL;
+  if (!ctx->have_params || !ctx->have_fields) return fail(ctx, PF_ESTATE, "pf_step before pf_set_params/pf_init_fields");
+  if (nsteps < 0) return fail(ctx, PF_EINVAL, "nsteps < 0");
+  for (int64_t n = 0; n < nsteps; ++n) {
+    if (int r = step_impl(ctx, false)) return r;
+    if (int r = window_maybe(ctx)) return r;
+  }
+  return PF_OK;
+}
+
+int pf_step_phi_only(pf_ctx* ctx) {
+  if (!ctx) return PF_EINVAL;
+  if (!ctx->have_params || !ctx->have_fields) return fail(ctx, PF_ESTATE, "step before params/fields");
+  return step_impl(ctx, true);
+}
+
+int pf_halo_exchange(pf_ctx* ctx, unsigned mask) {
+  if (!ctx) return PF_EINVAL;
+  if (!ctx->have_params) return fail(ctx, PF_ESTATE, "pf_halo_exchange before pf_set_params");
+  if (mask & PF_PHI)
+    if (int r = fill_ghosts(ctx, ctx->phi[ctx->cur], PF_N, false)) return r;
+  if (mask & PF_MU)
+    if (int r = fill_ghosts(ctx, ctx->mu[ctx->cur], PF_M, true)) return r;
+  return PF_OK;
+}
+
+// ---------------------------------------------------------------------------
+int pf_init_fields(pf_ctx* ctx, const double* phi, const double* mu, int where) {
+  if (!ctx || !phi || !mu) return PF_EINVAL;
+  if (!ctx->have_params) return fail(ctx, PF_ESTATE, "pf_init_fields before pf_set_params");
+  const Geom& g = ctx->g;
+  const size_t cells = (size_t)g.nx * g.ny * g.nz;
+  const cudaMemcpyKind kind = where == PF_HOST ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
+  ctx->cur = 0;
+  // stage the packed arrays in the (scratch) second time level, then scatter
+  CU(cudaMemcpyAsync(ctx->phi[1], phi, cells * PF_N * sizeof(double), kind, ctx->stream));
+  CU(cudaMemcpyAsync(ctx->mu[1], mu, cells * PF_M * sizeof(double), kind, ctx->stream));
+  launch_copy_interior(g, PF_N, ctx->phi[1], ctx->phi[0], 0, ctx->stream);
+  launch_copy_interior(g, PF_M, ctx->mu[1], ctx->mu[0], 0, ctx->stream);
+  if (int r = check_launch(ctx, "init copy")) return r;
+  ctx->step = 0;
+  ctx->z_off = 0;
+  ctx->have_fields = true;
+  // invariants of the input: |sum phi - 1| <= 1e-12, phi >= 0
+  double mon[2];
+  if (int r = pf_monitor(ctx, mon)) return r;
+  if (!(mon[0] <= 1e-12) || !(mon[1] >= 0.0)) {
+    ctx->have_fields = false;
+    return fail(ctx, PF_EINVAL, "initial phi off the Gibbs simplex: max|sum-1| = %g, min = %g", mon[0], mon[1]);
+  }
+  if (int r = pf_halo_exchange(ctx, PF_PHI | PF_MU)) return r;
+  CU(cudaStreamSynchronize(ctx->stream));
+  return PF_OK;
+}
+
+int pf_download(pf_ctx* ctx, double* phi, double* mu, int where) {
+  if (!ctx || (!phi && !mu)) return PF_EINVAL;
+  if (!ctx->have_fields) return fail(ctx, PF_ESTATE, "pf_download before pf_init_fields");
+  const Geom& g = ctx->g;
+  const size_t cells = (size_t)g.nx * g.ny * g.nz;
+  const cudaMemcpyKind kind = where == PF_HOST ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice;
+  // pack into the scratch time level, then copy out
+  if (phi) {
+    launch_copy_interior(g, PF_N, ctx->phi[ctx->cur], ctx->phi[1 - ctx->cur], 1, ctx->stream);
+    if (int r = check_launch(ctx, "download copy")) return r;
+    CU(cudaMemcpyAsync(phi, ctx->phi[1 - ctx->cur], cells * PF_N * sizeof(double), kind, ctx->stream));
+  }
+  if (mu) {
+    launch_copy_interior(g, PF_M, ctx->mu[ctx->cur], ctx->mu[1 - ctx->cur], 1, ctx->stream);
+    if (int r = check_launch(ctx, "download copy")) return r;
+    CU(cudaMemcpyAsync(mu, ctx->mu[1 - ctx->cur], cells * PF_M * sizeof(double), kind, ctx->stream));
+  }
+  CU(cudaStreamSynchronize(ctx->stream));
+  return PF_OK;
+}
+
+int pf_get_state(const pf_ctx* ctx, pf_state* out) {
+  if (!ctx || !out) return PF_EINVAL;
+  out->step = ctx->step;
+  out->z_off = ctx->z_off;
+  return PF_OK;
+}
+
+int pf_set_state(pf_ctx* ctx, const pf_state* s) {
+  if (!ctx || !s || s->step < 0) return PF_EINVAL;
+  ctx->step = s->step;
+  ctx->z_off = s->z_off;
+  return PF_OK;
+}
+
+int pf_set_variant(pf_ctx* ctx, int variant) {
+  if (!ctx || (variant != PF_VARIANT_TUNED && variant != PF_VARIANT_NAIVE)) return PF_EINVAL;
+  ctx->variant = variant;
+  return PF_OK;
+}
+
+// ---------------------------------------------------------------------------
+// reductions (collective over ranks)
+// ---------------------------------------------------------------------------
+static int allreduce_max_u64(pf_ctx* ctx, unsigned long long* dbuf, int n) {
+  if (!ctx->comm) return PF_OK;
+  NC(g_nccl.AllReduce(dbuf, dbuf, n, ncclUint64, ncclMax, ctx->comm, ctx->stream));
+  return PF_OK;
+}
+
+static int front_height_impl(pf_ctx* ctx, int* H) {
+  // encode H + 1 >= 0 as u64 so that -1 ("no solid") is the identity of max
+  CU(cudaMemsetAsync(ctx->red, 0, 16, ctx->stream));
+  launch_front_height(ctx->g, ctx->cfg.liquid, ctx->phi[ctx->cur], (int*)ctx->red, ctx->stream);
+  ctx->nlaunch[3] += 1;
+  if (int r = check_launch(ctx, "front_height")) return r;
+  if (int r = allreduce_max_u64(ctx, ctx->red, 1)) return r;
+  CU(cudaMemcpyAsync(ctx->pinned, ctx->red, 8, cudaMemcpyDeviceToHost, ctx->stream));
+  CU(cudaStreamSynchronize(ctx->stream));
+  *H = (int)(ctx->pinned[0] & 0xffffffffull) - 1;
+  return PF_OK;
+}
+
+int pf_front_height(pf_ctx* ctx, int* H) {
+  if (!ctx || !H) return PF_EINVAL;
+  if (!ctx->have_fields) return fail(ctx, PF_ESTATE, "no fields");
+  return front_height_impl(ctx, H);
+}
+
+int pf_monitor(pf_ctx* ctx, double out[2]) {
+  if (!ctx || !out) return PF_EINVAL;
+  if (!ctx->have_fields) return fail(ctx, PF_ESTATE, "no fields");
+  CU(cudaMemsetAsync(ctx->red, 0, 16, ctx->stream));
+  launch_monitor(ctx->g, ctx->phi[ctx->cur], ctx->red, ctx->stream);
+  if (int r = check_launch(ctx, "monitor")) return r;
+  if (int r = allreduce_max_u64(ctx, ctx->red, 2)) return r;
+  CU(cudaMemcpyAsync(ctx->pinned, ctx->red, 16, cudaMemcpyDeviceToHost, ctx->stream));
+  CU(cudaStreamSynchronize(ctx->stream));
+  auto dec = [](unsigned long long b) {
+    b = (b & 0x8000000000000000ull) ? (b & 0x7fffffffffffffffull) : ~b;
+    double v;
+    memcpy(&v, &b, 8);
+    return v;
+  };
+  out[0] = dec(ctx->pinned[0]);
+  out[1] = -dec(ctx->pinned[1]);
+  return PF_OK;
+}
+
+// ---------------------------------------------------------------------------
+// moving window (S6) [A16]
+// ---------------------------------------------------------------------------
+int pf_shift_window(pf_ctx* ctx, int k) {
+  if (!ctx) return PF_EINVAL;
+  if (!ctx->have_fields) return fail(ctx, PF_ESTATE, "no fields");
+  const int pz = ctx->cfg.procs[2] < 1 ? 1 : ctx->cfg.procs[2];
+  if (pz != 1) return fail(ctx, PF_EINVAL, "the moving window needs the growth axis unsplit (procs[2] == 1)");
+  if (k < 0 || k > ctx->g.nz) return fail(ctx, PF_EINVAL, "shift %d out of range", k);
+  if (k == 0) return PF_OK;
+  cudaEvent_t e0 = nullptr;
+  prof_begin(ctx, 3, &e0);
+  launch_shift(ctx->g, k, ctx->cfg.liquid, ctx->hp.mu_inf, ctx->phi[ctx->cur], ctx->mu[ctx->cur],
+               ctx->phi[1 - ctx->cur], ctx->mu[1 - ctx->cur], ctx->stream);
+  ctx->nlaunch[3] += 1;
+  prof_end(ctx, 3, e0);
+  if (int r = check_launch(ctx, "shift")) return r;
+  ctx->cur = 1 - ctx->cur;
+  ctx->z_off += k;
+  return pf_halo_exchange(ctx, PF_PHI | PF_MU);
+}
+
+static int window_maybe(pf_ctx* ctx) {
+  const int nc = ctx->hp.window_check;
+  if (nc <= 0 || ctx->step % nc != 0) return PF_OK;
+  int H = -1;
+  if (int r = front_height_impl(ctx, &H)) return r;
+  const int thr = (int)floor(ctx->hp.window_frac * (double)ctx->cfg.global[2]);
+  if (H > thr) return pf_shift_window(ctx, H - thr);
+  return PF_OK;
+}
+
+// ---------------------------------------------------------------------------
+int pf_profile(pf_ctx* ctx, int enable) {
+  if (!ctx) return PF_EINVAL;
+  CU(cudaStreamSynchronize(ctx->stream));
+  for (auto& o : ctx->ev_open) {
+    ctx->ev_pool.push_back(o.second.first);
+    ctx->ev_pool.push_back(o.second.second);
+  }
+  ctx->ev_open.clear();
+  for (int i = 0; i < 4; ++i) {
+    ctx->prof_ms[i] = 0;
+    ctx->prof_n[i] = 0;
+    ctx->nlaunch[i] = 0;
+  }
+  ctx->prof = enable != 0;
+  return PF_OK;
+}
+
+int pf_profile_read(pf_ctx* ctx, double ms[4], int64_t launches[4]) {
+  if (!ctx) return PF_EINVAL;
+  CU(cudaStreamSynchronize(ctx->stream));
+  for (auto& o : ctx->ev_open) {
+    float v = 0;
+    cudaEventElapsedTime(&v, o.second.first, o.second.second);
+    ctx->prof_ms[o.first] += v;
+    ctx->prof_n[o.first] += 1;
+    ctx->ev_pool.push_back(o.second.first);
+    ctx->ev_pool.push_back(o.second.second);
+  }
+  ctx->ev_open.clear();
+  for (int i = 0; i < 4; ++i) {
+    if (ms) ms[i] = ctx->prof_ms[i];
+    if (launches) launches[i] = ctx->nlaunch[i];
+  }
+  return PF_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,497 @@
+// pf_kernels.cu -- coefficient tables, the straightforward ("naive") sweeps,
+// ghost layers, moving window, reductions and field copies.
+//
+// The naive sweeps map one thread to one cell and compute every face flux
+// twice (the paper's "full" kernels).  They are the parity
+// baseline and the ncu reference for the tuned z-marching kernels
+// (pf_tuned.cu).
+#include <math.h>
+
+#include "pf_model.cuh"
+
+namespace pf {
+
+// ---------------------------------------------------------------------------
+// a1: frozen temperature T = T0 + G (z dx - v t) per plane [A13] and the
+// T-dependent coefficients A(T), B(T), C(T) (eq. 6), chi = dc/dmu = -(A+A^T)
+// [A6] and the mobility products P_a = D_a chi_a (eq. 9) [A7].
+// ---------------------------------------------------------------------------
+struct TabArgs {
+  pf_params p;
+  int liquid;
+  int nz, z0;
+  int64_t z_off;
+  double t;
+};
+
+__device__ void coef_at(const pf_params& p, int a, double T, double A[2][2], double B[2], double* C) {
+  for (int i = 0; i < 2; ++i) {
+    for (int j = 0; j < 2; ++j) A[i][j] = p.A0[a][i][j] + p.A1[a][i][j] * T;
+    B[i] = p.B0[a][i] + p.B1[a][i] * T;
+  }
+  *C = p.C0[a] + p.C1[a] * T;
+}
+
+__device__ void face_row(const pf_params& p, int L, double T, double* row) {
+  double chi[N][3], B[N][2];
+  for (int a = 0; a < N; ++a) {
+    double A[2][2], C;
+    coef_at(p, a, T, A, B[a], &C);
+    chi[a][0] = -(A[0][0] + A[0][0]);
+    chi[a][1] = -(A[0][1] + A[1][0]);
+    chi[a][2] = -(A[1][1] + A[1][1]);
+    const double x[2][2] = {{chi[a][0], chi[a][1]}, {chi[a][1], chi[a][2]}};
+    for (int i = 0; i < 2; ++i)
+      for (int j = 0; j < 2; ++j) row[TF_P + 4 * a + 2 * i + j] = p.D[a][i][0] * x[0][j] + p.D[a][i][1] * x[1][j];
+  }
+  for (int s = 0; s < NSOL; ++s) {
+    const int a = solid_phase(L, s);
+    for (int k = 0; k < 3; ++k) row[TF_DCHI + 3 * s + k] = chi[L][k] - chi[a][k];
+    for (int i = 0; i < 2; ++i) row[TF_DB + 2 * s + i] = B[L][i] - B[a][i];
+  }
+  row[TF_SIZE] = 0.0;
+}
+
+__global__ void k_tables(TabArgs A, double* __restrict__ tab) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  const pf_params& p = A.p;
+  const int nz = A.nz;
+  const int liquid = A.liquid;
+  double* cell = tab;
+  double* fxy = tab + (size_t)nz * TC_SIZE;
+  double* fz = fxy + (size_t)nz * TF_STRIDE;
+  auto Tz = [&](double zc) { return p.T0 + p.G * ((zc + (double)A.z0 + (double)A.z_off) * p.dx - p.v * A.t); };
+  if (i < nz) {
+    const double T = Tz((double)i);
+    double* row = cell + (size_t)i * TC_SIZE;
+    for (int a = 0; a < N; ++a) {
+      double Am[2][2], B[2], C;
+      coef_at(p, a, T, Am, B, &C);
+      row[TC_PSI + 6 * a + 0] = Am[0][0];
+      row[TC_PSI + 6 * a + 1] = Am[0][1] + Am[1][0];
+      row[TC_PSI + 6 * a + 2] = Am[1][1];
+      row[TC_PSI + 6 * a + 3] = B[0];
+      row[TC_PSI + 6 * a + 4] = B[1];
+      row[TC_PSI + 6 * a + 5] = C;
+      row[TC_CHI + 3 * a + 0] = -(Am[0][0] + Am[0][0]);
+      row[TC_CHI + 3 * a + 1] = -(Am[0][1] + Am[1][0]);
+      row[TC_CHI + 3 * a + 2] = -(Am[1][1] + Am[1][1]);
+      row[TC_B + 2 * a + 0] = B[0];
+      row[TC_B + 2 * a + 1] = B[1];
+    }
+    face_row(p, liquid, T, fxy + (size_t)i * TF_STRIDE);
+  }
+  if (i <= nz) face_row(p, liquid, Tz((double)i - 0.5), fz + (size_t)i * TF_STRIDE);
+}
+
+size_t table_doubles(int nz) { return (size_t)nz * TC_SIZE + (size_t)nz * TF_STRIDE + (size_t)(nz + 1) * TF_STRIDE; }
+
+Tables table_view(const double* tab, int nz) {
+  Tables T;
+  T.cell = tab;
+  T.fxy = tab + (size_t)nz * TC_SIZE;
+  T.fz = T.fxy + (size_t)nz * TF_STRIDE;
+  return T;
+}
+
+void launch_tables(const pf_params& p, int liquid, const Geom& g, double t, int64_t z_off, double* tab,
+                   cudaStream_t s) {
+  TabArgs A{p, liquid, g.nz, g.z0, z_off, t};
+  const int n = g.nz + 1;
+  k_tables<<<(n + 127) / 128, 128, 0, s>>>(A, tab);
+}
+
+// ---------------------------------------------------------------------------
+// Naive phi-sweep: one thread per cell, 6 faces each (Algorithm 1 line 1).
+// ---------------------------------------------------------------------------
+template <int L>
+__global__ void __launch_bounds__(256) k_phi_naive(DevParams P, Geom g, Tables T, const double* __restrict__ ps,
+                                                   const double* __restrict__ ms, double* __restrict__ pd) {
+  const int x = blockIdx.x * blockDim.x + threadIdx.x;
+  const int y = blockIdx.y * blockDim.y + threadIdx.y;
+  const int z = blockIdx.z * blockDim.z + threadIdx.z;
+  if (x >= g.nx || y >= g.ny || z >= g.nz) return;
+  const int64_t c = g.at(x, y, z);
+  const int64_t F = g.field;
+  const int64_t st[3] = {1, g.pitch, g.plane};
+  double ph[N], gd[N][3], divh[N] = {0.0, 0.0, 0.0, 0.0};
+#pragma unroll
+  for (int a = 0; a < N; ++a) ph[a] = __ldg(ps + a * F + c);
+#pragma unroll
+  for (int d = 0; d < 3; ++d) {
+    double fm[N], fpl[N], jp[N], jm[N];
+#pragma unroll
+    for (int a = 0; a < N; ++a) {
+      fm[a] = __ldg(ps + a * F + c - st[d]);
+      fpl[a] = __ldg(ps + a * F + c + st[d]);
+      gd[a][d] = fpl[a] - fm[a];
+    }
+    phi_face(P, ph, fpl, jp);
+    phi_face(P, fm, ph, jm);
+#pragma unroll
+    for (int a = 0; a < N; ++a) divh[a] += jp[a] - jm[a];
+  }
+  const double mu0 = __ldg(ms + c), mu1 = __ldg(ms + F + c);
+  double out[N];
+  phi_cell(P, T.cell + (size_t)z * TC_SIZE, ph, gd, divh, mu0, mu1, out);
+#pragma unroll
+  for (int a = 0; a < N; ++a) pd[a * F + c] = out[a];
+}
+
+// ---------------------------------------------------------------------------
+// Naive mu-sweep: one thread per cell, 6 faces each (Algorithm 1 line 3).
+// ---------------------------------------------------------------------------
+template <int L>
+__device__ __forceinline__ void mu_face_global(const DevParams& P, const double* __restrict__ frow, const Geom& g,
+                                               const double* __restrict__ ps, const double* __restrict__ pd,
+                                               const double* __restrict__ ms, int64_t p, int64_t sn, int64_t s1,
+                                               int64_t s2, double (&Fh)[M]) {
+  const int64_t F = g.field;
+  const int64_t q = p + sn;
+  double fp[N], fq[N], gt1[N], gt2[N], dsum[NSOL], mp[M], mq[M];
+#pragma unroll
+  for (int a = 0; a < N; ++a) {
+    const double* f = ps + a * F;
+    fp[a] = __ldg(f + p);
+    fq[a] = __ldg(f + q);
+    gt1[a] = 0.25 * ((__ldg(f + p + s1) - __ldg(f + p - s1)) + (__ldg(f + q + s1) - __ldg(f + q - s1)));
+    gt2[a] = 0.25 * ((__ldg(f + p + s2) - __ldg(f + p - s2)) + (__ldg(f + q + s2) - __ldg(f + q - s2)));
+  }
+#pragma unroll
+  for (int s = 0; s < NSOL; ++s) {
+    const int a = solid_phase(L, s);
+    dsum[s] = (__ldg(pd + a * F + p) - fp[a]) + (__ldg(pd + a * F + q) - fq[a]);
+  }
+#pragma unroll
+  for (int i = 0; i < M; ++i) {
+    mp[i] = __ldg(ms + i * F + p);
+    mq[i] = __ldg(ms + i * F + q);
+  }
+  mu_face<L>(P, frow, fp, fq, gt1, gt2, dsum, mp, mq, Fh);
+}
+
+template <int L>
+__global__ void __launch_bounds__(256) k_mu_naive(DevParams P, Geom g, Tables T, const double* __restrict__ ps,
+                                                  const double* __restrict__ pd, const double* __restrict__ ms,
+                                                  double* __restrict__ md) {
+  const int x = blockIdx.x * blockDim.x + threadIdx.x;
+  const int y = blockIdx.y * blockDim.y + threadIdx.y;
+  const int z = blockIdx.z * blockDim.z + threadIdx.z;
+  if (x >= g.nx || y >= g.ny || z >= g.nz) return;
+  const int64_t c = g.at(x, y, z);
+  const int64_t F = g.field;
+  const int64_t st[3] = {1, g.pitch, g.plane};
+  double divh[M] = {0.0, 0.0};
+  const double* fxy = T.fxy + (size_t)z * TF_STRIDE;
+#pragma unroll
+  for (int d = 0; d < 3; ++d) {
+    const int64_t s1 = st[d == 0 ? 1 : 0], s2 = st[d == 2 ? 1 : 2];
+    const double* fr_p = d == 2 ? T.fz + (size_t)(z + 1) * TF_STRIDE : fxy;
+    const double* fr_m = d == 2 ? T.fz + (size_t)z * TF_STRIDE : fxy;
+    double Fp[M], Fm[M];
+    mu_face_global<L>(P, fr_p, g, ps, pd, ms, c, st[d], s1, s2, Fp);
+    mu_face_global<L>(P, fr_m, g, ps, pd, ms, c - st[d], st[d], s1, s2, Fm);
+#pragma unroll
+    for (int i = 0; i < M; ++i) divh[i] += Fp[i] - Fm[i];
+  }
+  double ph[N], phn[N], mu[M], out[M];
+#pragma unroll
+  for (int a = 0; a < N; ++a) {
+    ph[a] = __ldg(ps + a * F + c);
+    phn[a] = __ldg(pd + a * F + c);
+  }
+#pragma unroll
+  for (int i = 0; i < M; ++i) mu[i] = __ldg(ms + i * F + c);
+  mu_cell(P, T.cell + (size_t)z * TC_SIZE, ph, phn, mu, divh, out);
+#pragma unroll
+  for (int i = 0; i < M; ++i) md[i * F + c] = out[i];
+}
+
+#define PF_DISPATCH_L(L, ...)                   \
+  switch (L) {                                  \
+    case 0: { constexpr int LL = 0; __VA_ARGS__; } break; \
+    case 1: { constexpr int LL = 1; __VA_ARGS__; } break; \
+    case 2: { constexpr int LL = 2; __VA_ARGS__; } break; \
+    default: { constexpr int LL = 3; __VA_ARGS__; } break; \
+  }
+
+void launch_phi_naive(const DevParams& P, const Geom& g, const Tables& T, const double* ps, const double* ms,
+                      double* pd, cudaStream_t s) {
+  dim3 b(32, 4, 2), gr((g.nx + 31) / 32, (g.ny + 3) / 4, (g.nz + 1) / 2);
+  PF_DISPATCH_L(P.liquid, (k_phi_naive<LL><<<gr, b, 0, s>>>(P, g, T, ps, ms, pd)));
+}
+
+void launch_mu_naive(const DevParams& P, const Geom& g, const Tables& T, const double* ps, const double* pd,
+                     const double* ms, double* md, cudaStream_t s) {
+  dim3 b(32, 4, 2), gr((g.nx + 31) / 32, (g.ny + 3) / 4, (g.nz + 1) / 2);
+  PF_DISPATCH_L(P.liquid, (k_mu_naive<LL><<<gr, b, 0, s>>>(P, g, T, ps, pd, ms, md)));
+}
+
+// ---------------------------------------------------------------------------
+// Ghost layers (Alg. 1 lines 2 and 4, "communication and boundary handling").
+// Every ghost cell is written from interior values by a per-axis index map,
+// which equals the ordered x -> y -> z fill (edges and corners consistent,
+// SURVEY C.6.6): periodic wrap, Neumann = adjacent interior; a ghost on a
+// Dirichlet side gets mu_inf [A15].  Sides with kind -1 are left alone
+// (filled by the halo exchange).
+// ---------------------------------------------------------------------------
+struct GhostArgs {
+  Geom g;
+  BCSpec bc;
+  int ncomp;
+  double dir[M];
+  int use_dir;
+};
+
+__device__ __forceinline__ int map_axis(int i, int n, int klo, int khi, bool* skip, bool* dirich) {
+  if (i < 0) {
+    if (klo < 0) { *skip = true; return i; }
+    if (klo == PF_BC_DIRICHLET_MU) *dirich = true;
+    return klo == PF_BC_PERIODIC ? n - 1 : 0;
+  }
+  if (i >= n) {
+    if (khi < 0) { *skip = true; return i; }
+    if (khi == PF_BC_DIRICHLET_MU) *dirich = true;
+    return khi == PF_BC_PERIODIC ? 0 : n - 1;
+  }
+  return i;
+}
+
+__global__ void k_ghost(GhostArgs A, double* __restrict__ f) {
+  const Geom& g = A.g;
+  const int64_t sx = g.nx + 2, sy = g.ny + 2;
+  const int64_t nzp = 2 * sx * sy;              // two z ghost planes
+  const int64_t nyr = 2 * sx * (int64_t)g.nz;   // two y ghost rows per interior z
+  const int64_t nxc = 2 * (int64_t)g.ny * g.nz; // two x ghost columns per interior (y,z)
+  const int64_t total = nzp + nyr + nxc;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    int x, y, z;
+    if (i < nzp) {
+      int64_t r = i;
+      z = (r / (sx * sy)) ? g.nz : -1;
+      r %= sx * sy;
+      y = (int)(r / sx) - 1;
+      x = (int)(r % sx) - 1;
+    } else if (i < nzp + nyr) {
+      int64_t r = i - nzp;
+      z = (int)(r / (2 * sx));
+      r %= 2 * sx;
+      y = (r / sx) ? g.ny : -1;
+      x = (int)(r % sx) - 1;
+    } else {
+      int64_t r = i - nzp - nyr;
+      z = (int)(r / (2 * g.ny));
+      r %= 2 * g.ny;
+      y = (int)(r / 2);
+      x = (r % 2) ? g.nx : -1;
+    }
+    bool skip = false, dir = false;
+    const int mx = map_axis(x, g.nx, A.bc.kind_lo[0], A.bc.kind_hi[0], &skip, &dir);
+    const int my = map_axis(y, g.ny, A.bc.kind_lo[1], A.bc.kind_hi[1], &skip, &dir);
+    const int mz = map_axis(z, g.nz, A.bc.kind_lo[2], A.bc.kind_hi[2], &skip, &dir);
+    if (skip) continue;
+    const int64_t dst = (int64_t)(z + 1) * g.plane + (int64_t)(y + 1) * g.pitch + g.xoff + x;
+    const int64_t src = (int64_t)(mz + 1) * g.plane + (int64_t)(my + 1) * g.pitch + g.xoff + mx;
+    for (int c = 0; c < A.ncomp; ++c)
+      f[c * g.field + dst] = (dir && A.use_dir) ? A.dir[c] : f[c * g.field + src];
+  }
+}
+
+void launch_ghost_fill(const Geom& g, const BCSpec& bc, double* f, int ncomp, const double* dirichlet, cudaStream_t s) {
+  GhostArgs A;
+  A.g = g;
+  A.bc = bc;
+  A.ncomp = ncomp;
+  A.use_dir = dirichlet != nullptr;
+  for (int i = 0; i < M; ++i) A.dir[i] = dirichlet ? dirichlet[i] : 0.0;
+  const int64_t total = 2 * (int64_t)(g.nx + 2) * (g.ny + 2) + 2 * (int64_t)(g.nx + 2) * g.nz + 2 * (int64_t)g.ny * g.nz;
+  int blocks = (int)((total + 255) / 256);
+  if (blocks > 148 * 8) blocks = 148 * 8;
+  k_ghost<<<blocks, 256, 0, s>>>(A, f);
+}
+
+// ---------------------------------------------------------------------------
+// Moving window [A16]: dst(z) = src(z + k) for z + k < nz, else inflow
+// (phi = e_l, mu = mu_inf).  Out-of-place; the caller swaps.
+// ---------------------------------------------------------------------------
+__global__ void k_shift(Geom g, int k, int L, double mi0, double mi1, const double* __restrict__ ps,
+                        const double* __restrict__ ms, double* __restrict__ pd, double* __restrict__ md) {
+  const int x = blockIdx.x * blockDim.x + threadIdx.x;
+  const int y = blockIdx.y;
+  const int z = blockIdx.z;
+  if (x >= g.nx) return;
+  const int64_t c = g.at(x, y, z);
+  const bool in = z + k < g.nz;
+  const int64_t sidx = in ? g.at(x, y, z + k) : 0;
+  for (int a = 0; a < N; ++a) pd[a * g.field + c] = in ? ps[a * g.field + sidx] : (a == L ? 1.0 : 0.0);
+  md[c] = in ? ms[sidx] : mi0;
+  md[g.field + c] = in ? ms[g.field + sidx] : mi1;
+}
+
+void launch_shift(const Geom& g, int k, int liquid, const double* mu_inf, const double* ps, const double* ms,
+                  double* pd, double* md, cudaStream_t s) {
+  dim3 b(128), gr((g.nx + 127) / 128, g.ny, g.nz);
+  k_shift<<<gr, b, 0, s>>>(g, k, liquid, mu_inf[0], mu_inf[1], ps, ms, pd, md);
+}
+
+// front height: max z with phi_l < 1/2 (deterministic integer max)
+__global__ void k_front(Geom g, const double* __restrict__ phl, int* out) {
+  const int x = blockIdx.x * blockDim.x + threadIdx.x;
+  const int y = blockIdx.y, z = blockIdx.z;
+  bool hit = x < g.nx && phl[g.at(x, y, z)] < 0.5;
+  if (__any_sync(0xffffffffu, hit) && (threadIdx.x & 31) == 0) atomicMax(out, z + g.z0 + 1);  // H + 1
+}
+
+void launch_front_height(const Geom& g, int liquid, const double* phi, int* out, cudaStream_t s) {
+  dim3 b(128), gr((g.nx + 127) / 128, g.ny, g.nz);
+  k_front<<<gr, b, 0, s>>>(g, phi + (int64_t)liquid * g.field, out);
+}
+
+// monitors: out[0] = max |sum phi - 1| (as ordered bits), out[1] = max(-min phi) encoded
+__device__ __forceinline__ unsigned long long ord_bits(double v) {
+  // order-preserving map of doubles to unsigned (max over the map = max over values)
+  unsigned long long b = (unsigned long long)__double_as_longlong(v);
+  return (b & 0x8000000000000000ull) ? ~b : (b | 0x8000000000000000ull);
+}
+
+__global__ void k_monitor(Geom g, const double* __restrict__ ph, unsigned long long* out) {
+  const int x = blockIdx.x * blockDim.x + threadIdx.x;
+  const int y = blockIdx.y, z = blockIdx.z;
+  double e = -1.0, neg = -INFINITY;
+  if (x < g.nx) {
+    const int64_t c = g.at(x, y, z);
+    double s = 0.0, mn = INFINITY;
+    for (int a = 0; a < N; ++a) {
+      const double v = ph[a * g.field + c];
+      s += v;
+      mn = fmin(mn, v);
+    }
+    e = fabs(s - 1.0);
+    neg = -mn;
+  }
+  for (int o = 16; o > 0; o >>= 1) {
+    e = fmax(e, __shfl_xor_sync(0xffffffffu, e, o));
+    neg = fmax(neg, __shfl_xor_sync(0xffffffffu, neg, o));
+  }
+  if ((threadIdx.x & 31) == 0) {
+    atomicMax(out, ord_bits(e));
+    atomicMax(out + 1, ord_bits(neg));
+  }
+}
+
+void launch_monitor(const Geom& g, const double* phi, unsigned long long* out2, cudaStream_t s) {
+  dim3 b(128), gr((g.nx + 127) / 128, g.ny, g.nz);
+  k_monitor<<<gr, b, 0, s>>>(g, phi, out2);
+}
+
+// interior <-> packed [comp][z][y][x] copies
+__global__ void k_copy(Geom g, int ncomp, const double* __restrict__ src, double* __restrict__ dst, int to_packed) {
+  const int x = blockIdx.x * blockDim.x + threadIdx.x;
+  const int y = blockIdx.y, z = blockIdx.z;
+  if (x >= g.nx) return;
+  const int64_t c = g.at(x, y, z);
+  const int64_t pk = ((int64_t)z * g.ny + y) * g.nx + x;
+  const int64_t pstride = (int64_t)g.nx * g.ny * g.nz;
+  for (int a = 0; a < ncomp; ++a) {
+    if (to_packed)
+      dst[a * pstride + pk] = src[a * g.field + c];
+    else
+      dst[a * g.field + c] = src[a * pstride + pk];
+  }
+}
+
+void launch_copy_interior(const Geom& g, int ncomp, const double* src, double* dst, int to_packed, cudaStream_t s) {
+  dim3 b(128), gr((g.nx + 127) / 128, g.ny, g.nz);
+  k_copy<<<gr, b, 0, s>>>(g, ncomp, src, dst, to_packed);
+}
+
+// ---------------------------------------------------------------------------
+// Halo pack / unpack along dimension d for the ordered x -> y -> z exchange:
+// the slab covers the interior range of the dimensions after d and the full
+// ghosted range of the dimensions before d, so that edge ghosts travel.
+// ---------------------------------------------------------------------------
+__host__ __device__ inline void slab_dims(const Geom& g, int d, int* n0, int* n1, int* o0, int* o1) {
+  // (u, w) = the two other axes in ascending order
+  const int n[3] = {g.nx, g.ny, g.nz};
+  const int u = d == 0 ? 1 : 0, w = d == 2 ? 1 : 2;
+  *n0 = u < d ? n[u] + 2 : n[u];
+  *o0 = u < d ? -1 : 0;
+  *n1 = w < d ? n[w] + 2 : n[w];
+  *o1 = w < d ? -1 : 0;
+}
+
+size_t halo_slab_elems(const Geom& g, int d) {
+  int n0, n1, o0, o1;
+  slab_dims(g, d, &n0, &n1, &o0, &o1);
+  return (size_t)n0 * n1;
+}
+
+__global__ void k_pack(Geom g, int d, int idx, int ncomp, double* __restrict__ f, double* __restrict__ buf, int unpack) {
+  int n0, n1, o0, o1;
+  slab_dims(g, d, &n0, &n1, &o0, &o1);
+  const int64_t tot = (int64_t)n0 * n1;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < tot; i += (int64_t)gridDim.x * blockDim.x) {
+    const int i0 = (int)(i % n0) + o0, i1 = (int)(i / n0) + o1;
+    int c[3];
+    c[d] = idx;
+    c[d == 0 ? 1 : 0] = i0;
+    c[d == 2 ? 1 : 2] = i1;
+    const int64_t li = (int64_t)(c[2] + 1) * g.plane + (int64_t)(c[1] + 1) * g.pitch + g.xoff + c[0];
+    for (int a = 0; a < ncomp; ++a) {
+      if (unpack)
+        f[a * g.field + li] = buf[a * tot + i];
+      else
+        buf[a * tot + i] = f[a * g.field + li];
+    }
+  }
+}
+
+void launch_pack(const Geom& g, int d, int idx, int ncomp, const double* f, double* buf, cudaStream_t s) {
+  const size_t tot = halo_slab_elems(g, d);
+  int blocks = (int)((tot + 255) / 256);
+  if (blocks > 148 * 4) blocks = 148 * 4;
+  k_pack<<<blocks, 256, 0, s>>>(g, d, idx, ncomp, const_cast<double*>(f), buf, 0);
+}
+
+// one stage of the ordered ghost fill: the d-ghost slabs (extended ranges of
+// the dimensions before d), kinds per side (-1 = leave alone)
+__global__ void k_ghost_stage(Geom g, int d, int klo, int khi, int ncomp, double* __restrict__ f, double dir0,
+                              double dir1, int use_dir) {
+  int n0, n1, o0, o1;
+  slab_dims(g, d, &n0, &n1, &o0, &o1);
+  const int n[3] = {g.nx, g.ny, g.nz};
+  const int64_t tot = (int64_t)n0 * n1;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < 2 * tot; i += (int64_t)gridDim.x * blockDim.x) {
+    const int side = i >= tot;
+    const int kind = side ? khi : klo;
+    if (kind < 0) continue;
+    const int64_t j = i - side * tot;
+    int c[3], s[3];
+    c[d == 0 ? 1 : 0] = s[d == 0 ? 1 : 0] = (int)(j % n0) + o0;
+    c[d == 2 ? 1 : 2] = s[d == 2 ? 1 : 2] = (int)(j / n0) + o1;
+    c[d] = side ? n[d] : -1;
+    s[d] = kind == PF_BC_PERIODIC ? (side ? 0 : n[d] - 1) : (side ? n[d] - 1 : 0);
+    const bool dirich = kind == PF_BC_DIRICHLET_MU && use_dir;
+    const int64_t li = (int64_t)(c[2] + 1) * g.plane + (int64_t)(c[1] + 1) * g.pitch + g.xoff + c[0];
+    const int64_t si = (int64_t)(s[2] + 1) * g.plane + (int64_t)(s[1] + 1) * g.pitch + g.xoff + s[0];
+    for (int a = 0; a < ncomp; ++a) f[a * g.field + li] = dirich ? (a == 0 ? dir0 : dir1) : f[a * g.field + si];
+  }
+}
+
+void launch_ghost_stage(const Geom& g, int d, int klo, int khi, double* f, int ncomp, const double* dirichlet,
+                        cudaStream_t s) {
+  const size_t tot = 2 * halo_slab_elems(g, d);
+  int blocks = (int)((tot + 255) / 256);
+  if (blocks > 148 * 4) blocks = 148 * 4;
+  k_ghost_stage<<<blocks, 256, 0, s>>>(g, d, klo, khi, ncomp, f, dirichlet ? dirichlet[0] : 0.0,
+                                       dirichlet ? dirichlet[1] : 0.0, dirichlet != nullptr);
+}
+
+void launch_unpack(const Geom& g, int d, int idx, int ncomp, double* f, const double* buf, cudaStream_t s) {
+  const size_t tot = halo_slab_elems(g, d);
+  int blocks = (int)((tot + 255) / 256);
+  if (blocks > 148 * 4) blocks = 148 * 4;
+  k_pack<<<blocks, 256, 0, s>>>(g, d, idx, ncomp, f, const_cast<double*>(buf), 1);
+}
+
+}  // namespace pf

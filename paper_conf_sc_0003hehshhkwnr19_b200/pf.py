@@ -1,0 +1,308 @@
+"""Thin ctypes binding of the C ABI in include/pf.h (argument marshalling only).
+
+Every step of the method runs in the CUDA kernels of libpf.so; PyTorch only
+provides device memory (the caller-owned buffers of pf_config), the stream
+and, for world > 1, the process group used to broadcast the NCCL id.  There
+is no CPU fallback: if libpf.so or a CUDA device is missing, this module
+raises.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(PKG, "libpf.so")
+
+PF_OK, PF_EINVAL, PF_ENOMEM, PF_ECUDA, PF_ENCCL, PF_ESTATE, PF_ENUMERIC = 0, -1, -2, -3, -4, -5, -6
+BC = {"periodic": 0, "neumann": 1, "dirichlet_mu": 2}
+PF_HOST, PF_DEVICE = 0, 1
+PF_PHI, PF_MU = 1, 2
+VARIANT = {"tuned": 0, "naive": 1}
+N, M = 4, 2
+
+
+class PFConfig(C.Structure):
+    _fields_ = [("n_phases", C.c_int), ("n_mu", C.c_int), ("liquid", C.c_int),
+                ("global_", C.c_int * 3), ("procs", C.c_int * 3),
+                ("bc_lo", C.c_int * 3), ("bc_hi", C.c_int * 3),
+                ("rank", C.c_int), ("world", C.c_int),
+                ("nccl_uid", C.c_ubyte * 128), ("device", C.c_int), ("stream", C.c_void_p),
+                ("phi", C.c_void_p * 2), ("mu", C.c_void_p * 2), ("workspace", C.c_void_p)]
+
+
+class PFLayout(C.Structure):
+    _fields_ = [("local", C.c_int * 3), ("offset", C.c_int * 3),
+                ("pitch", C.c_int64), ("plane", C.c_int64), ("field", C.c_int64), ("x_off", C.c_int64),
+                ("phi_bytes", C.c_size_t), ("mu_bytes", C.c_size_t), ("workspace_bytes", C.c_size_t)]
+
+
+class PFParams(C.Structure):
+    _fields_ = [("dx", C.c_double), ("dt", C.c_double), ("eps", C.c_double),
+                ("gamma", C.c_double * N * N), ("gamma3", C.c_double * N * N * N), ("tau", C.c_double * N * N),
+                ("A0", C.c_double * M * M * N), ("A1", C.c_double * M * M * N),
+                ("B0", C.c_double * M * N), ("B1", C.c_double * M * N),
+                ("C0", C.c_double * N), ("C1", C.c_double * N),
+                ("D", C.c_double * M * M * N),
+                ("T0", C.c_double), ("G", C.c_double), ("v", C.c_double),
+                ("mu_inf", C.c_double * M), ("window_frac", C.c_double), ("window_check", C.c_int)]
+
+
+class PFState(C.Structure):
+    _fields_ = [("step", C.c_int64), ("z_off", C.c_int64)]
+
+
+# every symbol include/pf.h declares (checked by tests/test_abi.py)
+ABI_SYMBOLS = ["pf_query_layout", "pf_create", "pf_destroy", "pf_set_params", "pf_init_fields", "pf_step",
+               "pf_step_phi_only", "pf_halo_exchange", "pf_shift_window", "pf_front_height", "pf_monitor",
+               "pf_download", "pf_get_state", "pf_set_state", "pf_set_variant", "pf_profile", "pf_profile_read",
+               "pf_nccl_unique_id", "pf_last_error", "pf_version"]
+
+_lib = None
+
+
+def load_library(path: str = LIB_PATH):
+    """Load libpf.so (no CUDA device needed just to load it)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(path):
+        raise RuntimeError(f"CUDA extension missing: {path} (run __graft_entry__.build())")
+    L = C.CDLL(path)
+    vp, ip = C.c_void_p, C.c_int
+    dp = C.POINTER(C.c_double)
+    L.pf_query_layout.argtypes = [C.POINTER(PFConfig), C.POINTER(PFLayout)]
+    L.pf_create.argtypes = [C.POINTER(PFConfig), C.POINTER(vp)]
+    L.pf_destroy.argtypes = [vp]
+    L.pf_set_params.argtypes = [vp, C.POINTER(PFParams)]
+    L.pf_init_fields.argtypes = [vp, vp, vp, ip]
+    L.pf_step.argtypes = [vp, C.c_int64]
+    L.pf_step_phi_only.argtypes = [vp]
+    L.pf_halo_exchange.argtypes = [vp, C.c_uint]
+    L.pf_shift_window.argtypes = [vp, ip]
+    L.pf_front_height.argtypes = [vp, C.POINTER(ip)]
+    L.pf_monitor.argtypes = [vp, dp]
+    L.pf_download.argtypes = [vp, vp, vp, ip]
+    L.pf_get_state.argtypes = [vp, C.POINTER(PFState)]
+    L.pf_set_state.argtypes = [vp, C.POINTER(PFState)]
+    L.pf_set_variant.argtypes = [vp, ip]
+    L.pf_profile.argtypes = [vp, ip]
+    L.pf_profile_read.argtypes = [vp, dp, C.POINTER(C.c_int64)]
+    L.pf_nccl_unique_id.argtypes = [C.POINTER(C.c_ubyte)]
+    L.pf_last_error.argtypes = [vp]
+    L.pf_last_error.restype = C.c_char_p
+    L.pf_version.restype = C.c_char_p
+    _lib = L
+    return L
+
+
+class PFError(RuntimeError):
+    pass
+
+
+def make_params(P: dict) -> PFParams:
+    p = PFParams()
+    assert int(P["N"]) == N and int(P["M"]) == M, "the CUDA path is specialised to N = 4, M = 2"
+
+    def put(dst, arr, shape):
+        arr = np.asarray(arr, dtype=np.float64)
+        assert arr.shape == shape, (arr.shape, shape)
+        for ix in np.ndindex(*shape):
+            o = dst
+            for k in ix[:-1]:
+                o = o[k]
+            o[ix[-1]] = float(arr[ix])
+
+    p.dx, p.dt, p.eps = float(P["dx"]), float(P["dt"]), float(P["eps"])
+    put(p.gamma, P["gamma"], (N, N))
+    put(p.gamma3, P["gamma3"], (N, N, N))
+    put(p.tau, P["tau"], (N, N))
+    put(p.A0, P["A0"], (N, M, M))
+    put(p.A1, P["A1"], (N, M, M))
+    put(p.B0, P["B0"], (N, M))
+    put(p.B1, P["B1"], (N, M))
+    put(p.C0, P["C0"], (N,))
+    put(p.C1, P["C1"], (N,))
+    put(p.D, P["D"], (N, M, M))
+    p.T0, p.G, p.v = float(P["T0"]), float(P["G"]), float(P["v"])
+    put(p.mu_inf, P["mu_inf"], (M,))
+    p.window_frac = float(P.get("window_frac", 0.5))
+    p.window_check = int(P.get("window_check", 0))
+    return p
+
+
+def nccl_unique_id() -> bytes:
+    buf = (C.c_ubyte * 128)()
+    r = load_library().pf_nccl_unique_id(buf)
+    if r != PF_OK:
+        raise PFError(f"pf_nccl_unique_id failed ({r})")
+    return bytes(buf)
+
+
+class PhaseField:
+    """One block of the global domain on one GPU (one rank).
+
+    shape = global (nz, ny, nx); procs = rank grid (px, py, pz); bc = dict
+    {"lo": (x, y, z), "hi": (x, y, z)} of "periodic" / "neumann" /
+    "dirichlet_mu".  Buffers are torch tensors owned by this object.
+    """
+
+    def __init__(self, shape, params: dict, bc=None, liquid: int = 3, procs=(1, 1, 1), rank: int = 0,
+                 world: int = 1, device: int | None = None, nccl_uid: bytes | None = None, stream=None):
+        import torch
+        if not torch.cuda.is_available():
+            raise PFError("no CUDA device: the phase-field step has no CPU fallback")
+        self.lib = load_library()
+        self.torch = torch
+        dev = torch.cuda.current_device() if device is None else int(device)
+        self.device = torch.device("cuda", dev)
+        self.stream = stream if stream is not None else torch.cuda.current_stream(self.device)
+        nz, ny, nx = shape
+        bc = bc or {"lo": ("periodic",) * 3, "hi": ("periodic",) * 3}
+        cfg = PFConfig()
+        cfg.n_phases, cfg.n_mu, cfg.liquid = N, M, int(liquid)
+        for d, n in enumerate((nx, ny, nz)):
+            cfg.global_[d] = n
+            cfg.procs[d] = int(procs[d])
+            cfg.bc_lo[d] = BC[bc["lo"][d]]
+            cfg.bc_hi[d] = BC[bc["hi"][d]]
+        cfg.rank, cfg.world = int(rank), int(world)
+        if nccl_uid is not None:
+            for i, b in enumerate(nccl_uid[:128]):
+                cfg.nccl_uid[i] = b
+        cfg.device = dev
+        cfg.stream = self.stream.cuda_stream
+        lay = PFLayout()
+        self._check(self.lib.pf_query_layout(C.byref(cfg), C.byref(lay)), "pf_query_layout", ctx=False)
+        self.layout = lay
+        self.local = (lay.local[2], lay.local[1], lay.local[0])
+        self.offset = (lay.offset[2], lay.offset[1], lay.offset[0])
+        u8 = torch.uint8
+        self._phi = [torch.empty(lay.phi_bytes, dtype=u8, device=self.device) for _ in range(2)]
+        self._mu = [torch.empty(lay.mu_bytes, dtype=u8, device=self.device) for _ in range(2)]
+        self._ws = torch.zeros(lay.workspace_bytes, dtype=u8, device=self.device)
+        for i in range(2):
+            self._phi[i].zero_()
+            self._mu[i].zero_()
+            cfg.phi[i] = self._phi[i].data_ptr()
+            cfg.mu[i] = self._mu[i].data_ptr()
+        cfg.workspace = self._ws.data_ptr()
+        self._cfg = cfg
+        h = C.c_void_p()
+        r = self.lib.pf_create(C.byref(cfg), C.byref(h))
+        self._h = h
+        if r != PF_OK:
+            msg = self.lib.pf_last_error(h).decode() if h.value else ""
+            raise PFError(f"pf_create failed ({r}): {msg}")
+        self.set_params(params)
+
+    # -- helpers ---------------------------------------------------------
+    def _check(self, r, what, ctx=True):
+        if r != PF_OK:
+            msg = self.lib.pf_last_error(self._h).decode() if ctx else ""
+            raise PFError(f"{what} failed ({r}): {msg}")
+
+    def close(self):
+        if getattr(self, "_h", None) is not None and self._h.value:
+            self.lib.pf_destroy(self._h)
+            self._h = C.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # -- the ABI ---------------------------------------------------------
+    def set_params(self, params: dict):
+        self.params = dict(params)
+        self._p = make_params(params)
+        self._check(self.lib.pf_set_params(self._h, C.byref(self._p)), "pf_set_params")
+
+    def init_fields(self, phi, mu):
+        """phi [4][nz][ny][nx], mu [2][nz][ny][nx] block-local; numpy (host)
+        or torch (host or cuda) float64, C-contiguous."""
+        torch = self.torch
+        if isinstance(phi, torch.Tensor):
+            assert phi.dtype == torch.float64 and mu.dtype == torch.float64
+            phi, mu = phi.contiguous(), mu.contiguous()
+            where = PF_DEVICE if phi.is_cuda else PF_HOST
+            pp, mp = phi.data_ptr(), mu.data_ptr()
+            keep = (phi, mu)
+        else:
+            phi = np.ascontiguousarray(phi, dtype=np.float64)
+            mu = np.ascontiguousarray(mu, dtype=np.float64)
+            where = PF_HOST
+            pp, mp = phi.ctypes.data, mu.ctypes.data
+            keep = (phi, mu)
+        assert tuple(phi.shape) == (N,) + self.local and tuple(mu.shape) == (M,) + self.local, (phi.shape, self.local)
+        self._check(self.lib.pf_init_fields(self._h, C.c_void_p(pp), C.c_void_p(mp), where), "pf_init_fields")
+        del keep
+
+    def step(self, n: int = 1):
+        self._check(self.lib.pf_step(self._h, int(n)), "pf_step")
+
+    def step_phi_only(self):
+        self._check(self.lib.pf_step_phi_only(self._h), "pf_step_phi_only")
+
+    def halo_exchange(self, mask: int = PF_PHI | PF_MU):
+        self._check(self.lib.pf_halo_exchange(self._h, int(mask)), "pf_halo_exchange")
+
+    def shift_window(self, k: int):
+        self._check(self.lib.pf_shift_window(self._h, int(k)), "pf_shift_window")
+
+    def front_height(self) -> int:
+        h = C.c_int(0)
+        self._check(self.lib.pf_front_height(self._h, C.byref(h)), "pf_front_height")
+        return h.value
+
+    def monitor(self):
+        out = (C.c_double * 2)()
+        self._check(self.lib.pf_monitor(self._h, out), "pf_monitor")
+        return float(out[0]), float(out[1])
+
+    def download(self, out=None, device: bool = False):
+        """Interior fields; numpy by default, torch cuda tensors if device=True,
+        or into given pinned/cuda torch tensors `out=(phi, mu)`."""
+        torch = self.torch
+        if out is not None:
+            phi, mu = out
+            where = PF_DEVICE if phi.is_cuda else PF_HOST
+            self._check(self.lib.pf_download(self._h, C.c_void_p(phi.data_ptr()), C.c_void_p(mu.data_ptr()), where),
+                        "pf_download")
+            return phi, mu
+        if device:
+            phi = torch.empty((N,) + self.local, dtype=torch.float64, device=self.device)
+            mu = torch.empty((M,) + self.local, dtype=torch.float64, device=self.device)
+            self._check(self.lib.pf_download(self._h, C.c_void_p(phi.data_ptr()), C.c_void_p(mu.data_ptr()),
+                                             PF_DEVICE), "pf_download")
+            return phi, mu
+        phi = np.empty((N,) + self.local)
+        mu = np.empty((M,) + self.local)
+        self._check(self.lib.pf_download(self._h, C.c_void_p(phi.ctypes.data), C.c_void_p(mu.ctypes.data), PF_HOST),
+                    "pf_download")
+        return phi, mu
+
+    def state(self):
+        s = PFState()
+        self._check(self.lib.pf_get_state(self._h, C.byref(s)), "pf_get_state")
+        return {"step": s.step, "z_off": s.z_off}
+
+    def set_state(self, step: int, z_off: int):
+        s = PFState(int(step), int(z_off))
+        self._check(self.lib.pf_set_state(self._h, C.byref(s)), "pf_set_state")
+
+    def set_variant(self, name: str):
+        self._check(self.lib.pf_set_variant(self._h, VARIANT[name]), "pf_set_variant")
+
+    def profile(self, enable: bool = True):
+        self._check(self.lib.pf_profile(self._h, int(enable)), "pf_profile")
+
+    def profile_read(self):
+        ms = (C.c_double * 4)()
+        n = (C.c_int64 * 4)()
+        self._check(self.lib.pf_profile_read(self._h, ms, n), "pf_profile_read")
+        keys = ("phi_sweep", "mu_sweep", "ghost", "window")
+        return {k: (float(ms[i]), int(n[i])) for i, k in enumerate(keys)}

@@ -1,0 +1,88 @@
+"""CPU-side checks of the C ABI (-m "not gpu"): libpf.so builds for sm_100a,
+loads without a GPU, exports every function include/pf.h declares, and the
+ctypes mirrors of the ABI structs match the C layout (sizes and offsets
+measured by compiling a probe against include/pf.h with the host compiler).
+No compute calls are made here."""
+import ctypes as C
+import os
+import re
+import subprocess
+import tempfile
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HDR = os.path.join(ROOT, "include", "pf.h")
+
+
+def declared_functions():
+    src = open(HDR).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"^\s*(?:const\s+)?\w+\**\s+\**(pf_\w+)\s*\(", src, flags=re.M)))
+
+
+@pytest.fixture(scope="module")
+def lib():
+    from paper_conf_sc_0003hehshhkwnr19_b200 import build, pf
+    build.build()
+    return pf.load_library()
+
+
+def test_header_declares_the_north_star_calls():
+    f = declared_functions()
+    for name in ("pf_create", "pf_set_params", "pf_init_fields", "pf_step", "pf_halo_exchange",
+                 "pf_shift_window", "pf_download"):
+        assert name in f
+
+
+def test_library_exports_every_declared_symbol(lib):
+    from paper_conf_sc_0003hehshhkwnr19_b200 import pf
+    decl = declared_functions()
+    assert sorted(pf.ABI_SYMBOLS) == decl
+    for name in decl:
+        assert hasattr(lib, name), name
+    assert b"sm_100a" in lib.pf_version()
+
+
+def test_library_is_sm100a_cubin():
+    from paper_conf_sc_0003hehshhkwnr19_b200 import build
+    so = build.build()
+    out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "--list-elf", so], capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+
+
+def test_struct_layout_matches_c(lib):
+    from paper_conf_sc_0003hehshhkwnr19_b200 import pf
+    probe = r'''
+#include <stdio.h>
+#include <stddef.h>
+#include "pf.h"
+int main(void) {
+  printf("%zu %zu %zu %zu\n", sizeof(pf_config), sizeof(pf_layout), sizeof(pf_params), sizeof(pf_state));
+  printf("%zu %zu %zu %zu\n", offsetof(pf_config, stream), offsetof(pf_config, workspace),
+         offsetof(pf_params, D), offsetof(pf_params, window_check));
+  printf("%zu %zu\n", offsetof(pf_layout, pitch), offsetof(pf_layout, workspace_bytes));
+  return 0;
+}
+'''
+    with tempfile.TemporaryDirectory() as d:
+        c = os.path.join(d, "probe.c")
+        open(c, "w").write(probe)
+        exe = os.path.join(d, "probe")
+        subprocess.check_call(["gcc", "-std=c99", "-I", os.path.dirname(HDR), c, "-o", exe])
+        vals = [int(v) for v in subprocess.check_output([exe], text=True).split()]
+    got = [C.sizeof(pf.PFConfig), C.sizeof(pf.PFLayout), C.sizeof(pf.PFParams), C.sizeof(pf.PFState),
+           pf.PFConfig.stream.offset, pf.PFConfig.workspace.offset, pf.PFParams.D.offset,
+           pf.PFParams.window_check.offset, pf.PFLayout.pitch.offset, pf.PFLayout.workspace_bytes.offset]
+    assert got == vals
+
+
+def test_no_oracle_in_product_path():
+    """The product package never imports or links the oracle (task rule 3)."""
+    pkg = os.path.join(ROOT, "paper_conf_sc_0003hehshhkwnr19_b200")
+    for dp, _, files in os.walk(pkg):
+        for f in files:
+            if f.endswith((".py", ".cu", ".cuh", ".h")):
+                s = open(os.path.join(dp, f)).read()
+                for pat in (r"^\s*(from|import)\s+oracle", r"#include\s+[<\"].*oracle", r"pf_oracle", r"oracle_\w+\("):
+                    assert not re.search(pat, s, flags=re.M), (f, pat)

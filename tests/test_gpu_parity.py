@@ -1,0 +1,213 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on
+the same seeded inputs (pin P13).  -m gpu.
+
+Bar (BASELINE.json north_star): relative L-inf per field, max|x - x_ref| /
+max|x_ref| [A21], <= 1e-12 after one step and <= 1e-9 after 1000 steps.
+"""
+import os
+
+import numpy as np
+import pytest
+
+from paper_conf_sc_0003hehshhkwnr19_b200 import inputs as I
+
+pytestmark = pytest.mark.gpu
+
+TOL_1 = 1e-12
+TOL_1000 = 1e-9
+
+
+def rel_linf(a, b):
+    return float(np.abs(a - b).max() / max(np.abs(b).max(), 1e-300))
+
+
+@pytest.fixture(scope="module")
+def pfmod():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.fail("GPU test without a CUDA device")
+    from paper_conf_sc_0003hehshhkwnr19_b200 import build, pf
+    build.build()
+    return pf
+
+
+@pytest.fixture(scope="module")
+def omod():
+    from oracle import oracle as O
+    O.build()
+    O.set_threads(min(16, os.cpu_count() or 1))
+    return O
+
+
+def run_pair(pfmod, omod, shape, P, ic, steps, bc=None, seed=20191117, variant="tuned", chunks=None, ic_kw=None):
+    phi, mu = I.make_ic(ic, shape, seed=seed, **(ic_kw or {}))
+    g = pfmod.PhaseField(shape, P, bc=bc)
+    g.set_variant(variant)
+    g.init_fields(phi, mu)
+    o = omod.Oracle(shape, P, bc)
+    o.init(phi, mu)
+    out = []
+    done = 0
+    for target in (chunks or [steps]):
+        g.step(target - done)
+        o.step(target - done)
+        done = target
+        gp, gm = g.download()
+        op, om = o.download()
+        out.append((target, rel_linf(gp, op), rel_linf(gm, om), g.state(), o.state()))
+    return out
+
+
+@pytest.mark.parametrize("variant", ["tuned", "naive"])
+@pytest.mark.parametrize("pset", ["c4", "stress"])
+@pytest.mark.parametrize("ic", ["R", "V", "L"])
+def test_one_step_parity(pfmod, omod, variant, pset, ic):
+    P = I.params_c4() if pset == "c4" else I.params_stress()
+    shape = (20, 24, 40)  # several tiles and a ragged tail in x
+    for t, ep, em, gs, os_ in run_pair(pfmod, omod, shape, P, ic, 1, variant=variant):
+        assert ep <= TOL_1 and em <= TOL_1, (ep, em)
+
+
+@pytest.mark.parametrize("shape", [(1, 1, 1), (3, 5, 7), (17, 9, 33), (8, 8, 130)])
+def test_ragged_and_tiny_shapes(pfmod, omod, shape):
+    P = I.params_stress()
+    for t, ep, em, *_ in run_pair(pfmod, omod, shape, P, "R", 2):
+        assert ep <= TOL_1 and em <= TOL_1, (shape, ep, em)
+
+
+def test_config1_50_steps(pfmod, omod):
+    """config 1: 32^3 periodic, 50 explicit steps, single device vs oracle."""
+    P = I.params_c4()
+    res = run_pair(pfmod, omod, (32, 32, 32), P, "V", 50, chunks=[1, 2, 5, 10, 50])
+    for t, ep, em, *_ in res:
+        assert ep <= 1e-11 and em <= 1e-11, (t, ep, em)
+
+
+def test_1000_steps(pfmod, omod):
+    P = I.params_stress()
+    res = run_pair(pfmod, omod, (16, 16, 16), P, "V", 1000, chunks=[1, 100, 1000])
+    for t, ep, em, *_ in res:
+        tol = TOL_1 if t == 1 else TOL_1000
+        assert ep <= tol and em <= tol, (t, ep, em)
+
+
+def test_ds_window_parity(pfmod, omod):
+    """config 2 structure at small size: DS BCs, frozen T, moving window."""
+    P = I.params_c4("ds", window_check=5, window_frac=0.5, v=0.05)
+    P["T0"] = I.ds_T0(20, P["G"])
+    shape = (32, 12, 16)  # front above nz/2: the first check shifts
+    res = run_pair(pfmod, omod, shape, P, "L", 60, bc=I.BC_DS, chunks=[1, 20, 60], ic_kw={"z_front": 20})
+    for t, ep, em, gs, os_ in res:
+        assert gs == os_, (gs, os_)
+        assert ep <= 1e-11 and em <= 1e-11, (t, ep, em)
+    assert res[-1][3]["z_off"] > 0
+
+
+def test_step_phi_only(pfmod, omod):
+    P = I.params_stress()
+    shape = (12, 10, 14)
+    phi, mu = I.ic_voronoi(shape, seed=4)
+    g = pfmod.PhaseField(shape, P)
+    g.init_fields(phi, mu)
+    g.step_phi_only()
+    o = omod.Oracle(shape, P)
+    o.init(phi, mu)
+    o.step_phi_only()
+    gp, gm = g.download()
+    op, om = o.download()
+    assert rel_linf(gp, op) <= TOL_1 and np.array_equal(gm, mu)
+
+
+def test_bitwise_reproducible_and_variants(pfmod):
+    P = I.params_stress()
+    shape = (24, 20, 36)
+    phi, mu = I.ic_voronoi(shape, seed=5)
+    outs = []
+    for _ in range(2):
+        g = pfmod.PhaseField(shape, P)
+        g.init_fields(phi, mu)
+        g.step(7)
+        outs.append(g.download())
+    assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
+
+
+def test_forced_exchange_path_bitwise(pfmod, monkeypatch):
+    """The pack / exchange / unpack path (used across ranks) gives bitwise
+    the same ghosts as the local periodic fill."""
+    P = I.params_stress()
+    shape = (10, 12, 14)
+    phi, mu = I.ic_voronoi(shape, seed=6)
+    g = pfmod.PhaseField(shape, P)
+    g.init_fields(phi, mu)
+    g.step(3)
+    ref = g.download()
+    monkeypatch.setenv("PF_FORCE_EXCHANGE", "1")
+    h = pfmod.PhaseField(shape, P)
+    h.init_fields(phi, mu)
+    h.step(3)
+    got = h.download()
+    assert np.array_equal(ref[0], got[0]) and np.array_equal(ref[1], got[1])
+
+
+def test_translation_invariance_bitwise(pfmod):
+    P = I.params_stress(G=0.0, v=0.0)
+    shape = (16, 12, 20)
+    phi, mu = I.ic_voronoi(shape, seed=7)
+    roll = lambda a: np.roll(a, (3, 2, 5), axis=(1, 2, 3))
+    g = pfmod.PhaseField(shape, P)
+    g.init_fields(phi, mu)
+    g.step(4)
+    a = g.download()
+    h = pfmod.PhaseField(shape, P)
+    h.init_fields(roll(phi), roll(mu))
+    h.step(4)
+    b = h.download()
+    assert np.array_equal(roll(a[0]), b[0]) and np.array_equal(roll(a[1]), b[1])
+
+
+def test_monitors_front_and_shift(pfmod, omod):
+    P = I.params_c4("ds")
+    shape = (24, 8, 12)
+    phi, mu = I.ic_lamellar(shape, seed=3, z_front=10)
+    g = pfmod.PhaseField(shape, P, bc=I.BC_DS)
+    g.init_fields(phi, mu)
+    o = omod.Oracle(shape, P, I.BC_DS)
+    o.init(phi, mu)
+    assert g.front_height() == o.front_height()
+    e, mn = g.monitor()
+    assert e == np.abs(phi.sum(0) - 1).max() and mn == phi.min()
+    g.shift_window(4)
+    o.shift_window(4)
+    gp, gm = g.download()
+    op, om = o.download()
+    assert np.array_equal(gp, op) and np.array_equal(gm, om)
+    assert g.state() == o.state()
+
+
+def test_rejects_bad_input(pfmod):
+    P = I.params_c4()
+    shape = (4, 4, 4)
+    g = pfmod.PhaseField(shape, P)
+    phi, mu = I.ic_random(shape)
+    phi[0, 0, 0, 0] += 1e-9
+    with pytest.raises(pfmod.PFError):
+        g.init_fields(phi, mu)
+    with pytest.raises(pfmod.PFError):
+        g.set_params(dict(P, dt=0.2))  # above the explicit stability bound
+    with pytest.raises(pfmod.PFError):
+        g.step(1)  # no fields yet
+
+
+def test_e2e_pinned_roundtrip(pfmod):
+    import torch
+    P = I.params_c4()
+    shape = (8, 8, 8)
+    phi, mu = I.ic_random(shape)
+    g = pfmod.PhaseField(shape, P)
+    tp = torch.from_numpy(phi).pin_memory()
+    tm = torch.from_numpy(mu).pin_memory()
+    g.init_fields(tp, tm)
+    op = torch.empty_like(tp).pin_memory()
+    om = torch.empty_like(tm).pin_memory()
+    g.download(out=(op, om))
+    assert np.array_equal(op.numpy(), phi) and np.array_equal(om.numpy(), mu)
