@@ -84,10 +84,12 @@ typedef struct {
 typedef struct {
   int local[3];           /* this rank's interior extents nx, ny, nz          */
   int offset[3];          /* global index of its first interior cell          */
-  int64_t pitch;          /* doubles per padded row (ghosts included)         */
-  int64_t plane;          /* doubles per z-plane = pitch * (ny + 2)           */
-  int64_t field;          /* doubles per component = plane * (nz + 2)         */
+  int64_t pitch;          /* doubles per padded row (>= x_off + nx + 2)       */
+  int64_t plane;          /* doubles per z-plane = pitch * (ny + 4)           */
+  int64_t field;          /* doubles per component = plane * (nz + 4)         */
   int64_t x_off;          /* row offset of interior x = 0 (128-B aligned)     */
+  /* cell (x,y,z) of component c is at c*field + (z+2)*plane + (y+2)*pitch +
+   * x_off + x: one ghost layer (index -1, n) inside a guard ring of 2.      */
   size_t phi_bytes;       /* one time level of phi: PF_N * field * 8          */
   size_t mu_bytes;        /* one time level of mu:  PF_M * field * 8          */
   size_t workspace_bytes; /* tables, pack buffers, reduction scratch          */

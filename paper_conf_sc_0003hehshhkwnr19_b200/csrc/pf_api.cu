@@ -20,14 +20,6 @@
 
 using namespace pf;
 
-namespace pf {
-void launch_tuned_phi(const DevParams& P, const Geom& g, const Tables& T, const double* ps, const double* ms,
-                      double* pd, cudaStream_t s);
-void launch_tuned_mu(const DevParams& P, const Geom& g, const Tables& T, const double* ps, const double* pd,
-                     const double* ms, double* md, cudaStream_t s);
-void launch_ghost_stage(const Geom& g, int d, int klo, int khi, double* f, int ncomp, const double* dirichlet,
-                        cudaStream_t s);
-}  // namespace pf
 
 // ---------------------------------------------------------------------------
 // NCCL, loaded on demand (dlopen) so that the library loads and runs without
@@ -91,7 +83,6 @@ struct pf_ctx {
   double* mu[2];
   int cur = 0;
   // workspace carve-up
-  double* tab = nullptr;
   unsigned long long* red = nullptr;  // reduction scratch (4 x u64)
   double* sendbuf[3][2] = {};
   double* recvbuf[3][2] = {};
@@ -171,13 +162,13 @@ int layout_of(const pf_config* cfg, pf_layout* L, int coord[3]) {
     if (L->local[d] < 1) return PF_EINVAL;
   }
   const int nx = L->local[0], ny = L->local[1], nz = L->local[2];
-  L->x_off = 16;  // interior x = 0 at a 128-B boundary
-  L->pitch = ((L->x_off + nx + 1) + 15) / 16 * 16;
-  L->plane = L->pitch * (ny + 2);
-  L->field = L->plane * (nz + 2);
+  L->x_off = 16;  // interior x = 0 at a 128-B boundary; x in [-16, ...) addressable
+  L->pitch = ((L->x_off + nx + GUARD) + 15) / 16 * 16;
+  L->plane = L->pitch * (ny + 2 * GUARD);
+  L->field = L->plane * (nz + 2 * GUARD);
   L->phi_bytes = (size_t)PF_N * L->field * sizeof(double) + 256;  // +256: tail slack for vector loads
   L->mu_bytes = (size_t)PF_M * L->field * sizeof(double) + 256;
-  size_t ws = align256(table_doubles(nz) * sizeof(double)) + 256;  // tables + reduction scratch
+  size_t ws = 256;  // reduction scratch
   Geom g{nx, ny, nz, L->offset[2], L->pitch, L->plane, L->field, L->x_off};
   for (int d = 0; d < 3; ++d) ws += 4 * align256(halo_slab_elems(g, d) * PF_N * sizeof(double));
   L->workspace_bytes = ws;
@@ -282,8 +273,6 @@ int pf_create(const pf_config* cfg, pf_ctx** out) {
   }
   // workspace carve-up
   char* w = (char*)cfg->workspace;
-  ctx->tab = (double*)w;
-  w += align256(table_doubles(ctx->g.nz) * sizeof(double));
   ctx->red = (unsigned long long*)w;
   w += 256;
   for (int d = 0; d < 3; ++d) {
@@ -437,7 +426,7 @@ int pf_set_params(pf_ctx* ctx, const pf_params* p) {
   if (p->dt > dt_phi || p->dt > dt_mu)
     return fail(ctx, PF_EINVAL, "dt = %g exceeds the explicit stability bound min(%g [phi], %g [mu])", p->dt, dt_phi,
                 dt_mu);
-  // device scalars
+  // device scalars and coefficients (kernel-parameter constant bank)
   DevParams& D = ctx->dp;
   memset(&D, 0, sizeof D);
   D.dx = p->dx;
@@ -449,6 +438,11 @@ int pf_set_params(pf_ctx* ctx, const pf_params* p) {
   D.inv_eps = 1.0 / p->eps;
   D.dt_over_eps = p->dt / p->eps;
   const double pi = 3.14159265358979323846;
+  D.at_c = p->dx * pi * p->eps / (8.0 * p->dt);
+  D.dTdt = -p->G * p->v;
+  D.Tdz = p->G * p->dx;
+  D.mu_inf[0] = p->mu_inf[0];
+  D.mu_inf[1] = p->mu_inf[1];
   for (int a = 0; a < PF_N; ++a)
     for (int b = 0; b < PF_N; ++b) {
       D.g[a][b] = a == b ? 0.0 : p->gamma[a][b];
@@ -468,22 +462,58 @@ int pf_set_params(pf_ctx* ctx, const pf_params* p) {
       D.tau[k++] = p->tau[a][b];
       tm += p->tau[a][b];
     }
-  D.tau_mean = tm / 6.0;
+  D.inv_tau_mean = 6.0 / tm;
+  bool ta = false;
   for (int a = 0; a < PF_N; ++a) {
-    D.dcT[a][0] = -(p->A1[a][0][0] + p->A1[a][0][0]);
-    D.dcT[a][1] = -(p->A1[a][0][1] + p->A1[a][1][0]);
-    D.dcT[a][2] = -(p->A1[a][1][1] + p->A1[a][1][1]);
+    const double(*A0)[2] = p->A0[a];
+    const double(*A1)[2] = p->A1[a];
+    D.psiA[a][0] = A0[0][0];
+    D.psiA[a][1] = A0[0][1] + A0[1][0];
+    D.psiA[a][2] = A0[1][1];
+    D.psiA1[a][0] = A1[0][0];
+    D.psiA1[a][1] = A1[0][1] + A1[1][0];
+    D.psiA1[a][2] = A1[1][1];
+    for (int i = 0; i < 2; ++i) {
+      D.B0[a][i] = p->B0[a][i];
+      D.B1[a][i] = p->B1[a][i];
+      for (int j = 0; j < 2; ++j) ta |= A1[i][j] != 0.0;
+    }
+    D.C0[a] = p->C0[a];
+    D.C1[a] = p->C1[a];
+    // chi = -(A + A^T)  [A6]
+    D.chi0[a][0] = -(A0[0][0] + A0[0][0]);
+    D.chi0[a][1] = -(A0[0][1] + A0[1][0]);
+    D.chi0[a][2] = -(A0[1][1] + A0[1][1]);
+    D.chi1[a][0] = -(A1[0][0] + A1[0][0]);
+    D.chi1[a][1] = -(A1[0][1] + A1[1][0]);
+    D.chi1[a][2] = -(A1[1][1] + A1[1][1]);
+    // P = D_a chi_a (eq. 9, D left-multiplied [A7]), split in c0 + T c1
+    const double X0[2][2] = {{D.chi0[a][0], D.chi0[a][1]}, {D.chi0[a][1], D.chi0[a][2]}};
+    const double X1[2][2] = {{D.chi1[a][0], D.chi1[a][1]}, {D.chi1[a][1], D.chi1[a][2]}};
+    for (int i = 0; i < 2; ++i)
+      for (int j = 0; j < 2; ++j) {
+        D.P0[a][2 * i + j] = p->D[a][i][0] * X0[0][j] + p->D[a][i][1] * X0[1][j];
+        D.P1[a][2 * i + j] = p->D[a][i][0] * X1[0][j] + p->D[a][i][1] * X1[1][j];
+      }
+    D.dcT[a][0] = D.chi1[a][0];
+    D.dcT[a][1] = D.chi1[a][1];
+    D.dcT[a][2] = D.chi1[a][2];
     D.dcT[a][3] = -p->B1[a][0];
     D.dcT[a][4] = -p->B1[a][1];
   }
-  D.dTdt = -p->G * p->v;
-  D.at_c = p->dx * pi * p->eps / (8.0 * p->dt);
-  D.mu_inf[0] = p->mu_inf[0];
-  D.mu_inf[1] = p->mu_inf[1];
-  D.T0 = p->T0;
-  D.G = p->G;
-  D.v = p->v;
+  for (int s = 0; s < PF_N - 1; ++s) {
+    const int a = s < L ? s : s + 1;
+    for (int i = 0; i < 3; ++i) {
+      D.dchi0[s][i] = D.chi0[L][i] - D.chi0[a][i];
+      D.dchi1[s][i] = D.chi1[L][i] - D.chi1[a][i];
+    }
+    for (int i = 0; i < 2; ++i) {
+      D.dB0[s][i] = p->B0[L][i] - p->B0[a][i];
+      D.dB1[s][i] = p->B1[L][i] - p->B1[a][i];
+    }
+  }
   D.liquid = L;
+  D.TA = ta ? 1 : 0;
   ctx->hp = *p;
   ctx->have_params = true;
   return PF_OK;
@@ -591,20 +621,16 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
   double* pd = ctx->phi[1 - ctx->cur];
   double* ms = ctx->mu[ctx->cur];
   double* md = ctx->mu[1 - ctx->cur];
+  // frozen temperature of this step: T(k) = T0 + G ((k + z0 + z_off) dx - v t_n), t_n = step dt  [A13]
   const double t = (double)ctx->step * ctx->hp.dt;
+  ctx->dp.Tbase = ctx->hp.T0 + ctx->hp.G * (((double)g.z0 + (double)ctx->z_off) * ctx->hp.dx - ctx->hp.v * t);
   cudaEvent_t e0 = nullptr;
-  prof_begin(ctx, 3, &e0);
-  launch_tables(ctx->hp, ctx->cfg.liquid, g, t, ctx->z_off, ctx->tab, ctx->stream);
-  ctx->nlaunch[3] += 1;
-  prof_end(ctx, 3, e0);
-  if (int r = check_launch(ctx, "tables")) return r;
-  const Tables T = table_view(ctx->tab, g.nz);
   // Algorithm 1, line 1: phi-sweep
   prof_begin(ctx, 0, &e0);
   if (ctx->variant == PF_VARIANT_NAIVE)
-    launch_phi_naive(ctx->dp, g, T, ps, ms, pd, ctx->stream);
+    launch_phi_naive(ctx->dp, g, ps, ms, pd, ctx->stream);
   else
-    launch_tuned_phi(ctx->dp, g, T, ps, ms, pd, ctx->stream);
+    launch_phi_tuned(ctx->dp, g, ps, ms, pd, ctx->stream);
   ctx->nlaunch[0] += 1;
   prof_end(ctx, 0, e0);
   if (int r = check_launch(ctx, "phi_sweep")) return r;
@@ -619,9 +645,9 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
     // line 3: mu-sweep
     prof_begin(ctx, 1, &e0);
     if (ctx->variant == PF_VARIANT_NAIVE)
-      launch_mu_naive(ctx->dp, g, T, ps, pd, ms, md, ctx->stream);
+      launch_mu_naive(ctx->dp, g, ps, pd, ms, md, ctx->stream);
     else
-      launch_tuned_mu(ctx->dp, g, T, ps, pd, ms, md, ctx->stream);
+      launch_mu_tuned(ctx->dp, g, ps, pd, ms, md, ctx->stream);
     ctx->nlaunch[1] += 1;
     prof_end(ctx, 1, e0);
     if (int r2 = check_launch(ctx, "mu_sweep")) return r2;

@@ -12,100 +12,10 @@
 namespace pf {
 
 // ---------------------------------------------------------------------------
-// a1: frozen temperature T = T0 + G (z dx - v t) per plane [A13] and the
-// T-dependent coefficients A(T), B(T), C(T) (eq. 6), chi = dc/dmu = -(A+A^T)
-// [A6] and the mobility products P_a = D_a chi_a (eq. 9) [A7].
-// ---------------------------------------------------------------------------
-struct TabArgs {
-  pf_params p;
-  int liquid;
-  int nz, z0;
-  int64_t z_off;
-  double t;
-};
-
-__device__ void coef_at(const pf_params& p, int a, double T, double A[2][2], double B[2], double* C) {
-  for (int i = 0; i < 2; ++i) {
-    for (int j = 0; j < 2; ++j) A[i][j] = p.A0[a][i][j] + p.A1[a][i][j] * T;
-    B[i] = p.B0[a][i] + p.B1[a][i] * T;
-  }
-  *C = p.C0[a] + p.C1[a] * T;
-}
-
-__device__ void face_row(const pf_params& p, int L, double T, double* row) {
-  double chi[N][3], B[N][2];
-  for (int a = 0; a < N; ++a) {
-    double A[2][2], C;
-    coef_at(p, a, T, A, B[a], &C);
-    chi[a][0] = -(A[0][0] + A[0][0]);
-    chi[a][1] = -(A[0][1] + A[1][0]);
-    chi[a][2] = -(A[1][1] + A[1][1]);
-    const double x[2][2] = {{chi[a][0], chi[a][1]}, {chi[a][1], chi[a][2]}};
-    for (int i = 0; i < 2; ++i)
-      for (int j = 0; j < 2; ++j) row[TF_P + 4 * a + 2 * i + j] = p.D[a][i][0] * x[0][j] + p.D[a][i][1] * x[1][j];
-  }
-  for (int s = 0; s < NSOL; ++s) {
-    const int a = solid_phase(L, s);
-    for (int k = 0; k < 3; ++k) row[TF_DCHI + 3 * s + k] = chi[L][k] - chi[a][k];
-    for (int i = 0; i < 2; ++i) row[TF_DB + 2 * s + i] = B[L][i] - B[a][i];
-  }
-  row[TF_SIZE] = 0.0;
-}
-
-__global__ void k_tables(TabArgs A, double* __restrict__ tab) {
-  const int i = blockIdx.x * blockDim.x + threadIdx.x;
-  const pf_params& p = A.p;
-  const int nz = A.nz;
-  const int liquid = A.liquid;
-  double* cell = tab;
-  double* fxy = tab + (size_t)nz * TC_SIZE;
-  double* fz = fxy + (size_t)nz * TF_STRIDE;
-  auto Tz = [&](double zc) { return p.T0 + p.G * ((zc + (double)A.z0 + (double)A.z_off) * p.dx - p.v * A.t); };
-  if (i < nz) {
-    const double T = Tz((double)i);
-    double* row = cell + (size_t)i * TC_SIZE;
-    for (int a = 0; a < N; ++a) {
-      double Am[2][2], B[2], C;
-      coef_at(p, a, T, Am, B, &C);
-      row[TC_PSI + 6 * a + 0] = Am[0][0];
-      row[TC_PSI + 6 * a + 1] = Am[0][1] + Am[1][0];
-      row[TC_PSI + 6 * a + 2] = Am[1][1];
-      row[TC_PSI + 6 * a + 3] = B[0];
-      row[TC_PSI + 6 * a + 4] = B[1];
-      row[TC_PSI + 6 * a + 5] = C;
-      row[TC_CHI + 3 * a + 0] = -(Am[0][0] + Am[0][0]);
-      row[TC_CHI + 3 * a + 1] = -(Am[0][1] + Am[1][0]);
-      row[TC_CHI + 3 * a + 2] = -(Am[1][1] + Am[1][1]);
-      row[TC_B + 2 * a + 0] = B[0];
-      row[TC_B + 2 * a + 1] = B[1];
-    }
-    face_row(p, liquid, T, fxy + (size_t)i * TF_STRIDE);
-  }
-  if (i <= nz) face_row(p, liquid, Tz((double)i - 0.5), fz + (size_t)i * TF_STRIDE);
-}
-
-size_t table_doubles(int nz) { return (size_t)nz * TC_SIZE + (size_t)nz * TF_STRIDE + (size_t)(nz + 1) * TF_STRIDE; }
-
-Tables table_view(const double* tab, int nz) {
-  Tables T;
-  T.cell = tab;
-  T.fxy = tab + (size_t)nz * TC_SIZE;
-  T.fz = T.fxy + (size_t)nz * TF_STRIDE;
-  return T;
-}
-
-void launch_tables(const pf_params& p, int liquid, const Geom& g, double t, int64_t z_off, double* tab,
-                   cudaStream_t s) {
-  TabArgs A{p, liquid, g.nz, g.z0, z_off, t};
-  const int n = g.nz + 1;
-  k_tables<<<(n + 127) / 128, 128, 0, s>>>(A, tab);
-}
-
-// ---------------------------------------------------------------------------
 // Naive phi-sweep: one thread per cell, 6 faces each (Algorithm 1 line 1).
 // ---------------------------------------------------------------------------
-template <int L>
-__global__ void __launch_bounds__(256) k_phi_naive(DevParams P, Geom g, Tables T, const double* __restrict__ ps,
+template <int L, bool TA>
+__global__ void __launch_bounds__(256) k_phi_naive(DevParams P, Geom g, const double* __restrict__ ps,
                                                    const double* __restrict__ ms, double* __restrict__ pd) {
   const int x = blockIdx.x * blockDim.x + threadIdx.x;
   const int y = blockIdx.y * blockDim.y + threadIdx.y;
@@ -113,17 +23,17 @@ __global__ void __launch_bounds__(256) k_phi_naive(DevParams P, Geom g, Tables T
   if (x >= g.nx || y >= g.ny || z >= g.nz) return;
   const int64_t c = g.at(x, y, z);
   const int64_t F = g.field;
-  const int64_t st[3] = {1, g.pitch, g.plane};
   double ph[N], gd[N][3], divh[N] = {0.0, 0.0, 0.0, 0.0};
 #pragma unroll
   for (int a = 0; a < N; ++a) ph[a] = __ldg(ps + a * F + c);
 #pragma unroll
   for (int d = 0; d < 3; ++d) {
+    const int64_t st = d == 0 ? 1 : (d == 1 ? g.pitch : g.plane);
     double fm[N], fpl[N], jp[N], jm[N];
 #pragma unroll
     for (int a = 0; a < N; ++a) {
-      fm[a] = __ldg(ps + a * F + c - st[d]);
-      fpl[a] = __ldg(ps + a * F + c + st[d]);
+      fm[a] = __ldg(ps + a * F + c - st);
+      fpl[a] = __ldg(ps + a * F + c + st);
       gd[a][d] = fpl[a] - fm[a];
     }
     phi_face(P, ph, fpl, jp);
@@ -133,7 +43,7 @@ __global__ void __launch_bounds__(256) k_phi_naive(DevParams P, Geom g, Tables T
   }
   const double mu0 = __ldg(ms + c), mu1 = __ldg(ms + F + c);
   double out[N];
-  phi_cell(P, T.cell + (size_t)z * TC_SIZE, ph, gd, divh, mu0, mu1, out);
+  phi_cell<TA>(P, plane_T(P, (double)z), ph, gd, divh, mu0, mu1, out);
 #pragma unroll
   for (int a = 0; a < N; ++a) pd[a * F + c] = out[a];
 }
@@ -142,36 +52,27 @@ __global__ void __launch_bounds__(256) k_phi_naive(DevParams P, Geom g, Tables T
 // Naive mu-sweep: one thread per cell, 6 faces each (Algorithm 1 line 3).
 // ---------------------------------------------------------------------------
 template <int L>
-__device__ __forceinline__ void mu_face_global(const DevParams& P, const double* __restrict__ frow, const Geom& g,
-                                               const double* __restrict__ ps, const double* __restrict__ pd,
-                                               const double* __restrict__ ms, int64_t p, int64_t sn, int64_t s1,
-                                               int64_t s2, double (&Fh)[M]) {
-  const int64_t F = g.field;
-  const int64_t q = p + sn;
-  double fp[N], fq[N], gt1[N], gt2[N], dsum[NSOL], mp[M], mq[M];
+__device__ __forceinline__ void load_side(const double* __restrict__ ps, const double* __restrict__ pd,
+                                          const double* __restrict__ ms, int64_t F, int64_t c, int64_t s1, int64_t s2,
+                                          FaceSide& o) {
 #pragma unroll
   for (int a = 0; a < N; ++a) {
     const double* f = ps + a * F;
-    fp[a] = __ldg(f + p);
-    fq[a] = __ldg(f + q);
-    gt1[a] = 0.25 * ((__ldg(f + p + s1) - __ldg(f + p - s1)) + (__ldg(f + q + s1) - __ldg(f + q - s1)));
-    gt2[a] = 0.25 * ((__ldg(f + p + s2) - __ldg(f + p - s2)) + (__ldg(f + q + s2) - __ldg(f + q - s2)));
+    o.f[a] = __ldg(f + c);
+    o.c1[a] = __ldg(f + c + s1) - __ldg(f + c - s1);
+    o.c2[a] = __ldg(f + c + s2) - __ldg(f + c - s2);
   }
 #pragma unroll
   for (int s = 0; s < NSOL; ++s) {
     const int a = solid_phase(L, s);
-    dsum[s] = (__ldg(pd + a * F + p) - fp[a]) + (__ldg(pd + a * F + q) - fq[a]);
+    o.ds[s] = __ldg(pd + a * F + c) - o.f[a];
   }
-#pragma unroll
-  for (int i = 0; i < M; ++i) {
-    mp[i] = __ldg(ms + i * F + p);
-    mq[i] = __ldg(ms + i * F + q);
-  }
-  mu_face<L>(P, frow, fp, fq, gt1, gt2, dsum, mp, mq, Fh);
+  o.m[0] = __ldg(ms + c);
+  o.m[1] = __ldg(ms + F + c);
 }
 
-template <int L>
-__global__ void __launch_bounds__(256) k_mu_naive(DevParams P, Geom g, Tables T, const double* __restrict__ ps,
+template <int L, bool TA>
+__global__ void __launch_bounds__(256) k_mu_naive(DevParams P, Geom g, const double* __restrict__ ps,
                                                   const double* __restrict__ pd, const double* __restrict__ ms,
                                                   double* __restrict__ md) {
   const int x = blockIdx.x * blockDim.x + threadIdx.x;
@@ -180,51 +81,48 @@ __global__ void __launch_bounds__(256) k_mu_naive(DevParams P, Geom g, Tables T,
   if (x >= g.nx || y >= g.ny || z >= g.nz) return;
   const int64_t c = g.at(x, y, z);
   const int64_t F = g.field;
-  const int64_t st[3] = {1, g.pitch, g.plane};
+  const double Tc = plane_T(P, (double)z);
   double divh[M] = {0.0, 0.0};
-  const double* fxy = T.fxy + (size_t)z * TF_STRIDE;
-#pragma unroll
+#pragma unroll 1
   for (int d = 0; d < 3; ++d) {
-    const int64_t s1 = st[d == 0 ? 1 : 0], s2 = st[d == 2 ? 1 : 2];
-    const double* fr_p = d == 2 ? T.fz + (size_t)(z + 1) * TF_STRIDE : fxy;
-    const double* fr_m = d == 2 ? T.fz + (size_t)z * TF_STRIDE : fxy;
+    const int64_t sn = d == 0 ? 1 : (d == 1 ? g.pitch : g.plane);
+    const int64_t s1 = d == 0 ? g.pitch : 1;
+    const int64_t s2 = d == 2 ? g.pitch : g.plane;
+    const double Tp = d == 2 ? plane_T(P, z + 0.5) : Tc;
+    const double Tm = d == 2 ? plane_T(P, z - 0.5) : Tc;
+    FaceSide sm, s0, sp;
+    load_side<L>(ps, pd, ms, F, c - sn, s1, s2, sm);
+    load_side<L>(ps, pd, ms, F, c, s1, s2, s0);
+    load_side<L>(ps, pd, ms, F, c + sn, s1, s2, sp);
     double Fp[M], Fm[M];
-    mu_face_global<L>(P, fr_p, g, ps, pd, ms, c, st[d], s1, s2, Fp);
-    mu_face_global<L>(P, fr_m, g, ps, pd, ms, c - st[d], st[d], s1, s2, Fm);
+    mu_face<L, TA>(P, Tp, s0, sp, Fp);
+    mu_face<L, TA>(P, Tm, sm, s0, Fm);
 #pragma unroll
     for (int i = 0; i < M; ++i) divh[i] += Fp[i] - Fm[i];
   }
-  double ph[N], phn[N], mu[M], out[M];
+  double ph[N], dph[N], mu[M], out[M];
 #pragma unroll
   for (int a = 0; a < N; ++a) {
     ph[a] = __ldg(ps + a * F + c);
-    phn[a] = __ldg(pd + a * F + c);
+    dph[a] = __ldg(pd + a * F + c) - ph[a];
   }
 #pragma unroll
   for (int i = 0; i < M; ++i) mu[i] = __ldg(ms + i * F + c);
-  mu_cell(P, T.cell + (size_t)z * TC_SIZE, ph, phn, mu, divh, out);
+  mu_cell<TA>(P, Tc, ph, dph, mu, divh, out);
 #pragma unroll
   for (int i = 0; i < M; ++i) md[i * F + c] = out[i];
 }
 
-#define PF_DISPATCH_L(L, ...)                   \
-  switch (L) {                                  \
-    case 0: { constexpr int LL = 0; __VA_ARGS__; } break; \
-    case 1: { constexpr int LL = 1; __VA_ARGS__; } break; \
-    case 2: { constexpr int LL = 2; __VA_ARGS__; } break; \
-    default: { constexpr int LL = 3; __VA_ARGS__; } break; \
-  }
-
-void launch_phi_naive(const DevParams& P, const Geom& g, const Tables& T, const double* ps, const double* ms,
-                      double* pd, cudaStream_t s) {
+void launch_phi_naive(const DevParams& P, const Geom& g, const double* ps, const double* ms, double* pd,
+                      cudaStream_t s) {
   dim3 b(32, 4, 2), gr((g.nx + 31) / 32, (g.ny + 3) / 4, (g.nz + 1) / 2);
-  PF_DISPATCH_L(P.liquid, (k_phi_naive<LL><<<gr, b, 0, s>>>(P, g, T, ps, ms, pd)));
+  PF_DISPATCH(P.liquid, P.TA, (k_phi_naive<LL, TT><<<gr, b, 0, s>>>(P, g, ps, ms, pd)));
 }
 
-void launch_mu_naive(const DevParams& P, const Geom& g, const Tables& T, const double* ps, const double* pd,
-                     const double* ms, double* md, cudaStream_t s) {
+void launch_mu_naive(const DevParams& P, const Geom& g, const double* ps, const double* pd, const double* ms,
+                     double* md, cudaStream_t s) {
   dim3 b(32, 4, 2), gr((g.nx + 31) / 32, (g.ny + 3) / 4, (g.nz + 1) / 2);
-  PF_DISPATCH_L(P.liquid, (k_mu_naive<LL><<<gr, b, 0, s>>>(P, g, T, ps, pd, ms, md)));
+  PF_DISPATCH(P.liquid, P.TA, (k_mu_naive<LL, TT><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md)));
 }
 
 // ---------------------------------------------------------------------------
@@ -290,8 +188,8 @@ __global__ void k_ghost(GhostArgs A, double* __restrict__ f) {
     const int my = map_axis(y, g.ny, A.bc.kind_lo[1], A.bc.kind_hi[1], &skip, &dir);
     const int mz = map_axis(z, g.nz, A.bc.kind_lo[2], A.bc.kind_hi[2], &skip, &dir);
     if (skip) continue;
-    const int64_t dst = (int64_t)(z + 1) * g.plane + (int64_t)(y + 1) * g.pitch + g.xoff + x;
-    const int64_t src = (int64_t)(mz + 1) * g.plane + (int64_t)(my + 1) * g.pitch + g.xoff + mx;
+    const int64_t dst = g.at(x, y, z);
+    const int64_t src = g.at(mx, my, mz);
     for (int c = 0; c < A.ncomp; ++c)
       f[c * g.field + dst] = (dir && A.use_dir) ? A.dir[c] : f[c * g.field + src];
   }
@@ -436,7 +334,7 @@ __global__ void k_pack(Geom g, int d, int idx, int ncomp, double* __restrict__ f
     c[d] = idx;
     c[d == 0 ? 1 : 0] = i0;
     c[d == 2 ? 1 : 2] = i1;
-    const int64_t li = (int64_t)(c[2] + 1) * g.plane + (int64_t)(c[1] + 1) * g.pitch + g.xoff + c[0];
+    const int64_t li = g.at(c[0], c[1], c[2]);
     for (int a = 0; a < ncomp; ++a) {
       if (unpack)
         f[a * g.field + li] = buf[a * tot + i];
@@ -472,8 +370,8 @@ __global__ void k_ghost_stage(Geom g, int d, int klo, int khi, int ncomp, double
     c[d] = side ? n[d] : -1;
     s[d] = kind == PF_BC_PERIODIC ? (side ? 0 : n[d] - 1) : (side ? n[d] - 1 : 0);
     const bool dirich = kind == PF_BC_DIRICHLET_MU && use_dir;
-    const int64_t li = (int64_t)(c[2] + 1) * g.plane + (int64_t)(c[1] + 1) * g.pitch + g.xoff + c[0];
-    const int64_t si = (int64_t)(s[2] + 1) * g.plane + (int64_t)(s[1] + 1) * g.pitch + g.xoff + s[0];
+    const int64_t li = g.at(c[0], c[1], c[2]);
+    const int64_t si = g.at(s[0], s[1], s[2]);
     for (int a = 0; a < ncomp; ++a) f[a * g.field + li] = dirich ? (a == 0 ? dir0 : dir1) : f[a * g.field + si];
   }
 }
