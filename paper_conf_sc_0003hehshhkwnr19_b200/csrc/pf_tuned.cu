@@ -40,15 +40,15 @@ __global__ void __launch_bounds__(TX* TY, 2) k_phi_tuned(DevParams P, Geom g, co
   const int z0 = blockIdx.z * ZC_PHI, z1 = min(z0 + ZC_PHI, g.nz);
   const int64_t F = g.field, SY = g.pitch, SZ = g.plane;
   // extra faces: warp 0 lanes < TY: +x face of row `lane`; warp 1: +y face of column `lane`
-  int64_t ep = 0, eq = 0;
+  int64_t ep = 0, eq = 0;  // the two cells of the extra face, at plane z0
   if (w == 0 && lane < TY) {
     const int ry = min(y0 + lane, g.ny);
-    ep = g.at(min(x0 + TX - 1, g.nx), ry, 0);
-    eq = g.at(min(x0 + TX, g.nx), ry, 0);
+    ep = g.at(min(x0 + TX - 1, g.nx), ry, z0);
+    eq = g.at(min(x0 + TX, g.nx), ry, z0);
   } else if (w == 1) {
     const int cx = min(x0 + lane, g.nx);
-    ep = g.at(cx, min(y0 + TY - 1, g.ny), 0);
-    eq = g.at(cx, min(y0 + TY, g.ny), 0);
+    ep = g.at(cx, min(y0 + TY - 1, g.ny), z0);
+    eq = g.at(cx, min(y0 + TY, g.ny), z0);
   }
   const bool extra = (w == 0 && lane < TY) || w == 1;
 
@@ -61,30 +61,33 @@ __global__ void __launch_bounds__(TX* TY, 2) k_phi_tuned(DevParams P, Geom g, co
   }
   phi_face(P, pm, p0, Fzm);
 
-  for (int z = z0; z < z1; ++z, c += SZ) {
+  for (int z = z0; z < z1; ++z, c += SZ, ep += SZ, eq += SZ) {
     const int buf = z & 1;
-    double pp[N], xm[N], xp[N], ym[N], yp[N];
+    double pp[N], Fxm[N], Fym[N], Fzp[N], gd[N][3];
+    {
+      double xm[N], xp[N], ym[N], yp[N];
 #pragma unroll
-    for (int a = 0; a < N; ++a) {
-      const double* f = ps + a * F + c;
-      pp[a] = __ldg(f + SZ);
-      xm[a] = __ldg(f - 1);
-      xp[a] = __ldg(f + 1);
-      ym[a] = __ldg(f - SY);
-      yp[a] = __ldg(f + SY);
+      for (int a = 0; a < N; ++a) {
+        const double* f = ps + a * F + c;
+        pp[a] = __ldg(f + SZ);
+        xm[a] = __ldg(f - 1);
+        xp[a] = __ldg(f + 1);
+        ym[a] = __ldg(f - SY);
+        yp[a] = __ldg(f + SY);
+        gd[a][0] = xp[a] - xm[a];
+        gd[a][1] = yp[a] - ym[a];
+        gd[a][2] = pp[a] - pm[a];
+      }
+      phi_face(P, xm, p0, Fxm);
+      phi_face(P, ym, p0, Fym);
     }
-    const double mu0 = __ldg(ms + c), mu1 = __ldg(ms + F + c);
-    double Fxm[N], Fym[N], Fzp[N];
-    phi_face(P, xm, p0, Fxm);
-    phi_face(P, ym, p0, Fym);
     phi_face(P, p0, pp, Fzp);
     if (extra) {
-      const int64_t zo = (int64_t)(z + GUARD) * SZ;
       double fa[N], fb[N], fe[N];
 #pragma unroll
       for (int a = 0; a < N; ++a) {
-        fa[a] = __ldg(ps + a * F + ep + zo);
-        fb[a] = __ldg(ps + a * F + eq + zo);
+        fa[a] = __ldg(ps + a * F + ep);
+        fb[a] = __ldg(ps + a * F + eq);
       }
       phi_face(P, fa, fb, fe);
       if (w == 0) {
@@ -97,17 +100,15 @@ __global__ void __launch_bounds__(TX* TY, 2) k_phi_tuned(DevParams P, Geom g, co
     }
 #pragma unroll
     for (int a = 0; a < N; ++a) fy[buf][a][w][lane] = Fym[a];
+    const double mu0 = __ldg(ms + c), mu1 = __ldg(ms + F + c);
     __syncthreads();
-    double divh[N], gd[N][3];
+    double divh[N];
 #pragma unroll
     for (int a = 0; a < N; ++a) {
       double fxp = __shfl_down_sync(0xffffffffu, Fxm[a], 1);
       if (lane == TX - 1) fxp = ex[buf][a][w];
       const double fyp = (w < TY - 1) ? fy[buf][a][w + 1][lane] : ey[buf][a][lane];
       divh[a] = ((fxp - Fxm[a]) + (fyp - Fym[a])) + (Fzp[a] - Fzm[a]);
-      gd[a][0] = xp[a] - xm[a];
-      gd[a][1] = yp[a] - ym[a];
-      gd[a][2] = pp[a] - pm[a];
     }
     double out[N];
     phi_cell<TA>(P, plane_T(P, (double)z), p0, gd, divh, mu0, mu1, out);
@@ -200,13 +201,15 @@ __global__ void __launch_bounds__(TX* TY, 2) k_mu_tuned(DevParams P, Geom g, con
   const int64_t F = g.field;
   const int me = hidx(lane + 1, w + 1);
   // halo ring cell owned by thread t < 2*TX + 2*TY (corners are not needed)
+  // (warps 4.. build the halo ring; warps 0, 1 compute the far-edge faces)
   int hx = 0, hy = 0, hs = -1;
   bool hwx = false, hwy = false;
-  if (t < TX) { hx = t + 1; hy = 0; hwx = true; }
-  else if (t < 2 * TX) { hx = t - TX + 1; hy = TY + 1; hwx = true; }
-  else if (t < 2 * TX + TY) { hx = 0; hy = t - 2 * TX + 1; hwy = true; }
-  else if (t < 2 * TX + 2 * TY) { hx = TX + 1; hy = t - 2 * TX - TY + 1; hwy = true; }
-  if (t < 2 * TX + 2 * TY) hs = hidx(hx, hy);
+  const int th = t - 4 * TX;
+  if (th >= 0 && th < TX) { hx = th + 1; hy = 0; hwx = true; }
+  else if (th >= TX && th < 2 * TX) { hx = th - TX + 1; hy = TY + 1; hwx = true; }
+  else if (th >= 2 * TX && th < 2 * TX + TY) { hx = 0; hy = th - 2 * TX + 1; hwy = true; }
+  else if (th >= 2 * TX + TY && th < 2 * TX + 2 * TY) { hx = TX + 1; hy = th - 2 * TX - TY + 1; hwy = true; }
+  if (hwx || hwy) hs = hidx(hx, hy);
   const int hgx = min(x0 + hx - 1, g.nx), hgy = min(y0 + hy - 1, g.ny);
 
   // z-face k-1/2 needs the previous plane's side (tangential: x, y)
@@ -277,14 +280,14 @@ __global__ void __launch_bounds__(TX* TY, 2) k_mu_tuned(DevParams P, Geom g, con
         fxs[(i * TY + w) * (TX + 1) + lane] = Fx[i];
         fys[(i * (TY + 1) + w) * TX + lane] = Fy[i];
       }
-      if (w == 3) {  // +y face of the top tile edge, column `lane`
+      if (w == 0) {  // +y face of the top tile edge, column `lane`
         double Fe[M];
         side_from_smem<L>(D, hidx(lane + 1, TY), D_CX, D_CZ, p);
         side_from_smem<L>(D, hidx(lane + 1, TY + 1), D_CX, D_CZ, s);
         mu_face<L, TA>(P, Tk, p, s, Fe);
 #pragma unroll
         for (int i = 0; i < M; ++i) fys[(i * (TY + 1) + TY) * TX + lane] = Fe[i];
-      } else if (w == 4 && lane < TY) {  // +x face of the right tile edge, row `lane`
+      } else if (w == 1 && lane < TY) {  // +x face of the right tile edge, row `lane`
         double Fe[M];
         side_from_smem<L>(D, hidx(TX, lane + 1), D_CY, D_CZ, p);
         side_from_smem<L>(D, hidx(TX + 1, lane + 1), D_CY, D_CZ, s);
