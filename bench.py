@@ -187,7 +187,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--n", type=int, default=256, help="block edge per GPU")
-    ap.add_argument("--variant", default="tuned", choices=["tuned", "naive"])
+    ap.add_argument("--variant", default="jit", choices=["jit", "tuned", "naive"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     args = ap.parse_args()

@@ -58,9 +58,12 @@ extern "C" {
 #define PF_N 4 /* phases (P1: 3 solids + liquid)  */
 #define PF_M 2 /* chemical potentials K-1 (3 components)        */
 
-/* kernel schedule (pf_set_variant); results are identical to <= 1e-12 */
-#define PF_VARIANT_TUNED 0 /* default: z-marching, face fluxes computed once */
+/* kernel schedule (pf_set_variant); all agree with the oracle to <= 1e-12 */
+#define PF_VARIANT_TUNED 0 /* z-marching, face fluxes computed once; generic */
 #define PF_VARIANT_NAIVE 1 /* one thread per cell, every face computed twice */
+#define PF_VARIANT_JIT 2   /* default: the tuned kernels specialised at run time
+                              (NVRTC) with the parameters and the block
+                              geometry as compile-time constants */
 
 typedef struct pf_ctx pf_ctx;
 
@@ -170,7 +173,9 @@ int pf_download(pf_ctx* ctx, double* phi, double* mu, int where);
 int pf_get_state(const pf_ctx* ctx, pf_state* out);
 int pf_set_state(pf_ctx* ctx, const pf_state* s);
 
-/* Kernel schedule selection (PF_VARIANT_*), for ablations and parity. */
+/* Kernel schedule selection (PF_VARIANT_*), for ablations and parity.  The
+ * JIT variant compiles on the first step after pf_set_params (~2 s, cached
+ * per process); PF_ECUDA with the NVRTC log if that fails.                 */
 int pf_set_variant(pf_ctx* ctx, int variant);
 
 /* Optional per-kernel timing with CUDA events on the compute stream:
@@ -187,6 +192,12 @@ int pf_profile_read(pf_ctx* ctx, double ms[4], int64_t launches[4]);
  * caller broadcasts (e.g. with torch.distributed) into every rank's
  * pf_config.nccl_uid before pf_create.  PF_ENCCL if NCCL cannot be loaded. */
 int pf_nccl_unique_id(unsigned char out[128]);
+
+/* Build check without a device: compile the run-time specialised kernels
+ * (PF_VARIANT_JIT) for parameters p, liquid index `liquid` and an n^3 block
+ * with NVRTC; optionally write the sm_100a cubin to cubin_path.  Returns the
+ * cubin size in bytes, or -1 with the compiler log in log[0..logn).       */
+int pf_jit_compile_only(const pf_params* p, int liquid, int n, const char* cubin_path, char* log, int logn);
 
 const char* pf_last_error(const pf_ctx* ctx);
 const char* pf_version(void);

@@ -16,7 +16,7 @@
 #include <string>
 #include <vector>
 
-#include "pf_model.cuh"
+#include "pf_internal.h"
 
 using namespace pf;
 
@@ -92,7 +92,8 @@ struct pf_ctx {
   DevParams dp;
   bool have_params = false, have_fields = false;
   int64_t step = 0, z_off = 0;
-  int variant = PF_VARIANT_TUNED;
+  int variant = PF_VARIANT_JIT;
+  JitModule* jit = nullptr;  // specialised kernels for (dp, g); reset by pf_set_params
   ncclComm_t comm = nullptr;
   // profiling
   bool prof = false;
@@ -209,6 +210,101 @@ double deff_at(const pf_params& p, const double* ph, double T) {
 }
 
 }  // namespace
+
+namespace pf {
+// device scalars and coefficients of pf_params (kernel-parameter constant
+// bank of the generic build, compile-time constants of the specialised one)
+void fill_dev_params(const pf_params& pr, int L, DevParams* out) {
+  const pf_params* p = &pr;
+  DevParams& D = *out;
+  memset(&D, 0, sizeof D);
+  D.dx = p->dx;
+  D.dt = p->dt;
+  D.eps = p->eps;
+  D.inv_dt = 1.0 / p->dt;
+  D.inv_dx2 = 1.0 / (p->dx * p->dx);
+  D.phi_grad_c = p->eps / (p->dx * p->dx);
+  D.inv_eps = 1.0 / p->eps;
+  D.dt_over_eps = p->dt / p->eps;
+  const double pi = 3.14159265358979323846;
+  D.at_c = p->dx * pi * p->eps / (8.0 * p->dt);
+  D.dTdt = -p->G * p->v;
+  D.Tdz = p->G * p->dx;
+  D.mu_inf[0] = p->mu_inf[0];
+  D.mu_inf[1] = p->mu_inf[1];
+  for (int a = 0; a < PF_N; ++a)
+    for (int b = 0; b < PF_N; ++b) {
+      D.g[a][b] = a == b ? 0.0 : p->gamma[a][b];
+      D.og[a][b] = a == b ? 0.0 : 16.0 / (pi * pi) * p->gamma[a][b];
+    }
+  const int others[4][3] = {{1, 2, 3}, {0, 2, 3}, {0, 1, 3}, {0, 1, 2}};
+  for (int a = 0; a < PF_N; ++a) {
+    const int* o = others[a];
+    D.g3[a][0] = p->gamma3[a][o[0]][o[1]];
+    D.g3[a][1] = p->gamma3[a][o[0]][o[2]];
+    D.g3[a][2] = p->gamma3[a][o[1]][o[2]];
+  }
+  int k = 0;
+  double tm = 0;
+  for (int a = 0; a < PF_N; ++a)
+    for (int b = a + 1; b < PF_N; ++b) {
+      D.tau[k++] = p->tau[a][b];
+      tm += p->tau[a][b];
+    }
+  D.inv_tau_mean = 6.0 / tm;
+  bool ta = false;
+  for (int a = 0; a < PF_N; ++a) {
+    const double(*A0)[2] = p->A0[a];
+    const double(*A1)[2] = p->A1[a];
+    D.psiA[a][0] = A0[0][0];
+    D.psiA[a][1] = A0[0][1] + A0[1][0];
+    D.psiA[a][2] = A0[1][1];
+    D.psiA1[a][0] = A1[0][0];
+    D.psiA1[a][1] = A1[0][1] + A1[1][0];
+    D.psiA1[a][2] = A1[1][1];
+    for (int i = 0; i < 2; ++i) {
+      D.B0[a][i] = p->B0[a][i];
+      D.B1[a][i] = p->B1[a][i];
+      for (int j = 0; j < 2; ++j) ta |= A1[i][j] != 0.0;
+    }
+    D.C0[a] = p->C0[a];
+    D.C1[a] = p->C1[a];
+    // chi = -(A + A^T)  [A6]
+    D.chi0[a][0] = -(A0[0][0] + A0[0][0]);
+    D.chi0[a][1] = -(A0[0][1] + A0[1][0]);
+    D.chi0[a][2] = -(A0[1][1] + A0[1][1]);
+    D.chi1[a][0] = -(A1[0][0] + A1[0][0]);
+    D.chi1[a][1] = -(A1[0][1] + A1[1][0]);
+    D.chi1[a][2] = -(A1[1][1] + A1[1][1]);
+    // P = D_a chi_a (eq. 9, D left-multiplied [A7]), split in c0 + T c1
+    const double X0[2][2] = {{D.chi0[a][0], D.chi0[a][1]}, {D.chi0[a][1], D.chi0[a][2]}};
+    const double X1[2][2] = {{D.chi1[a][0], D.chi1[a][1]}, {D.chi1[a][1], D.chi1[a][2]}};
+    for (int i = 0; i < 2; ++i)
+      for (int j = 0; j < 2; ++j) {
+        D.P0[a][2 * i + j] = p->D[a][i][0] * X0[0][j] + p->D[a][i][1] * X0[1][j];
+        D.P1[a][2 * i + j] = p->D[a][i][0] * X1[0][j] + p->D[a][i][1] * X1[1][j];
+      }
+    D.dcT[a][0] = D.chi1[a][0];
+    D.dcT[a][1] = D.chi1[a][1];
+    D.dcT[a][2] = D.chi1[a][2];
+    D.dcT[a][3] = -p->B1[a][0];
+    D.dcT[a][4] = -p->B1[a][1];
+  }
+  for (int s = 0; s < PF_N - 1; ++s) {
+    const int a = s < L ? s : s + 1;
+    for (int i = 0; i < 3; ++i) {
+      D.dchi0[s][i] = D.chi0[L][i] - D.chi0[a][i];
+      D.dchi1[s][i] = D.chi1[L][i] - D.chi1[a][i];
+    }
+    for (int i = 0; i < 2; ++i) {
+      D.dB0[s][i] = p->B0[L][i] - p->B0[a][i];
+      D.dB1[s][i] = p->B1[L][i] - p->B1[a][i];
+    }
+  }
+  D.liquid = L;
+  D.TA = ta ? 1 : 0;
+}
+}  // namespace pf
 
 // ===========================================================================
 extern "C" {
@@ -426,96 +522,10 @@ int pf_set_params(pf_ctx* ctx, const pf_params* p) {
   if (p->dt > dt_phi || p->dt > dt_mu)
     return fail(ctx, PF_EINVAL, "dt = %g exceeds the explicit stability bound min(%g [phi], %g [mu])", p->dt, dt_phi,
                 dt_mu);
-  // device scalars and coefficients (kernel-parameter constant bank)
-  DevParams& D = ctx->dp;
-  memset(&D, 0, sizeof D);
-  D.dx = p->dx;
-  D.dt = p->dt;
-  D.eps = p->eps;
-  D.inv_dt = 1.0 / p->dt;
-  D.inv_dx2 = 1.0 / (p->dx * p->dx);
-  D.phi_grad_c = p->eps / (p->dx * p->dx);
-  D.inv_eps = 1.0 / p->eps;
-  D.dt_over_eps = p->dt / p->eps;
-  const double pi = 3.14159265358979323846;
-  D.at_c = p->dx * pi * p->eps / (8.0 * p->dt);
-  D.dTdt = -p->G * p->v;
-  D.Tdz = p->G * p->dx;
-  D.mu_inf[0] = p->mu_inf[0];
-  D.mu_inf[1] = p->mu_inf[1];
-  for (int a = 0; a < PF_N; ++a)
-    for (int b = 0; b < PF_N; ++b) {
-      D.g[a][b] = a == b ? 0.0 : p->gamma[a][b];
-      D.og[a][b] = a == b ? 0.0 : 16.0 / (pi * pi) * p->gamma[a][b];
-    }
-  const int others[4][3] = {{1, 2, 3}, {0, 2, 3}, {0, 1, 3}, {0, 1, 2}};
-  for (int a = 0; a < PF_N; ++a) {
-    const int* o = others[a];
-    D.g3[a][0] = p->gamma3[a][o[0]][o[1]];
-    D.g3[a][1] = p->gamma3[a][o[0]][o[2]];
-    D.g3[a][2] = p->gamma3[a][o[1]][o[2]];
-  }
-  int k = 0;
-  double tm = 0;
-  for (int a = 0; a < PF_N; ++a)
-    for (int b = a + 1; b < PF_N; ++b) {
-      D.tau[k++] = p->tau[a][b];
-      tm += p->tau[a][b];
-    }
-  D.inv_tau_mean = 6.0 / tm;
-  bool ta = false;
-  for (int a = 0; a < PF_N; ++a) {
-    const double(*A0)[2] = p->A0[a];
-    const double(*A1)[2] = p->A1[a];
-    D.psiA[a][0] = A0[0][0];
-    D.psiA[a][1] = A0[0][1] + A0[1][0];
-    D.psiA[a][2] = A0[1][1];
-    D.psiA1[a][0] = A1[0][0];
-    D.psiA1[a][1] = A1[0][1] + A1[1][0];
-    D.psiA1[a][2] = A1[1][1];
-    for (int i = 0; i < 2; ++i) {
-      D.B0[a][i] = p->B0[a][i];
-      D.B1[a][i] = p->B1[a][i];
-      for (int j = 0; j < 2; ++j) ta |= A1[i][j] != 0.0;
-    }
-    D.C0[a] = p->C0[a];
-    D.C1[a] = p->C1[a];
-    // chi = -(A + A^T)  [A6]
-    D.chi0[a][0] = -(A0[0][0] + A0[0][0]);
-    D.chi0[a][1] = -(A0[0][1] + A0[1][0]);
-    D.chi0[a][2] = -(A0[1][1] + A0[1][1]);
-    D.chi1[a][0] = -(A1[0][0] + A1[0][0]);
-    D.chi1[a][1] = -(A1[0][1] + A1[1][0]);
-    D.chi1[a][2] = -(A1[1][1] + A1[1][1]);
-    // P = D_a chi_a (eq. 9, D left-multiplied [A7]), split in c0 + T c1
-    const double X0[2][2] = {{D.chi0[a][0], D.chi0[a][1]}, {D.chi0[a][1], D.chi0[a][2]}};
-    const double X1[2][2] = {{D.chi1[a][0], D.chi1[a][1]}, {D.chi1[a][1], D.chi1[a][2]}};
-    for (int i = 0; i < 2; ++i)
-      for (int j = 0; j < 2; ++j) {
-        D.P0[a][2 * i + j] = p->D[a][i][0] * X0[0][j] + p->D[a][i][1] * X0[1][j];
-        D.P1[a][2 * i + j] = p->D[a][i][0] * X1[0][j] + p->D[a][i][1] * X1[1][j];
-      }
-    D.dcT[a][0] = D.chi1[a][0];
-    D.dcT[a][1] = D.chi1[a][1];
-    D.dcT[a][2] = D.chi1[a][2];
-    D.dcT[a][3] = -p->B1[a][0];
-    D.dcT[a][4] = -p->B1[a][1];
-  }
-  for (int s = 0; s < PF_N - 1; ++s) {
-    const int a = s < L ? s : s + 1;
-    for (int i = 0; i < 3; ++i) {
-      D.dchi0[s][i] = D.chi0[L][i] - D.chi0[a][i];
-      D.dchi1[s][i] = D.chi1[L][i] - D.chi1[a][i];
-    }
-    for (int i = 0; i < 2; ++i) {
-      D.dB0[s][i] = p->B0[L][i] - p->B0[a][i];
-      D.dB1[s][i] = p->B1[L][i] - p->B1[a][i];
-    }
-  }
-  D.liquid = L;
-  D.TA = ta ? 1 : 0;
+  pf::fill_dev_params(*p, L, &ctx->dp);
   ctx->hp = *p;
   ctx->have_params = true;
+  ctx->jit = nullptr;
   return PF_OK;
 }
 
@@ -627,8 +637,15 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
   cudaEvent_t e0 = nullptr;
   // Algorithm 1, line 1: phi-sweep
   prof_begin(ctx, 0, &e0);
+  if (ctx->variant == PF_VARIANT_JIT && !ctx->jit) {
+    std::string err;
+    ctx->jit = jit_get(ctx->dp, g, &err);
+    if (!ctx->jit) return fail(ctx, PF_ECUDA, "run-time specialisation failed: %s", err.c_str());
+  }
   if (ctx->variant == PF_VARIANT_NAIVE)
     launch_phi_naive(ctx->dp, g, ps, ms, pd, ctx->stream);
+  else if (ctx->variant == PF_VARIANT_JIT)
+    CU(jit_launch_phi(ctx->jit, ctx->dp, ps, ms, pd, ctx->stream));
   else
     launch_phi_tuned(ctx->dp, g, ps, ms, pd, ctx->stream);
   ctx->nlaunch[0] += 1;
@@ -646,6 +663,8 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
     prof_begin(ctx, 1, &e0);
     if (ctx->variant == PF_VARIANT_NAIVE)
       launch_mu_naive(ctx->dp, g, ps, pd, ms, md, ctx->stream);
+    else if (ctx->variant == PF_VARIANT_JIT)
+      CU(jit_launch_mu(ctx->jit, ctx->dp, ps, pd, ms, md, ctx->stream));
     else
       launch_mu_tuned(ctx->dp, g, ps, pd, ms, md, ctx->stream);
     ctx->nlaunch[1] += 1;
@@ -755,7 +774,8 @@ int pf_set_state(pf_ctx* ctx, const pf_state* s) {
 }
 
 int pf_set_variant(pf_ctx* ctx, int variant) {
-  if (!ctx || (variant != PF_VARIANT_TUNED && variant != PF_VARIANT_NAIVE)) return PF_EINVAL;
+  if (!ctx || (variant != PF_VARIANT_TUNED && variant != PF_VARIANT_NAIVE && variant != PF_VARIANT_JIT))
+    return PF_EINVAL;
   ctx->variant = variant;
   return PF_OK;
 }

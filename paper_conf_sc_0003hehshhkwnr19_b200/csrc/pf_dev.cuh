@@ -1,0 +1,66 @@
+// pf_dev.cuh -- device-side types shared by the ahead-of-time (nvcc) build
+// and the run-time specialised (NVRTC) build of the sweep kernels.  Must
+// stay free of host headers: NVRTC compiles it as-is.
+#pragma once
+
+namespace pf {
+
+typedef long long i64;
+
+constexpr int N = 4;  // phases (P1: 3 solids + liquid)
+constexpr int M = 2;  // chemical potentials, K - 1
+constexpr int NSOL = N - 1;
+
+// One ghost layer (indices -1 and n) inside an allocated guard ring of width
+// 2 in y and z (and >= 2 in x), so that kernels may read any index in
+// [-2, n+1] without bounds checks (edge threads of ragged tiles clamp to the
+// ghost cell).
+constexpr int GUARD = 2;
+
+// Geometry of one block in the padded ghosted layout (pf_layout), run-time
+// values.  The specialised build uses a type with the same members as
+// compile-time constants.
+struct Geom {
+  int nx, ny, nz;
+  int z0;  // global z index of local interior plane 0
+  i64 pitch, plane, field, xoff;
+  __host__ __device__ __forceinline__ i64 at(int x, int y, int z) const {
+    return (i64)(z + GUARD) * plane + (i64)(y + GUARD) * pitch + xoff + x;
+  }
+};
+
+// Scalars and coefficients of the model.  Passed by value to every kernel
+// (kernel-parameter constant bank) in the generic build; folded into the
+// code as compile-time constants in the specialised build.  T-dependent
+// coefficients are stored as value = c0 + T c1 (eq. 6: A, B, C affine in T).
+struct DevParams {
+  double dx, dt, eps;
+  double inv_dt;
+  double inv_dx2;       // 1 / dx^2
+  double phi_grad_c;    // eps / dx^2
+  double inv_eps;
+  double dt_over_eps;
+  double at_c;          // dx * pi eps / (8 dt): anti-trapping prefactor in unscaled units
+  double dTdt;          // -G v
+  double Tbase, Tdz;    // T(local plane k) = Tbase + Tdz k; Tbase is set per step  [A13]
+  double mu_inf[M];
+  // phi-sweep
+  double g[N][N];       // gamma_ab (diag 0)
+  double og[N][N];      // 16/pi^2 gamma_ab
+  double g3[N][3];      // gamma_abd for the 3 pairs (b<d, b,d != a) of phase a, see kOtherPair()
+  double tau[6];        // tau_ab for pairs (0,1),(0,2),(0,3),(1,2),(1,3),(2,3)
+  double inv_tau_mean;  // 1 / mean tau_ab (tau of a pure cell, reading A5)
+  double psiA[N][3], psiA1[N][3];  // mu.A mu = a00 m0^2 + (a01+a10) m0 m1 + a11 m1^2
+  double B0[N][M], B1[N][M];
+  double C0[N], C1[N];
+  // mu-sweep
+  double chi0[N][3], chi1[N][3];   // chi_a = dc_a/dmu = -(A + A^T) (sym: 00, 01, 11)  [A6]
+  double P0[N][4], P1[N][4];       // D_a chi_a (row-major 00 01 10 11), eq. 9  [A7]
+  double dchi0[NSOL][3], dchi1[NSOL][3];  // chi_l - chi_s
+  double dB0[NSOL][M], dB1[NSOL][M];      // B_l - B_s
+  double dcT[N][5];     // dc_a/dT = -(A1 + A1^T) mu - B1: [s00, s01, s11, -B1_0, -B1_1]
+  int liquid;
+  int TA;               // A1 != 0: chi and the mobility depend on T
+};
+
+}  // namespace pf

@@ -7,9 +7,29 @@
 // (pf_tuned.cu).
 #include <math.h>
 
+#include "pf_internal.h"
 #include "pf_model.cuh"
 
 namespace pf {
+
+// dispatch on the liquid index (compile-time L) and the T-dependence of A (TA)
+#define PF_DISPATCH_TA(TA, ...)                  \
+  if (TA) {                                      \
+    constexpr bool TT = true;                    \
+    __VA_ARGS__;                                 \
+  } else {                                       \
+    constexpr bool TT = false;                   \
+    __VA_ARGS__;                                 \
+  }
+#define PF_DISPATCH(L, TA, ...)                                        \
+  switch (L) {                                                         \
+    case 0: { constexpr int LL = 0; PF_DISPATCH_TA(TA, __VA_ARGS__); } break; \
+    case 1: { constexpr int LL = 1; PF_DISPATCH_TA(TA, __VA_ARGS__); } break; \
+    case 2: { constexpr int LL = 2; PF_DISPATCH_TA(TA, __VA_ARGS__); } break; \
+    default: { constexpr int LL = 3; PF_DISPATCH_TA(TA, __VA_ARGS__); } break; \
+  }
+
+
 
 // ---------------------------------------------------------------------------
 // Naive phi-sweep: one thread per cell, 6 faces each (Algorithm 1 line 1).
@@ -43,7 +63,7 @@ __global__ void __launch_bounds__(256) k_phi_naive(DevParams P, Geom g, const do
   }
   const double mu0 = __ldg(ms + c), mu1 = __ldg(ms + F + c);
   double out[N];
-  phi_cell<TA>(P, plane_T(P, (double)z), ph, gd, divh, mu0, mu1, out);
+  phi_cell<TA>(P, plane_T(P, P, (double)z), ph, gd, divh, mu0, mu1, out);
 #pragma unroll
   for (int a = 0; a < N; ++a) pd[a * F + c] = out[a];
 }
@@ -81,15 +101,15 @@ __global__ void __launch_bounds__(256) k_mu_naive(DevParams P, Geom g, const dou
   if (x >= g.nx || y >= g.ny || z >= g.nz) return;
   const int64_t c = g.at(x, y, z);
   const int64_t F = g.field;
-  const double Tc = plane_T(P, (double)z);
+  const double Tc = plane_T(P, P, (double)z);
   double divh[M] = {0.0, 0.0};
 #pragma unroll 1
   for (int d = 0; d < 3; ++d) {
     const int64_t sn = d == 0 ? 1 : (d == 1 ? g.pitch : g.plane);
     const int64_t s1 = d == 0 ? g.pitch : 1;
     const int64_t s2 = d == 2 ? g.pitch : g.plane;
-    const double Tp = d == 2 ? plane_T(P, z + 0.5) : Tc;
-    const double Tm = d == 2 ? plane_T(P, z - 0.5) : Tc;
+    const double Tp = d == 2 ? plane_T(P, P, z + 0.5) : Tc;
+    const double Tm = d == 2 ? plane_T(P, P, z - 0.5) : Tc;
     FaceSide sm, s0, sp;
     load_side<L>(ps, pd, ms, F, c - sn, s1, s2, sm);
     load_side<L>(ps, pd, ms, F, c, s1, s2, s0);

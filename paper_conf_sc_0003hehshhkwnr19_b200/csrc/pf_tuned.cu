@@ -1,316 +1,51 @@
-// pf_tuned.cu -- the tuned phi- and mu-sweeps for sm_100a.
-//
-// Both kernels are bound by the fp64 pipe (Table 1: ~1.5 kFLOP per cell vs
-// 96 B of compulsory traffic), so the design goal is to issue
-// as few fp64 instructions per cell as possible and to keep the L1/shared
-// memory pipe below the fp64 pipe:
-//   * a CTA owns a 32 x 8 column tile and marches along z (2.5-D blocking);
-//   * every staggered face flux is computed ONCE: each thread computes the
-//     -x, -y and +z faces of its cell, the +x / +y faces come from the
-//     neighbour thread (warp shuffle / shared memory), and the two faces on
-//     the far tile edges are computed by one extra warp each;
-//   * the z-face flux is carried in registers to the next plane.
-// The paper's "split" kernels cache fluxes in a global staggered array
-// (P:L709-721); here they never leave the SM.
-#include "pf_model.cuh"
+// pf_tuned.cu -- generic (ahead-of-time) instantiation of the tuned sweeps
+// of pf_sweeps.cuh: parameters in the kernel-parameter constant bank,
+// geometry at run time.  The specialised build (pf_jit.cu) compiles the same
+// bodies with both folded in.
+#include "pf_internal.h"
+#include "pf_sweeps.cuh"
 
 namespace pf {
 
-constexpr int TX = 32;
-constexpr int TY = 8;
-constexpr int ZC_PHI = 32;  // z-chunk per CTA
-constexpr int ZC_MU = 32;
+// dispatch on the liquid index (compile-time L) and the T-dependence of A (TA)
+#define PF_DISPATCH_TA(TA, ...)                  \
+  if (TA) {                                      \
+    constexpr bool TT = true;                    \
+    __VA_ARGS__;                                 \
+  } else {                                       \
+    constexpr bool TT = false;                   \
+    __VA_ARGS__;                                 \
+  }
+#define PF_DISPATCH(L, TA, ...)                                        \
+  switch (L) {                                                         \
+    case 0: { constexpr int LL = 0; PF_DISPATCH_TA(TA, __VA_ARGS__); } break; \
+    case 1: { constexpr int LL = 1; PF_DISPATCH_TA(TA, __VA_ARGS__); } break; \
+    case 2: { constexpr int LL = 2; PF_DISPATCH_TA(TA, __VA_ARGS__); } break; \
+    default: { constexpr int LL = 3; PF_DISPATCH_TA(TA, __VA_ARGS__); } break; \
+  }
 
-// ===========================================================================
-// phi-sweep (Algorithm 1 line 1): D3C7 of phi_src, D3C1 of mu_src.
-// ===========================================================================
+
 template <int L, bool TA>
 __global__ void __launch_bounds__(TX* TY, 2) k_phi_tuned(DevParams P, Geom g, const double* __restrict__ ps,
                                                          const double* __restrict__ ms, double* __restrict__ pd) {
-  __shared__ double fy[2][N][TY][TX];  // -y face flux of every thread, by plane parity
-  __shared__ double ex[2][N][TY];      // +x flux on the right tile edge
-  __shared__ double ey[2][N][TX];      // +y flux on the top tile edge
-  const int lane = threadIdx.x, w = threadIdx.y;
-  const int x0 = blockIdx.x * TX, y0 = blockIdx.y * TY;
-  const int x = x0 + lane, y = y0 + w;
-  const bool active = x < g.nx && y < g.ny;
-  // ragged tiles: clamp to the ghost cell, whose -x / -y face is the +x / +y
-  // face of the last interior cell
-  const int xc = min(x, g.nx), yc = min(y, g.ny);
-  const int z0 = blockIdx.z * ZC_PHI, z1 = min(z0 + ZC_PHI, g.nz);
-  const int64_t F = g.field, SY = g.pitch, SZ = g.plane;
-  // extra faces: warp 0 lanes < TY: +x face of row `lane`; warp 1: +y face of column `lane`
-  int64_t ep = 0, eq = 0;  // the two cells of the extra face, at plane z0
-  if (w == 0 && lane < TY) {
-    const int ry = min(y0 + lane, g.ny);
-    ep = g.at(min(x0 + TX - 1, g.nx), ry, z0);
-    eq = g.at(min(x0 + TX, g.nx), ry, z0);
-  } else if (w == 1) {
-    const int cx = min(x0 + lane, g.nx);
-    ep = g.at(cx, min(y0 + TY - 1, g.ny), z0);
-    eq = g.at(cx, min(y0 + TY, g.ny), z0);
-  }
-  const bool extra = (w == 0 && lane < TY) || w == 1;
-
-  int64_t c = g.at(xc, yc, z0);
-  double pm[N], p0[N], Fzm[N];
-#pragma unroll
-  for (int a = 0; a < N; ++a) {
-    pm[a] = __ldg(ps + a * F + c - SZ);
-    p0[a] = __ldg(ps + a * F + c);
-  }
-  phi_face(P, pm, p0, Fzm);
-
-  for (int z = z0; z < z1; ++z, c += SZ, ep += SZ, eq += SZ) {
-    const int buf = z & 1;
-    double pp[N], Fxm[N], Fym[N], Fzp[N], gd[N][3];
-    {
-      double xm[N], xp[N], ym[N], yp[N];
-#pragma unroll
-      for (int a = 0; a < N; ++a) {
-        const double* f = ps + a * F + c;
-        pp[a] = __ldg(f + SZ);
-        xm[a] = __ldg(f - 1);
-        xp[a] = __ldg(f + 1);
-        ym[a] = __ldg(f - SY);
-        yp[a] = __ldg(f + SY);
-        gd[a][0] = xp[a] - xm[a];
-        gd[a][1] = yp[a] - ym[a];
-        gd[a][2] = pp[a] - pm[a];
-      }
-      phi_face(P, xm, p0, Fxm);
-      phi_face(P, ym, p0, Fym);
-    }
-    phi_face(P, p0, pp, Fzp);
-    if (extra) {
-      double fa[N], fb[N], fe[N];
-#pragma unroll
-      for (int a = 0; a < N; ++a) {
-        fa[a] = __ldg(ps + a * F + ep);
-        fb[a] = __ldg(ps + a * F + eq);
-      }
-      phi_face(P, fa, fb, fe);
-      if (w == 0) {
-#pragma unroll
-        for (int a = 0; a < N; ++a) ex[buf][a][lane] = fe[a];
-      } else {
-#pragma unroll
-        for (int a = 0; a < N; ++a) ey[buf][a][lane] = fe[a];
-      }
-    }
-#pragma unroll
-    for (int a = 0; a < N; ++a) fy[buf][a][w][lane] = Fym[a];
-    const double mu0 = __ldg(ms + c), mu1 = __ldg(ms + F + c);
-    __syncthreads();
-    double divh[N];
-#pragma unroll
-    for (int a = 0; a < N; ++a) {
-      double fxp = __shfl_down_sync(0xffffffffu, Fxm[a], 1);
-      if (lane == TX - 1) fxp = ex[buf][a][w];
-      const double fyp = (w < TY - 1) ? fy[buf][a][w + 1][lane] : ey[buf][a][lane];
-      divh[a] = ((fxp - Fxm[a]) + (fyp - Fym[a])) + (Fzp[a] - Fzm[a]);
-    }
-    double out[N];
-    phi_cell<TA>(P, plane_T(P, (double)z), p0, gd, divh, mu0, mu1, out);
-    if (active) {
-#pragma unroll
-      for (int a = 0; a < N; ++a) pd[a * F + c] = out[a];
-    }
-#pragma unroll
-    for (int a = 0; a < N; ++a) {
-      pm[a] = p0[a];
-      p0[a] = pp[a];
-      Fzm[a] = Fzp[a];
-    }
-  }
-}
-
-// ===========================================================================
-// mu-sweep (Algorithm 1 line 3): D3C19 of phi_src, D3C7 of phi_dst and mu.
-//
-// Per plane k every cell of the tile and of its 1-cell halo ring publishes
-// its "face side" data D (phi, the three central differences, dphi, mu) to
-// shared memory once; the -x / -y faces read both sides from there, the
-// z-face k-1/2 pairs the previous plane's D (registers) with the current
-// one, and the cell update of plane k-1 is done as soon as that z-face is
-// known (one-plane lag).
-// ===========================================================================
-constexpr int HX = TX + 2, HY = TY + 2, NC = HX * HY;
-// shared-memory D layout, structure of arrays over the NC halo-tile cells
-constexpr int D_F = 0;            // phi      [N]
-constexpr int D_CX = D_F + N;     // cd_x     [N]
-constexpr int D_CY = D_CX + N;    // cd_y     [N]
-constexpr int D_CZ = D_CY + N;    // cd_z     [N]
-constexpr int D_DP = D_CZ + N;    // dphi     [N] (phi_dst - phi_src)
-constexpr int D_MU = D_DP + N;    // mu       [M]
-constexpr int D_NV = D_MU + M;    // 22 doubles per cell
-constexpr size_t MU_SMEM = (size_t)(D_NV * NC + M * TY * (TX + 1) + M * (TY + 1) * TX) * sizeof(double);
-
-__device__ __forceinline__ int hidx(int hx, int hy) { return hy * HX + hx; }  // halo-tile coords (0..HX-1, 0..HY-1)
-
-// build D of cell (x,y,k) from global memory into shared slot i;
-// wx / wy / wz: compute cd_x / cd_y / cd_z (halo cells only need the
-// tangential ones, and must not read beyond the guard ring)
-__device__ __forceinline__ void build_cell(const Geom& g, const double* __restrict__ ps, const double* __restrict__ pd,
-                                           const double* __restrict__ ms, int x, int y, int k, bool wx, bool wy,
-                                           bool wz, double* __restrict__ D, int i) {
-  const int64_t F = g.field;
-  const int64_t c = g.at(x, y, k);
-#pragma unroll
-  for (int a = 0; a < N; ++a) {
-    const double* f = ps + a * F + c;
-    const double v = __ldg(f);
-    D[(D_F + a) * NC + i] = v;
-    if (wx) D[(D_CX + a) * NC + i] = __ldg(f + 1) - __ldg(f - 1);
-    if (wy) D[(D_CY + a) * NC + i] = __ldg(f + g.pitch) - __ldg(f - g.pitch);
-    if (wz) D[(D_CZ + a) * NC + i] = __ldg(f + g.plane) - __ldg(f - g.plane);
-    D[(D_DP + a) * NC + i] = __ldg(pd + a * F + c) - v;
-  }
-  D[(D_MU + 0) * NC + i] = __ldg(ms + c);
-  D[(D_MU + 1) * NC + i] = __ldg(ms + F + c);
-}
-
-template <int L>
-__device__ __forceinline__ void side_from_smem(const double* __restrict__ D, int i, int c1, int c2, FaceSide& s) {
-#pragma unroll
-  for (int a = 0; a < N; ++a) {
-    s.f[a] = D[(D_F + a) * NC + i];
-    s.c1[a] = D[(c1 + a) * NC + i];
-    s.c2[a] = D[(c2 + a) * NC + i];
-  }
-#pragma unroll
-  for (int t = 0; t < NSOL; ++t) s.ds[t] = D[(D_DP + solid_phase(L, t)) * NC + i];
-  s.m[0] = D[(D_MU + 0) * NC + i];
-  s.m[1] = D[(D_MU + 1) * NC + i];
+  phi_tuned_body<DevParams, Geom, L, TA>(P, P, g, ps, ms, pd);
 }
 
 template <int L, bool TA>
 __global__ void __launch_bounds__(TX* TY, 2) k_mu_tuned(DevParams P, Geom g, const double* __restrict__ ps,
                                                         const double* __restrict__ pd, const double* __restrict__ ms,
                                                         double* __restrict__ md) {
-  extern __shared__ double smem[];
-  double* D = smem;                          // [D_NV][NC]
-  double* fxs = D + D_NV * NC;               // [M][TY][TX+1]: x-face fluxes, face i = x0 - 1/2 + i
-  double* fys = fxs + M * TY * (TX + 1);     // [M][TY+1][TX]: y-face fluxes
-  const int lane = threadIdx.x, w = threadIdx.y, t = w * TX + lane;
-  const int x0 = blockIdx.x * TX, y0 = blockIdx.y * TY;
-  const int x = x0 + lane, y = y0 + w;
-  const bool active = x < g.nx && y < g.ny;
-  const int xc = min(x, g.nx), yc = min(y, g.ny);
-  const int z0 = blockIdx.z * ZC_MU, z1 = min(z0 + ZC_MU, g.nz);
-  const int64_t F = g.field;
-  const int me = hidx(lane + 1, w + 1);
-  // halo ring cell owned by thread t < 2*TX + 2*TY (corners are not needed)
-  // (warps 4.. build the halo ring; warps 0, 1 compute the far-edge faces)
-  int hx = 0, hy = 0, hs = -1;
-  bool hwx = false, hwy = false;
-  const int th = t - 4 * TX;
-  if (th >= 0 && th < TX) { hx = th + 1; hy = 0; hwx = true; }
-  else if (th >= TX && th < 2 * TX) { hx = th - TX + 1; hy = TY + 1; hwx = true; }
-  else if (th >= 2 * TX && th < 2 * TX + TY) { hx = 0; hy = th - 2 * TX + 1; hwy = true; }
-  else if (th >= 2 * TX + TY && th < 2 * TX + 2 * TY) { hx = TX + 1; hy = th - 2 * TX - TY + 1; hwy = true; }
-  if (hwx || hwy) hs = hidx(hx, hy);
-  const int hgx = min(x0 + hx - 1, g.nx), hgy = min(y0 + hy - 1, g.ny);
-
-  // z-face k-1/2 needs the previous plane's side (tangential: x, y)
-  FaceSide Dp;
-  double dpl = 0.0;  // dphi of the liquid at plane k-1 (for the cell update)
-  {
-    const int64_t c = g.at(xc, yc, z0 - 1);
-#pragma unroll
-    for (int a = 0; a < N; ++a) {
-      const double* f = ps + a * F + c;
-      Dp.f[a] = __ldg(f);
-      Dp.c1[a] = __ldg(f + 1) - __ldg(f - 1);
-      Dp.c2[a] = __ldg(f + g.pitch) - __ldg(f - g.pitch);
-    }
-#pragma unroll
-    for (int s = 0; s < NSOL; ++s) {
-      const int a = solid_phase(L, s);
-      Dp.ds[s] = __ldg(pd + a * F + c) - Dp.f[a];
-    }
-    Dp.m[0] = __ldg(ms + c);
-    Dp.m[1] = __ldg(ms + F + c);
-  }
-  double divxy[M] = {0.0, 0.0}, Fzm[M] = {0.0, 0.0};
-
-  for (int k = z0; k <= z1; ++k) {
-    const bool last = k == z1;
-    // (a) publish D(k) of the own cell and of the halo ring
-    build_cell(g, ps, pd, ms, xc, yc, k, true, true, !last, D, me);
-    if (hs >= 0 && !last) build_cell(g, ps, pd, ms, hgx, hgy, k, hwx, hwy, true, D, hs);
-    __syncthreads();
-    // (b) z-face k-1/2 from registers (plane k-1) and shared memory (plane k)
-    FaceSide q;
-    side_from_smem<L>(D, me, D_CX, D_CY, q);
-    double Fz[M];
-    mu_face<L, TA>(P, plane_T(P, k - 0.5), Dp, q, Fz);
-    // (c) cell update of plane k-1
-    if (k > z0 && active) {
-      double ph[N], dph[N], out[M];
-      const double divh[M] = {divxy[0] + (Fz[0] - Fzm[0]), divxy[1] + (Fz[1] - Fzm[1])};
-#pragma unroll
-      for (int a = 0; a < N; ++a) ph[a] = Dp.f[a];
-#pragma unroll
-      for (int s = 0; s < NSOL; ++s) dph[solid_phase(L, s)] = Dp.ds[s];
-      dph[L] = dpl;
-      mu_cell<TA>(P, plane_T(P, (double)(k - 1)), ph, dph, Dp.m, divh, out);
-      const int64_t c = g.at(xc, yc, k - 1);
-      md[c] = out[0];
-      md[F + c] = out[1];
-    }
-    Fzm[0] = Fz[0];
-    Fzm[1] = Fz[1];
-    // carry plane k's side for the next z-face
-    Dp = q;
-    dpl = D[(D_DP + L) * NC + me];
-    if (!last) {
-      // (d) faces of plane k: -x and -y of every thread, + the far tile edges
-      const double Tk = plane_T(P, (double)k);
-      FaceSide p, s;
-      double Fx[M], Fy[M];
-      side_from_smem<L>(D, me - 1, D_CY, D_CZ, p);
-      side_from_smem<L>(D, me, D_CY, D_CZ, s);
-      mu_face<L, TA>(P, Tk, p, s, Fx);
-      side_from_smem<L>(D, me - HX, D_CX, D_CZ, p);
-      side_from_smem<L>(D, me, D_CX, D_CZ, s);
-      mu_face<L, TA>(P, Tk, p, s, Fy);
-#pragma unroll
-      for (int i = 0; i < M; ++i) {
-        fxs[(i * TY + w) * (TX + 1) + lane] = Fx[i];
-        fys[(i * (TY + 1) + w) * TX + lane] = Fy[i];
-      }
-      if (w == 0) {  // +y face of the top tile edge, column `lane`
-        double Fe[M];
-        side_from_smem<L>(D, hidx(lane + 1, TY), D_CX, D_CZ, p);
-        side_from_smem<L>(D, hidx(lane + 1, TY + 1), D_CX, D_CZ, s);
-        mu_face<L, TA>(P, Tk, p, s, Fe);
-#pragma unroll
-        for (int i = 0; i < M; ++i) fys[(i * (TY + 1) + TY) * TX + lane] = Fe[i];
-      } else if (w == 1 && lane < TY) {  // +x face of the right tile edge, row `lane`
-        double Fe[M];
-        side_from_smem<L>(D, hidx(TX, lane + 1), D_CY, D_CZ, p);
-        side_from_smem<L>(D, hidx(TX + 1, lane + 1), D_CY, D_CZ, s);
-        mu_face<L, TA>(P, Tk, p, s, Fe);
-#pragma unroll
-        for (int i = 0; i < M; ++i) fxs[(i * TY + lane) * (TX + 1) + TX] = Fe[i];
-      }
-    }
-    __syncthreads();
-    if (!last) {
-#pragma unroll
-      for (int i = 0; i < M; ++i)
-        divxy[i] = (fxs[(i * TY + w) * (TX + 1) + lane + 1] - fxs[(i * TY + w) * (TX + 1) + lane]) +
-                   (fys[(i * (TY + 1) + w + 1) * TX + lane] - fys[(i * (TY + 1) + w) * TX + lane]);
-    }
-  }
+  mu_tuned_body<DevParams, Geom, L, TA>(P, P, g, ps, pd, ms, md);
 }
 
-// ===========================================================================
+dim3 tuned_block() { return dim3(TX, TY); }
+dim3 tuned_grid_phi(const Geom& g) { return dim3((g.nx + TX - 1) / TX, (g.ny + TY - 1) / TY, (g.nz + ZC_PHI - 1) / ZC_PHI); }
+dim3 tuned_grid_mu(const Geom& g) { return dim3((g.nx + TX - 1) / TX, (g.ny + TY - 1) / TY, (g.nz + ZC_MU - 1) / ZC_MU); }
+size_t tuned_mu_smem() { return MU_SMEM; }
+
 void launch_phi_tuned(const DevParams& P, const Geom& g, const double* ps, const double* ms, double* pd,
                       cudaStream_t s) {
-  dim3 b(TX, TY), gr((g.nx + TX - 1) / TX, (g.ny + TY - 1) / TY, (g.nz + ZC_PHI - 1) / ZC_PHI);
-  PF_DISPATCH(P.liquid, P.TA, (k_phi_tuned<LL, TT><<<gr, b, 0, s>>>(P, g, ps, ms, pd)));
+  PF_DISPATCH(P.liquid, P.TA, (k_phi_tuned<LL, TT><<<tuned_grid_phi(g), tuned_block(), 0, s>>>(P, g, ps, ms, pd)));
 }
 
 template <int L, bool TA>
@@ -321,8 +56,7 @@ static void mu_launch(const DevParams& P, const Geom& g, const double* ps, const
     cudaFuncSetAttribute(k_mu_tuned<L, TA>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)MU_SMEM);
     attr = true;
   }
-  dim3 b(TX, TY), gr((g.nx + TX - 1) / TX, (g.ny + TY - 1) / TY, (g.nz + ZC_MU - 1) / ZC_MU);
-  k_mu_tuned<L, TA><<<gr, b, MU_SMEM, s>>>(P, g, ps, pd, ms, md);
+  k_mu_tuned<L, TA><<<tuned_grid_mu(g), tuned_block(), MU_SMEM, s>>>(P, g, ps, pd, ms, md);
 }
 
 void launch_mu_tuned(const DevParams& P, const Geom& g, const double* ps, const double* pd, const double* ms,

@@ -20,7 +20,7 @@ PF_OK, PF_EINVAL, PF_ENOMEM, PF_ECUDA, PF_ENCCL, PF_ESTATE, PF_ENUMERIC = 0, -1,
 BC = {"periodic": 0, "neumann": 1, "dirichlet_mu": 2}
 PF_HOST, PF_DEVICE = 0, 1
 PF_PHI, PF_MU = 1, 2
-VARIANT = {"tuned": 0, "naive": 1}
+VARIANT = {"tuned": 0, "naive": 1, "jit": 2}
 N, M = 4, 2
 
 
@@ -58,7 +58,7 @@ class PFState(C.Structure):
 ABI_SYMBOLS = ["pf_query_layout", "pf_create", "pf_destroy", "pf_set_params", "pf_init_fields", "pf_step",
                "pf_step_phi_only", "pf_halo_exchange", "pf_shift_window", "pf_front_height", "pf_monitor",
                "pf_download", "pf_get_state", "pf_set_state", "pf_set_variant", "pf_profile", "pf_profile_read",
-               "pf_nccl_unique_id", "pf_last_error", "pf_version"]
+               "pf_nccl_unique_id", "pf_jit_compile_only", "pf_last_error", "pf_version"]
 
 _lib = None
 
@@ -91,6 +91,7 @@ def load_library(path: str = LIB_PATH):
     L.pf_profile.argtypes = [vp, ip]
     L.pf_profile_read.argtypes = [vp, dp, C.POINTER(C.c_int64)]
     L.pf_nccl_unique_id.argtypes = [C.POINTER(C.c_ubyte)]
+    L.pf_jit_compile_only.argtypes = [C.POINTER(PFParams), ip, ip, C.c_char_p, C.c_char_p, ip]
     L.pf_last_error.argtypes = [vp]
     L.pf_last_error.restype = C.c_char_p
     L.pf_version.restype = C.c_char_p
@@ -133,6 +134,18 @@ def make_params(P: dict) -> PFParams:
     return p
 
 
+def jit_compile_only(params: dict, n: int = 64, cubin_path: str | None = None) -> int:
+    """Compile the run-time specialised kernels for `params` and an n^3 block
+    without a GPU (NVRTC only); returns the cubin size."""
+    p = make_params(params)
+    log = C.create_string_buffer(8192)
+    r = load_library().pf_jit_compile_only(C.byref(p), int(params.get("liquid", 3)), int(n),
+                                           (cubin_path or "").encode(), log, 8192)
+    if r < 0:
+        raise PFError(f"specialised compile failed: {log.value.decode()}")
+    return r
+
+
 def nccl_unique_id() -> bytes:
     buf = (C.c_ubyte * 128)()
     r = load_library().pf_nccl_unique_id(buf)
@@ -149,7 +162,7 @@ class PhaseField:
     "dirichlet_mu".  Buffers are torch tensors owned by this object.
     """
 
-    def __init__(self, shape, params: dict, bc=None, liquid: int = 3, procs=(1, 1, 1), rank: int = 0,
+    def __init__(self, shape, params: dict, bc=None, liquid: int | None = None, procs=(1, 1, 1), rank: int = 0,
                  world: int = 1, device: int | None = None, nccl_uid: bytes | None = None, stream=None):
         import torch
         if not torch.cuda.is_available():
@@ -162,7 +175,8 @@ class PhaseField:
         nz, ny, nx = shape
         bc = bc or {"lo": ("periodic",) * 3, "hi": ("periodic",) * 3}
         cfg = PFConfig()
-        cfg.n_phases, cfg.n_mu, cfg.liquid = N, M, int(liquid)
+        liquid = int(params.get("liquid", 3)) if liquid is None else int(liquid)
+        cfg.n_phases, cfg.n_mu, cfg.liquid = N, M, liquid
         for d, n in enumerate((nx, ny, nz)):
             cfg.global_[d] = n
             cfg.procs[d] = int(procs[d])

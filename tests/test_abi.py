@@ -86,3 +86,15 @@ def test_no_oracle_in_product_path():
                 s = open(os.path.join(dp, f)).read()
                 for pat in (r"^\s*(from|import)\s+oracle", r"#include\s+[<\"].*oracle", r"pf_oracle", r"oracle_\w+\("):
                     assert not re.search(pat, s, flags=re.M), (f, pat)
+
+
+def test_specialised_kernels_compile_without_gpu(lib, tmp_path):
+    """The run-time specialisation (NVRTC, sm_100a) builds for the C.4 and
+    stress parameter sets and every liquid index, with no device present."""
+    from paper_conf_sc_0003hehshhkwnr19_b200 import inputs as I
+    from paper_conf_sc_0003hehshhkwnr19_b200 import pf
+    cub = str(tmp_path / "k.cubin")
+    assert pf.jit_compile_only(I.params_c4("ds"), n=48, cubin_path=cub) > 0
+    out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-sass", cub], capture_output=True, text=True).stdout
+    assert "pf_jit_phi" in out and "pf_jit_mu" in out and "DFMA" in out
+    assert pf.jit_compile_only(dict(I.params_stress(), liquid=1), n=17) > 0

@@ -39,7 +39,7 @@ def omod():
     return O
 
 
-def run_pair(pfmod, omod, shape, P, ic, steps, bc=None, seed=20191117, variant="tuned", chunks=None, ic_kw=None):
+def run_pair(pfmod, omod, shape, P, ic, steps, bc=None, seed=20191117, variant="jit", chunks=None, ic_kw=None):
     phi, mu = I.make_ic(ic, shape, seed=seed, **(ic_kw or {}))
     g = pfmod.PhaseField(shape, P, bc=bc)
     g.set_variant(variant)
@@ -58,7 +58,7 @@ def run_pair(pfmod, omod, shape, P, ic, steps, bc=None, seed=20191117, variant="
     return out
 
 
-@pytest.mark.parametrize("variant", ["tuned", "naive"])
+@pytest.mark.parametrize("variant", ["jit", "tuned", "naive"])
 @pytest.mark.parametrize("pset", ["c4", "stress"])
 @pytest.mark.parametrize("ic", ["R", "V", "L"])
 def test_one_step_parity(pfmod, omod, variant, pset, ic):
@@ -68,11 +68,42 @@ def test_one_step_parity(pfmod, omod, variant, pset, ic):
         assert ep <= TOL_1 and em <= TOL_1, (ep, em)
 
 
-@pytest.mark.parametrize("shape", [(1, 1, 1), (3, 5, 7), (17, 9, 33), (8, 8, 130)])
-def test_ragged_and_tiny_shapes(pfmod, omod, shape):
+@pytest.mark.parametrize("variant", ["jit", "tuned"])
+@pytest.mark.parametrize("shape", [(1, 1, 1), (3, 5, 7), (17, 9, 33), (8, 8, 130), (40, 70, 65)])
+def test_ragged_and_tiny_shapes(pfmod, omod, shape, variant):
     P = I.params_stress()
-    for t, ep, em, *_ in run_pair(pfmod, omod, shape, P, "R", 2):
+    for t, ep, em, *_ in run_pair(pfmod, omod, shape, P, "R", 2, variant=variant):
         assert ep <= TOL_1 and em <= TOL_1, (shape, ep, em)
+
+
+@pytest.mark.parametrize("liquid", [0, 2])
+def test_liquid_index_not_hardcoded(pfmod, omod, liquid):
+    """Any phase may be the liquid l of eq. 10: permute the C.4 set so that
+    phase `liquid` plays the liquid, on both sides."""
+    P = I.params_stress()
+    perm = list(range(4))
+    perm[3], perm[liquid] = perm[liquid], perm[3]
+    Q = dict(P, liquid=liquid)
+    for key in ("A0", "A1", "B0", "B1", "C0", "C1", "D"):
+        Q[key] = P[key][perm]
+    Q["gamma"] = P["gamma"][np.ix_(perm, perm)]
+    Q["tau"] = P["tau"][np.ix_(perm, perm)]
+    Q["gamma3"] = P["gamma3"][np.ix_(perm, perm, perm)]
+    shape = (10, 12, 14)
+    phi, mu = I.ic_voronoi(shape, seed=12)
+    outs = {}
+    for variant in ("jit", "tuned"):
+        g = pfmod.PhaseField(shape, Q, liquid=liquid)
+        g.set_variant(variant)
+        g.init_fields(phi, mu)
+        g.step(2)
+        outs[variant] = g.download()
+    o = omod.Oracle(shape, Q)
+    o.init(phi, mu)
+    o.step(2)
+    op, om = o.download()
+    for v, (gp, gm) in outs.items():
+        assert rel_linf(gp, op) <= TOL_1 and rel_linf(gm, om) <= TOL_1, v
 
 
 def test_config1_50_steps(pfmod, omod):

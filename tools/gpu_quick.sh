@@ -6,11 +6,11 @@ mkdir -p $OUT
 python -c "import __graft_entry__ as g; g.build()" > $OUT/build.log 2>&1
 timeout 900 python -m pytest tests -m gpu -x -q > $OUT/pytest_gpu.log 2>&1; echo "pytest exit $?" >> $OUT/pytest_gpu.log
 timeout 300 python bench.py --steps 100 --warmup 5 --no-cpu-baseline --no-e2e > $OUT/bench.json 2> $OUT/bench.err
-timeout 300 python bench.py --steps 50 --warmup 5 --no-cpu-baseline --no-e2e --variant naive > $OUT/bench_naive.json 2>> $OUT/bench.err
+timeout 300 python bench.py --steps 50 --warmup 5 --no-cpu-baseline --no-e2e --variant tuned > $OUT/bench_tuned.json 2>> $OUT/bench.err
 if [ "$2" == "ncu" ]; then
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_mu_tuned -s 3 -c 1 -o $OUT/prof_mu \
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:pf_jit_mu -s 3 -c 1 -o $OUT/prof_mu \
    python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_mu.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_phi_tuned -s 3 -c 1 -o $OUT/prof_phi \
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:pf_jit_phi -s 3 -c 1 -o $OUT/prof_phi \
    python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_phi.log 2>&1
 fi
 echo done > $OUT/DONE
