@@ -26,6 +26,7 @@ void launch_mu_tuned(const DevParams& P, const Geom& g, const double* ps, const 
                      double* md, cudaStream_t s);
 // launch geometry of the tuned kernels (shared with the specialised build)
 dim3 tuned_block();
+dim3 tuned_block_mu();
 dim3 tuned_grid_phi(const Geom& g);
 dim3 tuned_grid_mu(const Geom& g);
 size_t tuned_mu_smem();

@@ -24,6 +24,10 @@ constexpr int TX = 32;
 constexpr int TY = 8;
 constexpr int ZC_PHI = 32;  // z-chunk per CTA
 constexpr int ZC_MU = 32;
+#ifndef PF_MU_TY
+#define PF_MU_TY 4  // tile height of the mu-sweep (4: 4 CTAs of 128 threads per SM)
+#endif
+constexpr int MU_TY = PF_MU_TY;
 
 // ===========================================================================
 // phi-sweep (Algorithm 1 line 1): D3C7 of phi_src, D3C1 of mu_src.
@@ -140,7 +144,11 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, 
 // one, and the cell update of plane k-1 is done as soon as that z-face is
 // known (one-plane lag).
 // ===========================================================================
-constexpr int HX = TX + 2, HY = TY + 2, NC = HX * HY;
+// halo tile of a TX x MTY column tile (MTY: tile height of the mu-sweep)
+template <int MTY>
+struct MuTile {
+  static constexpr int HX = TX + 2, HY = MTY + 2, NC = HX * HY;
+};
 // shared-memory D layout, structure of arrays over the NC halo-tile cells
 constexpr int D_F = 0;            // phi      [N]
 constexpr int D_CX = D_F + N;     // cd_x     [N]
@@ -149,14 +157,17 @@ constexpr int D_CZ = D_CY + N;    // cd_z     [N]
 constexpr int D_DP = D_CZ + N;    // dphi     [N] (phi_dst - phi_src)
 constexpr int D_MU = D_DP + N;    // mu       [M]
 constexpr int D_NV = D_MU + M;    // 22 doubles per cell
-constexpr size_t MU_SMEM = (size_t)(D_NV * NC + M * TY * (TX + 1) + M * (TY + 1) * TX) * sizeof(double);
-
-__device__ __forceinline__ int hidx(int hx, int hy) { return hy * HX + hx; }  // halo-tile coords (0..HX-1, 0..HY-1)
+template <int MTY>
+__host__ __device__ constexpr size_t mu_smem_bytes() {
+  return (size_t)(D_NV * MuTile<MTY>::NC + M * MTY * (TX + 1) + M * (MTY + 1) * TX) * sizeof(double);
+}
+// halo-tile coords (0..HX-1, 0..HY-1) -> slot
+__device__ __forceinline__ int hidx(int hx, int hy) { return hy * (TX + 2) + hx; }
 
 // build D of cell (x,y,k) from global memory into shared slot i;
 // wx / wy / wz: compute cd_x / cd_y / cd_z (halo cells only need the
 // tangential ones, and must not read beyond the guard ring)
-template <class GT>
+template <int NC, class GT>
 __device__ __forceinline__ void build_cell(const GT& g, const double* __restrict__ ps, const double* __restrict__ pd,
                                            const double* __restrict__ ms, int x, int y, int k, bool wx, bool wy,
                                            bool wz, double* __restrict__ D, int i) {
@@ -176,7 +187,7 @@ __device__ __forceinline__ void build_cell(const GT& g, const double* __restrict
   D[(D_MU + 1) * NC + i] = __ldg(ms + F + c);
 }
 
-template <int L>
+template <int L, int NC>
 __device__ __forceinline__ void side_from_smem(const double* __restrict__ D, int i, int c1, int c2, FaceSide& s) {
 #pragma unroll
   for (int a = 0; a < N; ++a) {
@@ -190,31 +201,32 @@ __device__ __forceinline__ void side_from_smem(const double* __restrict__ D, int
   s.m[1] = D[(D_MU + 1) * NC + i];
 }
 
-template <class PT, class GT, int L, bool TA>
+template <class PT, class GT, int L, bool TA, int MTY>
 __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, const GT& g,
                                               const double* __restrict__ ps, const double* __restrict__ pd,
                                               const double* __restrict__ ms, double* __restrict__ md) {
+  constexpr int NC = MuTile<MTY>::NC, HX = MuTile<MTY>::HX;
   extern __shared__ double smem[];
   double* D = smem;                          // [D_NV][NC]
-  double* fxs = D + D_NV * NC;               // [M][TY][TX+1]: x-face fluxes, face i = x0 - 1/2 + i
-  double* fys = fxs + M * TY * (TX + 1);     // [M][TY+1][TX]: y-face fluxes
+  double* fxs = D + D_NV * NC;               // [M][MTY][TX+1]: x-face fluxes, face i = x0 - 1/2 + i
+  double* fys = fxs + M * MTY * (TX + 1);     // [M][MTY+1][TX]: y-face fluxes
   const int lane = threadIdx.x, w = threadIdx.y, t = w * TX + lane;
-  const int x0 = blockIdx.x * TX, y0 = blockIdx.y * TY;
+  const int x0 = blockIdx.x * TX, y0 = blockIdx.y * MTY;
   const int x = x0 + lane, y = y0 + w;
   const bool active = x < g.nx && y < g.ny;
   const int xc = min(x, g.nx), yc = min(y, g.ny);
   const int z0 = blockIdx.z * ZC_MU, z1 = min(z0 + ZC_MU, g.nz);
   const i64 F = g.field;
   const int me = hidx(lane + 1, w + 1);
-  // halo ring cell owned by thread t < 2*TX + 2*TY (corners are not needed)
-  // (warps 4.. build the halo ring; warps 0, 1 compute the far-edge faces)
+  // halo ring cell owned by thread t < 2*TX + 2*MTY (corners are not needed)
+  // (the last threads build the halo ring; warps 0, 1 compute the far-edge faces)
   int hx = 0, hy = 0, hs = -1;
   bool hwx = false, hwy = false;
-  const int th = t - 4 * TX;
+  const int th = t - (MTY * TX - (2 * TX + 2 * MTY));
   if (th >= 0 && th < TX) { hx = th + 1; hy = 0; hwx = true; }
-  else if (th >= TX && th < 2 * TX) { hx = th - TX + 1; hy = TY + 1; hwx = true; }
-  else if (th >= 2 * TX && th < 2 * TX + TY) { hx = 0; hy = th - 2 * TX + 1; hwy = true; }
-  else if (th >= 2 * TX + TY && th < 2 * TX + 2 * TY) { hx = TX + 1; hy = th - 2 * TX - TY + 1; hwy = true; }
+  else if (th >= TX && th < 2 * TX) { hx = th - TX + 1; hy = MTY + 1; hwx = true; }
+  else if (th >= 2 * TX && th < 2 * TX + MTY) { hx = 0; hy = th - 2 * TX + 1; hwy = true; }
+  else if (th >= 2 * TX + MTY && th < 2 * TX + 2 * MTY) { hx = TX + 1; hy = th - 2 * TX - MTY + 1; hwy = true; }
   if (hwx || hwy) hs = hidx(hx, hy);
   const int hgx = min(x0 + hx - 1, g.nx), hgy = min(y0 + hy - 1, g.ny);
 
@@ -243,12 +255,12 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
   for (int k = z0; k <= z1; ++k) {
     const bool last = k == z1;
     // (a) publish D(k) of the own cell and of the halo ring
-    build_cell(g, ps, pd, ms, xc, yc, k, true, true, !last, D, me);
-    if (hs >= 0 && !last) build_cell(g, ps, pd, ms, hgx, hgy, k, hwx, hwy, true, D, hs);
+    build_cell<NC>(g, ps, pd, ms, xc, yc, k, true, true, !last, D, me);
+    if (hs >= 0 && !last) build_cell<NC>(g, ps, pd, ms, hgx, hgy, k, hwx, hwy, true, D, hs);
     __syncthreads();
     // (b) z-face k-1/2 from registers (plane k-1) and shared memory (plane k)
     FaceSide q;
-    side_from_smem<L>(D, me, D_CX, D_CY, q);
+    side_from_smem<L, NC>(D, me, D_CX, D_CY, q);
     double Fz[M];
     mu_face<L, TA>(P, plane_T(P, R, k - 0.5), Dp, q, Fz);
     // (c) cell update of plane k-1
@@ -275,39 +287,39 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
       const double Tk = plane_T(P, R, (double)k);
       FaceSide p, s;
       double Fx[M], Fy[M];
-      side_from_smem<L>(D, me - 1, D_CY, D_CZ, p);
-      side_from_smem<L>(D, me, D_CY, D_CZ, s);
+      side_from_smem<L, NC>(D, me - 1, D_CY, D_CZ, p);
+      side_from_smem<L, NC>(D, me, D_CY, D_CZ, s);
       mu_face<L, TA>(P, Tk, p, s, Fx);
-      side_from_smem<L>(D, me - HX, D_CX, D_CZ, p);
-      side_from_smem<L>(D, me, D_CX, D_CZ, s);
+      side_from_smem<L, NC>(D, me - HX, D_CX, D_CZ, p);
+      side_from_smem<L, NC>(D, me, D_CX, D_CZ, s);
       mu_face<L, TA>(P, Tk, p, s, Fy);
 #pragma unroll
       for (int i = 0; i < M; ++i) {
-        fxs[(i * TY + w) * (TX + 1) + lane] = Fx[i];
-        fys[(i * (TY + 1) + w) * TX + lane] = Fy[i];
+        fxs[(i * MTY + w) * (TX + 1) + lane] = Fx[i];
+        fys[(i * (MTY + 1) + w) * TX + lane] = Fy[i];
       }
       if (w == 0) {  // +y face of the top tile edge, column `lane`
         double Fe[M];
-        side_from_smem<L>(D, hidx(lane + 1, TY), D_CX, D_CZ, p);
-        side_from_smem<L>(D, hidx(lane + 1, TY + 1), D_CX, D_CZ, s);
+        side_from_smem<L, NC>(D, hidx(lane + 1, MTY), D_CX, D_CZ, p);
+        side_from_smem<L, NC>(D, hidx(lane + 1, MTY + 1), D_CX, D_CZ, s);
         mu_face<L, TA>(P, Tk, p, s, Fe);
 #pragma unroll
-        for (int i = 0; i < M; ++i) fys[(i * (TY + 1) + TY) * TX + lane] = Fe[i];
-      } else if (w == 1 && lane < TY) {  // +x face of the right tile edge, row `lane`
+        for (int i = 0; i < M; ++i) fys[(i * (MTY + 1) + MTY) * TX + lane] = Fe[i];
+      } else if (w == 1 && lane < MTY) {  // +x face of the right tile edge, row `lane`
         double Fe[M];
-        side_from_smem<L>(D, hidx(TX, lane + 1), D_CY, D_CZ, p);
-        side_from_smem<L>(D, hidx(TX + 1, lane + 1), D_CY, D_CZ, s);
+        side_from_smem<L, NC>(D, hidx(TX, lane + 1), D_CY, D_CZ, p);
+        side_from_smem<L, NC>(D, hidx(TX + 1, lane + 1), D_CY, D_CZ, s);
         mu_face<L, TA>(P, Tk, p, s, Fe);
 #pragma unroll
-        for (int i = 0; i < M; ++i) fxs[(i * TY + lane) * (TX + 1) + TX] = Fe[i];
+        for (int i = 0; i < M; ++i) fxs[(i * MTY + lane) * (TX + 1) + TX] = Fe[i];
       }
     }
     __syncthreads();
     if (!last) {
 #pragma unroll
       for (int i = 0; i < M; ++i)
-        divxy[i] = (fxs[(i * TY + w) * (TX + 1) + lane + 1] - fxs[(i * TY + w) * (TX + 1) + lane]) +
-                   (fys[(i * (TY + 1) + w + 1) * TX + lane] - fys[(i * (TY + 1) + w) * TX + lane]);
+        divxy[i] = (fxs[(i * MTY + w) * (TX + 1) + lane + 1] - fxs[(i * MTY + w) * (TX + 1) + lane]) +
+                   (fys[(i * (MTY + 1) + w + 1) * TX + lane] - fys[(i * (MTY + 1) + w) * TX + lane]);
     }
   }
 }

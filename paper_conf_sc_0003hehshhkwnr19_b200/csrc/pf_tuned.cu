@@ -32,16 +32,20 @@ __global__ void __launch_bounds__(TX* TY, 2) k_phi_tuned(DevParams P, Geom g, co
 }
 
 template <int L, bool TA>
-__global__ void __launch_bounds__(TX* TY, 2) k_mu_tuned(DevParams P, Geom g, const double* __restrict__ ps,
-                                                        const double* __restrict__ pd, const double* __restrict__ ms,
-                                                        double* __restrict__ md) {
-  mu_tuned_body<DevParams, Geom, L, TA>(P, P, g, ps, pd, ms, md);
+__global__ void __launch_bounds__(TX* MU_TY, 16 / MU_TY) k_mu_tuned(DevParams P, Geom g, const double* __restrict__ ps,
+                                                                  const double* __restrict__ pd,
+                                                                  const double* __restrict__ ms,
+                                                                  double* __restrict__ md) {
+  mu_tuned_body<DevParams, Geom, L, TA, MU_TY>(P, P, g, ps, pd, ms, md);
 }
 
 dim3 tuned_block() { return dim3(TX, TY); }
+dim3 tuned_block_mu() { return dim3(TX, MU_TY); }
 dim3 tuned_grid_phi(const Geom& g) { return dim3((g.nx + TX - 1) / TX, (g.ny + TY - 1) / TY, (g.nz + ZC_PHI - 1) / ZC_PHI); }
-dim3 tuned_grid_mu(const Geom& g) { return dim3((g.nx + TX - 1) / TX, (g.ny + TY - 1) / TY, (g.nz + ZC_MU - 1) / ZC_MU); }
-size_t tuned_mu_smem() { return MU_SMEM; }
+dim3 tuned_grid_mu(const Geom& g) {
+  return dim3((g.nx + TX - 1) / TX, (g.ny + MU_TY - 1) / MU_TY, (g.nz + ZC_MU - 1) / ZC_MU);
+}
+size_t tuned_mu_smem() { return mu_smem_bytes<MU_TY>(); }
 
 void launch_phi_tuned(const DevParams& P, const Geom& g, const double* ps, const double* ms, double* pd,
                       cudaStream_t s) {
@@ -53,10 +57,10 @@ static void mu_launch(const DevParams& P, const Geom& g, const double* ps, const
                       double* md, cudaStream_t s) {
   static bool attr = false;  // per instantiation
   if (!attr) {
-    cudaFuncSetAttribute(k_mu_tuned<L, TA>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)MU_SMEM);
+    cudaFuncSetAttribute(k_mu_tuned<L, TA>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tuned_mu_smem());
     attr = true;
   }
-  k_mu_tuned<L, TA><<<tuned_grid_mu(g), tuned_block(), MU_SMEM, s>>>(P, g, ps, pd, ms, md);
+  k_mu_tuned<L, TA><<<tuned_grid_mu(g), tuned_block_mu(), tuned_mu_smem(), s>>>(P, g, ps, pd, ms, md);
 }
 
 void launch_mu_tuned(const DevParams& P, const Geom& g, const double* ps, const double* pd, const double* ms,
