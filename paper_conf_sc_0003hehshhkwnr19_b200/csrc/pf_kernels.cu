@@ -175,44 +175,42 @@ __device__ __forceinline__ int map_axis(int i, int n, int klo, int khi, bool* sk
   return i;
 }
 
+// One launch fills all ghosts of a field set: blockIdx.y selects the z ghost
+// planes (0), the y ghost rows of interior planes (1) or the x ghost columns
+// of interior rows (2); 32-bit index math, x fastest (coalesced for 0, 1).
 __global__ void k_ghost(GhostArgs A, double* __restrict__ f) {
   const Geom& g = A.g;
-  const int64_t sx = g.nx + 2, sy = g.ny + 2;
-  const int64_t nzp = 2 * sx * sy;              // two z ghost planes
-  const int64_t nyr = 2 * sx * (int64_t)g.nz;   // two y ghost rows per interior z
-  const int64_t nxc = 2 * (int64_t)g.ny * g.nz; // two x ghost columns per interior (y,z)
-  const int64_t total = nzp + nyr + nxc;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
-    int x, y, z;
-    if (i < nzp) {
-      int64_t r = i;
-      z = (r / (sx * sy)) ? g.nz : -1;
-      r %= sx * sy;
-      y = (int)(r / sx) - 1;
-      x = (int)(r % sx) - 1;
-    } else if (i < nzp + nyr) {
-      int64_t r = i - nzp;
-      z = (int)(r / (2 * sx));
-      r %= 2 * sx;
-      y = (r / sx) ? g.ny : -1;
-      x = (int)(r % sx) - 1;
-    } else {
-      int64_t r = i - nzp - nyr;
-      z = (int)(r / (2 * g.ny));
-      r %= 2 * g.ny;
-      y = (int)(r / 2);
-      x = (r % 2) ? g.nx : -1;
-    }
-    bool skip = false, dir = false;
-    const int mx = map_axis(x, g.nx, A.bc.kind_lo[0], A.bc.kind_hi[0], &skip, &dir);
-    const int my = map_axis(y, g.ny, A.bc.kind_lo[1], A.bc.kind_hi[1], &skip, &dir);
-    const int mz = map_axis(z, g.nz, A.bc.kind_lo[2], A.bc.kind_hi[2], &skip, &dir);
-    if (skip) continue;
-    const int64_t dst = g.at(x, y, z);
-    const int64_t src = g.at(mx, my, mz);
-    for (int c = 0; c < A.ncomp; ++c)
-      f[c * g.field + dst] = (dir && A.use_dir) ? A.dir[c] : f[c * g.field + src];
+  const int sx = g.nx + 2, sy = g.ny + 2;
+  const int seg = blockIdx.y;
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  int x, y, z;
+  if (seg == 0) {  // 2 planes of sx * sy
+    if (i >= 2 * sx * sy) return;
+    const int side = i / (sx * sy), r = i - side * sx * sy;
+    z = side ? g.nz : -1;
+    y = r / sx - 1;
+    x = r % sx - 1;
+  } else if (seg == 1) {  // 2 rows of sx per interior plane
+    if (i >= 2 * sx * g.nz) return;
+    const int zz = i / (2 * sx), r = i - zz * 2 * sx;
+    z = zz;
+    y = (r / sx) ? g.ny : -1;
+    x = r % sx - 1;
+  } else {  // 2 cells per interior row
+    if (i >= 2 * g.ny * g.nz) return;
+    const int row = i >> 1;
+    z = row / g.ny;
+    y = row - z * g.ny;
+    x = (i & 1) ? g.nx : -1;
   }
+  bool skip = false, dir = false;
+  const int mx = map_axis(x, g.nx, A.bc.kind_lo[0], A.bc.kind_hi[0], &skip, &dir);
+  const int my = map_axis(y, g.ny, A.bc.kind_lo[1], A.bc.kind_hi[1], &skip, &dir);
+  const int mz = map_axis(z, g.nz, A.bc.kind_lo[2], A.bc.kind_hi[2], &skip, &dir);
+  if (skip) return;
+  const int64_t dst = g.at(x, y, z);
+  const int64_t src = g.at(mx, my, mz);
+  for (int c = 0; c < A.ncomp; ++c) f[c * g.field + dst] = (dir && A.use_dir) ? A.dir[c] : f[c * g.field + src];
 }
 
 void launch_ghost_fill(const Geom& g, const BCSpec& bc, double* f, int ncomp, const double* dirichlet, cudaStream_t s) {
@@ -222,10 +220,11 @@ void launch_ghost_fill(const Geom& g, const BCSpec& bc, double* f, int ncomp, co
   A.ncomp = ncomp;
   A.use_dir = dirichlet != nullptr;
   for (int i = 0; i < M; ++i) A.dir[i] = dirichlet ? dirichlet[i] : 0.0;
-  const int64_t total = 2 * (int64_t)(g.nx + 2) * (g.ny + 2) + 2 * (int64_t)(g.nx + 2) * g.nz + 2 * (int64_t)g.ny * g.nz;
-  int blocks = (int)((total + 255) / 256);
-  if (blocks > 148 * 8) blocks = 148 * 8;
-  k_ghost<<<blocks, 256, 0, s>>>(A, f);
+  const int64_t n0 = 2 * (int64_t)(g.nx + 2) * (g.ny + 2), n1 = 2 * (int64_t)(g.nx + 2) * g.nz,
+                n2 = 2 * (int64_t)g.ny * g.nz;
+  const int64_t mx = n0 > n1 ? (n0 > n2 ? n0 : n2) : (n1 > n2 ? n1 : n2);
+  dim3 grid((unsigned)((mx + 255) / 256), 3);
+  k_ghost<<<grid, 256, 0, s>>>(A, f);
 }
 
 // ---------------------------------------------------------------------------

@@ -164,6 +164,10 @@ __host__ __device__ constexpr size_t mu_smem_bytes() {
 // halo-tile coords (0..HX-1, 0..HY-1) -> slot
 __device__ __forceinline__ int hidx(int hx, int hy) { return hy * (TX + 2) + hx; }
 
+// D is stored cell-major (array of structures, D_NV = 22 doubles = 176 B per
+// cell): the 16-B vector accesses of a warp then fall on distinct bank groups
+// (176 = 11 x 16, odd), and a face side is read with 9 LDS.128.
+
 // build D of cell (x,y,k) from global memory into shared slot i;
 // wx / wy / wz: compute cd_x / cd_y / cd_z (halo cells only need the
 // tangential ones, and must not read beyond the guard ring)
@@ -173,32 +177,51 @@ __device__ __forceinline__ void build_cell(const GT& g, const double* __restrict
                                            bool wz, double* __restrict__ D, int i) {
   const i64 F = g.field;
   const i64 c = g.at(x, y, k);
+  double v[D_NV];
 #pragma unroll
   for (int a = 0; a < N; ++a) {
     const double* f = ps + a * F + c;
-    const double v = __ldg(f);
-    D[(D_F + a) * NC + i] = v;
-    if (wx) D[(D_CX + a) * NC + i] = __ldg(f + 1) - __ldg(f - 1);
-    if (wy) D[(D_CY + a) * NC + i] = __ldg(f + g.pitch) - __ldg(f - g.pitch);
-    if (wz) D[(D_CZ + a) * NC + i] = __ldg(f + g.plane) - __ldg(f - g.plane);
-    D[(D_DP + a) * NC + i] = __ldg(pd + a * F + c) - v;
+    v[D_F + a] = __ldg(f);
+    v[D_CX + a] = wx ? __ldg(f + 1) - __ldg(f - 1) : 0.0;
+    v[D_CY + a] = wy ? __ldg(f + g.pitch) - __ldg(f - g.pitch) : 0.0;
+    v[D_CZ + a] = wz ? __ldg(f + g.plane) - __ldg(f - g.plane) : 0.0;
+    v[D_DP + a] = __ldg(pd + a * F + c) - v[D_F + a];
   }
-  D[(D_MU + 0) * NC + i] = __ldg(ms + c);
-  D[(D_MU + 1) * NC + i] = __ldg(ms + F + c);
+  v[D_MU + 0] = __ldg(ms + c);
+  v[D_MU + 1] = __ldg(ms + F + c);
+  double2* d = reinterpret_cast<double2*>(D + (size_t)i * D_NV);
+#pragma unroll
+  for (int j = 0; j < D_NV / 2; ++j) d[j] = make_double2(v[2 * j], v[2 * j + 1]);
 }
 
 template <int L, int NC>
 __device__ __forceinline__ void side_from_smem(const double* __restrict__ D, int i, int c1, int c2, FaceSide& s) {
+  const double2* d = reinterpret_cast<const double2*>(D + (size_t)i * D_NV);
+  double2 t;
 #pragma unroll
-  for (int a = 0; a < N; ++a) {
-    s.f[a] = D[(D_F + a) * NC + i];
-    s.c1[a] = D[(c1 + a) * NC + i];
-    s.c2[a] = D[(c2 + a) * NC + i];
+  for (int j = 0; j < N / 2; ++j) {
+    t = d[(D_F >> 1) + j];
+    s.f[2 * j] = t.x;
+    s.f[2 * j + 1] = t.y;
+    t = d[(c1 >> 1) + j];
+    s.c1[2 * j] = t.x;
+    s.c1[2 * j + 1] = t.y;
+    t = d[(c2 >> 1) + j];
+    s.c2[2 * j] = t.x;
+    s.c2[2 * j + 1] = t.y;
+  }
+  double dp[N];
+#pragma unroll
+  for (int j = 0; j < N / 2; ++j) {
+    t = d[(D_DP >> 1) + j];
+    dp[2 * j] = t.x;
+    dp[2 * j + 1] = t.y;
   }
 #pragma unroll
-  for (int t = 0; t < NSOL; ++t) s.ds[t] = D[(D_DP + solid_phase(L, t)) * NC + i];
-  s.m[0] = D[(D_MU + 0) * NC + i];
-  s.m[1] = D[(D_MU + 1) * NC + i];
+  for (int u = 0; u < NSOL; ++u) s.ds[u] = dp[solid_phase(L, u)];
+  t = d[D_MU >> 1];
+  s.m[0] = t.x;
+  s.m[1] = t.y;
 }
 
 template <class PT, class GT, int L, bool TA, int MTY>
@@ -281,7 +304,7 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
     Fzm[1] = Fz[1];
     // carry plane k's side for the next z-face
     Dp = q;
-    dpl = D[(D_DP + L) * NC + me];
+    dpl = D[(size_t)me * D_NV + D_DP + L];
     if (!last) {
       // (d) faces of plane k: -x and -y of every thread, + the far tile edges
       const double Tk = plane_T(P, R, (double)k);
