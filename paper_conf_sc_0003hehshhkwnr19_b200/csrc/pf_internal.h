@@ -30,6 +30,7 @@ dim3 tuned_block_mu();
 dim3 tuned_grid_phi(const Geom& g);
 dim3 tuned_grid_mu(const Geom& g);
 size_t tuned_mu_smem();
+size_t tuned_phi_smem();
 
 // ---- ghost layers, halo exchange, window, reductions, copies ------------
 // ghost fill of ncomp components; BC kind per side, -1 = filled by exchange

@@ -32,71 +32,99 @@ constexpr int MU_TY = PF_MU_TY;
 // ===========================================================================
 // phi-sweep (Algorithm 1 line 1): D3C7 of phi_src, D3C1 of mu_src.
 // ===========================================================================
+// cp.async (LDGSTS) helpers: 8-byte global -> shared copies that complete
+// in the background while the SM computes the previous plane
+__device__ __forceinline__ void cp_async8(void* smem, const void* gmem) {
+  const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(s), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
+
+// phi_src planes are staged in a 3-slot ring of (TX+2) x (TY+2) halo tiles
+constexpr int PHX = TX + 2, PHY = TY + 2, PNC = PHX * PHY;
+constexpr size_t PHI_SMEM = (size_t)(3 * N * PNC + 2 * N * TY * TX + 2 * N * TY + 2 * N * TX) * sizeof(double);
+
+template <class GT>
+__device__ __forceinline__ void phi_stage_plane(const GT& g, const double* __restrict__ ps, int x0, int y0, int z,
+                                                double* __restrict__ slot, int t) {
+  // N * PNC doubles; thread t copies elements t, t + 256, ...
+  for (int e = t; e < N * PNC; e += TX * TY) {
+    const int a = e / PNC, r = e - a * PNC;
+    const int hy = r / PHX, hx = r - hy * PHX;
+    const int gx = min(x0 - 1 + hx, g.nx + 1), gy = min(y0 - 1 + hy, g.ny + 1);
+    cp_async8(slot + e, ps + a * g.field + g.at(gx, gy, z));
+  }
+  cp_async_commit();
+}
+
 template <class PT, class GT, int L, bool TA>
 __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, const GT& g,
                                                const double* __restrict__ ps, const double* __restrict__ ms,
                                                double* __restrict__ pd) {
-  __shared__ double fy[2][N][TY][TX];  // -y face flux of every thread, by plane parity
-  __shared__ double ex[2][N][TY];      // +x flux on the right tile edge
-  __shared__ double ey[2][N][TX];      // +y flux on the top tile edge
-  const int lane = threadIdx.x, w = threadIdx.y;
+  extern __shared__ double psm[];
+  double* ring = psm;                                  // [3][N][PNC]
+  double(*fy)[N][TY][TX] = reinterpret_cast<double(*)[N][TY][TX]>(psm + 3 * N * PNC);  // [2][N][TY][TX]
+  double(*ex)[N][TY] = reinterpret_cast<double(*)[N][TY]>(psm + 3 * N * PNC + 2 * N * TY * TX);
+  double(*ey)[N][TX] = reinterpret_cast<double(*)[N][TX]>(psm + 3 * N * PNC + 2 * N * TY * TX + 2 * N * TY);
+  const int lane = threadIdx.x, w = threadIdx.y, t = w * TX + lane;
   const int x0 = blockIdx.x * TX, y0 = blockIdx.y * TY;
   const int x = x0 + lane, y = y0 + w;
   const bool active = x < g.nx && y < g.ny;
-  // ragged tiles: clamp to the ghost cell, whose -x / -y face is the +x / +y
-  // face of the last interior cell
+  // ragged tiles: threads beyond the domain read the ghost cell (or clamped
+  // guard values); the -x / -y face of the ghost cell is the +x / +y face of
+  // the last interior cell
   const int xc = min(x, g.nx), yc = min(y, g.ny);
   const int z0 = blockIdx.z * ZC_PHI, z1 = min(z0 + ZC_PHI, g.nz);
-  const i64 F = g.field, SY = g.pitch, SZ = g.plane;
-  // extra faces: warp 0 lanes < TY: +x face of row `lane`; warp 1: +y face of column `lane`
-  i64 ep = 0, eq = 0;  // the two cells of the extra face, at plane z0
-  if (w == 0 && lane < TY) {
-    const int ry = min(y0 + lane, g.ny);
-    ep = g.at(min(x0 + TX - 1, g.nx), ry, z0);
-    eq = g.at(min(x0 + TX, g.nx), ry, z0);
-  } else if (w == 1) {
-    const int cx = min(x0 + lane, g.nx);
-    ep = g.at(cx, min(y0 + TY - 1, g.ny), z0);
-    eq = g.at(cx, min(y0 + TY, g.ny), z0);
-  }
+  const i64 F = g.field;
+  const int me = (w + 1) * PHX + lane + 1;  // own cell in a halo tile
   const bool extra = (w == 0 && lane < TY) || w == 1;
+  // extra faces: warp 0 lanes < TY: +x face of row `lane`; warp 1: +y face of column `lane`
+  const int ea = w == 0 ? (lane + 1) * PHX + TX : TY * PHX + lane + 1;
+  const int eb = w == 0 ? ea + 1 : ea + PHX;
 
-  i64 c = g.at(xc, yc, z0);
+  // prologue: planes z0-1 and z0 synchronously, z0+1 in flight
+  phi_stage_plane(g, ps, x0, y0, z0 - 1, ring + ((z0 + 2) % 3) * N * PNC, t);
+  phi_stage_plane(g, ps, x0, y0, z0, ring + (z0 % 3) * N * PNC, t);
+  cp_async_wait_all();
+  __syncthreads();
+  phi_stage_plane(g, ps, x0, y0, z0 + 1, ring + ((z0 + 1) % 3) * N * PNC, t);
   double pm[N], p0[N], Fzm[N];
+  {
+    const double* sm1 = ring + ((z0 + 2) % 3) * N * PNC;
+    const double* s0 = ring + (z0 % 3) * N * PNC;
 #pragma unroll
-  for (int a = 0; a < N; ++a) {
-    pm[a] = __ldg(ps + a * F + c - SZ);
-    p0[a] = __ldg(ps + a * F + c);
+    for (int a = 0; a < N; ++a) {
+      pm[a] = sm1[a * PNC + me];
+      p0[a] = s0[a * PNC + me];
+    }
   }
   phi_face(P, pm, p0, Fzm);
+  i64 c = g.at(xc, yc, z0);
+  double mu0 = __ldg(ms + c), mu1 = __ldg(ms + F + c);
 
-  for (int z = z0; z < z1; ++z, c += SZ, ep += SZ, eq += SZ) {
+  for (int z = z0; z < z1; ++z, c += g.plane) {
     const int buf = z & 1;
-    double pp[N], Fxm[N], Fym[N], Fzp[N], gd[N][3];
+    const double* s0 = ring + (z % 3) * N * PNC;
+    double Fxm[N], Fym[N], gxy[N][2];
     {
-      double xm[N], xp[N], ym[N], yp[N];
+      double xm[N], ym[N];
 #pragma unroll
       for (int a = 0; a < N; ++a) {
-        const double* f = ps + a * F + c;
-        pp[a] = __ldg(f + SZ);
-        xm[a] = __ldg(f - 1);
-        xp[a] = __ldg(f + 1);
-        ym[a] = __ldg(f - SY);
-        yp[a] = __ldg(f + SY);
-        gd[a][0] = xp[a] - xm[a];
-        gd[a][1] = yp[a] - ym[a];
-        gd[a][2] = pp[a] - pm[a];
+        xm[a] = s0[a * PNC + me - 1];
+        ym[a] = s0[a * PNC + me - PHX];
+        gxy[a][0] = s0[a * PNC + me + 1] - xm[a];
+        gxy[a][1] = s0[a * PNC + me + PHX] - ym[a];
       }
       phi_face(P, xm, p0, Fxm);
       phi_face(P, ym, p0, Fym);
     }
-    phi_face(P, p0, pp, Fzp);
     if (extra) {
       double fa[N], fb[N], fe[N];
 #pragma unroll
       for (int a = 0; a < N; ++a) {
-        fa[a] = __ldg(ps + a * F + ep);
-        fb[a] = __ldg(ps + a * F + eq);
+        fa[a] = s0[a * PNC + ea];
+        fb[a] = s0[a * PNC + eb];
       }
       phi_face(P, fa, fb, fe);
       if (w == 0) {
@@ -109,15 +137,26 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, 
     }
 #pragma unroll
     for (int a = 0; a < N; ++a) fy[buf][a][w][lane] = Fym[a];
-    const double mu0 = __ldg(ms + c), mu1 = __ldg(ms + F + c);
+    // next plane's mu (prefetch) and plane z+1 of phi must have landed
+    const double nmu0 = z + 1 < z1 ? __ldg(ms + c + g.plane) : 0.0;
+    const double nmu1 = z + 1 < z1 ? __ldg(ms + F + c + g.plane) : 0.0;
+    cp_async_wait_all();
     __syncthreads();
-    double divh[N];
+    if (z + 2 <= z1) phi_stage_plane(g, ps, x0, y0, z + 2, ring + ((z + 2) % 3) * N * PNC, t);
+    const double* s1 = ring + ((z + 1) % 3) * N * PNC;
+    double pp[N], Fzp[N], divh[N], gd[N][3];
+#pragma unroll
+    for (int a = 0; a < N; ++a) pp[a] = s1[a * PNC + me];
+    phi_face(P, p0, pp, Fzp);
 #pragma unroll
     for (int a = 0; a < N; ++a) {
       double fxp = __shfl_down_sync(0xffffffffu, Fxm[a], 1);
       if (lane == TX - 1) fxp = ex[buf][a][w];
       const double fyp = (w < TY - 1) ? fy[buf][a][w + 1][lane] : ey[buf][a][lane];
       divh[a] = ((fxp - Fxm[a]) + (fyp - Fym[a])) + (Fzp[a] - Fzm[a]);
+      gd[a][0] = gxy[a][0];
+      gd[a][1] = gxy[a][1];
+      gd[a][2] = pp[a] - pm[a];
     }
     double out[N];
     phi_cell<TA>(P, plane_T(P, R, (double)z), p0, gd, divh, mu0, mu1, out);
@@ -131,6 +170,8 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, 
       p0[a] = pp[a];
       Fzm[a] = Fzp[a];
     }
+    mu0 = nmu0;
+    mu1 = nmu1;
   }
 }
 

@@ -13,4 +13,9 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:pf_j
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:pf_jit_phi -s 3 -c 1 -o $OUT/prof_phi \
    python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_phi.log 2>&1
 fi
+
+if [ "$3" == "launches" ]; then
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches.csv \
+   python bench.py --steps 10 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_launch.log 2>&1
+fi
 echo done > $OUT/DONE

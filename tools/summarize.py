@@ -33,3 +33,16 @@ for rep in sorted(glob.glob(os.path.join(d, "*.ncu-rep"))):
     st = {n.replace("smsp__average_warps_issue_stalled_", "").replace("_per_issue_active.ratio", ""): float(v[i] or 0)
           for i, n in enumerate(h) if n.startswith("smsp__average_warps_issue_stalled") and n.endswith("per_issue_active.ratio")}
     print("   stalls", {k: round(x, 2) for k, x in sorted(st.items(), key=lambda kv: -kv[1])[:7]})
+lp = os.path.join(d, "launches.csv")
+if os.path.exists(lp):
+    import collections
+    lines = open(lp).read().splitlines()
+    st = [i for i, l in enumerate(lines) if l.startswith('"ID"')]
+    if st:
+        agg = collections.defaultdict(list)
+        for r in csv.DictReader(lines[st[0]:]):
+            agg[r["Kernel Name"][:60]].append(float(r["Metric Value"]))
+        tot = sum(sum(v) for v in agg.values())
+        print("== launch list (ncu, serialized)")
+        for k, v in sorted(agg.items(), key=lambda kv: -sum(kv[1])):
+            print(f"   {sum(v)/1e3:9.1f} us  {100*sum(v)/tot:5.1f}%  n={len(v):3d} avg={sum(v)/len(v)/1e3:8.1f} us  {k}")
