@@ -32,48 +32,60 @@ constexpr int MU_TY = PF_MU_TY;
 // ===========================================================================
 // phi-sweep (Algorithm 1 line 1): D3C7 of phi_src, D3C1 of mu_src.
 // ===========================================================================
-// cp.async (LDGSTS) helpers: 8-byte global -> shared copies that complete
-// in the background while the SM computes the previous plane
-__device__ __forceinline__ void cp_async8(void* smem, const void* gmem) {
-  const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(s), "l"(gmem) : "memory");
+// ---------------------------------------------------------------------------
+// TMA + mbarrier helpers (sm_90+ PTX, the Blackwell async copy engine)
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ unsigned smem_u32(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(unsigned long long* bar, unsigned count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(smem_u32(bar)), "r"(count) : "memory");
 }
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
-__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
+__device__ __forceinline__ void mbar_fence_init() { asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory"); }
+__device__ __forceinline__ void mbar_expect_tx(unsigned long long* bar, unsigned bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(unsigned long long* bar, unsigned parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n WAIT_%=:\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      " @!p bra WAIT_%=;\n}\n" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+// 4-D tile load (x, y, z, component) of the padded field array into shared memory
+__device__ __forceinline__ void tma_load_4d(void* dst, const TmaDesc* desc, int x, int y, int z, int c,
+                                            unsigned long long* bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.4d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%2, %3, %4, %5}], [%6];\n" ::"r"(smem_u32(dst)),
+      "l"(desc), "r"(x), "r"(y), "r"(z), "r"(c), "r"(smem_u32(bar))
+      : "memory");
+}
 
-// phi_src planes are staged in a 3-slot ring of (TX+2) x (TY+2) halo tiles
+// phi_src planes are staged in a 3-slot ring of (TX+2) x (TY+2) halo tiles,
+// one TMA box of (TX+2, TY+2, 1, N) per plane issued by one thread
 constexpr int PHX = TX + 2, PHY = TY + 2, PNC = PHX * PHY;
-constexpr size_t PHI_SMEM = (size_t)(3 * N * PNC + 2 * N * TY * TX + 2 * N * TY + 2 * N * TX) * sizeof(double);
-
-template <class GT>
-__device__ __forceinline__ void phi_stage_plane(const GT& g, const double* __restrict__ ps, int x0, int y0, int z,
-                                                double* __restrict__ slot, int t) {
-  // N * PNC doubles; thread t copies elements t, t + 256, ...
-  for (int e = t; e < N * PNC; e += TX * TY) {
-    const int a = e / PNC, r = e - a * PNC;
-    const int hy = r / PHX, hx = r - hy * PHX;
-    const int gx = min(x0 - 1 + hx, g.nx + 1), gy = min(y0 - 1 + hy, g.ny + 1);
-    cp_async8(slot + e, ps + a * g.field + g.at(gx, gy, z));
-  }
-  cp_async_commit();
-}
+constexpr int PHI_TILE_BYTES = N * PNC * 8;
+constexpr int PHI_SLOT = (N * PNC + 15) / 16 * 16;  // doubles; slots 128-B aligned
+constexpr size_t PHI_SMEM =
+    (size_t)(3 * PHI_SLOT + 2 * N * TY * TX + 2 * N * TY + 2 * N * TX + 4) * sizeof(double);
 
 template <class PT, class GT, int L, bool TA>
-__device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, const GT& g,
-                                               const double* __restrict__ ps, const double* __restrict__ ms,
-                                               double* __restrict__ pd) {
-  extern __shared__ double psm[];
-  double* ring = psm;                                  // [3][N][PNC]
-  double(*fy)[N][TY][TX] = reinterpret_cast<double(*)[N][TY][TX]>(psm + 3 * N * PNC);  // [2][N][TY][TX]
-  double(*ex)[N][TY] = reinterpret_cast<double(*)[N][TY]>(psm + 3 * N * PNC + 2 * N * TY * TX);
-  double(*ey)[N][TX] = reinterpret_cast<double(*)[N][TX]>(psm + 3 * N * PNC + 2 * N * TY * TX + 2 * N * TY);
+__device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, const GT& g, const TmaDesc* tmap,
+                                               const double* __restrict__ ms, double* __restrict__ pd) {
+  extern __shared__ __align__(128) double psm[];
+  double* ring = psm;                                  // [3][PHI_SLOT]: [N][PHY][PHX]
+  double(*fy)[N][TY][TX] = reinterpret_cast<double(*)[N][TY][TX]>(psm + 3 * PHI_SLOT);  // [2][N][TY][TX]
+  double(*ex)[N][TY] = reinterpret_cast<double(*)[N][TY]>(psm + 3 * PHI_SLOT + 2 * N * TY * TX);
+  double(*ey)[N][TX] = reinterpret_cast<double(*)[N][TX]>(psm + 3 * PHI_SLOT + 2 * N * TY * TX + 2 * N * TY);
+  unsigned long long* bar =
+      reinterpret_cast<unsigned long long*>(psm + 3 * PHI_SLOT + 2 * N * TY * TX + 2 * N * TY + 2 * N * TX);
   const int lane = threadIdx.x, w = threadIdx.y, t = w * TX + lane;
   const int x0 = blockIdx.x * TX, y0 = blockIdx.y * TY;
   const int x = x0 + lane, y = y0 + w;
   const bool active = x < g.nx && y < g.ny;
-  // ragged tiles: threads beyond the domain read the ghost cell (or clamped
-  // guard values); the -x / -y face of the ghost cell is the +x / +y face of
-  // the last interior cell
+  // ragged tiles: threads beyond the domain read the ghost cell (or guard
+  // values); the -x / -y face of the ghost cell is the +x / +y face of the
+  // last interior cell
   const int xc = min(x, g.nx), yc = min(y, g.ny);
   const int z0 = blockIdx.z * ZC_PHI, z1 = min(z0 + ZC_PHI, g.nz);
   const i64 F = g.field;
@@ -82,30 +94,39 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, 
   // extra faces: warp 0 lanes < TY: +x face of row `lane`; warp 1: +y face of column `lane`
   const int ea = w == 0 ? (lane + 1) * PHX + TX : TY * PHX + lane + 1;
   const int eb = w == 0 ? ea + 1 : ea + PHX;
-
-  // prologue: planes z0-1 and z0 synchronously, z0+1 in flight
-  phi_stage_plane(g, ps, x0, y0, z0 - 1, ring + ((z0 + 2) % 3) * N * PNC, t);
-  phi_stage_plane(g, ps, x0, y0, z0, ring + (z0 % 3) * N * PNC, t);
-  cp_async_wait_all();
+  // tensor coordinates of the halo tile origin (x - 1, y - 1) in the padded array
+  const int tx = (int)g.xoff + x0 - 1, ty = GUARD + y0 - 1;
+  // plane j of this CTA (j = 0 <-> z0 - 1) lives in slot j % 3; its barrier phase is (j / 3) & 1
+  auto issue = [&](int j) {
+    mbar_expect_tx(&bar[j % 3], PHI_TILE_BYTES);
+    tma_load_4d(ring + (j % 3) * PHI_SLOT, tmap, tx, ty, GUARD + z0 - 1 + j, 0, &bar[j % 3]);
+  };
+  if (t == 0) {
+    for (int i = 0; i < 3; ++i) mbar_init(&bar[i], 1);
+    mbar_fence_init();
+  }
   __syncthreads();
-  phi_stage_plane(g, ps, x0, y0, z0 + 1, ring + ((z0 + 1) % 3) * N * PNC, t);
+  if (t == 0) {
+    issue(0);
+    issue(1);
+    issue(2);
+  }
+  mbar_wait(&bar[0], 0);
+  mbar_wait(&bar[1], 0);
   double pm[N], p0[N], Fzm[N];
-  {
-    const double* sm1 = ring + ((z0 + 2) % 3) * N * PNC;
-    const double* s0 = ring + (z0 % 3) * N * PNC;
 #pragma unroll
-    for (int a = 0; a < N; ++a) {
-      pm[a] = sm1[a * PNC + me];
-      p0[a] = s0[a * PNC + me];
-    }
+  for (int a = 0; a < N; ++a) {
+    pm[a] = ring[0 * PHI_SLOT + a * PNC + me];
+    p0[a] = ring[1 * PHI_SLOT + a * PNC + me];
   }
   phi_face(P, pm, p0, Fzm);
   i64 c = g.at(xc, yc, z0);
   double mu0 = __ldg(ms + c), mu1 = __ldg(ms + F + c);
 
   for (int z = z0; z < z1; ++z, c += g.plane) {
+    const int j = z - z0 + 1;  // plane z is j, plane z+1 is j+1
     const int buf = z & 1;
-    const double* s0 = ring + (z % 3) * N * PNC;
+    const double* s0 = ring + (j % 3) * PHI_SLOT;
     double Fxm[N], Fym[N], gxy[N][2];
     {
       double xm[N], ym[N];
@@ -137,13 +158,13 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, 
     }
 #pragma unroll
     for (int a = 0; a < N; ++a) fy[buf][a][w][lane] = Fym[a];
-    // next plane's mu (prefetch) and plane z+1 of phi must have landed
-    const double nmu0 = z + 1 < z1 ? __ldg(ms + c + g.plane) : 0.0;
+    const double nmu0 = z + 1 < z1 ? __ldg(ms + c + g.plane) : 0.0;  // prefetch the next plane's mu
     const double nmu1 = z + 1 < z1 ? __ldg(ms + F + c + g.plane) : 0.0;
-    cp_async_wait_all();
+    // all threads are done with plane j-1 (slot of j+2) and have published fy
     __syncthreads();
-    if (z + 2 <= z1) phi_stage_plane(g, ps, x0, y0, z + 2, ring + ((z + 2) % 3) * N * PNC, t);
-    const double* s1 = ring + ((z + 1) % 3) * N * PNC;
+    if (t == 0 && z + 2 <= z1) issue(j + 2);
+    mbar_wait(&bar[(j + 1) % 3], ((j + 1) / 3) & 1);
+    const double* s1 = ring + ((j + 1) % 3) * PHI_SLOT;
     double pp[N], Fzp[N], divh[N], gd[N][3];
 #pragma unroll
     for (int a = 0; a < N; ++a) pp[a] = s1[a * PNC + me];
