@@ -93,7 +93,6 @@ struct pf_ctx {
   bool have_params = false, have_fields = false;
   int64_t step = 0, z_off = 0;
   int variant = PF_VARIANT_JIT;
-  TmaDesc tm_phi[2];  // TMA descriptors of the two phi time levels
   JitModule* jit = nullptr;  // specialised kernels for (dp, g); reset by pf_set_params
   ncclComm_t comm = nullptr;
   // profiling
@@ -418,12 +417,6 @@ int pf_create(const pf_config* cfg, pf_ctx** out) {
       return PF_ENCCL;
     }
   }
-  for (int i = 0; i < 2; ++i) {
-    if (!make_tma_field(ctx->g, ctx->phi[i], PF_N, &ctx->tm_phi[i], &ctx->err)) {
-      *out = ctx;
-      return PF_ECUDA;
-    }
-  }
   {
     const char* fe = getenv("PF_FORCE_EXCHANGE");  // debug: periodic self-exchange through pack/unpack
     ctx->force_exchange = fe && fe[0] == '1';
@@ -652,9 +645,9 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
   if (ctx->variant == PF_VARIANT_NAIVE)
     launch_phi_naive(ctx->dp, g, ps, ms, pd, ctx->stream);
   else if (ctx->variant == PF_VARIANT_JIT)
-    CU(jit_launch_phi(ctx->jit, ctx->dp, ctx->tm_phi[ctx->cur], ms, pd, ctx->stream));
+    CU(jit_launch_phi(ctx->jit, ctx->dp, ps, ms, pd, ctx->stream));
   else
-    launch_phi_tuned(ctx->dp, g, ctx->tm_phi[ctx->cur], ms, pd, ctx->stream);
+    launch_phi_tuned(ctx->dp, g, ps, ms, pd, ctx->stream);
   ctx->nlaunch[0] += 1;
   prof_end(ctx, 0, e0);
   if (int r = check_launch(ctx, "phi_sweep")) return r;

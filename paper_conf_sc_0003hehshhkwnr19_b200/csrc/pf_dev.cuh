@@ -29,12 +29,6 @@ struct Geom {
   }
 };
 
-// Opaque TMA tensor descriptor (CUtensorMap, 128 B), built on the host by
-// cuTensorMapEncodeTiled and passed to kernels as a __grid_constant__.
-struct alignas(64) TmaDesc {
-  unsigned long long v[16];
-};
-
 // Scalars and coefficients of the model.  Passed by value to every kernel
 // (kernel-parameter constant bank) in the generic build; folded into the
 // code as compile-time constants in the specialised build.  T-dependent

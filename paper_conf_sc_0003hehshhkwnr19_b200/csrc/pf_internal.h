@@ -20,10 +20,8 @@ void launch_phi_naive(const DevParams& P, const Geom& g, const double* ps, const
                       cudaStream_t s);
 void launch_mu_naive(const DevParams& P, const Geom& g, const double* ps, const double* pd, const double* ms,
                      double* md, cudaStream_t s);
-void launch_phi_tuned(const DevParams& P, const Geom& g, const TmaDesc& tm, const double* ms, double* pd,
+void launch_phi_tuned(const DevParams& P, const Geom& g, const double* ps, const double* ms, double* pd,
                       cudaStream_t s);
-// TMA descriptor of a padded field array with ncomp components (phi halo-tile box)
-bool make_tma_field(const Geom& g, const double* base, int ncomp, TmaDesc* out, std::string* err);
 void launch_mu_tuned(const DevParams& P, const Geom& g, const double* ps, const double* pd, const double* ms,
                      double* md, cudaStream_t s);
 // launch geometry of the tuned kernels (shared with the specialised build)
@@ -61,7 +59,7 @@ struct JitModule;  // compiled sweep kernels for one (geometry, parameters)
 // build (or fetch from the process cache) the specialised kernels; returns
 // nullptr and sets *err on failure
 JitModule* jit_get(const DevParams& P, const Geom& g, std::string* err);
-cudaError_t jit_launch_phi(JitModule* m, const DevParams& P, const TmaDesc& tm, const double* ms, double* pd,
+cudaError_t jit_launch_phi(JitModule* m, const DevParams& P, const double* ps, const double* ms, double* pd,
                            cudaStream_t s);
 cudaError_t jit_launch_mu(JitModule* m, const DevParams& P, const double* ps, const double* pd, const double* ms,
                           double* md, cudaStream_t s);

@@ -51,27 +51,29 @@ __device__ __forceinline__ void mbar_wait(unsigned long long* bar, unsigned pari
       "r"(parity)
       : "memory");
 }
-// 4-D tile load (x, y, z, component) of the padded field array into shared memory
-__device__ __forceinline__ void tma_load_4d(void* dst, const TmaDesc* desc, int x, int y, int z, int c,
-                                            unsigned long long* bar) {
-  asm volatile(
-      "cp.async.bulk.tensor.4d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
-      " [%0], [%1, {%2, %3, %4, %5}], [%6];\n" ::"r"(smem_u32(dst)),
-      "l"(desc), "r"(x), "r"(y), "r"(z), "r"(c), "r"(smem_u32(bar))
-      : "memory");
+// 1-D bulk async copy (TMA engine, cp.async.bulk) of `bytes` contiguous
+// bytes global -> shared, completing on an mbarrier; src/dst 16-B aligned
+__device__ __forceinline__ void bulk_load(void* dst, const void* src, unsigned bytes, unsigned long long* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n" ::"r"(
+                   smem_u32(dst)),
+               "l"(src), "r"(bytes), "r"(smem_u32(bar))
+               : "memory");
 }
 
-// phi_src planes are staged in a 3-slot ring of (TX+2) x (TY+2) halo tiles,
-// one TMA box of (TX+2, TY+2, 1, N) per plane issued by one thread
-constexpr int PHX = TX + 2, PHY = TY + 2, PNC = PHX * PHY;
+// phi_src planes are staged in a 3-slot ring of halo tiles: rows of
+// PHX = TX + 4 doubles starting at x0 - 2 (16-B aligned: x_off = 16,
+// pitch % 16 == 0), PHY = TY + 2 rows, N components; one bulk copy per row
+// and component (N * PHY per plane) issued by warp 0
+constexpr int PHX = TX + 4, PHY = TY + 2, PNC = PHX * PHY;
 constexpr int PHI_TILE_BYTES = N * PNC * 8;
 constexpr int PHI_SLOT = (N * PNC + 15) / 16 * 16;  // doubles; slots 128-B aligned
 constexpr size_t PHI_SMEM =
     (size_t)(3 * PHI_SLOT + 2 * N * TY * TX + 2 * N * TY + 2 * N * TX + 4) * sizeof(double);
 
 template <class PT, class GT, int L, bool TA>
-__device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, const GT& g, const TmaDesc* tmap,
-                                               const double* __restrict__ ms, double* __restrict__ pd) {
+__device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, const GT& g,
+                                               const double* __restrict__ ps, const double* __restrict__ ms,
+                                               double* __restrict__ pd) {
   extern __shared__ __align__(128) double psm[];
   double* ring = psm;                                  // [3][PHI_SLOT]: [N][PHY][PHX]
   double(*fy)[N][TY][TX] = reinterpret_cast<double(*)[N][TY][TX]>(psm + 3 * PHI_SLOT);  // [2][N][TY][TX]
@@ -89,24 +91,30 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, 
   const int xc = min(x, g.nx), yc = min(y, g.ny);
   const int z0 = blockIdx.z * ZC_PHI, z1 = min(z0 + ZC_PHI, g.nz);
   const i64 F = g.field;
-  const int me = (w + 1) * PHX + lane + 1;  // own cell in a halo tile
+  const int me = (w + 1) * PHX + lane + 2;  // own cell in a halo tile (origin x0 - 2, y0 - 1)
   const bool extra = (w == 0 && lane < TY) || w == 1;
   // extra faces: warp 0 lanes < TY: +x face of row `lane`; warp 1: +y face of column `lane`
-  const int ea = w == 0 ? (lane + 1) * PHX + TX : TY * PHX + lane + 1;
+  const int ea = w == 0 ? (lane + 1) * PHX + TX + 1 : TY * PHX + lane + 2;
   const int eb = w == 0 ? ea + 1 : ea + PHX;
-  // tensor coordinates of the halo tile origin (x - 1, y - 1) in the padded array
-  const int tx = (int)g.xoff + x0 - 1, ty = GUARD + y0 - 1;
-  // plane j of this CTA (j = 0 <-> z0 - 1) lives in slot j % 3; its barrier phase is (j / 3) & 1
+  // plane j of this CTA (j = 0 <-> z0 - 1) lives in slot j % 3; its barrier phase is (j / 3) & 1.
+  // Warp 0 issues the N * PHY row copies of a plane (lane l: rows l, l + 32, ...).
   auto issue = [&](int j) {
-    mbar_expect_tx(&bar[j % 3], PHI_TILE_BYTES);
-    tma_load_4d(ring + (j % 3) * PHI_SLOT, tmap, tx, ty, GUARD + z0 - 1 + j, 0, &bar[j % 3]);
+    if (lane == 0) mbar_expect_tx(&bar[j % 3], PHI_TILE_BYTES);
+    __syncwarp();
+    const int zz = z0 - 1 + j;
+    for (int r = lane; r < N * PHY; r += TX) {
+      const int a = r / PHY, hy = r - a * PHY;
+      const int gy = min(y0 - 1 + hy, g.ny + 1);
+      bulk_load(ring + (j % 3) * PHI_SLOT + a * PNC + hy * PHX, ps + a * g.field + g.at(x0 - 2, gy, zz),
+                PHX * 8, &bar[j % 3]);
+    }
   };
   if (t == 0) {
     for (int i = 0; i < 3; ++i) mbar_init(&bar[i], 1);
     mbar_fence_init();
   }
   __syncthreads();
-  if (t == 0) {
+  if (w == 0) {
     issue(0);
     issue(1);
     issue(2);
@@ -162,7 +170,7 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, 
     const double nmu1 = z + 1 < z1 ? __ldg(ms + F + c + g.plane) : 0.0;
     // all threads are done with plane j-1 (slot of j+2) and have published fy
     __syncthreads();
-    if (t == 0 && z + 2 <= z1) issue(j + 2);
+    if (w == 0 && z + 2 <= z1) issue(j + 2);
     mbar_wait(&bar[(j + 1) % 3], ((j + 1) / 3) & 1);
     const double* s1 = ring + ((j + 1) % 3) * PHI_SLOT;
     double pp[N], Fzp[N], divh[N], gd[N][3];

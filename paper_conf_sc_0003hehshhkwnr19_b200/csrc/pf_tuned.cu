@@ -26,9 +26,9 @@ namespace pf {
 
 
 template <int L, bool TA>
-__global__ void __launch_bounds__(TX* TY, 2) k_phi_tuned(DevParams P, Geom g, const __grid_constant__ TmaDesc tm,
+__global__ void __launch_bounds__(TX* TY, 2) k_phi_tuned(DevParams P, Geom g, const double* __restrict__ ps,
                                                          const double* __restrict__ ms, double* __restrict__ pd) {
-  phi_tuned_body<DevParams, Geom, L, TA>(P, P, g, &tm, ms, pd);
+  phi_tuned_body<DevParams, Geom, L, TA>(P, P, g, ps, ms, pd);
 }
 
 template <int L, bool TA>
@@ -50,50 +50,19 @@ size_t tuned_mu_smem() { return mu_smem_bytes<MU_TY>(); }
 size_t tuned_phi_smem() { return PHI_SMEM; }
 
 template <int L, bool TA>
-static void phi_launch(const DevParams& P, const Geom& g, const TmaDesc& tm, const double* ms, double* pd,
+static void phi_launch(const DevParams& P, const Geom& g, const double* ps, const double* ms, double* pd,
                        cudaStream_t s) {
   static bool attr = false;  // per instantiation
   if (!attr) {
     cudaFuncSetAttribute(k_phi_tuned<L, TA>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PHI_SMEM);
     attr = true;
   }
-  k_phi_tuned<L, TA><<<tuned_grid_phi(g), tuned_block(), PHI_SMEM, s>>>(P, g, tm, ms, pd);
+  k_phi_tuned<L, TA><<<tuned_grid_phi(g), tuned_block(), PHI_SMEM, s>>>(P, g, ps, ms, pd);
 }
 
-void launch_phi_tuned(const DevParams& P, const Geom& g, const TmaDesc& tm, const double* ms, double* pd,
+void launch_phi_tuned(const DevParams& P, const Geom& g, const double* ps, const double* ms, double* pd,
                       cudaStream_t s) {
-  PF_DISPATCH(P.liquid, P.TA, (phi_launch<LL, TT>(P, g, tm, ms, pd, s)));
-}
-
-// TMA descriptor of one padded field array [N][nz+4][ny+4][pitch] (fp64),
-// box (TX+2, TY+2, 1, N): the phi_src halo tile of one plane
-bool make_tma_field(const Geom& g, const double* base, int ncomp, TmaDesc* out, std::string* err) {
-  typedef int (*Encode)(void*, int, unsigned, void*, const unsigned long long*, const unsigned long long*,
-                        const unsigned*, const unsigned*, int, int, int, int);
-  static Encode enc = nullptr;
-  if (!enc) {
-    void* fn = nullptr;
-    cudaDriverEntryPointQueryResult q;
-    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess || !fn) {
-      *err = "cuTensorMapEncodeTiled unavailable";
-      return false;
-    }
-    enc = (Encode)fn;
-  }
-  const unsigned long long dims[4] = {(unsigned long long)g.pitch, (unsigned long long)(g.ny + 2 * GUARD),
-                                      (unsigned long long)(g.nz + 2 * GUARD), (unsigned long long)ncomp};
-  const unsigned long long strides[3] = {(unsigned long long)g.pitch * 8, (unsigned long long)g.plane * 8,
-                                         (unsigned long long)g.field * 8};
-  const unsigned box[4] = {(unsigned)PHX, (unsigned)PHY, 1u, (unsigned)ncomp};
-  const unsigned estr[4] = {1, 1, 1, 1};
-  // CU_TENSOR_MAP_DATA_TYPE_FLOAT64 = 8, interleave none = 0, swizzle none = 0,
-  // L2 promotion 256B = 3, OOB fill none = 0
-  const int r = enc(out, 8, 4, (void*)base, dims, strides, box, estr, 0, 0, 3, 0);
-  if (r != 0) {
-    *err = "cuTensorMapEncodeTiled failed (" + std::to_string(r) + ")";
-    return false;
-  }
-  return true;
+  PF_DISPATCH(P.liquid, P.TA, (phi_launch<LL, TT>(P, g, ps, ms, pd, s)));
 }
 
 
@@ -112,5 +81,6 @@ void launch_mu_tuned(const DevParams& P, const Geom& g, const double* ps, const 
                      double* md, cudaStream_t s) {
   PF_DISPATCH(P.liquid, P.TA, (mu_launch<LL, TT>(P, g, ps, pd, ms, md, s)));
 }
+
 
 }  // namespace pf
