@@ -32,128 +32,71 @@ constexpr int MU_TY = PF_MU_TY;
 // ===========================================================================
 // phi-sweep (Algorithm 1 line 1): D3C7 of phi_src, D3C1 of mu_src.
 // ===========================================================================
-// ---------------------------------------------------------------------------
-// TMA + mbarrier helpers (sm_90+ PTX, the Blackwell async copy engine)
-// ---------------------------------------------------------------------------
-__device__ __forceinline__ unsigned smem_u32(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
-__device__ __forceinline__ void mbar_init(unsigned long long* bar, unsigned count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(smem_u32(bar)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_fence_init() { asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory"); }
-__device__ __forceinline__ void mbar_expect_tx(unsigned long long* bar, unsigned bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(unsigned long long* bar, unsigned parity) {
-  asm volatile(
-      "{\n .reg .pred p;\n WAIT_%=:\n"
-      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
-      " @!p bra WAIT_%=;\n}\n" ::"r"(smem_u32(bar)),
-      "r"(parity)
-      : "memory");
-}
-// 1-D bulk async copy (TMA engine, cp.async.bulk) of `bytes` contiguous
-// bytes global -> shared, completing on an mbarrier; src/dst 16-B aligned
-__device__ __forceinline__ void bulk_load(void* dst, const void* src, unsigned bytes, unsigned long long* bar) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n" ::"r"(
-                   smem_u32(dst)),
-               "l"(src), "r"(bytes), "r"(smem_u32(bar))
-               : "memory");
-}
-
-// phi_src planes are staged in a 3-slot ring of halo tiles: rows of
-// PHX = TX + 4 doubles starting at x0 - 2 (16-B aligned: x_off = 16,
-// pitch % 16 == 0), PHY = TY + 2 rows, N components; one bulk copy per row
-// and component (N * PHY per plane) issued by warp 0
-constexpr int PHX = TX + 4, PHY = TY + 2, PNC = PHX * PHY;
-constexpr int PHI_TILE_BYTES = N * PNC * 8;
-constexpr int PHI_SLOT = (N * PNC + 15) / 16 * 16;  // doubles; slots 128-B aligned
-constexpr size_t PHI_SMEM =
-    (size_t)(3 * PHI_SLOT + 2 * N * TY * TX + 2 * N * TY + 2 * N * TX + 4) * sizeof(double);
-
 template <class PT, class GT, int L, bool TA>
 __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, const GT& g,
                                                const double* __restrict__ ps, const double* __restrict__ ms,
                                                double* __restrict__ pd) {
-  extern __shared__ __align__(128) double psm[];
-  double* ring = psm;                                  // [3][PHI_SLOT]: [N][PHY][PHX]
-  double(*fy)[N][TY][TX] = reinterpret_cast<double(*)[N][TY][TX]>(psm + 3 * PHI_SLOT);  // [2][N][TY][TX]
-  double(*ex)[N][TY] = reinterpret_cast<double(*)[N][TY]>(psm + 3 * PHI_SLOT + 2 * N * TY * TX);
-  double(*ey)[N][TX] = reinterpret_cast<double(*)[N][TX]>(psm + 3 * PHI_SLOT + 2 * N * TY * TX + 2 * N * TY);
-  unsigned long long* bar =
-      reinterpret_cast<unsigned long long*>(psm + 3 * PHI_SLOT + 2 * N * TY * TX + 2 * N * TY + 2 * N * TX);
-  const int lane = threadIdx.x, w = threadIdx.y, t = w * TX + lane;
+  __shared__ double fy[2][N][TY][TX];  // -y face flux of every thread, by plane parity
+  __shared__ double ex[2][N][TY];      // +x flux on the right tile edge
+  __shared__ double ey[2][N][TX];      // +y flux on the top tile edge
+  const int lane = threadIdx.x, w = threadIdx.y;
   const int x0 = blockIdx.x * TX, y0 = blockIdx.y * TY;
   const int x = x0 + lane, y = y0 + w;
   const bool active = x < g.nx && y < g.ny;
-  // ragged tiles: threads beyond the domain read the ghost cell (or guard
-  // values); the -x / -y face of the ghost cell is the +x / +y face of the
-  // last interior cell
+  // ragged tiles: clamp to the ghost cell, whose -x / -y face is the +x / +y
+  // face of the last interior cell
   const int xc = min(x, g.nx), yc = min(y, g.ny);
   const int z0 = blockIdx.z * ZC_PHI, z1 = min(z0 + ZC_PHI, g.nz);
-  const i64 F = g.field;
-  const int me = (w + 1) * PHX + lane + 2;  // own cell in a halo tile (origin x0 - 2, y0 - 1)
-  const bool extra = (w == 0 && lane < TY) || w == 1;
+  const i64 F = g.field, SY = g.pitch, SZ = g.plane;
   // extra faces: warp 0 lanes < TY: +x face of row `lane`; warp 1: +y face of column `lane`
-  const int ea = w == 0 ? (lane + 1) * PHX + TX + 1 : TY * PHX + lane + 2;
-  const int eb = w == 0 ? ea + 1 : ea + PHX;
-  // plane j of this CTA (j = 0 <-> z0 - 1) lives in slot j % 3; its barrier phase is (j / 3) & 1.
-  // Warp 0 issues the N * PHY row copies of a plane (lane l: rows l, l + 32, ...).
-  auto issue = [&](int j) {
-    if (lane == 0) mbar_expect_tx(&bar[j % 3], PHI_TILE_BYTES);
-    __syncwarp();
-    const int zz = z0 - 1 + j;
-    for (int r = lane; r < N * PHY; r += TX) {
-      const int a = r / PHY, hy = r - a * PHY;
-      const int gy = min(y0 - 1 + hy, g.ny + 1);
-      bulk_load(ring + (j % 3) * PHI_SLOT + a * PNC + hy * PHX, ps + a * g.field + g.at(x0 - 2, gy, zz),
-                PHX * 8, &bar[j % 3]);
-    }
-  };
-  if (t == 0) {
-    for (int i = 0; i < 3; ++i) mbar_init(&bar[i], 1);
-    mbar_fence_init();
+  i64 ep = 0, eq = 0;  // the two cells of the extra face, at plane z0
+  if (w == 0 && lane < TY) {
+    const int ry = min(y0 + lane, g.ny);
+    ep = g.at(min(x0 + TX - 1, g.nx), ry, z0);
+    eq = g.at(min(x0 + TX, g.nx), ry, z0);
+  } else if (w == 1) {
+    const int cx = min(x0 + lane, g.nx);
+    ep = g.at(cx, min(y0 + TY - 1, g.ny), z0);
+    eq = g.at(cx, min(y0 + TY, g.ny), z0);
   }
-  __syncthreads();
-  if (w == 0) {
-    issue(0);
-    issue(1);
-    issue(2);
-  }
-  mbar_wait(&bar[0], 0);
-  mbar_wait(&bar[1], 0);
+  const bool extra = (w == 0 && lane < TY) || w == 1;
+
+  i64 c = g.at(xc, yc, z0);
   double pm[N], p0[N], Fzm[N];
 #pragma unroll
   for (int a = 0; a < N; ++a) {
-    pm[a] = ring[0 * PHI_SLOT + a * PNC + me];
-    p0[a] = ring[1 * PHI_SLOT + a * PNC + me];
+    pm[a] = __ldg(ps + a * F + c - SZ);
+    p0[a] = __ldg(ps + a * F + c);
   }
   phi_face(P, pm, p0, Fzm);
-  i64 c = g.at(xc, yc, z0);
-  double mu0 = __ldg(ms + c), mu1 = __ldg(ms + F + c);
 
-  for (int z = z0; z < z1; ++z, c += g.plane) {
-    const int j = z - z0 + 1;  // plane z is j, plane z+1 is j+1
+  for (int z = z0; z < z1; ++z, c += SZ, ep += SZ, eq += SZ) {
     const int buf = z & 1;
-    const double* s0 = ring + (j % 3) * PHI_SLOT;
-    double Fxm[N], Fym[N], gxy[N][2];
+    double pp[N], Fxm[N], Fym[N], Fzp[N], gd[N][3];
     {
-      double xm[N], ym[N];
+      double xm[N], xp[N], ym[N], yp[N];
 #pragma unroll
       for (int a = 0; a < N; ++a) {
-        xm[a] = s0[a * PNC + me - 1];
-        ym[a] = s0[a * PNC + me - PHX];
-        gxy[a][0] = s0[a * PNC + me + 1] - xm[a];
-        gxy[a][1] = s0[a * PNC + me + PHX] - ym[a];
+        const double* f = ps + a * F + c;
+        pp[a] = __ldg(f + SZ);
+        xm[a] = __ldg(f - 1);
+        xp[a] = __ldg(f + 1);
+        ym[a] = __ldg(f - SY);
+        yp[a] = __ldg(f + SY);
+        gd[a][0] = xp[a] - xm[a];
+        gd[a][1] = yp[a] - ym[a];
+        gd[a][2] = pp[a] - pm[a];
       }
       phi_face(P, xm, p0, Fxm);
       phi_face(P, ym, p0, Fym);
     }
+    phi_face(P, p0, pp, Fzp);
     if (extra) {
       double fa[N], fb[N], fe[N];
 #pragma unroll
       for (int a = 0; a < N; ++a) {
-        fa[a] = s0[a * PNC + ea];
-        fb[a] = s0[a * PNC + eb];
+        fa[a] = __ldg(ps + a * F + ep);
+        fb[a] = __ldg(ps + a * F + eq);
       }
       phi_face(P, fa, fb, fe);
       if (w == 0) {
@@ -166,26 +109,15 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, 
     }
 #pragma unroll
     for (int a = 0; a < N; ++a) fy[buf][a][w][lane] = Fym[a];
-    const double nmu0 = z + 1 < z1 ? __ldg(ms + c + g.plane) : 0.0;  // prefetch the next plane's mu
-    const double nmu1 = z + 1 < z1 ? __ldg(ms + F + c + g.plane) : 0.0;
-    // all threads are done with plane j-1 (slot of j+2) and have published fy
+    const double mu0 = __ldg(ms + c), mu1 = __ldg(ms + F + c);
     __syncthreads();
-    if (w == 0 && z + 2 <= z1) issue(j + 2);
-    mbar_wait(&bar[(j + 1) % 3], ((j + 1) / 3) & 1);
-    const double* s1 = ring + ((j + 1) % 3) * PHI_SLOT;
-    double pp[N], Fzp[N], divh[N], gd[N][3];
-#pragma unroll
-    for (int a = 0; a < N; ++a) pp[a] = s1[a * PNC + me];
-    phi_face(P, p0, pp, Fzp);
+    double divh[N];
 #pragma unroll
     for (int a = 0; a < N; ++a) {
       double fxp = __shfl_down_sync(0xffffffffu, Fxm[a], 1);
       if (lane == TX - 1) fxp = ex[buf][a][w];
       const double fyp = (w < TY - 1) ? fy[buf][a][w + 1][lane] : ey[buf][a][lane];
       divh[a] = ((fxp - Fxm[a]) + (fyp - Fym[a])) + (Fzp[a] - Fzm[a]);
-      gd[a][0] = gxy[a][0];
-      gd[a][1] = gxy[a][1];
-      gd[a][2] = pp[a] - pm[a];
     }
     double out[N];
     phi_cell<TA>(P, plane_T(P, R, (double)z), p0, gd, divh, mu0, mu1, out);
@@ -199,8 +131,6 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, 
       p0[a] = pp[a];
       Fzm[a] = Fzp[a];
     }
-    mu0 = nmu0;
-    mu1 = nmu1;
   }
 }
 

@@ -47,17 +47,12 @@ dim3 tuned_grid_mu(const Geom& g) {
 }
 size_t tuned_mu_smem() { return mu_smem_bytes<MU_TY>(); }
 
-size_t tuned_phi_smem() { return PHI_SMEM; }
+size_t tuned_phi_smem() { return 0; }  // static shared memory only
 
 template <int L, bool TA>
 static void phi_launch(const DevParams& P, const Geom& g, const double* ps, const double* ms, double* pd,
                        cudaStream_t s) {
-  static bool attr = false;  // per instantiation
-  if (!attr) {
-    cudaFuncSetAttribute(k_phi_tuned<L, TA>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)PHI_SMEM);
-    attr = true;
-  }
-  k_phi_tuned<L, TA><<<tuned_grid_phi(g), tuned_block(), PHI_SMEM, s>>>(P, g, ps, ms, pd);
+  k_phi_tuned<L, TA><<<tuned_grid_phi(g), tuned_block(), 0, s>>>(P, g, ps, ms, pd);
 }
 
 void launch_phi_tuned(const DevParams& P, const Geom& g, const double* ps, const double* ms, double* pd,

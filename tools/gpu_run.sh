@@ -12,8 +12,8 @@ timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $OUT/smoke.log 
 timeout 600 python bench.py --steps 100 --warmup 5 > $OUT/bench.json 2> $OUT/bench.err
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches.csv \
    python bench.py --steps 10 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_launch.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_mu_tuned -s 3 -c 1 -o $OUT/prof_mu \
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:pf_jit_mu -s 3 -c 1 -o $OUT/prof_mu \
    python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_mu.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_phi_tuned -s 3 -c 1 -o $OUT/prof_phi \
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:pf_jit_phi -s 3 -c 1 -o $OUT/prof_phi \
    python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_phi.log 2>&1
 echo done > $OUT/DONE
