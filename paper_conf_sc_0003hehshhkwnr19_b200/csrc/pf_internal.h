@@ -26,10 +26,11 @@ void launch_mu_tuned(const DevParams& P, const Geom& g, const double* ps, const 
                      double* md, cudaStream_t s);
 // launch geometry of the tuned kernels (shared with the specialised build)
 dim3 tuned_block();
-dim3 tuned_block_mu();
+dim3 tuned_block_mu(int mty);
 dim3 tuned_grid_phi(const Geom& g);
-dim3 tuned_grid_mu(const Geom& g);
-size_t tuned_mu_smem();
+dim3 tuned_grid_mu(const Geom& g, int mty);
+size_t tuned_mu_smem(int mty);  // mty: tile height of the mu-sweep (2, 4, 8)
+int tuned_mu_ty_default();
 size_t tuned_phi_smem();
 
 // ---- ghost layers, halo exchange, window, reductions, copies ------------

@@ -40,12 +40,15 @@ __global__ void __launch_bounds__(TX* MU_TY, 16 / MU_TY) k_mu_tuned(DevParams P,
 }
 
 dim3 tuned_block() { return dim3(TX, TY); }
-dim3 tuned_block_mu() { return dim3(TX, MU_TY); }
+dim3 tuned_block_mu(int mty) { return dim3(TX, mty); }
 dim3 tuned_grid_phi(const Geom& g) { return dim3((g.nx + TX - 1) / TX, (g.ny + TY - 1) / TY, (g.nz + ZC_PHI - 1) / ZC_PHI); }
-dim3 tuned_grid_mu(const Geom& g) {
-  return dim3((g.nx + TX - 1) / TX, (g.ny + MU_TY - 1) / MU_TY, (g.nz + ZC_MU - 1) / ZC_MU);
+dim3 tuned_grid_mu(const Geom& g, int mty) {
+  return dim3((g.nx + TX - 1) / TX, (g.ny + mty - 1) / mty, (g.nz + ZC_MU - 1) / ZC_MU);
 }
-size_t tuned_mu_smem() { return mu_smem_bytes<MU_TY>(); }
+size_t tuned_mu_smem(int mty) {
+  return mty == 8 ? mu_smem_bytes<8>() : (mty == 4 ? mu_smem_bytes<4>() : (mty == 2 ? mu_smem_bytes<2>() : 0));
+}
+int tuned_mu_ty_default() { return MU_TY; }
 
 size_t tuned_phi_smem() { return 0; }  // static shared memory only
 
@@ -66,10 +69,10 @@ static void mu_launch(const DevParams& P, const Geom& g, const double* ps, const
                       double* md, cudaStream_t s) {
   static bool attr = false;  // per instantiation
   if (!attr) {
-    cudaFuncSetAttribute(k_mu_tuned<L, TA>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tuned_mu_smem());
+    cudaFuncSetAttribute(k_mu_tuned<L, TA>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tuned_mu_smem(MU_TY));
     attr = true;
   }
-  k_mu_tuned<L, TA><<<tuned_grid_mu(g), tuned_block_mu(), tuned_mu_smem(), s>>>(P, g, ps, pd, ms, md);
+  k_mu_tuned<L, TA><<<tuned_grid_mu(g, MU_TY), tuned_block_mu(MU_TY), tuned_mu_smem(MU_TY), s>>>(P, g, ps, pd, ms, md);
 }
 
 void launch_mu_tuned(const DevParams& P, const Geom& g, const double* ps, const double* pd, const double* ms,
