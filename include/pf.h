@@ -123,6 +123,14 @@ typedef struct {
  * Reads cfg->global/procs/rank only.  PF_EINVAL on a bad decomposition. */
 int pf_query_layout(const pf_config* cfg, pf_layout* out);
 
+/* Host-only: neighbour ranks of this rank's block per dimension (nb_lo,
+ * nb_hi; -1 = physical boundary, periodic dimensions wrap, possibly onto the
+ * rank itself).  The halo exchange of dimension d sends the hi face to nb_hi
+ * and the lo face to nb_lo, then receives the lo ghost from nb_lo and the hi
+ * ghost from nb_hi (x, then y, then z; earlier dimensions' ghosts included
+ * so that edges travel).  Reads cfg->global/procs/rank/world/bc_lo.        */
+int pf_query_neighbors(const pf_config* cfg, int nb_lo[3], int nb_hi[3]);
+
 /* Validate cfg, bind the caller's buffers, create streams/events and (world > 1)
  * the NCCL communicator from cfg->nccl_uid.  Collective when world > 1.     */
 int pf_create(const pf_config* cfg, pf_ctx** out);

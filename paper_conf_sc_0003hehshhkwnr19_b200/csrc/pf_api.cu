@@ -176,6 +176,27 @@ int layout_of(const pf_config* cfg, pf_layout* L, int coord[3]) {
   return PF_OK;
 }
 
+// Neighbour ranks of the block at rank-grid coordinates coord (-1 = physical
+// boundary; periodic dimensions wrap, also onto the rank itself).
+void neighbours_of(const pf_config* cfg, const int coord[3], int nb_lo[3], int nb_hi[3]) {
+  int pr[3];
+  for (int d = 0; d < 3; ++d) pr[d] = cfg->procs[d] < 1 ? 1 : cfg->procs[d];
+  auto rank_of = [&](const int c[3]) { return c[0] + pr[0] * (c[1] + pr[1] * c[2]); };
+  for (int d = 0; d < 3; ++d) {
+    const bool periodic = cfg->bc_lo[d] == PF_BC_PERIODIC;
+    int lo = coord[d] - 1, hi = coord[d] + 1;
+    if (periodic) {
+      lo = (lo + pr[d]) % pr[d];
+      hi = hi % pr[d];
+    }
+    int cl[3] = {coord[0], coord[1], coord[2]}, ch[3] = {coord[0], coord[1], coord[2]};
+    cl[d] = lo;
+    ch[d] = hi;
+    nb_lo[d] = (lo >= 0 && lo < pr[d]) ? rank_of(cl) : -1;
+    nb_hi[d] = (hi >= 0 && hi < pr[d]) ? rank_of(ch) : -1;
+  }
+}
+
 // Explicit (FTCS) stability bounds (SURVEY C.4 "dt"), in time units.
 //  phi: linearised diffusivity of the gradient flux 2 sum_b gamma_ab phi_b^2 / tau <= 2 gamma_max / tau_min
 //  mu:  D_eff = spectral radius of chi^{-1} M over sample points of the simplex
@@ -328,6 +349,15 @@ int pf_query_layout(const pf_config* cfg, pf_layout* out) {
   return layout_of(cfg, out, coord);
 }
 
+int pf_query_neighbors(const pf_config* cfg, int nb_lo[3], int nb_hi[3]) {
+  pf_layout L;
+  int coord[3];
+  if (!nb_lo || !nb_hi) return PF_EINVAL;
+  if (int r = layout_of(cfg, &L, coord)) return r;
+  neighbours_of(cfg, coord, nb_lo, nb_hi);
+  return PF_OK;
+}
+
 int pf_create(const pf_config* cfg, pf_ctx** out) {
   if (!cfg || !out) return PF_EINVAL;
   *out = nullptr;
@@ -382,23 +412,10 @@ int pf_create(const pf_config* cfg, pf_ctx** out) {
   }
   // neighbours and BC kinds
   const int world = cfg->world < 1 ? 1 : cfg->world;
-  int pr[3];
-  for (int d = 0; d < 3; ++d) pr[d] = cfg->procs[d] < 1 ? 1 : cfg->procs[d];
-  auto rank_of = [&](int cx, int cy, int cz) { return cx + pr[0] * (cy + pr[1] * cz); };
+  neighbours_of(cfg, ctx->coord, ctx->nb_lo, ctx->nb_hi);
   for (int d = 0; d < 3; ++d) {
-    const bool periodic = cfg->bc_lo[d] == PF_BC_PERIODIC;
-    int c[3] = {ctx->coord[0], ctx->coord[1], ctx->coord[2]};
-    int lo = c[d] - 1, hi = c[d] + 1;
-    if (periodic) {
-      lo = (lo + pr[d]) % pr[d];
-      hi = hi % pr[d];
-    }
-    int cl[3] = {c[0], c[1], c[2]}, ch[3] = {c[0], c[1], c[2]};
-    cl[d] = lo;
-    ch[d] = hi;
-    ctx->nb_lo[d] = (lo >= 0 && lo < pr[d]) ? rank_of(cl[0], cl[1], cl[2]) : -1;
-    ctx->nb_hi[d] = (hi >= 0 && hi < pr[d]) ? rank_of(ch[0], ch[1], ch[2]) : -1;
-    ctx->exchange[d] = pr[d] > 1;
+    const int pr = cfg->procs[d] < 1 ? 1 : cfg->procs[d];
+    ctx->exchange[d] = pr > 1;
     ctx->bc_all.kind_lo[d] = (ctx->exchange[d] && ctx->nb_lo[d] >= 0) ? -1 : cfg->bc_lo[d];
     ctx->bc_all.kind_hi[d] = (ctx->exchange[d] && ctx->nb_hi[d] >= 0) ? -1 : cfg->bc_hi[d];
   }

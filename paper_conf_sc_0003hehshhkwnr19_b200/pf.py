@@ -55,7 +55,7 @@ class PFState(C.Structure):
 
 
 # every symbol include/pf.h declares (checked by tests/test_abi.py)
-ABI_SYMBOLS = ["pf_query_layout", "pf_create", "pf_destroy", "pf_set_params", "pf_init_fields", "pf_step",
+ABI_SYMBOLS = ["pf_query_layout", "pf_query_neighbors", "pf_create", "pf_destroy", "pf_set_params", "pf_init_fields", "pf_step",
                "pf_step_phi_only", "pf_halo_exchange", "pf_shift_window", "pf_front_height", "pf_monitor",
                "pf_download", "pf_get_state", "pf_set_state", "pf_set_variant", "pf_profile", "pf_profile_read",
                "pf_nccl_unique_id", "pf_jit_compile_only", "pf_last_error", "pf_version"]
@@ -74,6 +74,7 @@ def load_library(path: str = LIB_PATH):
     vp, ip = C.c_void_p, C.c_int
     dp = C.POINTER(C.c_double)
     L.pf_query_layout.argtypes = [C.POINTER(PFConfig), C.POINTER(PFLayout)]
+    L.pf_query_neighbors.argtypes = [C.POINTER(PFConfig), C.POINTER(ip), C.POINTER(ip)]
     L.pf_create.argtypes = [C.POINTER(PFConfig), C.POINTER(vp)]
     L.pf_destroy.argtypes = [vp]
     L.pf_set_params.argtypes = [vp, C.POINTER(PFParams)]
@@ -144,6 +145,39 @@ def jit_compile_only(params: dict, n: int = 64, cubin_path: str | None = None) -
     if r < 0:
         raise PFError(f"specialised compile failed: {log.value.decode()}")
     return r
+
+
+def make_config(shape, bc=None, liquid: int = 3, procs=(1, 1, 1), rank: int = 0, world: int = 1) -> PFConfig:
+    """pf_config for a global (nz, ny, nx) domain (no buffers bound)."""
+    nz, ny, nx = shape
+    bc = bc or {"lo": ("periodic",) * 3, "hi": ("periodic",) * 3}
+    cfg = PFConfig()
+    cfg.n_phases, cfg.n_mu, cfg.liquid = N, M, int(liquid)
+    for d, n in enumerate((nx, ny, nz)):
+        cfg.global_[d] = n
+        cfg.procs[d] = int(procs[d])
+        cfg.bc_lo[d] = BC[bc["lo"][d]]
+        cfg.bc_hi[d] = BC[bc["hi"][d]]
+    cfg.rank, cfg.world = int(rank), int(world)
+    return cfg
+
+
+def query_layout(shape, procs=(1, 1, 1), rank: int = 0, world: int = 1, bc=None) -> PFLayout:
+    """Host-only block layout of `rank` (no GPU needed)."""
+    lay = PFLayout()
+    r = load_library().pf_query_layout(C.byref(make_config(shape, bc, 3, procs, rank, world)), C.byref(lay))
+    if r != PF_OK:
+        raise PFError(f"pf_query_layout failed ({r})")
+    return lay
+
+
+def query_neighbors(shape, procs=(1, 1, 1), rank: int = 0, world: int = 1, bc=None):
+    """Host-only neighbour ranks (x, y, z) of `rank`: (lo, hi), -1 = boundary."""
+    lo, hi = (C.c_int * 3)(), (C.c_int * 3)()
+    r = load_library().pf_query_neighbors(C.byref(make_config(shape, bc, 3, procs, rank, world)), lo, hi)
+    if r != PF_OK:
+        raise PFError(f"pf_query_neighbors failed ({r})")
+    return tuple(lo), tuple(hi)
 
 
 def nccl_unique_id() -> bytes:
