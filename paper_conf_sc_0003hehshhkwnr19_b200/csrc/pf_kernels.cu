@@ -251,54 +251,72 @@ void launch_shift(const Geom& g, int k, int liquid, const double* mu_inf, const 
   k_shift<<<gr, b, 0, s>>>(g, k, liquid, mu_inf[0], mu_inf[1], ps, ms, pd, md);
 }
 
-// front height: max z with phi_l < 1/2 (deterministic integer max)
+// front height: max z with phi_l < 1/2 (deterministic integer max).  One
+// block per (y-slab, z) plane: block-level OR, one atomic per block.
 __global__ void k_front(Geom g, const double* __restrict__ phl, int* out) {
-  const int x = blockIdx.x * blockDim.x + threadIdx.x;
-  const int y = blockIdx.y, z = blockIdx.z;
-  bool hit = x < g.nx && phl[g.at(x, y, z)] < 0.5;
-  if (__any_sync(0xffffffffu, hit) && (threadIdx.x & 31) == 0) atomicMax(out, z + g.z0 + 1);  // H + 1
+  const int z = blockIdx.y;
+  bool hit = false;
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < g.nx * g.ny; i += gridDim.x * blockDim.x) {
+    const int y = i / g.nx, x = i - y * g.nx;
+    hit |= phl[g.at(x, y, z)] < 0.5;
+  }
+  if (__syncthreads_or(hit) && threadIdx.x == 0) atomicMax(out, z + g.z0 + 1);  // H + 1
 }
 
 void launch_front_height(const Geom& g, int liquid, const double* phi, int* out, cudaStream_t s) {
-  dim3 b(128), gr((g.nx + 127) / 128, g.ny, g.nz);
-  k_front<<<gr, b, 0, s>>>(g, phi + (int64_t)liquid * g.field, out);
+  int bx = (g.nx * g.ny + 255) / 256;
+  if (bx > 64) bx = 64;
+  dim3 gr(bx, g.nz);
+  k_front<<<gr, 256, 0, s>>>(g, phi + (int64_t)liquid * g.field, out);
 }
 
-// monitors: out[0] = max |sum phi - 1| (as ordered bits), out[1] = max(-min phi) encoded
+// monitors: out[0] = max |sum phi - 1|, out[1] = max(-min phi), as
+// order-preserving bit patterns; block-level reduction, one atomic per block
 __device__ __forceinline__ unsigned long long ord_bits(double v) {
-  // order-preserving map of doubles to unsigned (max over the map = max over values)
   unsigned long long b = (unsigned long long)__double_as_longlong(v);
   return (b & 0x8000000000000000ull) ? ~b : (b | 0x8000000000000000ull);
 }
 
 __global__ void k_monitor(Geom g, const double* __restrict__ ph, unsigned long long* out) {
-  const int x = blockIdx.x * blockDim.x + threadIdx.x;
-  const int y = blockIdx.y, z = blockIdx.z;
+  const int z = blockIdx.y;
   double e = -1.0, neg = -INFINITY;
-  if (x < g.nx) {
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < g.nx * g.ny; i += gridDim.x * blockDim.x) {
+    const int y = i / g.nx, x = i - y * g.nx;
     const int64_t c = g.at(x, y, z);
-    double s = 0.0, mn = INFINITY;
+    double sum = 0.0, mn = INFINITY;
     for (int a = 0; a < N; ++a) {
       const double v = ph[a * g.field + c];
-      s += v;
+      sum += v;
       mn = fmin(mn, v);
     }
-    e = fabs(s - 1.0);
-    neg = -mn;
+    e = fmax(e, fabs(sum - 1.0));
+    neg = fmax(neg, -mn);
   }
   for (int o = 16; o > 0; o >>= 1) {
     e = fmax(e, __shfl_xor_sync(0xffffffffu, e, o));
     neg = fmax(neg, __shfl_xor_sync(0xffffffffu, neg, o));
   }
+  __shared__ double se[8], sn[8];
   if ((threadIdx.x & 31) == 0) {
+    se[threadIdx.x >> 5] = e;
+    sn[threadIdx.x >> 5] = neg;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    for (int w = 1; w < (int)(blockDim.x >> 5); ++w) {
+      e = fmax(e, se[w]);
+      neg = fmax(neg, sn[w]);
+    }
     atomicMax(out, ord_bits(e));
     atomicMax(out + 1, ord_bits(neg));
   }
 }
 
 void launch_monitor(const Geom& g, const double* phi, unsigned long long* out2, cudaStream_t s) {
-  dim3 b(128), gr((g.nx + 127) / 128, g.ny, g.nz);
-  k_monitor<<<gr, b, 0, s>>>(g, phi, out2);
+  int bx = (g.nx * g.ny + 255) / 256;
+  if (bx > 64) bx = 64;
+  dim3 gr(bx, g.nz);
+  k_monitor<<<gr, 256, 0, s>>>(g, phi, out2);
 }
 
 // interior <-> packed [comp][z][y][x] copies

@@ -1,0 +1,75 @@
+"""Copy the evidence of one GPU session into profiles/ (tracked):
+bench line, ncu launch list, ncu --set full summaries of the sweeps (key
+metrics, stall reasons, dynamic instruction mix), fp64 micro-benchmarks, and
+profiles/ncu_summary.json (dram bytes per launch, read by bench.py).
+usage: python tools/write_profiles.py gpurun_out/<dir> <round-tag>"""
+import collections
+import csv
+import json
+import os
+import re
+import shutil
+import subprocess
+import sys
+
+src, tag = sys.argv[1], sys.argv[2]
+dst = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles")
+os.makedirs(dst, exist_ok=True)
+for name, out in (("bench.json", f"{tag}_bench.json"), ("launches.csv", f"{tag}_launches.csv"),
+                  ("fp64_micro.json", f"{tag}_fp64_micro.json"), ("pytest_gpu.log", f"{tag}_pytest_gpu.log"),
+                  ("smoke.log", f"{tag}_smoke.log"), ("nvidia-smi.txt", f"{tag}_nvidia-smi.txt")):
+    p = os.path.join(src, name)
+    if os.path.exists(p):
+        shutil.copy(p, os.path.join(dst, out))
+
+KEYS = ["gpu__time_duration.sum", "launch__registers_per_thread", "launch__occupancy_limit_registers",
+        "launch__occupancy_limit_shared_mem", "sm__warps_active.avg.pct_of_peak_sustained_active",
+        "sm__pipe_fp64_cycles_active.avg.pct_of_peak_sustained_active",
+        "smsp__issue_active.avg.pct_of_peak_sustained_active", "l1tex__throughput.avg.pct_of_peak_sustained_active",
+        "dram__bytes_read.sum", "dram__bytes_write.sum", "dram__throughput.avg.pct_of_peak_sustained_elapsed",
+        "lts__t_sector_hit_rate.pct", "smsp__inst_executed.sum", "smsp__sass_inst_executed_op_global_ld.sum",
+        "smsp__sass_inst_executed_op_shared_ld.sum", "smsp__sass_inst_executed_op_local_ld.sum"]
+summary = {}
+for kern in ("mu", "phi"):
+    rep = os.path.join(src, f"prof_{kern}.ncu-rep")
+    if not os.path.exists(rep):
+        continue
+    raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    rows = list(csv.reader(raw.splitlines()))
+    h, u, v = rows[0], rows[1], rows[2]
+    m = {n: (v[i], u[i]) for i, n in enumerate(h)}
+    lines = [f"ncu --set full summary: {m.get('Kernel Name', ('?',))[0]}  (session {os.path.basename(src)})", ""]
+    for k in KEYS:
+        if k in m:
+            lines.append(f"  {k:70s} {m[k][0]} {m[k][1]}")
+    st = {n.replace("smsp__average_warps_issue_stalled_", "").replace("_per_issue_active.ratio", ""): float(v[i] or 0)
+          for i, n in enumerate(h)
+          if n.startswith("smsp__average_warps_issue_stalled") and n.endswith("per_issue_active.ratio")}
+    lines += ["", "  warp stall reasons (cycles per issued instruction):"]
+    lines += [f"    {k:28s} {x:6.2f}" for k, x in sorted(st.items(), key=lambda kv: -kv[1]) if x > 0.05]
+    srcp = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
+                          capture_output=True, text=True).stdout
+    srows = list(csv.reader(srcp.splitlines()))
+    if len(srows) > 2:
+        hh = srows[1]
+        iE = hh.index("Instructions Executed")
+        ops = collections.Counter()
+        for r in srows[2:]:
+            mm = re.match(r"(@!?U?P\w+\s+)?([A-Z0-9_]+)", r[1].strip())
+            if mm:
+                ops[mm.group(2)] += int(r[iE] or 0)
+        tot = sum(ops.values())
+        fp64 = sum(ops[o] for o in ("DFMA", "DMUL", "DADD", "DSETP", "DMNMX", "MUFU"))
+        lines += ["", f"  dynamic instruction mix (warp-level, total {tot}, fp64-pipe share {fp64 / max(tot, 1):.1%}):"]
+        lines += [f"    {k:10s} {c / tot:6.1%}" for k, c in ops.most_common(20)]
+    open(os.path.join(dst, f"{tag}_ncu_{kern}.txt"), "w").write("\n".join(lines) + "\n")
+    rd = float(m["dram__bytes_read.sum"][0]) * {"Gbyte": 1e9, "Mbyte": 1e6, "Kbyte": 1e3, "byte": 1}[m["dram__bytes_read.sum"][1]]
+    wr = float(m["dram__bytes_write.sum"][0]) * {"Gbyte": 1e9, "Mbyte": 1e6, "Kbyte": 1e3, "byte": 1}[m["dram__bytes_write.sum"][1]]
+    summary[f"{kern}_sweep"] = {"dram_bytes_per_launch": rd + wr, "dram_read": rd, "dram_write": wr,
+                                "session": os.path.basename(src), "round": tag}
+if summary:
+    p = os.path.join(dst, "ncu_summary.json")
+    old = json.load(open(p)) if os.path.exists(p) else {}
+    old.update(summary)
+    json.dump(old, open(p, "w"), indent=1)
+print("wrote", sorted(os.listdir(dst)))
