@@ -71,7 +71,7 @@ class ClockSampler:
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
-                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+                 "-lms", "50"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
         except Exception:
@@ -81,7 +81,7 @@ class ClockSampler:
         for line in self.proc.stdout:
             self.lines.append(line.strip())
 
-    def stop(self):
+    def stop(self, first: int = 0):
         if not self.proc:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
         self.proc.terminate()
@@ -92,7 +92,7 @@ class ClockSampler:
         self.t.join(timeout=2)
         sm, smax, reasons, power = [], [], set(), []
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for ln in self.lines:
+        for ln in self.lines[max(first - 1, 0):]:
             f = [x.strip() for x in ln.split(",")]
             if len(f) < 9:
                 continue
@@ -245,13 +245,18 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
-    # ---- warm-up ----
-    g.step(args.warmup)
-    barrier()
-    # ---- timed region (device events on the library's stream) ----
-    g.profile(True)
+    # ---- warm-up (the clock sampler spins up meanwhile) ----
     clocks = ClockSampler(local_rank)
     clocks.start()
+    g.step(args.warmup)
+    barrier()
+    t_wait = time.time()
+    while len(clocks.lines) < 2 and time.time() - t_wait < 3.0:
+        g.step(1)
+        torch.cuda.synchronize()
+    # ---- timed region (device events on the library's stream) ----
+    g.profile(True)
+    n_clk0 = len(clocks.lines)
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
     barrier()
@@ -261,7 +266,7 @@ def main():
     e1.synchronize()
     barrier()
     ms = e0.elapsed_time(e1)
-    clk = clocks.stop()
+    clk = clocks.stop(n_clk0)
     prof = g.profile_read()
     ms_max = max_over_ranks(ms)
     launches = sum(v[1] for v in prof.values())
