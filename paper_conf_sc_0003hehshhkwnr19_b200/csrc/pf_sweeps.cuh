@@ -241,30 +241,21 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
   const int z0 = blockIdx.z * ZC_MU, z1 = min(z0 + ZC_MU, g.nz);
   const i64 F = g.field;
   const int me = hidx(lane + 1, w + 1);
-  // halo ring (+ its 4 corners, whose phi the ring's tangential differences
-  // need) owned by the last 2*TX + 2*MTY + 4 threads; warps 0, 1 compute the
-  // far-edge faces
-  int hx = -1, hy = -1, hs = -1, hkind = 0;  // hkind: 1 = row (needs cd_x), 2 = column (cd_y), 3 = corner
-  {
-    const int th = t - (MTY * TX - (2 * TX + 2 * MTY + 4));
-    if (th >= 0 && th < TX) { hx = th + 1; hy = 0; hkind = 1; }
-    else if (th >= TX && th < 2 * TX) { hx = th - TX + 1; hy = MTY + 1; hkind = 1; }
-    else if (th >= 2 * TX && th < 2 * TX + MTY) { hx = 0; hy = th - 2 * TX + 1; hkind = 2; }
-    else if (th >= 2 * TX + MTY && th < 2 * TX + 2 * MTY) { hx = TX + 1; hy = th - 2 * TX - MTY + 1; hkind = 2; }
-    else if (th >= 2 * TX + 2 * MTY && th < 2 * TX + 2 * MTY + 4) {
-      const int cc = th - 2 * TX - 2 * MTY;
-      hx = (cc & 1) ? TX + 1 : 0;
-      hy = (cc & 2) ? MTY + 1 : 0;
-      hkind = 3;
-    }
-    if (hkind) hs = hidx(hx, hy);
-  }
-  const int hgx = min(x0 + hx - 1, g.nx + 1), hgy = min(y0 + hy - 1, g.ny + 1);
+  // halo ring cell owned by thread t < 2*TX + 2*MTY (corners are not needed)
+  // (the last threads build the halo ring; warps 0, 1 compute the far-edge faces)
+  int hx = 0, hy = 0, hs = -1;
+  bool hwx = false, hwy = false;
+  const int th = t - (MTY * TX - (2 * TX + 2 * MTY));
+  if (th >= 0 && th < TX) { hx = th + 1; hy = 0; hwx = true; }
+  else if (th >= TX && th < 2 * TX) { hx = th - TX + 1; hy = MTY + 1; hwx = true; }
+  else if (th >= 2 * TX && th < 2 * TX + MTY) { hx = 0; hy = th - 2 * TX + 1; hwy = true; }
+  else if (th >= 2 * TX + MTY && th < 2 * TX + 2 * MTY) { hx = TX + 1; hy = th - 2 * TX - MTY + 1; hwy = true; }
+  if (hwx || hwy) hs = hidx(hx, hy);
+  const int hgx = min(x0 + hx - 1, g.nx), hgy = min(y0 + hy - 1, g.ny);
 
   // z-face k-1/2 needs the previous plane's side (tangential: x, y)
   FaceSide Dp;
   double dpl = 0.0;  // dphi of the liquid at plane k-1 (for the cell update)
-  double pnx[N];     // phi_src of the own cell at the plane being built (carried, one load per plane)
   {
     const i64 c = g.at(xc, yc, z0 - 1);
 #pragma unroll
@@ -273,7 +264,6 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
       Dp.f[a] = __ldg(f);
       Dp.c1[a] = __ldg(f + 1) - __ldg(f - 1);
       Dp.c2[a] = __ldg(f + g.pitch) - __ldg(f - g.pitch);
-      pnx[a] = __ldg(f + g.plane);
     }
 #pragma unroll
     for (int s = 0; s < NSOL; ++s) {
@@ -287,73 +277,9 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
 
   for (int k = z0; k <= z1; ++k) {
     const bool last = k == z1;
-    // (a1) publish phi, cd_z, dphi, mu of plane k: own cell (phi(k) carried,
-    //      phi(k-1) = Dp.f) and the halo ring (+ corners) from global memory
-    {
-      const i64 c = g.at(xc, yc, k);
-      double v[D_NV];
-#pragma unroll
-      for (int a = 0; a < N; ++a) {
-        const double pk1 = last ? 0.0 : __ldg(ps + a * F + c + g.plane);
-        v[D_F + a] = pnx[a];
-        v[D_CZ + a] = pk1 - Dp.f[a];
-        v[D_DP + a] = __ldg(pd + a * F + c) - pnx[a];
-        pnx[a] = pk1;
-      }
-      v[D_MU + 0] = __ldg(ms + c);
-      v[D_MU + 1] = __ldg(ms + F + c);
-      double2* d = reinterpret_cast<double2*>(D + (size_t)me * D_NV);
-#pragma unroll
-      for (int a = 0; a < N / 2; ++a) {
-        d[(D_F >> 1) + a] = make_double2(v[D_F + 2 * a], v[D_F + 2 * a + 1]);
-        d[(D_CZ >> 1) + a] = make_double2(v[D_CZ + 2 * a], v[D_CZ + 2 * a + 1]);
-        d[(D_DP >> 1) + a] = make_double2(v[D_DP + 2 * a], v[D_DP + 2 * a + 1]);
-      }
-      d[D_MU >> 1] = make_double2(v[D_MU], v[D_MU + 1]);
-    }
-    if (hkind) {
-      const i64 c = g.at(hgx, hgy, k);
-      double2* d = reinterpret_cast<double2*>(D + (size_t)hs * D_NV);
-#pragma unroll
-      for (int a = 0; a < N; a += 2) {
-        const double f0 = __ldg(ps + a * F + c), f1 = __ldg(ps + (a + 1) * F + c);
-        d[(D_F + a) >> 1] = make_double2(f0, f1);
-        if (hkind != 3) {
-          d[(D_CZ + a) >> 1] = make_double2(__ldg(ps + a * F + c + g.plane) - __ldg(ps + a * F + c - g.plane),
-                                            __ldg(ps + (a + 1) * F + c + g.plane) -
-                                                __ldg(ps + (a + 1) * F + c - g.plane));
-          d[(D_DP + a) >> 1] = make_double2(__ldg(pd + a * F + c) - f0, __ldg(pd + (a + 1) * F + c) - f1);
-        }
-      }
-      if (hkind != 3) d[D_MU >> 1] = make_double2(__ldg(ms + c), __ldg(ms + F + c));
-    }
-    __syncthreads();
-    // (a2) in-plane central differences from the published phi (own: x and y;
-    //      ring rows: x; ring columns: y)
-    {
-      const double2* dm = reinterpret_cast<const double2*>(D);
-      double2* d = reinterpret_cast<double2*>(D + (size_t)me * D_NV);
-#pragma unroll
-      for (int a = 0; a < N / 2; ++a) {
-        const double2 xp = dm[(size_t)(me + 1) * (D_NV / 2) + (D_F >> 1) + a];
-        const double2 xm = dm[(size_t)(me - 1) * (D_NV / 2) + (D_F >> 1) + a];
-        const double2 yp = dm[(size_t)(me + HX) * (D_NV / 2) + (D_F >> 1) + a];
-        const double2 ym = dm[(size_t)(me - HX) * (D_NV / 2) + (D_F >> 1) + a];
-        d[(D_CX >> 1) + a] = make_double2(xp.x - xm.x, xp.y - xm.y);
-        d[(D_CY >> 1) + a] = make_double2(yp.x - ym.x, yp.y - ym.y);
-      }
-      if (hkind == 1 || hkind == 2) {
-        const int st = hkind == 1 ? 1 : HX;
-        const int off = hkind == 1 ? (D_CX >> 1) : (D_CY >> 1);
-        double2* dh = reinterpret_cast<double2*>(D + (size_t)hs * D_NV);
-#pragma unroll
-        for (int a = 0; a < N / 2; ++a) {
-          const double2 p1 = dm[(size_t)(hs + st) * (D_NV / 2) + (D_F >> 1) + a];
-          const double2 m1 = dm[(size_t)(hs - st) * (D_NV / 2) + (D_F >> 1) + a];
-          dh[off + a] = make_double2(p1.x - m1.x, p1.y - m1.y);
-        }
-      }
-    }
+    // (a) publish D(k) of the own cell and of the halo ring
+    build_cell<NC>(g, ps, pd, ms, xc, yc, k, true, true, !last, D, me);
+    if (hs >= 0 && !last) build_cell<NC>(g, ps, pd, ms, hgx, hgy, k, hwx, hwy, true, D, hs);
     __syncthreads();
     // (b) z-face k-1/2 from registers (plane k-1) and shared memory (plane k)
     FaceSide q;
