@@ -194,31 +194,6 @@ __device__ __forceinline__ void build_cell(const GT& g, const double* __restrict
   for (int j = 0; j < D_NV / 2; ++j) d[j] = make_double2(v[2 * j], v[2 * j + 1]);
 }
 
-// the own cell's D computed into registers (prefetch for the next plane)
-template <class GT>
-__device__ __forceinline__ void load_cell(const GT& g, const double* __restrict__ ps, const double* __restrict__ pd,
-                                          const double* __restrict__ ms, int x, int y, int k, bool wz,
-                                          double (&v)[D_NV]) {
-  const i64 F = g.field;
-  const i64 c = g.at(x, y, k);
-#pragma unroll
-  for (int a = 0; a < N; ++a) {
-    const double* f = ps + a * F + c;
-    v[D_F + a] = __ldg(f);
-    v[D_CX + a] = __ldg(f + 1) - __ldg(f - 1);
-    v[D_CY + a] = __ldg(f + g.pitch) - __ldg(f - g.pitch);
-    v[D_CZ + a] = wz ? __ldg(f + g.plane) - __ldg(f - g.plane) : 0.0;
-    v[D_DP + a] = __ldg(pd + a * F + c) - v[D_F + a];
-  }
-  v[D_MU + 0] = __ldg(ms + c);
-  v[D_MU + 1] = __ldg(ms + F + c);
-}
-__device__ __forceinline__ void store_cell(double* __restrict__ D, int i, const double (&v)[D_NV]) {
-  double2* d = reinterpret_cast<double2*>(D + (size_t)i * D_NV);
-#pragma unroll
-  for (int j = 0; j < D_NV / 2; ++j) d[j] = make_double2(v[2 * j], v[2 * j + 1]);
-}
-
 template <int L, int NC>
 __device__ __forceinline__ void side_from_smem(const double* __restrict__ D, int i, int c1, int c2, FaceSide& s) {
   const double2* d = reinterpret_cast<const double2*>(D + (size_t)i * D_NV);
@@ -299,13 +274,11 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
     Dp.m[1] = __ldg(ms + F + c);
   }
   double divxy[M] = {0.0, 0.0}, Fzm[M] = {0.0, 0.0};
-  double nxt[D_NV];  // own D of the next plane, loaded at the end of the previous iteration
-  load_cell(g, ps, pd, ms, xc, yc, z0, z0 < z1, nxt);
 
   for (int k = z0; k <= z1; ++k) {
     const bool last = k == z1;
-    // (a) publish D(k) of the own cell (prefetched) and of the halo ring
-    store_cell(D, me, nxt);
+    // (a) publish D(k) of the own cell and of the halo ring
+    build_cell<NC>(g, ps, pd, ms, xc, yc, k, true, true, !last, D, me);
     if (hs >= 0 && !last) build_cell<NC>(g, ps, pd, ms, hgx, hgy, k, hwx, hwy, true, D, hs);
     __syncthreads();
     // (b) z-face k-1/2 from registers (plane k-1) and shared memory (plane k)
@@ -363,8 +336,6 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
 #pragma unroll
         for (int i = 0; i < M; ++i) fxs[(i * MTY + lane) * (TX + 1) + TX] = Fe[i];
       }
-      // prefetch the own cell of the next plane (its loads overlap the barrier)
-      load_cell(g, ps, pd, ms, xc, yc, k + 1, k + 1 < z1, nxt);
     }
     __syncthreads();
     if (!last) {
