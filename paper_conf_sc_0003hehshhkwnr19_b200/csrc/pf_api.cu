@@ -93,7 +93,6 @@ struct pf_ctx {
   bool have_params = false, have_fields = false;
   int64_t step = 0, z_off = 0;
   int variant = PF_VARIANT_JIT;
-  int epi_dims = 0;  // leading dimensions whose ghosts the tuned sweeps write (fused BC)
   JitModule* jit = nullptr;  // specialised kernels for (dp, g); reset by pf_set_params
   ncclComm_t comm = nullptr;
   // profiling
@@ -105,10 +104,6 @@ struct pf_ctx {
   int64_t nlaunch[4] = {0, 0, 0, 0};  // kernels launched per category since pf_profile()
   std::string err;
 };
-
-static bool dim_exchanged(const pf_ctx* ctx, int d) {
-  return ctx->exchange[d] || (ctx->force_exchange && ctx->cfg.bc_lo[d] == PF_BC_PERIODIC);
-}
 
 namespace {
 
@@ -443,14 +438,6 @@ int pf_create(const pf_config* cfg, pf_ctx** out) {
     const char* fe = getenv("PF_FORCE_EXCHANGE");  // debug: periodic self-exchange through pack/unpack
     ctx->force_exchange = fe && fe[0] == '1';
   }
-  // the tuned sweeps fill the ghosts of the leading local dimensions in their
-  // epilogue; from the first exchanged dimension on, the ordered stages run
-  ctx->epi_dims = 3;
-  for (int d = 0; d < 3; ++d)
-    if (dim_exchanged(ctx, d)) {
-      ctx->epi_dims = d;
-      break;
-    }
   e = cudaMallocHost(&ctx->pinned, 64);
   if (e != cudaSuccess) {
     ctx->err = cudaGetErrorString(e);
@@ -553,10 +540,6 @@ int pf_set_params(pf_ctx* ctx, const pf_params* p) {
     return fail(ctx, PF_EINVAL, "dt = %g exceeds the explicit stability bound min(%g [phi], %g [mu])", p->dt, dt_phi,
                 dt_mu);
   pf::fill_dev_params(*p, L, &ctx->dp);
-  for (int d = 0; d < 3; ++d) {
-    ctx->dp.epi_lo[d] = d < ctx->epi_dims ? ctx->cfg.bc_lo[d] : -1;
-    ctx->dp.epi_hi[d] = d < ctx->epi_dims ? ctx->cfg.bc_hi[d] : -1;
-  }
   ctx->hp = *p;
   ctx->have_params = true;
   ctx->jit = nullptr;
@@ -566,20 +549,17 @@ int pf_set_params(pf_ctx* ctx, const pf_params* p) {
 // ---------------------------------------------------------------------------
 // ghost layers of one field set (Alg. 1 lines 2 / 4): local BCs + halo exchange
 // ---------------------------------------------------------------------------
-// first_dim > 0: dimensions before it were already filled by the sweep
-// epilogue (fused boundary handling)
-static int fill_ghosts(pf_ctx* ctx, double* f, int ncomp, bool is_mu, int first_dim = 0) {
+static int fill_ghosts(pf_ctx* ctx, double* f, int ncomp, bool is_mu) {
   const double* dir = is_mu ? ctx->hp.mu_inf : nullptr;
-  const bool any_ex = dim_exchanged(ctx, 0) || dim_exchanged(ctx, 1) || dim_exchanged(ctx, 2);
-  if (first_dim >= 3) return PF_OK;
-  if (!any_ex && first_dim == 0) {
+  const bool any_ex = ctx->exchange[0] || ctx->exchange[1] || ctx->exchange[2] || ctx->force_exchange;
+  if (!any_ex) {
     launch_ghost_fill(ctx->g, ctx->bc_all, f, ncomp, dir, ctx->stream);
     ctx->nlaunch[2] += 1;
     return check_launch(ctx, "ghost_fill");
   }
   // ordered x -> y -> z stages so that edge ghosts travel with the slabs
-  for (int d = first_dim; d < 3; ++d) {
-    const bool ex = dim_exchanged(ctx, d);
+  for (int d = 0; d < 3; ++d) {
+    const bool ex = ctx->exchange[d] || (ctx->force_exchange && ctx->cfg.bc_lo[d] == PF_BC_PERIODIC);
     if (!ex) {
       launch_ghost_stage(ctx->g, d, ctx->cfg.bc_lo[d], ctx->cfg.bc_hi[d], f, ncomp, dir, ctx->stream);
       ctx->nlaunch[2] += 1;
@@ -690,8 +670,7 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
   if (int r = check_launch(ctx, "phi_sweep")) return r;
   // line 2: phi_dst communication and boundary handling
   prof_begin(ctx, 2, &e0);
-  const int first = ctx->variant == PF_VARIANT_NAIVE ? 0 : ctx->epi_dims;
-  int r = fill_ghosts(ctx, pd, PF_N, false, first);
+  int r = fill_ghosts(ctx, pd, PF_N, false);
   prof_end(ctx, 2, e0);
   if (r) return r;
   if (phi_only) {
@@ -710,7 +689,7 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
     if (int r2 = check_launch(ctx, "mu_sweep")) return r2;
     // line 4
     prof_begin(ctx, 2, &e0);
-    r = fill_ghosts(ctx, md, PF_M, true, first);
+    r = fill_ghosts(ctx, md, PF_M, true);
     prof_end(ctx, 2, e0);
     if (r) return r;
   }
@@ -742,12 +721,8 @@ int pf_halo_exchange(pf_ctx* ctx, unsigned mask) {
   if (!ctx->have_params) return fail(ctx, PF_ESTATE, "pf_halo_exchange before pf_set_params");
   if (mask & PF_PHI)
     if (int r = fill_ghosts(ctx, ctx->phi[ctx->cur], PF_N, false)) return r;
-  if (mask & PF_MU) {
+  if (mask & PF_MU)
     if (int r = fill_ghosts(ctx, ctx->mu[ctx->cur], PF_M, true)) return r;
-    // the fused epilogue never writes Dirichlet ghosts: set them on the
-    // other time level too (its interior is stale; it is overwritten next step)
-    if (int r = fill_ghosts(ctx, ctx->mu[1 - ctx->cur], PF_M, true)) return r;
-  }
   return PF_OK;
 }
 

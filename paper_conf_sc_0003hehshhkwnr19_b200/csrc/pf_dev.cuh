@@ -61,10 +61,6 @@ struct DevParams {
   double dcT[N][5];     // dc_a/dT = -(A1 + A1^T) mu - B1: [s00, s01, s11, -B1_0, -B1_1]
   int liquid;
   int TA;               // A1 != 0: chi and the mobility depend on T
-  // ghost images written by the sweep epilogues (fused "boundary handling",
-  // Alg. 1 lines 2 and 4): BC kind per side (0 periodic, 1 Neumann,
-  // 2 Dirichlet-mu), -1 = filled by a halo exchange / separate kernel
-  int epi_lo[3], epi_hi[3];
 };
 
 }  // namespace pf

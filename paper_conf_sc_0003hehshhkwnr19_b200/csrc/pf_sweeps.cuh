@@ -124,7 +124,6 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, 
     if (active) {
 #pragma unroll
       for (int a = 0; a < N; ++a) pd[a * F + c] = out[a];
-      store_ghost_images<N>(P, g, pd, x, y, z, out, false);
     }
 #pragma unroll
     for (int a = 0; a < N; ++a) {
@@ -300,7 +299,6 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
       const i64 c = g.at(xc, yc, k - 1);
       md[c] = out[0];
       md[F + c] = out[1];
-      store_ghost_images<M>(P, g, md, x, y, k - 1, out, true);
     }
     Fzm[0] = Fz[0];
     Fzm[1] = Fz[1];
