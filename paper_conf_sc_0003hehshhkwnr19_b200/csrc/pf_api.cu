@@ -248,7 +248,7 @@ void fill_dev_params(const pf_params& pr, int L, DevParams* out) {
   D.inv_eps = 1.0 / p->eps;
   D.dt_over_eps = p->dt / p->eps;
   const double pi = 3.14159265358979323846;
-  D.at_c = p->dx * pi * p->eps / (8.0 * p->dt);
+  D.at_c = 4.0 * p->dx * pi * p->eps / (8.0 * p->dt);  // x 4: gradients scaled by 4 in mu_face
   D.dTdt = -p->G * p->v;
   D.Tdz = p->G * p->dx;
   D.mu_inf[0] = p->mu_inf[0];
@@ -302,8 +302,9 @@ void fill_dev_params(const pf_params& pr, int L, DevParams* out) {
     const double X1[2][2] = {{D.chi1[a][0], D.chi1[a][1]}, {D.chi1[a][1], D.chi1[a][2]}};
     for (int i = 0; i < 2; ++i)
       for (int j = 0; j < 2; ++j) {
-        D.P0[a][2 * i + j] = p->D[a][i][0] * X0[0][j] + p->D[a][i][1] * X0[1][j];
-        D.P1[a][2 * i + j] = p->D[a][i][0] * X1[0][j] + p->D[a][i][1] * X1[1][j];
+        // x 1/2: the mu face uses face sums, not means
+        D.P0[a][2 * i + j] = 0.5 * (p->D[a][i][0] * X0[0][j] + p->D[a][i][1] * X0[1][j]);
+        D.P1[a][2 * i + j] = 0.5 * (p->D[a][i][0] * X1[0][j] + p->D[a][i][1] * X1[1][j]);
       }
     D.dcT[a][0] = D.chi1[a][0];
     D.dcT[a][1] = D.chi1[a][1];
@@ -314,8 +315,8 @@ void fill_dev_params(const pf_params& pr, int L, DevParams* out) {
   for (int s = 0; s < PF_N - 1; ++s) {
     const int a = s < L ? s : s + 1;
     for (int i = 0; i < 3; ++i) {
-      D.dchi0[s][i] = D.chi0[L][i] - D.chi0[a][i];
-      D.dchi1[s][i] = D.chi1[L][i] - D.chi1[a][i];
+      D.dchi0[s][i] = 0.5 * (D.chi0[L][i] - D.chi0[a][i]);  // x 1/2: face sums of mu
+      D.dchi1[s][i] = 0.5 * (D.chi1[L][i] - D.chi1[a][i]);
     }
     for (int i = 0; i < 2; ++i) {
       D.dB0[s][i] = p->B0[L][i] - p->B0[a][i];

@@ -40,7 +40,7 @@ struct DevParams {
   double phi_grad_c;    // eps / dx^2
   double inv_eps;
   double dt_over_eps;
-  double at_c;          // dx * pi eps / (8 dt): anti-trapping prefactor in unscaled units
+  double at_c;          // 4 dx pi eps / (8 dt): anti-trapping prefactor in the units of mu_face
   double dTdt;          // -G v
   double Tbase, Tdz;    // T(local plane k) = Tbase + Tdz k; Tbase is set per step  [A13]
   double mu_inf[M];
@@ -55,8 +55,8 @@ struct DevParams {
   double C0[N], C1[N];
   // mu-sweep
   double chi0[N][3], chi1[N][3];   // chi_a = dc_a/dmu = -(A + A^T) (sym: 00, 01, 11)  [A6]
-  double P0[N][4], P1[N][4];       // D_a chi_a (row-major 00 01 10 11), eq. 9  [A7]
-  double dchi0[NSOL][3], dchi1[NSOL][3];  // chi_l - chi_s
+  double P0[N][4], P1[N][4];       // D_a chi_a / 2 (row-major 00 01 10 11), eq. 9 [A7]; /2: face sums
+  double dchi0[NSOL][3], dchi1[NSOL][3];  // (chi_l - chi_s) / 2 (face sums of mu)
   double dB0[NSOL][M], dB1[NSOL][M];      // B_l - B_s
   double dcT[N][5];     // dc_a/dT = -(A1 + A1^T) mu - B1: [s00, s01, s11, -B1_0, -B1_1]
   int liquid;
