@@ -62,34 +62,23 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, 
   const bool extra = (w == 0 && lane < TY) || w == 1;
 
   i64 c = g.at(xc, yc, z0);
-  double pm[N], p0[N], Fzm[N], pn[N];
+  double pm[N], p0[N], Fzm[N];
 #pragma unroll
   for (int a = 0; a < N; ++a) {
     pm[a] = __ldg(ps + a * F + c - SZ);
     p0[a] = __ldg(ps + a * F + c);
-    pn[a] = __ldg(ps + a * F + c + SZ);
   }
-  double mn0 = __ldg(ms + c), mn1 = __ldg(ms + F + c);
   phi_face(P, pm, p0, Fzm);
 
   for (int z = z0; z < z1; ++z, c += SZ, ep += SZ, eq += SZ) {
     const int buf = z & 1;
     double pp[N], Fxm[N], Fym[N], Fzp[N], gd[N][3];
-    // own column of the next plane and mu were prefetched one plane ahead;
-    // issue the loads of plane z+2 (<= nz+1, inside the guard ring) now
-    const double mu0 = mn0, mu1 = mn1;
-    mn0 = __ldg(ms + c + SZ);
-    mn1 = __ldg(ms + F + c + SZ);
-#pragma unroll
-    for (int a = 0; a < N; ++a) {
-      pp[a] = pn[a];
-      pn[a] = __ldg(ps + a * F + c + 2 * SZ);
-    }
     {
       double xm[N], xp[N], ym[N], yp[N];
 #pragma unroll
       for (int a = 0; a < N; ++a) {
         const double* f = ps + a * F + c;
+        pp[a] = __ldg(f + SZ);
         xm[a] = __ldg(f - 1);
         xp[a] = __ldg(f + 1);
         ym[a] = __ldg(f - SY);
@@ -120,6 +109,7 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, 
     }
 #pragma unroll
     for (int a = 0; a < N; ++a) fy[buf][a][w][lane] = Fym[a];
+    const double mu0 = __ldg(ms + c), mu1 = __ldg(ms + F + c);
     __syncthreads();
     double divh[N];
 #pragma unroll
