@@ -210,7 +210,15 @@ __global__ void k_ghost(GhostArgs A, double* __restrict__ f) {
   if (skip) return;
   const int64_t dst = g.at(x, y, z);
   const int64_t src = g.at(mx, my, mz);
-  for (int c = 0; c < A.ncomp; ++c) f[c * g.field + dst] = (dir && A.use_dir) ? A.dir[c] : f[c * g.field + src];
+  // all loads first (the source and destination share the array, so a
+  // load-store loop would serialise on the possible alias)
+  double v[N];
+#pragma unroll
+  for (int c = 0; c < N; ++c)
+    if (c < A.ncomp) v[c] = (dir && A.use_dir) ? A.dir[c < M ? c : 0] : __ldg(f + c * g.field + src);
+#pragma unroll
+  for (int c = 0; c < N; ++c)
+    if (c < A.ncomp) f[c * g.field + dst] = v[c];
 }
 
 void launch_ghost_fill(const Geom& g, const BCSpec& bc, double* f, int ncomp, const double* dirichlet, cudaStream_t s) {
@@ -372,12 +380,18 @@ __global__ void k_pack(Geom g, int d, int idx, int ncomp, double* __restrict__ f
     c[d == 0 ? 1 : 0] = i0;
     c[d == 2 ? 1 : 2] = i1;
     const int64_t li = g.at(c[0], c[1], c[2]);
-    for (int a = 0; a < ncomp; ++a) {
-      if (unpack)
-        f[a * g.field + li] = buf[a * tot + i];
-      else
-        buf[a * tot + i] = f[a * g.field + li];
-    }
+    double v[N];
+#pragma unroll
+    for (int a = 0; a < N; ++a)
+      if (a < ncomp) v[a] = unpack ? buf[a * tot + i] : f[a * g.field + li];
+#pragma unroll
+    for (int a = 0; a < N; ++a)
+      if (a < ncomp) {
+        if (unpack)
+          f[a * g.field + li] = v[a];
+        else
+          buf[a * tot + i] = v[a];
+      }
   }
 }
 
@@ -409,7 +423,13 @@ __global__ void k_ghost_stage(Geom g, int d, int klo, int khi, int ncomp, double
     const bool dirich = kind == PF_BC_DIRICHLET_MU && use_dir;
     const int64_t li = g.at(c[0], c[1], c[2]);
     const int64_t si = g.at(s[0], s[1], s[2]);
-    for (int a = 0; a < ncomp; ++a) f[a * g.field + li] = dirich ? (a == 0 ? dir0 : dir1) : f[a * g.field + si];
+    double v[N];
+#pragma unroll
+    for (int a = 0; a < N; ++a)
+      if (a < ncomp) v[a] = dirich ? (a == 0 ? dir0 : dir1) : __ldg(f + a * g.field + si);
+#pragma unroll
+    for (int a = 0; a < N; ++a)
+      if (a < ncomp) f[a * g.field + li] = v[a];
   }
 }
 
