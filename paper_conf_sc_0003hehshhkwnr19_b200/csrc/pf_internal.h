@@ -27,7 +27,8 @@ void launch_mu_tuned(const DevParams& P, const Geom& g, const double* ps, const 
 // launch geometry of the tuned kernels (shared with the specialised build)
 dim3 tuned_block();
 dim3 tuned_block_mu(int mty);
-dim3 tuned_grid_phi(const Geom& g);
+dim3 tuned_grid_phi(const Geom& g, int pty);
+dim3 tuned_block_phi(int pty);
 dim3 tuned_grid_mu(const Geom& g, int mty);
 size_t tuned_mu_smem(int mty);  // mty: tile height of the mu-sweep (2, 4, 8)
 int tuned_mu_ty_default();

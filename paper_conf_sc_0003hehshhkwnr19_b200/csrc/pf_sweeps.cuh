@@ -32,15 +32,15 @@ constexpr int MU_TY = PF_MU_TY;
 // ===========================================================================
 // phi-sweep (Algorithm 1 line 1): D3C7 of phi_src, D3C1 of mu_src.
 // ===========================================================================
-template <class PT, class GT, int L, bool TA>
+template <class PT, class GT, int L, bool TA, int PTY = TY>
 __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, const GT& g,
                                                const double* __restrict__ ps, const double* __restrict__ ms,
                                                double* __restrict__ pd) {
-  __shared__ double fy[2][N][TY][TX];  // -y face flux of every thread, by plane parity
-  __shared__ double ex[2][N][TY];      // +x flux on the right tile edge
+  __shared__ double fy[2][N][PTY][TX];  // -y face flux of every thread, by plane parity
+  __shared__ double ex[2][N][PTY];      // +x flux on the right tile edge
   __shared__ double ey[2][N][TX];      // +y flux on the top tile edge
   const int lane = threadIdx.x, w = threadIdx.y;
-  const int x0 = blockIdx.x * TX, y0 = blockIdx.y * TY;
+  const int x0 = blockIdx.x * TX, y0 = blockIdx.y * PTY;
   const int x = x0 + lane, y = y0 + w;
   const bool active = x < g.nx && y < g.ny;
   // ragged tiles: clamp to the ghost cell, whose -x / -y face is the +x / +y
@@ -48,18 +48,18 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, 
   const int xc = min(x, g.nx), yc = min(y, g.ny);
   const int z0 = blockIdx.z * ZC_PHI, z1 = min(z0 + ZC_PHI, g.nz);
   const i64 F = g.field, SY = g.pitch, SZ = g.plane;
-  // extra faces: warp 0 lanes < TY: +x face of row `lane`; warp 1: +y face of column `lane`
+  // extra faces: warp 0 lanes < PTY: +x face of row `lane`; warp 1: +y face of column `lane`
   i64 ep = 0, eq = 0;  // the two cells of the extra face, at plane z0
-  if (w == 0 && lane < TY) {
+  if (w == 0 && lane < PTY) {
     const int ry = min(y0 + lane, g.ny);
     ep = g.at(min(x0 + TX - 1, g.nx), ry, z0);
     eq = g.at(min(x0 + TX, g.nx), ry, z0);
   } else if (w == 1) {
     const int cx = min(x0 + lane, g.nx);
-    ep = g.at(cx, min(y0 + TY - 1, g.ny), z0);
-    eq = g.at(cx, min(y0 + TY, g.ny), z0);
+    ep = g.at(cx, min(y0 + PTY - 1, g.ny), z0);
+    eq = g.at(cx, min(y0 + PTY, g.ny), z0);
   }
-  const bool extra = (w == 0 && lane < TY) || w == 1;
+  const bool extra = (w == 0 && lane < PTY) || w == 1;
 
   i64 c = g.at(xc, yc, z0);
   double pm[N], p0[N], Fzm[N];
@@ -116,7 +116,7 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, 
     for (int a = 0; a < N; ++a) {
       double fxp = __shfl_down_sync(0xffffffffu, Fxm[a], 1);
       if (lane == TX - 1) fxp = ex[buf][a][w];
-      const double fyp = (w < TY - 1) ? fy[buf][a][w + 1][lane] : ey[buf][a][lane];
+      const double fyp = (w < PTY - 1) ? fy[buf][a][w + 1][lane] : ey[buf][a][lane];
       divh[a] = ((fxp - Fxm[a]) + (fyp - Fym[a])) + (Fzp[a] - Fzm[a]);
     }
     double out[N];

@@ -40,8 +40,11 @@ __global__ void __launch_bounds__(TX* MU_TY, 16 / MU_TY) k_mu_tuned(DevParams P,
 }
 
 dim3 tuned_block() { return dim3(TX, TY); }
+dim3 tuned_block_phi(int pty) { return dim3(TX, pty); }
 dim3 tuned_block_mu(int mty) { return dim3(TX, mty); }
-dim3 tuned_grid_phi(const Geom& g) { return dim3((g.nx + TX - 1) / TX, (g.ny + TY - 1) / TY, (g.nz + ZC_PHI - 1) / ZC_PHI); }
+dim3 tuned_grid_phi(const Geom& g, int pty) {
+  return dim3((g.nx + TX - 1) / TX, (g.ny + pty - 1) / pty, (g.nz + ZC_PHI - 1) / ZC_PHI);
+}
 dim3 tuned_grid_mu(const Geom& g, int mty) {
   return dim3((g.nx + TX - 1) / TX, (g.ny + mty - 1) / mty, (g.nz + ZC_MU - 1) / ZC_MU);
 }
@@ -55,7 +58,7 @@ size_t tuned_phi_smem() { return 0; }  // static shared memory only
 template <int L, bool TA>
 static void phi_launch(const DevParams& P, const Geom& g, const double* ps, const double* ms, double* pd,
                        cudaStream_t s) {
-  k_phi_tuned<L, TA><<<tuned_grid_phi(g), tuned_block(), 0, s>>>(P, g, ps, ms, pd);
+  k_phi_tuned<L, TA><<<tuned_grid_phi(g, TY), tuned_block(), 0, s>>>(P, g, ps, ms, pd);
 }
 
 void launch_phi_tuned(const DevParams& P, const Geom& g, const double* ps, const double* ms, double* pd,
