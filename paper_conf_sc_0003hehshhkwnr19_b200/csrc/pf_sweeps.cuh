@@ -20,6 +20,21 @@
 
 namespace pf {
 
+// software prefetch distance (planes) into L2 / L1 of the z-marching sweeps:
+// PF_PREFETCH 0 = off, 1 = L2, 2 = L1
+#ifndef PF_PREFETCH
+#define PF_PREFETCH 0
+#endif
+__device__ __forceinline__ void prefetch_line(const void* p) {
+#if PF_PREFETCH == 1
+  asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
+#elif PF_PREFETCH == 2
+  asm volatile("prefetch.global.L1 [%0];" ::"l"(p));
+#else
+  (void)p;
+#endif
+}
+
 constexpr int TX = 32;
 constexpr int TY = 8;
 constexpr int ZC_PHI = 32;  // z-chunk per CTA
@@ -72,6 +87,12 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, 
 
   for (int z = z0; z < z1; ++z, c += SZ, ep += SZ, eq += SZ) {
     const int buf = z & 1;
+    if (PF_PREFETCH && z + 3 <= z1 + 1) {  // own column two planes ahead (<= nz + 1: guard ring)
+#pragma unroll
+      for (int a = 0; a < N; ++a) prefetch_line(ps + a * F + c + 2 * SZ);
+      prefetch_line(ms + c + 2 * SZ);
+      prefetch_line(ms + F + c + 2 * SZ);
+    }
     double pp[N], Fxm[N], Fym[N], Fzp[N], gd[N][3];
     {
       double xm[N], xp[N], ym[N], yp[N];
@@ -277,6 +298,16 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
 
   for (int k = z0; k <= z1; ++k) {
     const bool last = k == z1;
+    if (PF_PREFETCH && !last) {  // own cell's lines of the next planes
+      const i64 cp = g.at(xc, yc, k);
+#pragma unroll
+      for (int a = 0; a < N; ++a) {
+        prefetch_line(ps + a * F + cp + 2 * g.plane);
+        prefetch_line(pd + a * F + cp + g.plane);
+      }
+      prefetch_line(ms + cp + g.plane);
+      prefetch_line(ms + F + cp + g.plane);
+    }
     // (a) publish D(k) of the own cell and of the halo ring
     build_cell<NC>(g, ps, pd, ms, xc, yc, k, true, true, !last, D, me);
     if (hs >= 0 && !last) build_cell<NC>(g, ps, pd, ms, hgx, hgy, k, hwx, hwy, true, D, hs);
