@@ -23,7 +23,10 @@ namespace pf {
 // software prefetch distance (planes) into L2 / L1 of the z-marching sweeps:
 // PF_PREFETCH 0 = off, 1 = L2, 2 = L1
 #ifndef PF_PREFETCH
-#define PF_PREFETCH 0
+#define PF_PREFETCH 1
+#endif
+#ifndef PF_PREFETCH_D
+#define PF_PREFETCH_D 2  // planes ahead
 #endif
 __device__ __forceinline__ void prefetch_line(const void* p) {
 #if PF_PREFETCH == 1
@@ -87,11 +90,11 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, 
 
   for (int z = z0; z < z1; ++z, c += SZ, ep += SZ, eq += SZ) {
     const int buf = z & 1;
-    if (PF_PREFETCH && z + 3 <= z1 + 1) {  // own column two planes ahead (<= nz + 1: guard ring)
+    if (PF_PREFETCH && z + PF_PREFETCH_D <= z1 + 1) {  // own column ahead (<= nz + 1: guard ring)
 #pragma unroll
-      for (int a = 0; a < N; ++a) prefetch_line(ps + a * F + c + 2 * SZ);
-      prefetch_line(ms + c + 2 * SZ);
-      prefetch_line(ms + F + c + 2 * SZ);
+      for (int a = 0; a < N; ++a) prefetch_line(ps + a * F + c + PF_PREFETCH_D * SZ);
+      prefetch_line(ms + c + PF_PREFETCH_D * SZ);
+      prefetch_line(ms + F + c + PF_PREFETCH_D * SZ);
     }
     double pp[N], Fxm[N], Fym[N], Fzp[N], gd[N][3];
     {
@@ -298,15 +301,15 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
 
   for (int k = z0; k <= z1; ++k) {
     const bool last = k == z1;
-    if (PF_PREFETCH && !last) {  // own cell's lines of the next planes
+    if (PF_PREFETCH && k + PF_PREFETCH_D <= z1 + 1) {  // own cell's lines of the next planes
       const i64 cp = g.at(xc, yc, k);
 #pragma unroll
       for (int a = 0; a < N; ++a) {
-        prefetch_line(ps + a * F + cp + 2 * g.plane);
-        prefetch_line(pd + a * F + cp + g.plane);
+        prefetch_line(ps + a * F + cp + PF_PREFETCH_D * g.plane);
+        prefetch_line(pd + a * F + cp + (PF_PREFETCH_D - 1) * g.plane);
       }
-      prefetch_line(ms + cp + g.plane);
-      prefetch_line(ms + F + cp + g.plane);
+      prefetch_line(ms + cp + (PF_PREFETCH_D - 1) * g.plane);
+      prefetch_line(ms + F + cp + (PF_PREFETCH_D - 1) * g.plane);
     }
     // (a) publish D(k) of the own cell and of the halo ring
     build_cell<NC>(g, ps, pd, ms, xc, yc, k, true, true, !last, D, me);
