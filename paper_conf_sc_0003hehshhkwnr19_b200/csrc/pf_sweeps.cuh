@@ -310,15 +310,6 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
       }
       prefetch_line(ms + cp + (PF_PREFETCH_D - 1) * g.plane);
       prefetch_line(ms + F + cp + (PF_PREFETCH_D - 1) * g.plane);
-      if (hs >= 0) {  // and the halo cell this thread builds
-        const i64 ch = g.at(hgx, hgy, k);
-#pragma unroll
-        for (int a = 0; a < N; ++a) {
-          prefetch_line(ps + a * F + ch + PF_PREFETCH_D * g.plane);
-          prefetch_line(pd + a * F + ch + (PF_PREFETCH_D - 1) * g.plane);
-        }
-        prefetch_line(ms + ch + (PF_PREFETCH_D - 1) * g.plane);
-      }
     }
     // (a) publish D(k) of the own cell and of the halo ring
     build_cell<NC>(g, ps, pd, ms, xc, yc, k, true, true, !last, D, me);
