@@ -93,6 +93,12 @@ struct pf_ctx {
   bool have_params = false, have_fields = false;
   int64_t step = 0, z_off = 0;
   int variant = PF_VARIANT_JIT;
+  // overlap of the halo exchange with interior work
+  int first_ex = 3;                 // first exchanged dimension (3 = none)
+  cudaStream_t comm_s = nullptr;    // exchange stream
+  cudaEvent_t ev_phi = nullptr, ev_phix = nullptr, ev_mu = nullptr, ev_mux = nullptr;
+  bool mux_pending = false;         // mu exchange in flight on comm_s
+  bool overlap = true;
   JitModule* jit = nullptr;  // specialised kernels for (dp, g); reset by pf_set_params
   ncclComm_t comm = nullptr;
   // profiling
@@ -439,6 +445,25 @@ int pf_create(const pf_config* cfg, pf_ctx** out) {
     const char* fe = getenv("PF_FORCE_EXCHANGE");  // debug: periodic self-exchange through pack/unpack
     ctx->force_exchange = fe && fe[0] == '1';
   }
+  ctx->first_ex = 3;
+  for (int d = 0; d < 3; ++d)
+    if (ctx->exchange[d] || (ctx->force_exchange && cfg->bc_lo[d] == PF_BC_PERIODIC)) {
+      ctx->first_ex = d;
+      break;
+    }
+  if (ctx->first_ex < 3) {
+    const char* ov = getenv("PF_OVERLAP");
+    ctx->overlap = !(ov && ov[0] == '0');
+    e = cudaStreamCreateWithFlags(&ctx->comm_s, cudaStreamNonBlocking);
+    cudaEvent_t* evs[4] = {&ctx->ev_phi, &ctx->ev_phix, &ctx->ev_mu, &ctx->ev_mux};
+    for (cudaEvent_t* ev : evs)
+      if (e == cudaSuccess) e = cudaEventCreateWithFlags(ev, cudaEventDisableTiming);
+    if (e != cudaSuccess) {
+      ctx->err = cudaGetErrorString(e);
+      *out = ctx;
+      return PF_ECUDA;
+    }
+  }
   e = cudaMallocHost(&ctx->pinned, 64);
   if (e != cudaSuccess) {
     ctx->err = cudaGetErrorString(e);
@@ -458,6 +483,12 @@ int pf_destroy(pf_ctx* ctx) {
     cudaEventDestroy(o.second.second);
   }
   if (ctx->comm) g_nccl.CommDestroy(ctx->comm);
+  if (ctx->comm_s) {
+    cudaStreamSynchronize(ctx->comm_s);
+    cudaStreamDestroy(ctx->comm_s);
+  }
+  for (cudaEvent_t ev : {ctx->ev_phi, ctx->ev_phix, ctx->ev_mu, ctx->ev_mux})
+    if (ev) cudaEventDestroy(ev);
   if (ctx->pinned) cudaFreeHost(ctx->pinned);
   delete ctx;
   return PF_OK;
@@ -550,19 +581,20 @@ int pf_set_params(pf_ctx* ctx, const pf_params* p) {
 // ---------------------------------------------------------------------------
 // ghost layers of one field set (Alg. 1 lines 2 / 4): local BCs + halo exchange
 // ---------------------------------------------------------------------------
-static int fill_ghosts(pf_ctx* ctx, double* f, int ncomp, bool is_mu) {
+// dimensions [d0, d1) of the ordered x -> y -> z ghost fill, on stream `st`
+static int fill_ghost_dims(pf_ctx* ctx, double* f, int ncomp, bool is_mu, int d0, int d1, cudaStream_t st) {
   const double* dir = is_mu ? ctx->hp.mu_inf : nullptr;
-  const bool any_ex = ctx->exchange[0] || ctx->exchange[1] || ctx->exchange[2] || ctx->force_exchange;
-  if (!any_ex) {
-    launch_ghost_fill(ctx->g, ctx->bc_all, f, ncomp, dir, ctx->stream);
+  const bool any_ex = ctx->first_ex < 3;
+  if (!any_ex && d0 == 0 && d1 == 3) {
+    launch_ghost_fill(ctx->g, ctx->bc_all, f, ncomp, dir, st);
     ctx->nlaunch[2] += 1;
     return check_launch(ctx, "ghost_fill");
   }
   // ordered x -> y -> z stages so that edge ghosts travel with the slabs
-  for (int d = 0; d < 3; ++d) {
+  for (int d = d0; d < d1; ++d) {
     const bool ex = ctx->exchange[d] || (ctx->force_exchange && ctx->cfg.bc_lo[d] == PF_BC_PERIODIC);
     if (!ex) {
-      launch_ghost_stage(ctx->g, d, ctx->cfg.bc_lo[d], ctx->cfg.bc_hi[d], f, ncomp, dir, ctx->stream);
+      launch_ghost_stage(ctx->g, d, ctx->cfg.bc_lo[d], ctx->cfg.bc_hi[d], f, ncomp, dir, st);
       ctx->nlaunch[2] += 1;
       if (int r = check_launch(ctx, "ghost_stage")) return r;
       continue;
@@ -571,38 +603,52 @@ static int fill_ghosts(pf_ctx* ctx, double* f, int ncomp, bool is_mu) {
     const size_t cnt = halo_slab_elems(ctx->g, d) * ncomp;
     const int lo = ctx->nb_lo[d] >= 0 ? ctx->nb_lo[d] : -1;
     const int hi = ctx->nb_hi[d] >= 0 ? ctx->nb_hi[d] : -1;
-    if (hi >= 0) launch_pack(ctx->g, d, n - 1, ncomp, f, ctx->sendbuf[d][1], ctx->stream);
-    if (lo >= 0) launch_pack(ctx->g, d, 0, ncomp, f, ctx->sendbuf[d][0], ctx->stream);
+    if (hi >= 0) launch_pack(ctx->g, d, n - 1, ncomp, f, ctx->sendbuf[d][1], st);
+    if (lo >= 0) launch_pack(ctx->g, d, 0, ncomp, f, ctx->sendbuf[d][0], st);
     ctx->nlaunch[2] += (hi >= 0) + (lo >= 0);
     if (int r = check_launch(ctx, "pack")) return r;
     if (ctx->comm) {
       // per peer pair the k-th send matches the k-th recv: send (hi, lo), recv (lo, hi)
       NC(g_nccl.GroupStart());
-      if (hi >= 0) NC(g_nccl.Send(ctx->sendbuf[d][1], cnt, ncclDouble, hi, ctx->comm, ctx->stream));
-      if (lo >= 0) NC(g_nccl.Send(ctx->sendbuf[d][0], cnt, ncclDouble, lo, ctx->comm, ctx->stream));
-      if (lo >= 0) NC(g_nccl.Recv(ctx->recvbuf[d][0], cnt, ncclDouble, lo, ctx->comm, ctx->stream));
-      if (hi >= 0) NC(g_nccl.Recv(ctx->recvbuf[d][1], cnt, ncclDouble, hi, ctx->comm, ctx->stream));
+      if (hi >= 0) NC(g_nccl.Send(ctx->sendbuf[d][1], cnt, ncclDouble, hi, ctx->comm, st));
+      if (lo >= 0) NC(g_nccl.Send(ctx->sendbuf[d][0], cnt, ncclDouble, lo, ctx->comm, st));
+      if (lo >= 0) NC(g_nccl.Recv(ctx->recvbuf[d][0], cnt, ncclDouble, lo, ctx->comm, st));
+      if (hi >= 0) NC(g_nccl.Recv(ctx->recvbuf[d][1], cnt, ncclDouble, hi, ctx->comm, st));
       NC(g_nccl.GroupEnd());
     } else {
       // world == 1, periodic self-exchange through the same pack/unpack path
       CU(cudaMemcpyAsync(ctx->recvbuf[d][0], ctx->sendbuf[d][1], cnt * sizeof(double), cudaMemcpyDeviceToDevice,
-                         ctx->stream));
+                         st));
       CU(cudaMemcpyAsync(ctx->recvbuf[d][1], ctx->sendbuf[d][0], cnt * sizeof(double), cudaMemcpyDeviceToDevice,
-                         ctx->stream));
+                         st));
     }
-    if (lo >= 0) launch_unpack(ctx->g, d, -1, ncomp, f, ctx->recvbuf[d][0], ctx->stream);
-    if (hi >= 0) launch_unpack(ctx->g, d, n, ncomp, f, ctx->recvbuf[d][1], ctx->stream);
+    if (lo >= 0) launch_unpack(ctx->g, d, -1, ncomp, f, ctx->recvbuf[d][0], st);
+    if (hi >= 0) launch_unpack(ctx->g, d, n, ncomp, f, ctx->recvbuf[d][1], st);
     ctx->nlaunch[2] += (hi >= 0) + (lo >= 0);
     if (int r = check_launch(ctx, "unpack")) return r;
     if (lo < 0 || hi < 0) {  // physical boundary on one side of an exchanged dimension
       launch_ghost_stage(ctx->g, d, lo < 0 ? ctx->cfg.bc_lo[d] : -1, hi < 0 ? ctx->cfg.bc_hi[d] : -1, f, ncomp, dir,
-                         ctx->stream);
+                         st);
       ctx->nlaunch[2] += 1;
       if (int r = check_launch(ctx, "ghost_stage")) return r;
     }
   }
   return PF_OK;
 }
+
+static int fill_ghosts(pf_ctx* ctx, double* f, int ncomp, bool is_mu) {
+  return fill_ghost_dims(ctx, f, ncomp, is_mu, 0, 3, ctx->stream);
+}
+
+// make the compute stream wait for an exchange still in flight on comm_s
+static int join_comm(pf_ctx* ctx) {
+  if (ctx->mux_pending) {
+    CU(cudaStreamWaitEvent(ctx->stream, ctx->ev_mux, 0));
+    ctx->mux_pending = false;
+  }
+  return PF_OK;
+}
+
 
 // ---------------------------------------------------------------------------
 static cudaEvent_t ev_get(pf_ctx* ctx) {
@@ -643,6 +689,18 @@ static void prof_end(pf_ctx* ctx, int k, cudaEvent_t a) {
 static int window_maybe(pf_ctx* ctx);
 static int front_height_impl(pf_ctx* ctx, int* H);
 
+static int launch_mu(pf_ctx* ctx, const TileSel* ts, dim3 grid, const double* ps, const double* pd,
+                     const double* ms, double* md) {
+  if (ctx->variant == PF_VARIANT_NAIVE)
+    launch_mu_naive(ctx->dp, ctx->g, ps, pd, ms, md, ctx->stream);
+  else if (ctx->variant == PF_VARIANT_JIT)
+    CU(jit_launch_mu(ctx->jit, ctx->dp, ts, grid, ps, pd, ms, md, ctx->stream));
+  else
+    launch_mu_tuned(ctx->dp, ctx->g, ts, grid, ps, pd, ms, md, ctx->stream);
+  ctx->nlaunch[1] += 1;
+  return check_launch(ctx, "mu_sweep");
+}
+
 static int step_impl(pf_ctx* ctx, bool phi_only) {
   const Geom& g = ctx->g;
   double* ps = ctx->phi[ctx->cur];
@@ -653,13 +711,16 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
   const double t = (double)ctx->step * ctx->hp.dt;
   ctx->dp.Tbase = ctx->hp.T0 + ctx->hp.G * (((double)g.z0 + (double)ctx->z_off) * ctx->hp.dx - ctx->hp.v * t);
   cudaEvent_t e0 = nullptr;
-  // Algorithm 1, line 1: phi-sweep
-  prof_begin(ctx, 0, &e0);
   if (ctx->variant == PF_VARIANT_JIT && !ctx->jit) {
     std::string err;
     ctx->jit = jit_get(ctx->dp, g, &err);
     if (!ctx->jit) return fail(ctx, PF_ECUDA, "run-time specialisation failed: %s", err.c_str());
   }
+  // overlap: the exchanged dimensions' ghosts travel on the
+  // comm stream while the mu-sweep updates the tiles that do not read them
+  const bool ov = ctx->overlap && ctx->first_ex < 3 && ctx->variant != PF_VARIANT_NAIVE && !phi_only;
+  // Algorithm 1, line 1: phi-sweep (reads no mu ghosts: may overlap the previous mu exchange)
+  prof_begin(ctx, 0, &e0);
   if (ctx->variant == PF_VARIANT_NAIVE)
     launch_phi_naive(ctx->dp, g, ps, ms, pd, ctx->stream);
   else if (ctx->variant == PF_VARIANT_JIT)
@@ -669,30 +730,67 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
   ctx->nlaunch[0] += 1;
   prof_end(ctx, 0, e0);
   if (int r = check_launch(ctx, "phi_sweep")) return r;
-  // line 2: phi_dst communication and boundary handling
-  prof_begin(ctx, 2, &e0);
-  int r = fill_ghosts(ctx, pd, PF_N, false);
-  prof_end(ctx, 2, e0);
-  if (r) return r;
-  if (phi_only) {
-    CU(cudaMemcpyAsync(md, ms, ctx->lay.mu_bytes - 256, cudaMemcpyDeviceToDevice, ctx->stream));
-  } else {
-    // line 3: mu-sweep
-    prof_begin(ctx, 1, &e0);
-    if (ctx->variant == PF_VARIANT_NAIVE)
-      launch_mu_naive(ctx->dp, g, ps, pd, ms, md, ctx->stream);
-    else if (ctx->variant == PF_VARIANT_JIT)
-      CU(jit_launch_mu(ctx->jit, ctx->dp, ps, pd, ms, md, ctx->stream));
-    else
-      launch_mu_tuned(ctx->dp, g, ps, pd, ms, md, ctx->stream);
-    ctx->nlaunch[1] += 1;
-    prof_end(ctx, 1, e0);
-    if (int r2 = check_launch(ctx, "mu_sweep")) return r2;
-    // line 4
+  if (!ov) {
+    if (int r = join_comm(ctx)) return r;
+    // line 2: phi_dst communication and boundary handling
     prof_begin(ctx, 2, &e0);
-    r = fill_ghosts(ctx, md, PF_M, true);
+    int r = fill_ghosts(ctx, pd, PF_N, false);
     prof_end(ctx, 2, e0);
     if (r) return r;
+    if (phi_only) {
+      CU(cudaMemcpyAsync(md, ms, ctx->lay.mu_bytes - 256, cudaMemcpyDeviceToDevice, ctx->stream));
+    } else {
+      // line 3: mu-sweep
+      prof_begin(ctx, 1, &e0);
+      if (int r2 = launch_mu(ctx, nullptr, dim3(), ps, pd, ms, md)) return r2;
+      prof_end(ctx, 1, e0);
+      // line 4
+      prof_begin(ctx, 2, &e0);
+      r = fill_ghosts(ctx, md, PF_M, true);
+      prof_end(ctx, 2, e0);
+      if (r) return r;
+    }
+  } else {
+    // line 2: local dimensions before the first exchanged one on the compute
+    // stream, the rest (exchanges in x -> y -> z order) on the comm stream
+    const int fe = ctx->first_ex;
+    if (int r = fill_ghost_dims(ctx, pd, PF_N, false, 0, fe, ctx->stream)) return r;
+    CU(cudaEventRecord(ctx->ev_phi, ctx->stream));
+    CU(cudaStreamWaitEvent(ctx->comm_s, ctx->ev_phi, 0));
+    if (int r = fill_ghost_dims(ctx, pd, PF_N, false, fe, 3, ctx->comm_s)) return r;
+    CU(cudaEventRecord(ctx->ev_phix, ctx->comm_s));
+    // the mu-sweep reads mu ghosts: the previous mu exchange must be done
+    if (int r = join_comm(ctx)) return r;
+    // line 3: interior tiles (no phi_dst ghost of an exchanged dimension is read)
+    const int mty = ctx->variant == PF_VARIANT_JIT ? jit_mu_ty_of(ctx->jit) : tuned_mu_ty_default();
+    const dim3 full = tuned_grid_mu(g, mty);
+    const int nb[3] = {(int)full.x, (int)full.y, (int)full.z};
+    TileSel in = {{0, 0, 0}, {0, 0, 0}, {nb[0], nb[1], nb[2]}, 0};
+    bool any_in = true;
+    for (int d = fe; d < 3; ++d) {
+      in.lo[d] = 1;
+      in.hi[d] = nb[d] - 1;
+      any_in &= in.hi[d] > in.lo[d];
+    }
+    prof_begin(ctx, 1, &e0);
+    if (any_in) {
+      TileSel ti = {{in.lo[0], in.lo[1], in.lo[2]}, {0, 0, 0}, {0, 0, 0}, 0};
+      const dim3 gi(in.hi[0] - in.lo[0], in.hi[1] - in.lo[1], in.hi[2] - in.lo[2]);
+      if (int r = launch_mu(ctx, &ti, gi, ps, pd, ms, md)) return r;
+    }
+    // shell tiles once the phi ghosts have arrived
+    CU(cudaStreamWaitEvent(ctx->stream, ctx->ev_phix, 0));
+    TileSel sh = in;
+    sh.skip = any_in ? 1 : 0;
+    if (int r = launch_mu(ctx, &sh, full, ps, pd, ms, md)) return r;
+    prof_end(ctx, 1, e0);
+    // line 4: mu ghosts; the exchange overlaps the next phi-sweep
+    if (int r = fill_ghost_dims(ctx, md, PF_M, true, 0, fe, ctx->stream)) return r;
+    CU(cudaEventRecord(ctx->ev_mu, ctx->stream));
+    CU(cudaStreamWaitEvent(ctx->comm_s, ctx->ev_mu, 0));
+    if (int r = fill_ghost_dims(ctx, md, PF_M, true, fe, 3, ctx->comm_s)) return r;
+    CU(cudaEventRecord(ctx->ev_mux, ctx->comm_s));
+    ctx->mux_pending = true;
   }
   // line 5: swap
   ctx->cur = 1 - ctx->cur;
@@ -708,7 +806,7 @@ int pf_step(pf_ctx* ctx, int64_t nsteps) {
     if (int r = step_impl(ctx, false)) return r;
     if (int r = window_maybe(ctx)) return r;
   }
-  return PF_OK;
+  return join_comm(ctx);
 }
 
 int pf_step_phi_only(pf_ctx* ctx) {
@@ -720,6 +818,7 @@ int pf_step_phi_only(pf_ctx* ctx) {
 int pf_halo_exchange(pf_ctx* ctx, unsigned mask) {
   if (!ctx) return PF_EINVAL;
   if (!ctx->have_params) return fail(ctx, PF_ESTATE, "pf_halo_exchange before pf_set_params");
+  if (int r = join_comm(ctx)) return r;
   if (mask & PF_PHI)
     if (int r = fill_ghosts(ctx, ctx->phi[ctx->cur], PF_N, false)) return r;
   if (mask & PF_MU)
@@ -856,6 +955,7 @@ int pf_shift_window(pf_ctx* ctx, int k) {
   if (pz != 1) return fail(ctx, PF_EINVAL, "the moving window needs the growth axis unsplit (procs[2] == 1)");
   if (k < 0 || k > ctx->g.nz) return fail(ctx, PF_EINVAL, "shift %d out of range", k);
   if (k == 0) return PF_OK;
+  if (int r = join_comm(ctx)) return r;
   cudaEvent_t e0 = nullptr;
   prof_begin(ctx, 3, &e0);
   launch_shift(ctx->g, k, ctx->cfg.liquid, ctx->hp.mu_inf, ctx->phi[ctx->cur], ctx->mu[ctx->cur],

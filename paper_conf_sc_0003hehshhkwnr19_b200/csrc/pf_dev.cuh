@@ -29,6 +29,15 @@ struct Geom {
   }
 };
 
+// Tile selection of a sweep launch (interior / shell split for overlapping
+// the halo exchange): tile = blockIdx + off; if skip, tiles
+// with lo <= tile < hi in all three dimensions return at once.
+struct TileSel {
+  int off[3];
+  int lo[3], hi[3];
+  int skip;
+};
+
 // Scalars and coefficients of the model.  Passed by value to every kernel
 // (kernel-parameter constant bank) in the generic build; folded into the
 // code as compile-time constants in the specialised build.  T-dependent

@@ -22,8 +22,9 @@ void launch_mu_naive(const DevParams& P, const Geom& g, const double* ps, const 
                      double* md, cudaStream_t s);
 void launch_phi_tuned(const DevParams& P, const Geom& g, const double* ps, const double* ms, double* pd,
                       cudaStream_t s);
-void launch_mu_tuned(const DevParams& P, const Geom& g, const double* ps, const double* pd, const double* ms,
-                     double* md, cudaStream_t s);
+// ts == nullptr: all tiles (grid ignored); else the selected tiles of `grid`
+void launch_mu_tuned(const DevParams& P, const Geom& g, const TileSel* ts, dim3 grid, const double* ps,
+                     const double* pd, const double* ms, double* md, cudaStream_t s);
 // launch geometry of the tuned kernels (shared with the specialised build)
 dim3 tuned_block();
 dim3 tuned_block_mu(int mty);
@@ -63,7 +64,8 @@ struct JitModule;  // compiled sweep kernels for one (geometry, parameters)
 JitModule* jit_get(const DevParams& P, const Geom& g, std::string* err);
 cudaError_t jit_launch_phi(JitModule* m, const DevParams& P, const double* ps, const double* ms, double* pd,
                            cudaStream_t s);
-cudaError_t jit_launch_mu(JitModule* m, const DevParams& P, const double* ps, const double* pd, const double* ms,
-                          double* md, cudaStream_t s);
+cudaError_t jit_launch_mu(JitModule* m, const DevParams& P, const TileSel* ts, dim3 grid, const double* ps,
+                          const double* pd, const double* ms, double* md, cudaStream_t s);
+int jit_mu_ty_of(const JitModule* m);
 
 }  // namespace pf

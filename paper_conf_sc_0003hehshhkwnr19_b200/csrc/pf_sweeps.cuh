@@ -249,20 +249,24 @@ __device__ __forceinline__ void side_from_smem(const double* __restrict__ D, int
 }
 
 template <class PT, class GT, int L, bool TA, int MTY>
-__device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, const GT& g,
+__device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, const GT& g, const TileSel& ts,
                                               const double* __restrict__ ps, const double* __restrict__ pd,
                                               const double* __restrict__ ms, double* __restrict__ md) {
   constexpr int NC = MuTile<MTY>::NC, HX = MuTile<MTY>::HX;
+  const int tbx = blockIdx.x + ts.off[0], tby = blockIdx.y + ts.off[1], tbz = blockIdx.z + ts.off[2];
+  if (ts.skip && tbx >= ts.lo[0] && tbx < ts.hi[0] && tby >= ts.lo[1] && tby < ts.hi[1] && tbz >= ts.lo[2] &&
+      tbz < ts.hi[2])
+    return;  // interior tile, done by the other launch
   extern __shared__ double smem[];
   double* D = smem;                          // [D_NV][NC]
   double* fxs = D + D_NV * NC;               // [M][MTY][TX+1]: x-face fluxes, face i = x0 - 1/2 + i
   double* fys = fxs + M * MTY * (TX + 1);     // [M][MTY+1][TX]: y-face fluxes
   const int lane = threadIdx.x, w = threadIdx.y, t = w * TX + lane;
-  const int x0 = blockIdx.x * TX, y0 = blockIdx.y * MTY;
+  const int x0 = tbx * TX, y0 = tby * MTY;
   const int x = x0 + lane, y = y0 + w;
   const bool active = x < g.nx && y < g.ny;
   const int xc = min(x, g.nx), yc = min(y, g.ny);
-  const int z0 = blockIdx.z * ZC_MU, z1 = min(z0 + ZC_MU, g.nz);
+  const int z0 = tbz * ZC_MU, z1 = min(z0 + ZC_MU, g.nz);
   const i64 F = g.field;
   const int me = hidx(lane + 1, w + 1);
   // halo ring cell owned by thread t < 2*TX + 2*MTY (corners are not needed)

@@ -32,11 +32,12 @@ __global__ void __launch_bounds__(TX* TY, 2) k_phi_tuned(DevParams P, Geom g, co
 }
 
 template <int L, bool TA>
-__global__ void __launch_bounds__(TX* MU_TY, 16 / MU_TY) k_mu_tuned(DevParams P, Geom g, const double* __restrict__ ps,
+__global__ void __launch_bounds__(TX* MU_TY, 16 / MU_TY) k_mu_tuned(DevParams P, Geom g, TileSel ts,
+                                                                  const double* __restrict__ ps,
                                                                   const double* __restrict__ pd,
                                                                   const double* __restrict__ ms,
                                                                   double* __restrict__ md) {
-  mu_tuned_body<DevParams, Geom, L, TA, MU_TY>(P, P, g, ps, pd, ms, md);
+  mu_tuned_body<DevParams, Geom, L, TA, MU_TY>(P, P, g, ts, ps, pd, ms, md);
 }
 
 dim3 tuned_block() { return dim3(TX, TY); }
@@ -68,19 +69,22 @@ void launch_phi_tuned(const DevParams& P, const Geom& g, const double* ps, const
 
 
 template <int L, bool TA>
-static void mu_launch(const DevParams& P, const Geom& g, const double* ps, const double* pd, const double* ms,
-                      double* md, cudaStream_t s) {
+static void mu_launch(const DevParams& P, const Geom& g, const TileSel& ts, dim3 grid, const double* ps,
+                      const double* pd, const double* ms, double* md, cudaStream_t s) {
   static bool attr = false;  // per instantiation
   if (!attr) {
     cudaFuncSetAttribute(k_mu_tuned<L, TA>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tuned_mu_smem(MU_TY));
     attr = true;
   }
-  k_mu_tuned<L, TA><<<tuned_grid_mu(g, MU_TY), tuned_block_mu(MU_TY), tuned_mu_smem(MU_TY), s>>>(P, g, ps, pd, ms, md);
+  k_mu_tuned<L, TA><<<grid, tuned_block_mu(MU_TY), tuned_mu_smem(MU_TY), s>>>(P, g, ts, ps, pd, ms, md);
 }
 
-void launch_mu_tuned(const DevParams& P, const Geom& g, const double* ps, const double* pd, const double* ms,
-                     double* md, cudaStream_t s) {
-  PF_DISPATCH(P.liquid, P.TA, (mu_launch<LL, TT>(P, g, ps, pd, ms, md, s)));
+void launch_mu_tuned(const DevParams& P, const Geom& g, const TileSel* ts, dim3 grid, const double* ps,
+                     const double* pd, const double* ms, double* md, cudaStream_t s) {
+  TileSel all = {{0, 0, 0}, {0, 0, 0}, {0, 0, 0}, 0};
+  const TileSel& t = ts ? *ts : all;
+  const dim3 gr = ts ? grid : tuned_grid_mu(g, MU_TY);
+  PF_DISPATCH(P.liquid, P.TA, (mu_launch<LL, TT>(P, g, t, gr, ps, pd, ms, md, s)));
 }
 
 

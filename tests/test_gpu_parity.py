@@ -180,6 +180,27 @@ def test_forced_exchange_path_bitwise(pfmod, monkeypatch):
     assert np.array_equal(ref[0], got[0]) and np.array_equal(ref[1], got[1])
 
 
+@pytest.mark.parametrize("variant", ["jit", "tuned"])
+def test_overlapped_exchange_bitwise(pfmod, monkeypatch, variant):
+    """Interior/shell split of the mu-sweep with the phi exchange on a second
+    stream and the mu exchange overlapping the next phi-sweep:
+    bitwise equal to the serial schedule and to the local ghost fill."""
+    P = I.params_stress()
+    shape = (70, 20, 100)  # 4 x-tiles, 5 y-tiles, 3 z-chunks: non-empty interior
+    phi, mu = I.ic_voronoi(shape, seed=8)
+    outs = []
+    for force, overlap in (("0", "1"), ("1", "0"), ("1", "1")):
+        monkeypatch.setenv("PF_FORCE_EXCHANGE", force)
+        monkeypatch.setenv("PF_OVERLAP", overlap)
+        g = pfmod.PhaseField(shape, P)
+        g.set_variant(variant)
+        g.init_fields(phi, mu)
+        g.step(4)
+        outs.append(g.download())
+    for o in outs[1:]:
+        assert np.array_equal(outs[0][0], o[0]) and np.array_equal(outs[0][1], o[1])
+
+
 def test_translation_invariance_bitwise(pfmod):
     P = I.params_stress(G=0.0, v=0.0)
     shape = (16, 12, 20)
