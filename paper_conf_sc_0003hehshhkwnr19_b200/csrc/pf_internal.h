@@ -28,9 +28,9 @@ void launch_mu_tuned(const DevParams& P, const Geom& g, const TileSel* ts, dim3 
 // launch geometry of the tuned kernels (shared with the specialised build)
 dim3 tuned_block();
 dim3 tuned_block_mu(int mty);
-dim3 tuned_grid_phi(const Geom& g, int pty);
+dim3 tuned_grid_phi(const Geom& g, int pty, int zc = 0);  // zc <= 0: the built-in z-chunk
 dim3 tuned_block_phi(int pty);
-dim3 tuned_grid_mu(const Geom& g, int mty);
+dim3 tuned_grid_mu(const Geom& g, int mty, int zc = 0);
 size_t tuned_mu_smem(int mty);  // mty: tile height of the mu-sweep (2, 4, 8)
 int tuned_mu_ty_default();
 size_t tuned_phi_smem();
@@ -67,5 +67,6 @@ cudaError_t jit_launch_phi(JitModule* m, const DevParams& P, const double* ps, c
 cudaError_t jit_launch_mu(JitModule* m, const DevParams& P, const TileSel* ts, dim3 grid, const double* ps,
                           const double* pd, const double* ms, double* md, cudaStream_t s);
 int jit_mu_ty_of(const JitModule* m);
+int jit_mu_zc_of(const JitModule* m);
 
 }  // namespace pf

@@ -40,8 +40,14 @@ __device__ __forceinline__ void prefetch_line(const void* p) {
 
 constexpr int TX = 32;
 constexpr int TY = 8;
-constexpr int ZC_PHI = 32;  // z-chunk per CTA
-constexpr int ZC_MU = 32;
+#ifndef PF_ZC_PHI
+#define PF_ZC_PHI 32
+#endif
+#ifndef PF_ZC_MU
+#define PF_ZC_MU 32
+#endif
+constexpr int ZC_PHI = PF_ZC_PHI;  // z-chunk per CTA
+constexpr int ZC_MU = PF_ZC_MU;
 #ifndef PF_MU_TY
 #define PF_MU_TY 4  // tile height of the mu-sweep (4: 4 CTAs of 128 threads per SM)
 #endif

@@ -43,11 +43,13 @@ __global__ void __launch_bounds__(TX* MU_TY, 16 / MU_TY) k_mu_tuned(DevParams P,
 dim3 tuned_block() { return dim3(TX, TY); }
 dim3 tuned_block_phi(int pty) { return dim3(TX, pty); }
 dim3 tuned_block_mu(int mty) { return dim3(TX, mty); }
-dim3 tuned_grid_phi(const Geom& g, int pty) {
-  return dim3((g.nx + TX - 1) / TX, (g.ny + pty - 1) / pty, (g.nz + ZC_PHI - 1) / ZC_PHI);
+dim3 tuned_grid_phi(const Geom& g, int pty, int zc) {
+  if (zc <= 0) zc = ZC_PHI;
+  return dim3((g.nx + TX - 1) / TX, (g.ny + pty - 1) / pty, (g.nz + zc - 1) / zc);
 }
-dim3 tuned_grid_mu(const Geom& g, int mty) {
-  return dim3((g.nx + TX - 1) / TX, (g.ny + mty - 1) / mty, (g.nz + ZC_MU - 1) / ZC_MU);
+dim3 tuned_grid_mu(const Geom& g, int mty, int zc) {
+  if (zc <= 0) zc = ZC_MU;
+  return dim3((g.nx + TX - 1) / TX, (g.ny + mty - 1) / mty, (g.nz + zc - 1) / zc);
 }
 size_t tuned_mu_smem(int mty) {
   return mty == 8 ? mu_smem_bytes<8>() : (mty == 4 ? mu_smem_bytes<4>() : (mty == 2 ? mu_smem_bytes<2>() : 0));
@@ -59,7 +61,7 @@ size_t tuned_phi_smem() { return 0; }  // static shared memory only
 template <int L, bool TA>
 static void phi_launch(const DevParams& P, const Geom& g, const double* ps, const double* ms, double* pd,
                        cudaStream_t s) {
-  k_phi_tuned<L, TA><<<tuned_grid_phi(g, TY), tuned_block(), 0, s>>>(P, g, ps, ms, pd);
+  k_phi_tuned<L, TA><<<tuned_grid_phi(g, TY, 0), tuned_block(), 0, s>>>(P, g, ps, ms, pd);
 }
 
 void launch_phi_tuned(const DevParams& P, const Geom& g, const double* ps, const double* ms, double* pd,
@@ -83,7 +85,7 @@ void launch_mu_tuned(const DevParams& P, const Geom& g, const TileSel* ts, dim3 
                      const double* pd, const double* ms, double* md, cudaStream_t s) {
   TileSel all = {{0, 0, 0}, {0, 0, 0}, {0, 0, 0}, 0};
   const TileSel& t = ts ? *ts : all;
-  const dim3 gr = ts ? grid : tuned_grid_mu(g, MU_TY);
+  const dim3 gr = ts ? grid : tuned_grid_mu(g, MU_TY, 0);
   PF_DISPATCH(P.liquid, P.TA, (mu_launch<LL, TT>(P, g, t, gr, ps, pd, ms, md, s)));
 }
 
