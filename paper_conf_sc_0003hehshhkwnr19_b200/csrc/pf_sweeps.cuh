@@ -41,10 +41,10 @@ __device__ __forceinline__ void prefetch_line(const void* p) {
 constexpr int TX = 32;
 constexpr int TY = 8;
 #ifndef PF_ZC_PHI
-#define PF_ZC_PHI 32
+#define PF_ZC_PHI 12
 #endif
 #ifndef PF_ZC_MU
-#define PF_ZC_MU 32
+#define PF_ZC_MU 12
 #endif
 constexpr int ZC_PHI = PF_ZC_PHI;  // z-chunk per CTA
 constexpr int ZC_MU = PF_ZC_MU;
