@@ -264,7 +264,7 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
       tbz < ts.hi[2])
     return;  // interior tile, done by the other launch
   extern __shared__ double smem[];
-  double* D = smem;                          // [D_NV][NC]
+  double* D = smem;                          // [NC][D_NV] (AoS: LDS.128 per pair)
   double* fxs = D + D_NV * NC;               // [M][MTY][TX+1]: x-face fluxes, face i = x0 - 1/2 + i
   double* fys = fxs + M * MTY * (TX + 1);     // [M][MTY+1][TX]: y-face fluxes
   const int lane = threadIdx.x, w = threadIdx.y, t = w * TX + lane;
@@ -352,13 +352,29 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
     if (!last) {
       // (d) faces of plane k: -x and -y of every thread, + the far tile edges
       const double Tk = plane_T(P, R, (double)k);
+      // (the own side is Dp = plane k's {f, cx, cy, ds, mu}, already in
+      // registers: only its cz comes from shared memory)
       FaceSide p, s;
       double Fx[M], Fy[M];
+      {
+        const double2* d = reinterpret_cast<const double2*>(D + (size_t)me * D_NV + D_CZ);
+        const double2 z01 = d[0], z23 = d[1];
+        s.c2[0] = z01.x; s.c2[1] = z01.y; s.c2[2] = z23.x; s.c2[3] = z23.y;
+      }
+#pragma unroll
+      for (int a = 0; a < N; ++a) {
+        s.f[a] = Dp.f[a];
+        s.c1[a] = Dp.c2[a];
+      }
+#pragma unroll
+      for (int u = 0; u < NSOL; ++u) s.ds[u] = Dp.ds[u];
+      s.m[0] = Dp.m[0];
+      s.m[1] = Dp.m[1];
       side_from_smem<L, NC>(D, me - 1, D_CY, D_CZ, p);
-      side_from_smem<L, NC>(D, me, D_CY, D_CZ, s);
       mu_face<L, TA>(P, Tk, p, s, Fx);
+#pragma unroll
+      for (int a = 0; a < N; ++a) s.c1[a] = Dp.c1[a];
       side_from_smem<L, NC>(D, me - HX, D_CX, D_CZ, p);
-      side_from_smem<L, NC>(D, me, D_CX, D_CZ, s);
       mu_face<L, TA>(P, Tk, p, s, Fy);
 #pragma unroll
       for (int i = 0; i < M; ++i) {
