@@ -259,6 +259,7 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
                                               const double* __restrict__ ps, const double* __restrict__ pd,
                                               const double* __restrict__ ms, double* __restrict__ md) {
   constexpr int NC = MuTile<MTY>::NC, HX = MuTile<MTY>::HX;
+  static_assert(2 * TX + 2 * MTY <= MTY * TX, "the halo ring needs 2 TX + 2 MTY threads");
   const int tbx = blockIdx.x + ts.off[0], tby = blockIdx.y + ts.off[1], tbz = blockIdx.z + ts.off[2];
   if (ts.skip && tbx >= ts.lo[0] && tbx < ts.hi[0] && tby >= ts.lo[1] && tby < ts.hi[1] && tbz >= ts.lo[2] &&
       tbz < ts.hi[2])

@@ -52,7 +52,7 @@ dim3 tuned_grid_mu(const Geom& g, int mty, int zc) {
   return dim3((g.nx + TX - 1) / TX, (g.ny + mty - 1) / mty, (g.nz + zc - 1) / zc);
 }
 size_t tuned_mu_smem(int mty) {
-  return mty == 8 ? mu_smem_bytes<8>() : (mty == 4 ? mu_smem_bytes<4>() : (mty == 2 ? mu_smem_bytes<2>() : 0));
+  return (size_t)(D_NV * (TX + 2) * (mty + 2) + M * mty * (TX + 1) + M * (mty + 1) * TX) * sizeof(double);
 }
 int tuned_mu_ty_default() { return MU_TY; }
 
