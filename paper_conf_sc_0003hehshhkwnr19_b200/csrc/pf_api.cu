@@ -451,7 +451,7 @@ int pf_create(const pf_config* cfg, pf_ctx** out) {
       ctx->first_ex = d;
       break;
     }
-  if (ctx->first_ex < 3) {
+  {  // side stream: halo exchanges (N > 1) and the mu ghost fill (any N)
     const char* ov = getenv("PF_OVERLAP");
     ctx->overlap = !(ov && ov[0] == '0');
     e = cudaStreamCreateWithFlags(&ctx->comm_s, cudaStreamNonBlocking);
@@ -744,11 +744,21 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
       prof_begin(ctx, 1, &e0);
       if (int r2 = launch_mu(ctx, nullptr, dim3(), ps, pd, ms, md)) return r2;
       prof_end(ctx, 1, e0);
-      // line 4
-      prof_begin(ctx, 2, &e0);
-      r = fill_ghosts(ctx, md, PF_M, true);
-      prof_end(ctx, 2, e0);
-      if (r) return r;
+      // line 4: mu ghosts.  The next phi-sweep reads mu only at its own
+      // cells, so the fill runs on the side stream concurrently with it and
+      // the next mu-sweep (or any other use) joins first (join_comm).
+      if (ctx->overlap && ctx->comm_s) {
+        CU(cudaEventRecord(ctx->ev_mu, ctx->stream));
+        CU(cudaStreamWaitEvent(ctx->comm_s, ctx->ev_mu, 0));
+        if (int r2 = fill_ghost_dims(ctx, md, PF_M, true, 0, 3, ctx->comm_s)) return r2;
+        CU(cudaEventRecord(ctx->ev_mux, ctx->comm_s));
+        ctx->mux_pending = true;
+      } else {
+        prof_begin(ctx, 2, &e0);
+        r = fill_ghosts(ctx, md, PF_M, true);
+        prof_end(ctx, 2, e0);
+        if (r) return r;
+      }
     }
   } else {
     // line 2: local dimensions before the first exchanged one on the compute

@@ -183,13 +183,14 @@ def test_forced_exchange_path_bitwise(pfmod, monkeypatch):
 @pytest.mark.parametrize("variant", ["jit", "tuned"])
 def test_overlapped_exchange_bitwise(pfmod, monkeypatch, variant):
     """Interior/shell split of the mu-sweep with the phi exchange on a second
-    stream and the mu exchange overlapping the next phi-sweep:
-    bitwise equal to the serial schedule and to the local ghost fill."""
+    stream and the mu exchange overlapping the next phi-sweep,
+    and (no exchange) the local mu ghost fill on the side stream: bitwise
+    equal to the serial schedule and to the local ghost fill."""
     P = I.params_stress()
     shape = (70, 20, 100)  # 4 x-tiles, 5 y-tiles, 3 z-chunks: non-empty interior
     phi, mu = I.ic_voronoi(shape, seed=8)
     outs = []
-    for force, overlap in (("0", "1"), ("1", "0"), ("1", "1")):
+    for force, overlap in (("0", "0"), ("0", "1"), ("1", "0"), ("1", "1")):
         monkeypatch.setenv("PF_FORCE_EXCHANGE", force)
         monkeypatch.setenv("PF_OVERLAP", overlap)
         g = pfmod.PhaseField(shape, P)
