@@ -159,6 +159,7 @@ struct GhostArgs {
   int ncomp;
   double dir[M];
   int use_dir;
+  int vec_x;  // x ghost sectors 32-B aligned (nx % 4 == 0, xoff % 4 == 0): full-sector stores
 };
 
 __device__ __forceinline__ int map_axis(int i, int n, int klo, int khi, bool* skip, bool* dirich) {
@@ -216,6 +217,20 @@ __global__ void k_ghost(GhostArgs A, double* __restrict__ f) {
 #pragma unroll
   for (int c = 0; c < N; ++c)
     if (c < A.ncomp) v[c] = (dir && A.use_dir) ? A.dir[c < M ? c : 0] : __ldg(f + c * g.field + src);
+  if (seg == 2 && A.vec_x) {
+    // x ghost columns: store the whole 32-B sector (x = -4..-1, or nx..nx+3)
+    // with the ghost value so that L2 never merges a partial sector with
+    // DRAM; the other three slots are guard cells that no result depends on
+    const int64_t base = g.at(x < 0 ? -4 : g.nx, y, z);
+#pragma unroll
+    for (int c = 0; c < N; ++c)
+      if (c < A.ncomp) {
+        double2* q = reinterpret_cast<double2*>(f + c * g.field + base);
+        q[0] = make_double2(v[c], v[c]);
+        q[1] = make_double2(v[c], v[c]);
+      }
+    return;
+  }
 #pragma unroll
   for (int c = 0; c < N; ++c)
     if (c < A.ncomp) f[c * g.field + dst] = v[c];
@@ -228,6 +243,8 @@ void launch_ghost_fill(const Geom& g, const BCSpec& bc, double* f, int ncomp, co
   A.ncomp = ncomp;
   A.use_dir = dirichlet != nullptr;
   for (int i = 0; i < M; ++i) A.dir[i] = dirichlet ? dirichlet[i] : 0.0;
+  A.vec_x = (g.nx % 4 == 0 && g.xoff % 4 == 0 && g.pitch % 4 == 0 && g.xoff >= 4 &&
+             g.pitch - g.xoff >= (int64_t)g.nx + 4);
   const int64_t n0 = 2 * (int64_t)(g.nx + 2) * (g.ny + 2), n1 = 2 * (int64_t)(g.nx + 2) * g.nz,
                 n2 = 2 * (int64_t)g.ny * g.nz;
   const int64_t mx = n0 > n1 ? (n0 > n2 ? n0 : n2) : (n1 > n2 ? n1 : n2);
