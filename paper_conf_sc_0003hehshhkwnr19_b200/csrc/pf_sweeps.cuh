@@ -25,6 +25,9 @@ namespace pf {
 #ifndef PF_PREFETCH
 #define PF_PREFETCH 1
 #endif
+#ifndef PF_MU_ZCARRY  // own cell's phi_src z column carried in registers (8 loads fewer per cell)
+#define PF_MU_ZCARRY 1
+#endif
 #ifndef PF_PREFETCH_D
 #define PF_PREFETCH_D 2  // planes ahead
 #endif
@@ -224,6 +227,35 @@ __device__ __forceinline__ void build_cell(const GT& g, const double* __restrict
   for (int j = 0; j < D_NV / 2; ++j) d[j] = make_double2(v[2 * j], v[2 * j + 1]);
 }
 
+// build D of the own cell (x,y,k) into slot i with its z column carried in
+// registers: fc = phi_src(k) (loaded as the +z neighbour one plane earlier),
+// fm = phi_src(k-1); loads phi_src(k+1) into fc for the next plane.
+template <int NC, class GT>
+__device__ __forceinline__ void build_own_carry(const GT& g, const double* __restrict__ ps,
+                                                const double* __restrict__ pd, const double* __restrict__ ms, int x,
+                                                int y, int k, bool wz, const double (&fm)[N], double (&fc)[N],
+                                                double* __restrict__ D, int i) {
+  const i64 F = g.field;
+  const i64 c = g.at(x, y, k);
+  double v[D_NV];
+#pragma unroll
+  for (int a = 0; a < N; ++a) {
+    const double* f = ps + a * F + c;
+    const double fp = wz ? __ldg(f + g.plane) : 0.0;
+    v[D_F + a] = fc[a];
+    v[D_CX + a] = __ldg(f + 1) - __ldg(f - 1);
+    v[D_CY + a] = __ldg(f + g.pitch) - __ldg(f - g.pitch);
+    v[D_CZ + a] = wz ? fp - fm[a] : 0.0;
+    v[D_DP + a] = __ldg(pd + a * F + c) - fc[a];
+    fc[a] = fp;
+  }
+  v[D_MU + 0] = __ldg(ms + c);
+  v[D_MU + 1] = __ldg(ms + F + c);
+  double2* d = reinterpret_cast<double2*>(D + (size_t)i * D_NV);
+#pragma unroll
+  for (int j = 0; j < D_NV / 2; ++j) d[j] = make_double2(v[2 * j], v[2 * j + 1]);
+}
+
 template <int L, int NC>
 __device__ __forceinline__ void side_from_smem(const double* __restrict__ D, int i, int c1, int c2, FaceSide& s) {
   const double2* d = reinterpret_cast<const double2*>(D + (size_t)i * D_NV);
@@ -309,6 +341,14 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
     Dp.m[1] = __ldg(ms + F + c);
   }
   double divxy[M] = {0.0, 0.0}, Fzm[M] = {0.0, 0.0};
+#if PF_MU_ZCARRY
+  double fcar[N];  // phi_src(k) of the own cell, carried along z
+  {
+    const i64 c = g.at(xc, yc, z0);
+#pragma unroll
+    for (int a = 0; a < N; ++a) fcar[a] = __ldg(ps + a * F + c);
+  }
+#endif
 
   for (int k = z0; k <= z1; ++k) {
     const bool last = k == z1;
@@ -323,7 +363,11 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
       prefetch_line(ms + F + cp + (PF_PREFETCH_D - 1) * g.plane);
     }
     // (a) publish D(k) of the own cell and of the halo ring
+#if PF_MU_ZCARRY
+    build_own_carry<NC>(g, ps, pd, ms, xc, yc, k, !last, Dp.f, fcar, D, me);
+#else
     build_cell<NC>(g, ps, pd, ms, xc, yc, k, true, true, !last, D, me);
+#endif
     if (hs >= 0 && !last) build_cell<NC>(g, ps, pd, ms, hgx, hgy, k, hwx, hwy, true, D, hs);
     __syncthreads();
     // (b) z-face k-1/2 from registers (plane k-1) and shared memory (plane k)

@@ -32,7 +32,7 @@ __global__ void __launch_bounds__(TX* TY, 2) k_phi_tuned(DevParams P, Geom g, co
 }
 
 template <int L, bool TA>
-__global__ void __launch_bounds__(TX* MU_TY, 16 / MU_TY) k_mu_tuned(DevParams P, Geom g, TileSel ts,
+__global__ void __launch_bounds__(TX* MU_TY, MU_TY == 4 ? 3 : 16 / MU_TY) k_mu_tuned(DevParams P, Geom g, TileSel ts,
                                                                   const double* __restrict__ ps,
                                                                   const double* __restrict__ pd,
                                                                   const double* __restrict__ ms,
