@@ -16,4 +16,6 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:pf_j
    python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_mu.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:pf_jit_phi -s 3 -c 1 -o $OUT/prof_phi \
    python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_phi.log 2>&1
+timeout 600 ncu --set full --clock-control none -k regex:k_ghost -s 6 -c 1 -o $OUT/prof_ghost \
+   python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_ghost.log 2>&1
 echo done > $OUT/DONE

@@ -30,7 +30,7 @@ KEYS = ["gpu__time_duration.sum", "launch__registers_per_thread", "launch__occup
         "lts__t_sector_hit_rate.pct", "smsp__inst_executed.sum", "smsp__sass_inst_executed_op_global_ld.sum",
         "smsp__sass_inst_executed_op_shared_ld.sum", "smsp__sass_inst_executed_op_local_ld.sum"]
 summary = {}
-for kern in ("mu", "phi"):
+for kern in ("mu", "phi", "ghost"):
     rep = os.path.join(src, f"prof_{kern}.ncu-rep")
     if not os.path.exists(rep):
         continue
@@ -62,6 +62,29 @@ for kern in ("mu", "phi"):
         fp64 = sum(ops[o] for o in ("DFMA", "DMUL", "DADD", "DSETP", "DMNMX", "MUFU"))
         lines += ["", f"  dynamic instruction mix (warp-level, total {tot}, fp64-pipe share {fp64 / max(tot, 1):.1%}):"]
         lines += [f"    {k:10s} {c / tot:6.1%}" for k, c in ops.most_common(20)]
+        # stall samples per code region (regions end at a CTA barrier)
+        iS = hh.index("Warp Stall Sampling (All Samples)")
+        scol = [c for c in hh if c.startswith("stall_") and "Not Issued" not in c]
+        regs, cur = [], {"n": 0, "samples": 0.0, "exec": 0.0, "st": collections.Counter()}
+        for r in srows[2:]:
+            cur["n"] += 1
+            cur["samples"] += float(r[iS] or 0)
+            cur["exec"] += float(r[iE] or 0)
+            for c in scol:
+                cur["st"][c[6:]] += float(r[hh.index(c)] or 0)
+            if "BAR.SYNC" in r[1] or re.search(r"\bEXIT\b", r[1]):
+                cur["end"] = r[1].strip()[:28]
+                regs.append(cur)
+                cur = {"n": 0, "samples": 0.0, "exec": 0.0, "st": collections.Counter()}
+        ts = sum(x["samples"] for x in regs) or 1.0
+        te = sum(x["exec"] for x in regs) or 1.0
+        lines += ["", "  stall samples by code region (region = SASS up to a BAR.SYNC / EXIT):"]
+        for x in regs:
+            if x["samples"] / ts < 0.02:
+                continue
+            top = ", ".join(f"{k} {v / x['samples']:.0%}" for k, v in x["st"].most_common(4))
+            lines.append(f"    {x['n']:4d} instr ending '{x['end']}': {x['samples'] / ts:5.1%} of samples, "
+                         f"{x['exec'] / te:5.1%} of executed; top: {top}")
     open(os.path.join(dst, f"{tag}_ncu_{kern}.txt"), "w").write("\n".join(lines) + "\n")
     rd = float(m["dram__bytes_read.sum"][0]) * {"Gbyte": 1e9, "Mbyte": 1e6, "Kbyte": 1e3, "byte": 1}[m["dram__bytes_read.sum"][1]]
     wr = float(m["dram__bytes_write.sum"][0]) * {"Gbyte": 1e9, "Mbyte": 1e6, "Kbyte": 1e3, "byte": 1}[m["dram__bytes_write.sum"][1]]
