@@ -28,6 +28,9 @@ namespace pf {
 #ifndef PF_MU_ZCARRY  // own cell's phi_src z column carried in registers (8 loads fewer per cell)
 #define PF_MU_ZCARRY 1
 #endif
+#ifndef PF_MU_RPF  // own cell's L1-missing loads issued one plane ahead into registers
+#define PF_MU_RPF 1
+#endif
 #ifndef PF_PREFETCH_D
 #define PF_PREFETCH_D 2  // planes ahead
 #endif
@@ -256,6 +259,43 @@ __device__ __forceinline__ void build_own_carry(const GT& g, const double* __res
   for (int j = 0; j < D_NV / 2; ++j) d[j] = make_double2(v[2 * j], v[2 * j + 1]);
 }
 
+// as build_own_carry, with the loads that miss L1 (phi_src(k+1), phi_dst(k),
+// mu(k)) taken from registers loaded one plane earlier (nf, nd, nm); the
+// loads for plane k+1 are issued here, a whole face phase before their use
+template <int NC, class GT>
+__device__ __forceinline__ void build_own_rpf(const GT& g, const double* __restrict__ ps,
+                                              const double* __restrict__ pd, const double* __restrict__ ms, int x,
+                                              int y, int k, bool wz, const double (&fm)[N], double (&fc)[N],
+                                              double (&nf)[N], double (&nd)[N], double (&nm)[M],
+                                              double* __restrict__ D, int i) {
+  const i64 F = g.field;
+  const i64 c = g.at(x, y, k);
+  double v[D_NV];
+#pragma unroll
+  for (int a = 0; a < N; ++a) {
+    const double* f = ps + a * F + c;
+    v[D_F + a] = fc[a];
+    v[D_CX + a] = __ldg(f + 1) - __ldg(f - 1);
+    v[D_CY + a] = __ldg(f + g.pitch) - __ldg(f - g.pitch);
+    v[D_CZ + a] = wz ? nf[a] - fm[a] : 0.0;
+    v[D_DP + a] = nd[a] - fc[a];
+    fc[a] = nf[a];
+  }
+  v[D_MU + 0] = nm[0];
+  v[D_MU + 1] = nm[1];
+  double2* d = reinterpret_cast<double2*>(D + (size_t)i * D_NV);
+#pragma unroll
+  for (int j = 0; j < D_NV / 2; ++j) d[j] = make_double2(v[2 * j], v[2 * j + 1]);
+  // next plane (k + 2 <= nz + 1 and k + 1 <= nz + 1 stay inside the guard ring)
+#pragma unroll
+  for (int a = 0; a < N; ++a) {
+    nf[a] = __ldg(ps + a * F + c + 2 * g.plane);
+    nd[a] = __ldg(pd + a * F + c + g.plane);
+  }
+  nm[0] = __ldg(ms + c + g.plane);
+  nm[1] = __ldg(ms + F + c + g.plane);
+}
+
 template <int L, int NC>
 __device__ __forceinline__ void side_from_smem(const double* __restrict__ D, int i, int c1, int c2, FaceSide& s) {
   const double2* d = reinterpret_cast<const double2*>(D + (size_t)i * D_NV);
@@ -349,6 +389,19 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
     for (int a = 0; a < N; ++a) fcar[a] = __ldg(ps + a * F + c);
   }
 #endif
+#if PF_MU_RPF
+  double rnf[N], rnd[N], rnm[M];  // phi_src(k+1), phi_dst(k), mu(k) of the own cell
+  {
+    const i64 c = g.at(xc, yc, z0);
+#pragma unroll
+    for (int a = 0; a < N; ++a) {
+      rnf[a] = __ldg(ps + a * F + c + g.plane);
+      rnd[a] = __ldg(pd + a * F + c);
+    }
+    rnm[0] = __ldg(ms + c);
+    rnm[1] = __ldg(ms + F + c);
+  }
+#endif
 
   for (int k = z0; k <= z1; ++k) {
     const bool last = k == z1;
@@ -363,7 +416,9 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
       prefetch_line(ms + F + cp + (PF_PREFETCH_D - 1) * g.plane);
     }
     // (a) publish D(k) of the own cell and of the halo ring
-#if PF_MU_ZCARRY
+#if PF_MU_RPF
+    build_own_rpf<NC>(g, ps, pd, ms, xc, yc, k, !last, Dp.f, fcar, rnf, rnd, rnm, D, me);
+#elif PF_MU_ZCARRY
     build_own_carry<NC>(g, ps, pd, ms, xc, yc, k, !last, Dp.f, fcar, D, me);
 #else
     build_cell<NC>(g, ps, pd, ms, xc, yc, k, true, true, !last, D, me);

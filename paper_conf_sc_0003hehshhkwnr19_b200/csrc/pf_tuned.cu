@@ -3,6 +3,9 @@
 // geometry at run time.  The specialised build (pf_jit.cu) compiles the same
 // bodies with both folded in.
 #include "pf_internal.h"
+// the generic (run-time parameter) build has less register headroom than the
+// specialised one: no register prefetch of the next plane (it spills here)
+#define PF_MU_RPF 0
 #include "pf_sweeps.cuh"
 
 namespace pf {
