@@ -28,6 +28,10 @@ namespace pf {
 #ifndef PF_MU_ZCARRY  // own cell's phi_src z column carried in registers (8 loads fewer per cell)
 #define PF_MU_ZCARRY 1
 #endif
+#ifndef PF_PHI_UNROLL  // phi-sweep z loop unrolled: the plane rotation (pm <- p0 <- pp) becomes renaming
+#define PF_PHI_UNROLL 3
+#endif
+constexpr int kPhiUnroll = PF_PHI_UNROLL;
 #ifndef PF_MU_RPF  // own cell's L1-missing loads issued one plane ahead into registers
 #define PF_MU_RPF 1
 #endif
@@ -100,6 +104,7 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, 
   }
   phi_face(P, pm, p0, Fzm);
 
+#pragma unroll kPhiUnroll
   for (int z = z0; z < z1; ++z, c += SZ, ep += SZ, eq += SZ) {
     const int buf = z & 1;
     if (PF_PREFETCH && z + PF_PREFETCH_D <= z1 + 1) {  // own column ahead (<= nz + 1: guard ring)

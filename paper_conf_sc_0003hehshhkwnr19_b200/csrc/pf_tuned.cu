@@ -4,8 +4,10 @@
 // bodies with both folded in.
 #include "pf_internal.h"
 // the generic (run-time parameter) build has less register headroom than the
-// specialised one: no register prefetch of the next plane (it spills here)
+// specialised one: no register prefetch of the next plane and no unrolled
+// phi loop (both spill here)
 #define PF_MU_RPF 0
+#define PF_PHI_UNROLL 1
 #include "pf_sweeps.cuh"
 
 namespace pf {
