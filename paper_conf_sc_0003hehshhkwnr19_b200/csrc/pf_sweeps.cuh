@@ -301,6 +301,11 @@ __device__ __forceinline__ void build_own_rpf(const GT& g, const double* __restr
   nm[1] = __ldg(ms + F + c + g.plane);
 }
 
+template <bool B>
+struct BoolC {
+  static constexpr bool value = B;
+};
+
 template <int L, int NC>
 __device__ __forceinline__ void side_from_smem(const double* __restrict__ D, int i, int c1, int c2, FaceSide& s) {
   const double2* d = reinterpret_cast<const double2*>(D + (size_t)i * D_NV);
@@ -408,8 +413,10 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
   }
 #endif
 
-  for (int k = z0; k <= z1; ++k) {
-    const bool last = k == z1;
+  // one plane of the march; the last one (k = z1) only completes the cell
+  // updates of plane z1 - 1, peeled so that the main loop has no such tests
+  auto plane = [&](auto lastc, const int k) {
+    constexpr bool last = decltype(lastc)::value;
     if (PF_PREFETCH && k + PF_PREFETCH_D <= z1 + 1) {  // own cell's lines of the next planes
       const i64 cp = g.at(xc, yc, k);
 #pragma unroll
@@ -428,7 +435,7 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
 #else
     build_cell<NC>(g, ps, pd, ms, xc, yc, k, true, true, !last, D, me);
 #endif
-    if (hs >= 0 && !last) build_cell<NC>(g, ps, pd, ms, hgx, hgy, k, hwx, hwy, true, D, hs);
+    if (!last && hs >= 0) build_cell<NC>(g, ps, pd, ms, hgx, hgy, k, hwx, hwy, true, D, hs);
     __syncthreads();
     // (b) z-face k-1/2 from registers (plane k-1) and shared memory (plane k)
     FaceSide q;
@@ -454,7 +461,7 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
     // carry plane k's side for the next z-face
     Dp = q;
     dpl = D[(size_t)me * D_NV + D_DP + L];
-    if (!last) {
+    if constexpr (!last) {
       // (d) faces of plane k: -x and -y of every thread, + the far tile edges
       const double Tk = plane_T(P, R, (double)k);
       // (the own side is Dp = plane k's {f, cx, cy, ds, mu}, already in
@@ -502,14 +509,16 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
         for (int i = 0; i < M; ++i) fxs[(i * MTY + lane) * (TX + 1) + TX] = Fe[i];
       }
     }
-    __syncthreads();
-    if (!last) {
+    if constexpr (!last) {
+      __syncthreads();
 #pragma unroll
       for (int i = 0; i < M; ++i)
         divxy[i] = (fxs[(i * MTY + w) * (TX + 1) + lane + 1] - fxs[(i * MTY + w) * (TX + 1) + lane]) +
                    (fys[(i * (MTY + 1) + w + 1) * TX + lane] - fys[(i * (MTY + 1) + w) * TX + lane]);
     }
-  }
+  };
+  for (int k = z0; k < z1; ++k) plane(BoolC<false>{}, k);
+  plane(BoolC<true>{}, z1);
 }
 
 }  // namespace pf
