@@ -28,6 +28,9 @@ namespace pf {
 #ifndef PF_MU_ZCARRY  // own cell's phi_src z column carried in registers (8 loads fewer per cell)
 #define PF_MU_ZCARRY 1
 #endif
+#ifndef PF_HALO_L1
+#define PF_HALO_L1 1  // halo-ring cells: next plane's new lines prefetched into L1
+#endif
 #ifndef PF_PHI_UNROLL  // phi-sweep z loop unrolled: the plane rotation (pm <- p0 <- pp) becomes renaming
 #define PF_PHI_UNROLL 3
 #endif
@@ -426,6 +429,16 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
       }
       prefetch_line(ms + cp + (PF_PREFETCH_D - 1) * g.plane);
       prefetch_line(ms + F + cp + (PF_PREFETCH_D - 1) * g.plane);
+    }
+    if (PF_HALO_L1 && !last && hs >= 0) {  // halo-ring cell's lines of the next plane into L1
+      const i64 ch = g.at(hgx, hgy, k + 1);
+#pragma unroll
+      for (int a = 0; a < N; ++a) {
+        asm volatile("prefetch.global.L1 [%0];" ::"l"(ps + a * F + ch + g.plane));
+        asm volatile("prefetch.global.L1 [%0];" ::"l"(pd + a * F + ch));
+      }
+      asm volatile("prefetch.global.L1 [%0];" ::"l"(ms + ch));
+      asm volatile("prefetch.global.L1 [%0];" ::"l"(ms + F + ch));
     }
     // (a) publish D(k) of the own cell and of the halo ring
 #if PF_MU_RPF
