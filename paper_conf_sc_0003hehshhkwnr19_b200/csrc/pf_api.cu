@@ -774,7 +774,8 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
     // line 3: interior tiles (no phi_dst ghost of an exchanged dimension is read)
     const int mty = ctx->variant == PF_VARIANT_JIT ? jit_mu_ty_of(ctx->jit) : tuned_mu_ty_default();
     const int zc = ctx->variant == PF_VARIANT_JIT ? jit_mu_zc_of(ctx->jit) : 0;
-    const dim3 full = tuned_grid_mu(g, mty, zc);
+    const int mtx = ctx->variant == PF_VARIANT_JIT ? jit_mu_tx_of(ctx->jit) : 32;
+    const dim3 full = tuned_grid_mu(g, mty, zc, mtx);
     const int nb[3] = {(int)full.x, (int)full.y, (int)full.z};
     TileSel in = {{0, 0, 0}, {0, 0, 0}, {nb[0], nb[1], nb[2]}, 0};
     bool any_in = true;

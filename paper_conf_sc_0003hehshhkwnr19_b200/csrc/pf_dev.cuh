@@ -72,4 +72,15 @@ struct DevParams {
   int TA;               // A1 != 0: chi and the mobility depend on T
 };
 
+// Compile-time structure of a parameter set, known only to the specialised
+// build (pf_jit.cu specialises it for its constant struct): all gamma_ab
+// (a != b) equal, all gamma_abd equal.  The generic build keeps the general
+// expressions (the paper's "generic application ... would have to spend
+// FLOPs").
+template <class PT>
+struct ParamShape {
+  static constexpr bool guni = false;   // gamma_ab uniform
+  static constexpr bool g3uni = false;  // gamma_abd uniform
+};
+
 }  // namespace pf

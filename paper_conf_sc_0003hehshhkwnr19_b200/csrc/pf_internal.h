@@ -27,11 +27,11 @@ void launch_mu_tuned(const DevParams& P, const Geom& g, const TileSel* ts, dim3 
                      const double* pd, const double* ms, double* md, cudaStream_t s);
 // launch geometry of the tuned kernels (shared with the specialised build)
 dim3 tuned_block();
-dim3 tuned_block_mu(int mty);
+dim3 tuned_block_mu(int mty, int mtx = 32);
 dim3 tuned_grid_phi(const Geom& g, int pty, int zc = 0);  // zc <= 0: the built-in z-chunk
 dim3 tuned_block_phi(int pty);
-dim3 tuned_grid_mu(const Geom& g, int mty, int zc = 0);
-size_t tuned_mu_smem(int mty);  // mty: tile height of the mu-sweep (2, 4, 8)
+dim3 tuned_grid_mu(const Geom& g, int mty, int zc = 0, int mtx = 32);
+size_t tuned_mu_smem(int mty, int mtx = 32);  // mu-sweep tile: mtx x mty
 int tuned_mu_ty_default();
 size_t tuned_phi_smem();
 
@@ -67,6 +67,7 @@ cudaError_t jit_launch_phi(JitModule* m, const DevParams& P, const double* ps, c
 cudaError_t jit_launch_mu(JitModule* m, const DevParams& P, const TileSel* ts, dim3 grid, const double* ps,
                           const double* pd, const double* ms, double* md, cudaStream_t s);
 int jit_mu_ty_of(const JitModule* m);
+int jit_mu_tx_of(const JitModule* m);
 int jit_mu_zc_of(const JitModule* m);
 
 }  // namespace pf

@@ -69,10 +69,89 @@ constexpr int MU_TY = PF_MU_TY;
 // ===========================================================================
 // phi-sweep (Algorithm 1 line 1): D3C7 of phi_src, D3C1 of mu_src.
 // ===========================================================================
+#ifndef PF_PHI_FACES6  // every thread computes all six faces of its cell (no flux exchange, no barrier)
+#define PF_PHI_FACES6 0
+#endif
+#ifndef PF_PHI_ZREC
+#define PF_PHI_ZREC 0
+#endif
 template <class PT, class GT, int L, bool TA, int PTY = TY>
 __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, const GT& g,
                                                const double* __restrict__ ps, const double* __restrict__ ms,
                                                double* __restrict__ pd) {
+#if PF_PHI_FACES6
+  {
+    // The +x / +y face of a cell is the -x / -y face of its neighbour: both
+    // threads evaluate phi_face on the same (left, right) operands, so the
+    // two values are bitwise equal and the fluxes still telescope.  Costs
+    // two extra face evaluations per cell (the neighbour values are loaded
+    // for the central differences anyway) and saves the flux exchange, the
+    // per-plane barrier and the tile-edge faces.
+    const int x = blockIdx.x * TX + threadIdx.x, y = blockIdx.y * PTY + threadIdx.y;
+    if (x >= g.nx || y >= g.ny) return;
+    const int z0 = blockIdx.z * ZC_PHI, z1 = min(z0 + ZC_PHI, g.nz);
+    const i64 F = g.field, SY = g.pitch, SZ = g.plane;
+    i64 c = g.at(x, y, z0);
+    double pm[N], p0[N], Fzm[N];
+#pragma unroll
+    for (int a = 0; a < N; ++a) {
+      pm[a] = __ldg(ps + a * F + c - SZ);
+      p0[a] = __ldg(ps + a * F + c);
+    }
+    phi_face(P, pm, p0, Fzm);
+#pragma unroll kPhiUnroll
+    for (int z = z0; z < z1; ++z, c += SZ) {
+      if (PF_PREFETCH && z + PF_PREFETCH_D <= z1 + 1) {
+#pragma unroll
+        for (int a = 0; a < N; ++a) prefetch_line(ps + a * F + c + PF_PREFETCH_D * SZ);
+        prefetch_line(ms + c + PF_PREFETCH_D * SZ);
+        prefetch_line(ms + F + c + PF_PREFETCH_D * SZ);
+      }
+      double pp[N], Fzp[N], gd[N][3], divh[N];
+      {
+        double xm[N], xp[N], ym[N], yp[N], Fa[N], Fb[N];
+#pragma unroll
+        for (int a = 0; a < N; ++a) {
+          const double* f = ps + a * F + c;
+          pp[a] = __ldg(f + SZ);
+          xm[a] = __ldg(f - 1);
+          xp[a] = __ldg(f + 1);
+          ym[a] = __ldg(f - SY);
+          yp[a] = __ldg(f + SY);
+          gd[a][0] = xp[a] - xm[a];
+          gd[a][1] = yp[a] - ym[a];
+          gd[a][2] = pp[a] - pm[a];
+        }
+        phi_face(P, xm, p0, Fa);
+        phi_face(P, p0, xp, Fb);
+#pragma unroll
+        for (int a = 0; a < N; ++a) divh[a] = Fb[a] - Fa[a];
+        phi_face(P, ym, p0, Fa);
+        phi_face(P, p0, yp, Fb);
+#pragma unroll
+        for (int a = 0; a < N; ++a) divh[a] += Fb[a] - Fa[a];
+      }
+      phi_face(P, p0, pp, Fzp);
+#if PF_PHI_ZREC  // -z face recomputed instead of carried (8 registers fewer)
+      phi_face(P, pm, p0, Fzm);
+#endif
+#pragma unroll
+      for (int a = 0; a < N; ++a) divh[a] += Fzp[a] - Fzm[a];
+      const double mu0 = __ldg(ms + c), mu1 = __ldg(ms + F + c);
+      double out[N];
+      phi_cell<TA>(P, plane_T(P, R, (double)z), p0, gd, divh, mu0, mu1, out);
+#pragma unroll
+      for (int a = 0; a < N; ++a) pd[a * F + c] = out[a];
+#pragma unroll
+      for (int a = 0; a < N; ++a) {
+        pm[a] = p0[a];
+        p0[a] = pp[a];
+        Fzm[a] = Fzp[a];
+      }
+    }
+    return;
+  }
+#endif
   __shared__ double fy[2][N][PTY][TX];  // -y face flux of every thread, by plane parity
   __shared__ double ex[2][N][PTY];      // +x flux on the right tile edge
   __shared__ double ey[2][N][TX];      // +y flux on the top tile edge
@@ -188,10 +267,10 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, 
 // one, and the cell update of plane k-1 is done as soon as that z-face is
 // known (one-plane lag).
 // ===========================================================================
-// halo tile of a TX x MTY column tile (MTY: tile height of the mu-sweep)
-template <int MTY>
+// halo tile of an MTX x MTY column tile (MTX, MTY: tile width and height of the mu-sweep)
+template <int MTY, int MTX = TX>
 struct MuTile {
-  static constexpr int HX = TX + 2, HY = MTY + 2, NC = HX * HY;
+  static constexpr int HX = MTX + 2, HY = MTY + 2, NC = HX * HY;
 };
 // shared-memory D layout, structure of arrays over the NC halo-tile cells
 constexpr int D_F = 0;            // phi      [N]
@@ -201,12 +280,13 @@ constexpr int D_CZ = D_CY + N;    // cd_z     [N]
 constexpr int D_DP = D_CZ + N;    // dphi     [N] (phi_dst - phi_src)
 constexpr int D_MU = D_DP + N;    // mu       [M]
 constexpr int D_NV = D_MU + M;    // 22 doubles per cell
-template <int MTY>
+template <int MTY, int MTX = TX>
 __host__ __device__ constexpr size_t mu_smem_bytes() {
-  return (size_t)(D_NV * MuTile<MTY>::NC + M * MTY * (TX + 1) + M * (MTY + 1) * TX) * sizeof(double);
+  return (size_t)(D_NV * MuTile<MTY, MTX>::NC + M * MTY * (MTX + 1) + M * (MTY + 1) * MTX) * sizeof(double);
 }
 // halo-tile coords (0..HX-1, 0..HY-1) -> slot
-__device__ __forceinline__ int hidx(int hx, int hy) { return hy * (TX + 2) + hx; }
+template <int MTX = TX>
+__device__ __forceinline__ int hidx(int hx, int hy) { return hy * (MTX + 2) + hx; }
 
 // D is stored cell-major (array of structures, D_NV = 22 doubles = 176 B per
 // cell): the 16-B vector accesses of a warp then fall on distinct bank groups
@@ -311,6 +391,7 @@ struct BoolC {
 
 template <int L, int NC>
 __device__ __forceinline__ void side_from_smem(const double* __restrict__ D, int i, int c1, int c2, FaceSide& s) {
+  // (c1, c2: offsets of the two tangential central differences in D)
   const double2* d = reinterpret_cast<const double2*>(D + (size_t)i * D_NV);
   double2 t;
 #pragma unroll
@@ -339,39 +420,52 @@ __device__ __forceinline__ void side_from_smem(const double* __restrict__ D, int
   s.m[1] = t.y;
 }
 
-template <class PT, class GT, int L, bool TA, int MTY>
+template <class PT, class GT, int L, bool TA, int MTY, int MTX = TX>
 __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, const GT& g, const TileSel& ts,
                                               const double* __restrict__ ps, const double* __restrict__ pd,
                                               const double* __restrict__ ms, double* __restrict__ md) {
-  constexpr int NC = MuTile<MTY>::NC, HX = MuTile<MTY>::HX;
-  static_assert(2 * TX + 2 * MTY <= MTY * TX, "the halo ring needs 2 TX + 2 MTY threads");
+  constexpr int NC = MuTile<MTY, MTX>::NC, HX = MuTile<MTY, MTX>::HX;
+  static_assert(2 * MTX + 2 * MTY <= MTY * MTX, "the halo ring needs 2 MTX + 2 MTY threads");
+  static_assert(MTX % 16 == 0 && MTX <= 32, "tile rows of whole 128-B lines");
   const int tbx = blockIdx.x + ts.off[0], tby = blockIdx.y + ts.off[1], tbz = blockIdx.z + ts.off[2];
   if (ts.skip && tbx >= ts.lo[0] && tbx < ts.hi[0] && tby >= ts.lo[1] && tby < ts.hi[1] && tbz >= ts.lo[2] &&
       tbz < ts.hi[2])
     return;  // interior tile, done by the other launch
   extern __shared__ double smem[];
   double* D = smem;                          // [NC][D_NV] (AoS: LDS.128 per pair)
-  double* fxs = D + D_NV * NC;               // [M][MTY][TX+1]: x-face fluxes, face i = x0 - 1/2 + i
-  double* fys = fxs + M * MTY * (TX + 1);     // [M][MTY+1][TX]: y-face fluxes
-  const int lane = threadIdx.x, w = threadIdx.y, t = w * TX + lane;
-  const int x0 = tbx * TX, y0 = tby * MTY;
+  double* fxs = D + D_NV * NC;               // [M][MTY][MTX+1]: x-face fluxes, face i = x0 - 1/2 + i
+  double* fys = fxs + M * MTY * (MTX + 1);    // [M][MTY+1][MTX]: y-face fluxes
+  const int lane = threadIdx.x, w = threadIdx.y, t = w * MTX + lane;  // lane: x in the tile, w: row
+  const int x0 = tbx * MTX, y0 = tby * MTY;
   const int x = x0 + lane, y = y0 + w;
   const bool active = x < g.nx && y < g.ny;
   const int xc = min(x, g.nx), yc = min(y, g.ny);
   const int z0 = tbz * ZC_MU, z1 = min(z0 + ZC_MU, g.nz);
   const i64 F = g.field;
-  const int me = hidx(lane + 1, w + 1);
-  // halo ring cell owned by thread t < 2*TX + 2*MTY (corners are not needed)
-  // (the last threads build the halo ring; warps 0, 1 compute the far-edge faces)
+  const int me = hidx<MTX>(lane + 1, w + 1);
+  // halo ring cell owned by thread t >= MTX MTY - (2 MTX + 2 MTY) (corners
+  // are not needed): the last threads build the halo ring, the first ones
+  // compute the far-edge faces
   int hx = 0, hy = 0, hs = -1;
   bool hwx = false, hwy = false;
-  const int th = t - (MTY * TX - (2 * TX + 2 * MTY));
-  if (th >= 0 && th < TX) { hx = th + 1; hy = 0; hwx = true; }
-  else if (th >= TX && th < 2 * TX) { hx = th - TX + 1; hy = MTY + 1; hwx = true; }
-  else if (th >= 2 * TX && th < 2 * TX + MTY) { hx = 0; hy = th - 2 * TX + 1; hwy = true; }
-  else if (th >= 2 * TX + MTY && th < 2 * TX + 2 * MTY) { hx = TX + 1; hy = th - 2 * TX - MTY + 1; hwy = true; }
-  if (hwx || hwy) hs = hidx(hx, hy);
+  const int th = t - (MTY * MTX - (2 * MTX + 2 * MTY));
+  if (th >= 0 && th < MTX) { hx = th + 1; hy = 0; hwx = true; }
+  else if (th >= MTX && th < 2 * MTX) { hx = th - MTX + 1; hy = MTY + 1; hwx = true; }
+  else if (th >= 2 * MTX && th < 2 * MTX + MTY) { hx = 0; hy = th - 2 * MTX + 1; hwy = true; }
+  else if (th >= 2 * MTX + MTY && th < 2 * MTX + 2 * MTY) { hx = MTX + 1; hy = th - 2 * MTX - MTY + 1; hwy = true; }
+  if (hwx || hwy) hs = hidx<MTX>(hx, hy);
   const int hgx = min(x0 + hx - 1, g.nx), hgy = min(y0 + hy - 1, g.ny);
+  // far-edge face of thread t: t < MTX: +y face of the top tile row, column t;
+  // MTX <= t < MTX + MTY: +x face of the right tile column, row t - MTX.
+  // One code path for both (slots and tangential components per thread), so
+  // that a warp holding both kinds computes them in one pass.
+  const bool eyf = t < MTX, exf = t >= MTX && t < MTX + MTY;
+  const int ep = eyf ? hidx<MTX>(t + 1, MTY) : hidx<MTX>(MTX, t - MTX + 1);
+  const int eq = eyf ? hidx<MTX>(t + 1, MTY + 1) : hidx<MTX>(MTX + 1, t - MTX + 1);
+  const int ec1 = eyf ? D_CX : D_CY;
+  const int eo = eyf ? (MTY * MTX + t) : (t - MTX) * (MTX + 1) + MTX;  // flux slot (component 0)
+  double* const eout = eyf ? fys : fxs;
+  const int estr = eyf ? (MTY + 1) * MTX : MTY * (MTX + 1);           // component stride
 
   // z-face k-1/2 needs the previous plane's side (tangential: x, y)
   FaceSide Dp;
@@ -503,31 +597,40 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
       mu_face<L, TA>(P, Tk, p, s, Fy);
 #pragma unroll
       for (int i = 0; i < M; ++i) {
-        fxs[(i * MTY + w) * (TX + 1) + lane] = Fx[i];
-        fys[(i * (MTY + 1) + w) * TX + lane] = Fy[i];
+        fxs[(i * MTY + w) * (MTX + 1) + lane] = Fx[i];
+        fys[(i * (MTY + 1) + w) * MTX + lane] = Fy[i];
       }
-      if (w == 0) {  // +y face of the top tile edge, column `lane`
+      if constexpr (MTX == 32) {  // far tile edges in different warps: compile-time components
+        if (w == 0) {  // +y face of the top tile edge, column `lane`
+          double Fe[M];
+          side_from_smem<L, NC>(D, hidx<MTX>(lane + 1, MTY), D_CX, D_CZ, p);
+          side_from_smem<L, NC>(D, hidx<MTX>(lane + 1, MTY + 1), D_CX, D_CZ, s);
+          mu_face<L, TA>(P, Tk, p, s, Fe);
+#pragma unroll
+          for (int i = 0; i < M; ++i) fys[(i * (MTY + 1) + MTY) * MTX + lane] = Fe[i];
+        } else if (w == 1 && lane < MTY) {  // +x face of the right tile edge, row `lane`
+          double Fe[M];
+          side_from_smem<L, NC>(D, hidx<MTX>(MTX, lane + 1), D_CY, D_CZ, p);
+          side_from_smem<L, NC>(D, hidx<MTX>(MTX + 1, lane + 1), D_CY, D_CZ, s);
+          mu_face<L, TA>(P, Tk, p, s, Fe);
+#pragma unroll
+          for (int i = 0; i < M; ++i) fxs[(i * MTY + lane) * (MTX + 1) + MTX] = Fe[i];
+        }
+      } else if (eyf || exf) {  // both kinds in one warp: one pass
         double Fe[M];
-        side_from_smem<L, NC>(D, hidx(lane + 1, MTY), D_CX, D_CZ, p);
-        side_from_smem<L, NC>(D, hidx(lane + 1, MTY + 1), D_CX, D_CZ, s);
+        side_from_smem<L, NC>(D, ep, ec1, D_CZ, p);
+        side_from_smem<L, NC>(D, eq, ec1, D_CZ, s);
         mu_face<L, TA>(P, Tk, p, s, Fe);
 #pragma unroll
-        for (int i = 0; i < M; ++i) fys[(i * (MTY + 1) + MTY) * TX + lane] = Fe[i];
-      } else if (w == 1 && lane < MTY) {  // +x face of the right tile edge, row `lane`
-        double Fe[M];
-        side_from_smem<L, NC>(D, hidx(TX, lane + 1), D_CY, D_CZ, p);
-        side_from_smem<L, NC>(D, hidx(TX + 1, lane + 1), D_CY, D_CZ, s);
-        mu_face<L, TA>(P, Tk, p, s, Fe);
-#pragma unroll
-        for (int i = 0; i < M; ++i) fxs[(i * MTY + lane) * (TX + 1) + TX] = Fe[i];
+        for (int i = 0; i < M; ++i) eout[eo + i * estr] = Fe[i];
       }
     }
     if constexpr (!last) {
       __syncthreads();
 #pragma unroll
       for (int i = 0; i < M; ++i)
-        divxy[i] = (fxs[(i * MTY + w) * (TX + 1) + lane + 1] - fxs[(i * MTY + w) * (TX + 1) + lane]) +
-                   (fys[(i * (MTY + 1) + w + 1) * TX + lane] - fys[(i * (MTY + 1) + w) * TX + lane]);
+        divxy[i] = (fxs[(i * MTY + w) * (MTX + 1) + lane + 1] - fxs[(i * MTY + w) * (MTX + 1) + lane]) +
+                   (fys[(i * (MTY + 1) + w + 1) * MTX + lane] - fys[(i * (MTY + 1) + w) * MTX + lane]);
     }
   };
   for (int k = z0; k < z1; ++k) plane(BoolC<false>{}, k);

@@ -47,17 +47,17 @@ __global__ void __launch_bounds__(TX* MU_TY, MU_TY == 4 ? 3 : 16 / MU_TY) k_mu_t
 
 dim3 tuned_block() { return dim3(TX, TY); }
 dim3 tuned_block_phi(int pty) { return dim3(TX, pty); }
-dim3 tuned_block_mu(int mty) { return dim3(TX, mty); }
+dim3 tuned_block_mu(int mty, int mtx) { return dim3(mtx, mty); }
 dim3 tuned_grid_phi(const Geom& g, int pty, int zc) {
   if (zc <= 0) zc = ZC_PHI;
   return dim3((g.nx + TX - 1) / TX, (g.ny + pty - 1) / pty, (g.nz + zc - 1) / zc);
 }
-dim3 tuned_grid_mu(const Geom& g, int mty, int zc) {
+dim3 tuned_grid_mu(const Geom& g, int mty, int zc, int mtx) {
   if (zc <= 0) zc = ZC_MU;
-  return dim3((g.nx + TX - 1) / TX, (g.ny + mty - 1) / mty, (g.nz + zc - 1) / zc);
+  return dim3((g.nx + mtx - 1) / mtx, (g.ny + mty - 1) / mty, (g.nz + zc - 1) / zc);
 }
-size_t tuned_mu_smem(int mty) {
-  return (size_t)(D_NV * (TX + 2) * (mty + 2) + M * mty * (TX + 1) + M * (mty + 1) * TX) * sizeof(double);
+size_t tuned_mu_smem(int mty, int mtx) {
+  return (size_t)(D_NV * (mtx + 2) * (mty + 2) + M * mty * (mtx + 1) + M * (mty + 1) * mtx) * sizeof(double);
 }
 int tuned_mu_ty_default() { return MU_TY; }
 
