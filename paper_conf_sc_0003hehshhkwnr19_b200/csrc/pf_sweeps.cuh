@@ -445,14 +445,16 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
   const int me = hidx<MTX>(lane + 1, w + 1);
   // halo ring cell owned by thread t >= MTX MTY - (2 MTX + 2 MTY) (corners
   // are not needed): the last threads build the halo ring, the first ones
-  // compute the far-edge faces
+  // compute the far-edge faces.  The x-halo cells come first so that with
+  // 32-wide tiles each halo row is built by one whole warp (a warp's loads
+  // then touch the lines of one row, not of two rows and a column).
   int hx = 0, hy = 0, hs = -1;
   bool hwx = false, hwy = false;
   const int th = t - (MTY * MTX - (2 * MTX + 2 * MTY));
-  if (th >= 0 && th < MTX) { hx = th + 1; hy = 0; hwx = true; }
-  else if (th >= MTX && th < 2 * MTX) { hx = th - MTX + 1; hy = MTY + 1; hwx = true; }
-  else if (th >= 2 * MTX && th < 2 * MTX + MTY) { hx = 0; hy = th - 2 * MTX + 1; hwy = true; }
-  else if (th >= 2 * MTX + MTY && th < 2 * MTX + 2 * MTY) { hx = MTX + 1; hy = th - 2 * MTX - MTY + 1; hwy = true; }
+  if (th >= 0 && th < MTY) { hx = 0; hy = th + 1; hwy = true; }
+  else if (th >= MTY && th < 2 * MTY) { hx = MTX + 1; hy = th - MTY + 1; hwy = true; }
+  else if (th >= 2 * MTY && th < 2 * MTY + MTX) { hx = th - 2 * MTY + 1; hy = 0; hwx = true; }
+  else if (th >= 2 * MTY + MTX && th < 2 * MTY + 2 * MTX) { hx = th - 2 * MTY - MTX + 1; hy = MTY + 1; hwx = true; }
   if (hwx || hwy) hs = hidx<MTX>(hx, hy);
   const int hgx = min(x0 + hx - 1, g.nx), hgy = min(y0 + hy - 1, g.ny);
   // far-edge face of thread t: t < MTX: +y face of the top tile row, column t;
