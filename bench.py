@@ -121,14 +121,14 @@ def traffic_per_launch():
         return None
 
 
-def cpu_baseline(P, bc, seconds=12.0, shape=(64, 96, 96)):
+def cpu_baseline(P, bc, seconds=12.0, shape=(64, 96, 96), strong=False):
     """The oracle, as it stands, on the host cores (bounded sample)."""
     from oracle import oracle as O
     from paper_conf_sc_0003hehshhkwnr19_b200 import inputs as I
     O.build()
     cores = os.cpu_count() or 1
     O.set_threads(cores)
-    phi, mu = I.ic_lamellar(shape, seed=20191117)
+    phi, mu = I.ic_voronoi(shape, seed=20191117) if strong else I.ic_lamellar(shape, seed=20191117)
     o = O.Oracle(shape, P, bc)
     o.init(phi, mu)
     n = 0
@@ -142,8 +142,9 @@ def cpu_baseline(P, bc, seconds=12.0, shape=(64, 96, 96)):
     cells = shape[0] * shape[1] * shape[2]
     O.set_threads(0)
     return {"value": cells * n / el / 1e6, "unit": UNIT, "cores": cores, "kind": "oracle",
-            "sample": f"{n} step(s) of the config-2 workload on a {shape[2]}x{shape[1]}x{shape[0]} (x*y*z) "
-                      f"IC-L DS block, OpenMP over z on {cores} host threads, {el:.1f} s"}
+            "sample": f"{n} step(s) of the config-{4 if strong else 2} workload on a {shape[2]}x{shape[1]}x{shape[0]} "
+                      f"(x*y*z) {'IC-V periodic' if strong else 'IC-L DS'} block, OpenMP over z on {cores} host "
+                      f"threads, {el:.1f} s"}
 
 
 def run_reference(args, rank, world):
@@ -187,6 +188,9 @@ def main():
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--n", type=int, default=256, help="block edge per GPU")
+    ap.add_argument("--config", default="weak", choices=["weak", "strong"],
+                    help="weak: config 2/3 (n^3 DS block per GPU); strong: config 4 (fixed 512x512x1024 "
+                         "periodic domain, z-slabs)")
     ap.add_argument("--variant", default="jit", choices=["jit", "tuned", "naive"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
@@ -210,12 +214,20 @@ def main():
     if world > 1:
         import torch.distributed as dist
         dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
-    procs = grid_for(world)
+    strong = args.config == "strong"
     n = args.n
-    gshape = (n, n * procs[1], n * procs[0])  # (nz, ny, nx): growth axis z unsplit
-    P = I.params_c4("ds", window_check=10, window_frac=0.5)
-    z_front = n // 4
-    P["T0"] = I.ds_T0(z_front, P["G"])
+    if strong:  # config 4: fixed 512 x 512 x 1024 periodic domain in z-slabs, IC-V
+        procs = (1, 1, world)
+        gshape = (1024, 512, 512)
+        P = I.params_c4("periodic")
+        bc = I.BC_PERIODIC
+    else:  # configs 2/3: n^3 DS block per GPU, growth axis z unsplit
+        procs = grid_for(world)
+        gshape = (n, n * procs[1], n * procs[0])  # (nz, ny, nx)
+        P = I.params_c4("ds", window_check=10, window_frac=0.5)
+        z_front = n // 4
+        P["T0"] = I.ds_T0(z_front, P["G"])
+        bc = I.BC_DS
     uid = None
     if world > 1:
         t = torch.zeros(128, dtype=torch.uint8, device="cuda")
@@ -223,13 +235,31 @@ def main():
             t.copy_(torch.tensor(list(pf.nccl_unique_id()), dtype=torch.uint8))
         dist.broadcast(t, 0)
         uid = bytes(t.cpu().tolist())
-    g = pf.PhaseField(gshape, P, bc=I.BC_DS, procs=procs, rank=rank, world=world, device=local_rank, nccl_uid=uid)
+    g = pf.PhaseField(gshape, P, bc=bc, procs=procs, rank=rank, world=world, device=local_rank, nccl_uid=uid)
     g.set_variant(args.variant)
     lshape = g.local
-    phi, mu = I.ic_lamellar(lshape, seed=20191117 + rank, z_front=z_front)
-    phi_pin = torch.from_numpy(phi).pin_memory()
-    mu_pin = torch.from_numpy(mu).pin_memory()
-    g.init_fields(phi_pin, mu_pin)
+    if strong:
+        # IC-V on a 256^3 periodic tile (24 grains, S§8(d) density), tiled
+        # periodically over the global domain; this rank's slab
+        # (tiled on the device: the slab is up to 12.9 GB of fields)
+        tphi, tmu = I.ic_voronoi((256, 256, 256), seed=20191117)
+        dev = torch.device("cuda", local_rank)
+        z0 = g.offset[0]
+        iz = torch.tensor([(z0 + k) % 256 for k in range(lshape[0])], device=dev)
+        iy = torch.arange(lshape[1], device=dev) % 256
+        ix = torch.arange(lshape[2], device=dev) % 256
+        phi_d = torch.from_numpy(tphi).to(dev)[:, iz][:, :, iy][:, :, :, ix].contiguous()
+        mu_d = torch.from_numpy(tmu).to(dev)[:, iz][:, :, iy][:, :, :, ix].contiguous()
+        del tphi, tmu
+        g.init_fields(phi_d, mu_d)
+        del phi_d, mu_d
+        torch.cuda.empty_cache()
+        args.no_e2e = True  # no host copy of the slab (e2e is measured on the weak-scaling workload)
+    else:
+        phi, mu = I.ic_lamellar(lshape, seed=20191117 + rank, z_front=z_front)
+        phi_pin = torch.from_numpy(phi).pin_memory()
+        mu_pin = torch.from_numpy(mu).pin_memory()
+        g.init_fields(phi_pin, mu_pin)
     stream = g.stream
     cells_local = lshape[0] * lshape[1] * lshape[2]
 
@@ -286,10 +316,13 @@ def main():
     R = min(peak_tf * 1e12 / F_STEP, hbm * 1e9 / Q_STEP) / 1e6  # MLUP/s per GPU
     rec = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True, "scaling": "weak",
+        "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
+        "scaling": "strong" if strong else "weak",
         "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-        "config": {"workload": f"config 2: {n}^3 block per GPU, ternary eutectic N=4/K-1=2, frozen-T directional "
-                               f"solidification, moving window (check every 10 steps), IC-L, C.4 parameters",
+        "config": {"workload": ("config 4: fixed 512x512x1024 periodic domain in z-slabs, ternary eutectic "
+                                "N=4/K-1=2, IC-V (256^3 periodic tile), C.4 parameters") if strong else
+                               (f"config 2: {n}^3 block per GPU, ternary eutectic N=4/K-1=2, frozen-T directional "
+                                f"solidification, moving window (check every 10 steps), IC-L, C.4 parameters"),
                    "global_xyz": [gshape[2], gshape[1], gshape[0]], "procs_xyz": list(procs),
                    "parallelism": f"domain decomposition {procs[0]}x{procs[1]}x{procs[2]}",
                    "variant": args.variant,
@@ -298,7 +331,9 @@ def main():
         "step_roofline": {"R_mlups": R, "F_flop_per_cell": F_STEP, "Q_bytes_per_cell": Q_STEP,
                           "frac": (value / world) / R, "peak_fp64_tflops": peak_tf, "hbm_gbs": hbm},
         "roofline": {"bound": "alu", "kernel": "mu_sweep", "achieved": mu_tf, "peak": peak_tf, "unit": "TFLOP/s",
-                     "frac": (mu_tf / peak_tf) if mu_tf else None, "traffic": traffic_per_launch(),
+                     "frac": (mu_tf / peak_tf) if mu_tf else None,
+                     # the committed ncu capture is of the 256^3 block launch
+                     "traffic": traffic_per_launch() if cells_local == 256 ** 3 else None,
                      "flop_per_cell": F_MU, "cells_per_launch": cells_local,
                      "avg_launch_ms": mu_ms / mu_n if mu_n else None,
                      "peak_note": "derived: 148 SMs x 64 FP64 lanes x 2 x 1.965 GHz (DESIGN.md §6)"},
@@ -327,13 +362,13 @@ def main():
         f1.synchronize()
         barrier()
         ems = max_over_ranks(max(f0.elapsed_time(f1), (time.perf_counter() - t0) * 1e3))
-        bytes_state = (phi.nbytes + mu.nbytes)
+        bytes_state = (phi_pin.numel() + mu_pin.numel()) * 8
         rec["e2e"] = {"value": total_cells * args.steps / (ems * 1e-3) / 1e6, "unit": UNIT,
                       "h2d_bytes_per_step": bytes_state / args.steps, "d2h_bytes_per_step": bytes_state / args.steps,
                       "note": "one chunk = pf_init_fields from pinned host memory, K steps, pf_download to pinned "
                               "host memory, all inside the timed region"}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        rec["cpu_baseline"] = cpu_baseline(P, I.BC_DS)
+        rec["cpu_baseline"] = cpu_baseline(P, bc, strong=strong)
     if rank == 0:
         print(json.dumps(rec), flush=True)
     g.close()

@@ -35,6 +35,12 @@ namespace pf {
 #define PF_PHI_UNROLL 3
 #endif
 constexpr int kPhiUnroll = PF_PHI_UNROLL;
+#ifndef PF_MU_FXREG  // cell's own -x / -y face fluxes kept in registers for its divergence
+#define PF_MU_FXREG 0
+#endif
+#ifndef PF_MU_QREG  // own cell's D(k) kept in registers from the build (no shared-memory re-read)
+#define PF_MU_QREG 0
+#endif
 #ifndef PF_MU_RPF  // own cell's L1-missing loads issued one plane ahead into registers
 #define PF_MU_RPF 1
 #endif
@@ -325,10 +331,9 @@ template <int NC, class GT>
 __device__ __forceinline__ void build_own_carry(const GT& g, const double* __restrict__ ps,
                                                 const double* __restrict__ pd, const double* __restrict__ ms, int x,
                                                 int y, int k, bool wz, const double (&fm)[N], double (&fc)[N],
-                                                double* __restrict__ D, int i) {
+                                                double* __restrict__ D, int i, double (&v)[D_NV]) {
   const i64 F = g.field;
   const i64 c = g.at(x, y, k);
-  double v[D_NV];
 #pragma unroll
   for (int a = 0; a < N; ++a) {
     const double* f = ps + a * F + c;
@@ -355,10 +360,9 @@ __device__ __forceinline__ void build_own_rpf(const GT& g, const double* __restr
                                               const double* __restrict__ pd, const double* __restrict__ ms, int x,
                                               int y, int k, bool wz, const double (&fm)[N], double (&fc)[N],
                                               double (&nf)[N], double (&nd)[N], double (&nm)[M],
-                                              double* __restrict__ D, int i) {
+                                              double* __restrict__ D, int i, double (&v)[D_NV]) {
   const i64 F = g.field;
   const i64 c = g.at(x, y, k);
-  double v[D_NV];
 #pragma unroll
   for (int a = 0; a < N; ++a) {
     const double* f = ps + a * F + c;
@@ -537,10 +541,11 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
       asm volatile("prefetch.global.L1 [%0];" ::"l"(ms + F + ch));
     }
     // (a) publish D(k) of the own cell and of the halo ring
+    double vo[D_NV];  // own cell's D(k) (kept in registers with PF_MU_QREG)
 #if PF_MU_RPF
-    build_own_rpf<NC>(g, ps, pd, ms, xc, yc, k, !last, Dp.f, fcar, rnf, rnd, rnm, D, me);
+    build_own_rpf<NC>(g, ps, pd, ms, xc, yc, k, !last, Dp.f, fcar, rnf, rnd, rnm, D, me, vo);
 #elif PF_MU_ZCARRY
-    build_own_carry<NC>(g, ps, pd, ms, xc, yc, k, !last, Dp.f, fcar, D, me);
+    build_own_carry<NC>(g, ps, pd, ms, xc, yc, k, !last, Dp.f, fcar, D, me, vo);
 #else
     build_cell<NC>(g, ps, pd, ms, xc, yc, k, true, true, !last, D, me);
 #endif
@@ -548,7 +553,20 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
     __syncthreads();
     // (b) z-face k-1/2 from registers (plane k-1) and shared memory (plane k)
     FaceSide q;
+#if PF_MU_QREG && (PF_MU_RPF || PF_MU_ZCARRY)
+#pragma unroll
+    for (int a = 0; a < N; ++a) {
+      q.f[a] = vo[D_F + a];
+      q.c1[a] = vo[D_CX + a];
+      q.c2[a] = vo[D_CY + a];
+    }
+#pragma unroll
+    for (int u = 0; u < NSOL; ++u) q.ds[u] = vo[D_DP + solid_phase(L, u)];
+    q.m[0] = vo[D_MU];
+    q.m[1] = vo[D_MU + 1];
+#else
     side_from_smem<L, NC>(D, me, D_CX, D_CY, q);
+#endif
     double Fz[M];
     mu_face<L, TA>(P, plane_T(P, R, k - 0.5), Dp, q, Fz);
     // (c) cell update of plane k-1
@@ -569,19 +587,28 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
     Fzm[1] = Fz[1];
     // carry plane k's side for the next z-face
     Dp = q;
+#if PF_MU_QREG && (PF_MU_RPF || PF_MU_ZCARRY)
+    dpl = vo[D_DP + L];
+#else
     dpl = D[(size_t)me * D_NV + D_DP + L];
+#endif
+    double Fx[M], Fy[M];  // -x / -y face fluxes of the own cell, plane k
     if constexpr (!last) {
       // (d) faces of plane k: -x and -y of every thread, + the far tile edges
       const double Tk = plane_T(P, R, (double)k);
       // (the own side is Dp = plane k's {f, cx, cy, ds, mu}, already in
       // registers: only its cz comes from shared memory)
       FaceSide p, s;
-      double Fx[M], Fy[M];
+#if PF_MU_QREG && (PF_MU_RPF || PF_MU_ZCARRY)
+#pragma unroll
+      for (int a = 0; a < N; ++a) s.c2[a] = vo[D_CZ + a];
+#else
       {
         const double2* d = reinterpret_cast<const double2*>(D + (size_t)me * D_NV + D_CZ);
         const double2 z01 = d[0], z23 = d[1];
         s.c2[0] = z01.x; s.c2[1] = z01.y; s.c2[2] = z23.x; s.c2[3] = z23.y;
       }
+#endif
 #pragma unroll
       for (int a = 0; a < N; ++a) {
         s.f[a] = Dp.f[a];
@@ -631,8 +658,12 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
       __syncthreads();
 #pragma unroll
       for (int i = 0; i < M; ++i)
+#if PF_MU_FXREG  // own -x / -y fluxes from registers, only the +x / +y ones from shared memory
+        divxy[i] = (fxs[(i * MTY + w) * (MTX + 1) + lane + 1] - Fx[i]) + (fys[(i * (MTY + 1) + w + 1) * MTX + lane] - Fy[i]);
+#else
         divxy[i] = (fxs[(i * MTY + w) * (MTX + 1) + lane + 1] - fxs[(i * MTY + w) * (MTX + 1) + lane]) +
                    (fys[(i * (MTY + 1) + w + 1) * MTX + lane] - fys[(i * (MTY + 1) + w) * MTX + lane]);
+#endif
     }
   };
   for (int k = z0; k < z1; ++k) plane(BoolC<false>{}, k);
