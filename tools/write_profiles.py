@@ -15,7 +15,7 @@ import sys
 src, tag = sys.argv[1], sys.argv[2]
 dst = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles")
 os.makedirs(dst, exist_ok=True)
-for name, out in (("bench.json", f"{tag}_bench.json"), ("launches.csv", f"{tag}_launches.csv"),
+for name, out in (("bench.json", f"{tag}_bench.json"), ("bench_strong.json", f"{tag}_bench_strong.json"), ("launches.csv", f"{tag}_launches.csv"),
                   ("fp64_micro.json", f"{tag}_fp64_micro.json"), ("pytest_gpu.log", f"{tag}_pytest_gpu.log"),
                   ("smoke.log", f"{tag}_smoke.log"), ("nvidia-smi.txt", f"{tag}_nvidia-smi.txt")):
     p = os.path.join(src, name)
