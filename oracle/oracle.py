@@ -42,6 +42,7 @@ class OrParams(C.Structure):
         ("mu_inf", C.c_double * MAXM),
         ("window_frac", C.c_double), ("window_check", C.c_int),
         ("antitrapping", C.c_int), ("projection", C.c_int),
+        ("xi_amp", C.c_double), ("xi_seed", C.c_uint),
     ]
 
 
@@ -89,6 +90,9 @@ def lib():
         L.oracle_phi_rhs.argtypes = [C.c_void_p, dp]
         L.oracle_project_simplex.argtypes = [C.c_int, dp, dp]
         L.oracle_front_height.argtypes = [C.c_void_p]
+        u4 = C.POINTER(C.c_uint)
+        L.oracle_philox4x32_10.argtypes = [u4, u4, u4]
+        L.oracle_xi_uniforms.argtypes = [C.c_int, C.c_int, C.c_int, C.c_int64, C.c_uint, dp]
         L.oracle_footprint.argtypes = [C.c_void_p, C.c_int, C.c_int, C.c_int, C.c_int, C.POINTER(C.c_int)]
         _lib = L
     return _lib
@@ -130,7 +134,25 @@ def make_params(P: dict) -> OrParams:
     p.window_check = int(P.get("window_check", 0))
     p.antitrapping = int(P.get("antitrapping", 1))
     p.projection = int(P.get("projection", 1))
+    p.xi_amp = float(P.get("xi_amp", 0.0))
+    p.xi_seed = int(P.get("xi_seed", 0)) & 0xFFFFFFFF
     return p
+
+
+def philox4x32_10(ctr, key):
+    """Philox4x32-10 of the oracle (fluctuation term RNG)."""
+    c = (C.c_uint * 4)(*[int(v) & 0xFFFFFFFF for v in ctr])
+    k = (C.c_uint * 2)(*[int(v) & 0xFFFFFFFF for v in key])
+    o = (C.c_uint * 4)()
+    lib().oracle_philox4x32_10(c, k, o)
+    return tuple(int(v) for v in o)
+
+
+def xi_uniforms(x, y, z, step, seed) -> np.ndarray:
+    """The four uniforms in (-1, 1) of cell (x, y, z) at step n (reading B4)."""
+    out = np.empty(4)
+    lib().oracle_xi_uniforms(int(x), int(y), int(z), int(step), int(seed) & 0xFFFFFFFF, _dp(out))
+    return out
 
 
 def project_simplex(x) -> np.ndarray:

@@ -265,6 +265,44 @@ static void phi_rhs_cell(const pf_oracle* o, int x, int y, int z, double* r) {
   }
 }
 
+/* ------------------------------------------------------------------------ */
+/* Fluctuation term (eq. 7 "+ xi", listing P:L490-495: fluctuation =
+ * amplitude * random(-1, 1, kind='philox'); "the counter-based
+ * random number generator Philox [31] ... The global cell index and current
+ * time step are used as counters/keys").  Reading B4:
+ * counter = (x, y, z, step mod 2^32), key = (seed, step / 2^32); the four
+ * 32-bit words u_a give U_a = (u_a + 1/2) 2^-31 - 1 in (-1, 1) (exact in
+ * fp64) for phases a = 0..N-1.                                              */
+/* ------------------------------------------------------------------------ */
+static unsigned int mulhilo32(unsigned int a, unsigned int b, unsigned int* hi) {
+  const unsigned long long p = (unsigned long long)a * (unsigned long long)b;
+  *hi = (unsigned int)(p >> 32);
+  return (unsigned int)p;
+}
+
+void oracle_philox4x32_10(const unsigned int ctr[4], const unsigned int key[2], unsigned int out[4]) {
+  unsigned int c0 = ctr[0], c1 = ctr[1], c2 = ctr[2], c3 = ctr[3];
+  unsigned int k0 = key[0], k1 = key[1];
+  for (int round = 0; round < 10; ++round) {
+    unsigned int hi0, hi1;
+    const unsigned int lo0 = mulhilo32(0xD2511F53u, c0, &hi0);
+    const unsigned int lo1 = mulhilo32(0xCD9E8D57u, c2, &hi1);
+    const unsigned int n0 = hi1 ^ c1 ^ k0, n1 = lo1, n2 = hi0 ^ c3 ^ k1, n3 = lo0;
+    c0 = n0; c1 = n1; c2 = n2; c3 = n3;
+    k0 += 0x9E3779B9u; /* Weyl sequence key schedule */
+    k1 += 0xBB67AE85u;
+  }
+  out[0] = c0; out[1] = c1; out[2] = c2; out[3] = c3;
+}
+
+void oracle_xi_uniforms(int x, int y, int z, int64_t n, unsigned int seed, double U[4]) {
+  const unsigned int ctr[4] = {(unsigned int)x, (unsigned int)y, (unsigned int)z, (unsigned int)(uint64_t)n};
+  const unsigned int key[2] = {seed, (unsigned int)((uint64_t)n >> 32)};
+  unsigned int u[4];
+  oracle_philox4x32_10(ctr, key, u);
+  for (int a = 0; a < 4; ++a) U[a] = ((double)u[a] + 0.5) * (1.0 / 2147483648.0) - 1.0;
+}
+
 /* C.1 S2 steps 6-8 for one cell: tau, Euler + Lagrange multiplier, projection */
 static void phi_update_cell(pf_oracle* o, int x, int y, int z) {
   const or_params* p = &o->p;
@@ -288,7 +326,14 @@ static void phi_update_cell(pf_oracle* o, int x, int y, int z) {
   for (int b = 0; b < N; ++b) rs += r[b];
   double lam = rs / (double)N;
   double f = p->dt / (tau * p->eps);
-  for (int a = 0; a < N; ++a) xs[a] = ph[a] + f * (-r[a] + lam);
+  /* fluctuation xi_a (eq. 7) [B4]; 0 when off [A17] */
+  double xi[OR_MAXN] = {0.0, 0.0, 0.0, 0.0};
+  if (p->xi_amp != 0.0) {
+    double U[4];
+    oracle_xi_uniforms(x, y, z, o->st.step, p->xi_seed, U);
+    for (int a = 0; a < N; ++a) xi[a] = p->xi_amp * U[a];
+  }
+  for (int a = 0; a < N; ++a) xs[a] = ph[a] + f * (-r[a] + lam + xi[a]);
   /* 8. Gibbs-simplex projection [A14, A25] */
   if (p->projection)
     oracle_project_simplex(N, xs, out);

@@ -47,6 +47,11 @@ typedef struct {
   /* debug switches */
   int antitrapping; /* 1 = eq. 10 on (default), 0 = off                    */
   int projection;   /* 1 = Gibbs-simplex projection on (default), 0 = off  */
+  /* fluctuation term xi of eq. 7, reading B4:
+   * xi_a = xi_amp * U_a, U_a uniform in (-1, 1) from Philox4x32-10 keyed by
+   * the global cell index and the time step; 0 = off (reading A17)        */
+  double xi_amp;
+  unsigned int xi_seed;
 } or_params;
 
 typedef struct {
@@ -78,6 +83,11 @@ void oracle_set_threads(int n); /* OpenMP threads for timing only; 0 = serial */
 int oracle_phi_rhs(pf_oracle* o, double* r);
 /* Euclidean projection onto the Gibbs simplex (reading A14)               */
 void oracle_project_simplex(int N, const double* x, double* out);
+/* Philox4x32-10 (Salmon et al., SC'11), the counter-based RNG of P:L669-676:
+ * out = the 10-round bijection of counter ctr under key key.               */
+void oracle_philox4x32_10(const unsigned int ctr[4], const unsigned int key[2], unsigned int out[4]);
+/* The four uniforms U in (-1, 1) of cell (x, y, z) at step n (reading B4). */
+void oracle_xi_uniforms(int x, int y, int z, int64_t n, unsigned int seed, double U[4]);
 /* front height H of S6 (-1 if no solid cell) */
 int oracle_front_height(const pf_oracle* o);
 /* Table-1 footprint (pin P14): which = 0 phi-full, 1 phi-flux, 2 phi-cell,

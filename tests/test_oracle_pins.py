@@ -660,3 +660,95 @@ def test_window_auto_trigger(oracle_mod):
     o.step(2)
     st = o.state()
     assert st["z_off"] > 0 and o.front_height() <= 8
+
+
+# --------------------------------------------------------------------------
+# Fluctuation term xi (eq. 7 "+ xi(phi)", listing P:L490-495:
+# fluctuation = amplitude * random(-1, 1, kind='philox'); RNG P:L669-676),
+# reading B4: xi_a = A U_a, U_a = (u_a + 1/2) 2^-31 - 1 from Philox4x32-10
+# with counter (x, y, z, step) and key (seed, step >> 32).
+# --------------------------------------------------------------------------
+def _kat():
+    rows = []
+    for ln in open(os.path.join(GOLDEN, "philox4x32_10_kat.txt")):
+        if ln.strip() and not ln.startswith("#"):
+            w = [int(t, 16) for t in ln.split()]
+            rows.append((w[0:4], w[4:6], tuple(w[6:10])))
+    return rows
+
+
+def test_xi_philox_known_answers(oracle_mod):
+    """The oracle's Philox4x32-10 reproduces the published known-answer vectors."""
+    for ctr, key, out in _kat():
+        assert oracle_mod.philox4x32_10(ctr, key) == out
+
+
+def test_xi_uniforms_distribution(oracle_mod):
+    """U in (-1, 1): mean 0, variance 1/3, the four phases uncorrelated, a new
+    draw every step (counter = cell and step)."""
+    rng = np.random.default_rng(5)
+    cells = rng.integers(0, 400, size=(4000, 3))
+    U = np.array([oracle_mod.xi_uniforms(x, y, z, 7, 20191117) for x, y, z in cells])
+    assert np.all(np.abs(U) < 1.0)
+    assert np.abs(U.mean(0)).max() < 0.04
+    assert np.abs(U.var(0) - 1.0 / 3.0).max() < 0.03
+    C = np.corrcoef(U.T)
+    assert np.abs(C - np.eye(4)).max() < 0.06
+    V = np.array([oracle_mod.xi_uniforms(x, y, z, 8, 20191117) for x, y, z in cells])
+    assert np.abs(np.corrcoef(U[:, 0], V[:, 0])[0, 1]) < 0.06
+    # the mapping of the 32-bit words: u = 0 -> -1 + 2^-32, u = 2^32 - 1 -> 1 - 2^-32
+    words = oracle_mod.philox4x32_10((3, 4, 5, 6), (99, 0))
+    expect = np.array([(w + 0.5) / 2.0 ** 31 - 1.0 for w in words])
+    assert np.array_equal(oracle_mod.xi_uniforms(3, 4, 5, 6, 99), expect)
+
+
+def test_xi_enters_the_euler_step(oracle_mod):
+    """With all tau_ab equal (tau = tau0 exactly) and no projection, one step
+    with amplitude A differs from the step without noise by exactly
+    dt/(tau0 eps) A U_a(x, y, z, n=0) per phase (the noise is added to the
+    right-hand side of eq. 7, outside the Lagrange multiplier)."""
+    shape = (5, 6, 7)
+    P = I.params_stress()
+    P["tau"] = np.full((4, 4), 1.7)
+    phi, mu = I.ic_voronoi(shape, seed=9)
+    outs = []
+    for A in (0.0, 0.05):
+        o = oracle_mod.Oracle(shape, dict(P, projection=0, xi_amp=A, xi_seed=77))
+        o.init(phi, mu)
+        o.step_phi_only()
+        outs.append(o.download()[0])
+    f = P["dt"] / (1.7 * P["eps"])
+    z, y, x = np.meshgrid(range(shape[0]), range(shape[1]), range(shape[2]), indexing="ij")
+    U = np.array([oracle_mod.xi_uniforms(a, b, c, 0, 77) for a, b, c in zip(x.ravel(), y.ravel(), z.ravel())])
+    U = U.T.reshape((4,) + shape)
+    assert np.abs((outs[1] - outs[0]) - f * 0.05 * U).max() < 1e-15
+
+
+def test_xi_invariants_and_bulk(oracle_mod):
+    """With noise: sum phi = 1 and phi >= 0 every step (P2); an amplitude
+    below the obstacle margin keeps bulk cells bitwise pure (P3): in a pure
+    cell the other phases receive dt/(tau eps) (mean r - r_b + xi_b) < 0
+    when A < (16 gamma / pi^2)/(4 eps) (eq. 5)."""
+    shape = (24, 24, 24)
+    P = I.params_c4()
+    phi, mu = I.ic_voronoi(shape, seed=3, nseeds=3, blur=1)
+    A = 0.5 * (16.0 / np.pi ** 2) / (4.0 * P["eps"])
+    o = oracle_mod.Oracle(shape, dict(P, xi_amp=A, xi_seed=5))
+    o.init(phi, mu)
+    for _ in range(3):
+        o.step(1)
+        p, _ = o.download()
+        assert np.abs(p.sum(0) - 1.0).max() <= 8 * 2.2e-16
+        assert p.min() >= 0.0
+    pure0 = phi.max(0) == 1.0
+    far = pure0.copy()
+    for ax in (0, 1, 2):
+        for s in range(1, 5):
+            far &= np.roll(pure0, s, ax) & np.roll(pure0, -s, ax)
+    assert far.sum() > 100
+    assert np.array_equal(p[:, far], phi[:, far])
+    # and the noise does act in the interfaces
+    o2 = oracle_mod.Oracle(shape, P)
+    o2.init(phi, mu)
+    o2.step(3)
+    assert np.abs(o2.download()[0] - p).max() > 1e-4
