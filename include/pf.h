@@ -112,6 +112,13 @@ typedef struct {
   double mu_inf[PF_M];                 /* inflow / Dirichlet value of mu           */
   double window_frac;                  /* moving window threshold fraction [A16]   */
   int window_check;                    /* check every n steps; 0 = window off      */
+  /* Fluctuation term xi of eq. 7 (RNG P:L669-676), reading B4:
+   * xi_a = xi_amp * U_a, U_a in (-1, 1) from Philox4x32-10 with counter
+   * (global x, y, z, step mod 2^32) and key (xi_seed, step / 2^32), added to
+   * the right-hand side of the phi equation outside the Lagrange multiplier.
+   * xi_amp = 0: off (reading A17).  xi_amp >= 0 and finite.                  */
+  double xi_amp;
+  uint32_t xi_seed;
 } pf_params;
 
 typedef struct {

@@ -176,7 +176,7 @@ int layout_of(const pf_config* cfg, pf_layout* L, int coord[3]) {
   L->phi_bytes = (size_t)PF_N * L->field * sizeof(double) + 256;  // +256: tail slack for vector loads
   L->mu_bytes = (size_t)PF_M * L->field * sizeof(double) + 256;
   size_t ws = 256;  // reduction scratch
-  Geom g{nx, ny, nz, L->offset[2], L->pitch, L->plane, L->field, L->x_off};
+  Geom g{nx, ny, nz, L->offset[2], L->pitch, L->plane, L->field, L->x_off, L->offset[0], L->offset[1]};
   for (int d = 0; d < 3; ++d) ws += 4 * align256(halo_slab_elems(g, d) * PF_N * sizeof(double));
   L->workspace_bytes = ws;
   return PF_OK;
@@ -331,6 +331,8 @@ void fill_dev_params(const pf_params& pr, int L, DevParams* out) {
   }
   D.liquid = L;
   D.TA = ta ? 1 : 0;
+  D.xi_amp = p->xi_amp;
+  D.xi_seed = p->xi_seed;
 }
 }  // namespace pf
 
@@ -377,7 +379,8 @@ int pf_create(const pf_config* cfg, pf_ctx** out) {
     return PF_EINVAL;
   }
   const pf_layout& L = ctx->lay;
-  ctx->g = Geom{L.local[0], L.local[1], L.local[2], L.offset[2], L.pitch, L.plane, L.field, L.x_off};
+  ctx->g = Geom{L.local[0], L.local[1], L.local[2], L.offset[2], L.pitch, L.plane, L.field, L.x_off,
+                L.offset[0], L.offset[1]};
   for (int d = 0; d < 3; ++d) {
     const int blo = cfg->bc_lo[d], bhi = cfg->bc_hi[d];
     if (blo < 0 || blo > 2 || bhi < 0 || bhi > 2 || ((blo == PF_BC_PERIODIC) != (bhi == PF_BC_PERIODIC))) {
@@ -520,6 +523,8 @@ int pf_set_params(pf_ctx* ctx, const pf_params* p) {
           return fail(ctx, PF_EINVAL, "gamma3 must be symmetric");
   if (p->window_check < 0 || (p->window_check > 0 && !(p->window_frac > 0 && p->window_frac < 1)))
     return fail(ctx, PF_EINVAL, "window_check >= 0 and 0 < window_frac < 1");
+  if (!(std::isfinite(p->xi_amp) && p->xi_amp >= 0.0))
+    return fail(ctx, PF_EINVAL, "xi_amp must be finite and >= 0");
   // T range over the global domain at t = 0 (frozen gradient; window keeps it bounded)
   const double zmax = (double)ctx->cfg.global[2];
   const double Ts[2] = {p->T0 - fabs(p->G) * p->dx, p->T0 + fabs(p->G) * (zmax + 1) * p->dx};
@@ -710,6 +715,7 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
   // frozen temperature of this step: T(k) = T0 + G ((k + z0 + z_off) dx - v t_n), t_n = step dt  [A13]
   const double t = (double)ctx->step * ctx->hp.dt;
   ctx->dp.Tbase = ctx->hp.T0 + ctx->hp.G * (((double)g.z0 + (double)ctx->z_off) * ctx->hp.dx - ctx->hp.v * t);
+  ctx->dp.step = (unsigned long long)ctx->step;  // fluctuation counter [B4]
   cudaEvent_t e0 = nullptr;
   if (ctx->variant == PF_VARIANT_JIT && !ctx->jit) {
     std::string err;

@@ -24,6 +24,7 @@ struct Geom {
   int nx, ny, nz;
   int z0;  // global z index of local interior plane 0
   i64 pitch, plane, field, xoff;
+  int x0, y0;  // global x / y index of local interior cell 0 (fluctuation counters)
   __host__ __device__ __forceinline__ i64 at(int x, int y, int z) const {
     return (i64)(z + GUARD) * plane + (i64)(y + GUARD) * pitch + xoff + x;
   }
@@ -70,6 +71,10 @@ struct DevParams {
   double dcT[N][5];     // dc_a/dT = -(A1 + A1^T) mu - B1: [s00, s01, s11, -B1_0, -B1_1]
   int liquid;
   int TA;               // A1 != 0: chi and the mobility depend on T
+  // fluctuation term (eq. 7) [B4]; per-step: step
+  double xi_amp;        // 0 = off
+  unsigned int xi_seed;
+  unsigned long long step;  // time step n of the launch (Philox counter / key)
 };
 
 // Compile-time structure of a parameter set, known only to the specialised
@@ -81,6 +86,7 @@ template <class PT>
 struct ParamShape {
   static constexpr bool guni = false;   // gamma_ab uniform
   static constexpr bool g3uni = false;  // gamma_abd uniform
+  static constexpr bool xi = true;      // fluctuation term compiled in (run-time amplitude, may be 0)
 };
 
 }  // namespace pf

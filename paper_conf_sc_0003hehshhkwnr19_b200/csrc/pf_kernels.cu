@@ -63,7 +63,9 @@ __global__ void __launch_bounds__(256) k_phi_naive(DevParams P, Geom g, const do
   }
   const double mu0 = __ldg(ms + c), mu1 = __ldg(ms + F + c);
   double out[N];
-  phi_cell<TA>(P, plane_T(P, P, (double)z), ph, gd, divh, mu0, mu1, out);
+  double xi[N];
+  xi_of(P, P.step, x + g.x0, y + g.y0, z + g.z0, xi);
+  phi_cell<TA>(P, plane_T(P, P, (double)z), ph, gd, divh, mu0, mu1, xi, out);
 #pragma unroll
   for (int a = 0; a < N; ++a) pd[a * F + c] = out[a];
 }

@@ -144,8 +144,9 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, 
 #pragma unroll
       for (int a = 0; a < N; ++a) divh[a] += Fzp[a] - Fzm[a];
       const double mu0 = __ldg(ms + c), mu1 = __ldg(ms + F + c);
-      double out[N];
-      phi_cell<TA>(P, plane_T(P, R, (double)z), p0, gd, divh, mu0, mu1, out);
+      double out[N], xi[N];
+      if constexpr (ParamShape<PT>::xi) xi_of(P, R.step, x + g.x0, y + g.y0, z + g.z0, xi);
+      phi_cell<TA>(P, plane_T(P, R, (double)z), p0, gd, divh, mu0, mu1, xi, out);
 #pragma unroll
       for (int a = 0; a < N; ++a) pd[a * F + c] = out[a];
 #pragma unroll
@@ -248,8 +249,9 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, 
       const double fyp = (w < PTY - 1) ? fy[buf][a][w + 1][lane] : ey[buf][a][lane];
       divh[a] = ((fxp - Fxm[a]) + (fyp - Fym[a])) + (Fzp[a] - Fzm[a]);
     }
-    double out[N];
-    phi_cell<TA>(P, plane_T(P, R, (double)z), p0, gd, divh, mu0, mu1, out);
+    double out[N], xi[N];
+    if constexpr (ParamShape<PT>::xi) xi_of(P, R.step, x + g.x0, y + g.y0, z + g.z0, xi);
+    phi_cell<TA>(P, plane_T(P, R, (double)z), p0, gd, divh, mu0, mu1, xi, out);
     if (active) {
 #pragma unroll
       for (int a = 0; a < N; ++a) pd[a * F + c] = out[a];

@@ -47,7 +47,8 @@ class PFParams(C.Structure):
                 ("C0", C.c_double * N), ("C1", C.c_double * N),
                 ("D", C.c_double * M * M * N),
                 ("T0", C.c_double), ("G", C.c_double), ("v", C.c_double),
-                ("mu_inf", C.c_double * M), ("window_frac", C.c_double), ("window_check", C.c_int)]
+                ("mu_inf", C.c_double * M), ("window_frac", C.c_double), ("window_check", C.c_int),
+                ("xi_amp", C.c_double), ("xi_seed", C.c_uint32)]
 
 
 class PFState(C.Structure):
@@ -132,6 +133,8 @@ def make_params(P: dict) -> PFParams:
     put(p.mu_inf, P["mu_inf"], (M,))
     p.window_frac = float(P.get("window_frac", 0.5))
     p.window_check = int(P.get("window_check", 0))
+    p.xi_amp = float(P.get("xi_amp", 0.0))
+    p.xi_seed = int(P.get("xi_seed", 0)) & 0xFFFFFFFF
     return p
 
 

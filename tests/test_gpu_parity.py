@@ -134,6 +134,41 @@ def test_ds_window_parity(pfmod, omod):
     assert res[-1][3]["z_off"] > 0
 
 
+# Fluctuation term xi of eq. 7 (NEXT-3, Philox P:L669-676),
+# reading B4: both sides draw the same Philox4x32-10 uniforms per cell/step.
+@pytest.mark.parametrize("variant", ["jit", "tuned", "naive"])
+@pytest.mark.parametrize("pset", ["c4", "stress"])
+def test_fluctuation_parity(pfmod, omod, variant, pset):
+    P = I.params_c4() if pset == "c4" else I.params_stress()
+    P = dict(P, xi_amp=0.05, xi_seed=20191117)
+    shape = (20, 24, 40)
+    res = run_pair(pfmod, omod, shape, P, "V", 20, variant=variant, chunks=[1, 2, 20])
+    for t, ep, em, *_ in res:
+        tol = TOL_1 if t == 1 else 1e-11
+        assert ep <= tol and em <= tol, (t, ep, em)
+
+
+def test_fluctuation_ds_window_and_reproducible(pfmod, omod):
+    """xi with the DS boundary conditions, frozen T and window shifts (global
+    z counter = lattice index), 1000-step bar, and bitwise run-to-run."""
+    P = I.params_c4("ds", window_check=5, window_frac=0.5, v=0.05, xi_amp=0.03, xi_seed=7)
+    P["T0"] = I.ds_T0(20, P["G"])
+    shape = (32, 12, 16)
+    res = run_pair(pfmod, omod, shape, P, "L", 200, bc=I.BC_DS, chunks=[1, 200], ic_kw={"z_front": 20})
+    for t, ep, em, gs, os_ in res:
+        assert gs == os_
+        tol = TOL_1 if t == 1 else TOL_1000
+        assert ep <= tol and em <= tol, (t, ep, em)
+    phi, mu = I.ic_lamellar(shape, seed=20191117, z_front=20)
+    outs = []
+    for _ in range(2):
+        g = pfmod.PhaseField(shape, P, bc=I.BC_DS)
+        g.init_fields(phi, mu)
+        g.step(30)
+        outs.append(g.download())
+    assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
+
+
 def test_step_phi_only(pfmod, omod):
     P = I.params_stress()
     shape = (12, 10, 14)

@@ -1,0 +1,135 @@
+"""Config 5 of BASELINE.json on ONE B200: the 400 x 400 x 2000 directional-
+solidification run (ternary eutectic, frozen temperature, moving window) for
+20k steps, with the lamellae and sum(phi) = 1 checks of SURVEY §8(c)-C.3 P16
+every 1,000 steps.  (BASELINE.json names 8 GPUs; the whole domain, 32 GB of
+state, fits one 180 GB B200, so it runs here as a single block.)
+
+P16 is "parity unpinned": the paper prints no data for this run, so the
+checks are qualitative (S§8(c)-C.3): in the x-y slice 20 cells below the
+front all three solids are present and their area fractions are within
++-0.1 of the lever rule of the C.4 diagram; max|sum(phi) - 1| <= 8 ulp-ish
+(1e-14) and min(phi) >= 0 over the whole domain, every check.
+
+    python tools/config5.py [--steps 20000] [--check 1000] [--out gpurun_out/config5.jsonl]
+
+The IC is IC-L (S§8(c)-C.5) built on the device without the interface noise
+(an x-y Voronoi of the three solids in lever-rule proportions extruded below
+z_front = nz/4, liquid above, 3 box-blur passes), because the host copy of
+the 15 GB field set is not needed.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+from paper_conf_sc_0003hehshhkwnr19_b200 import inputs as I  # noqa: E402
+from paper_conf_sc_0003hehshhkwnr19_b200 import pf  # noqa: E402
+
+
+def ic_lamellar_device(shape, seed, z_front, dev):
+    """IC-L on the device (no noise): same construction as inputs.ic_lamellar."""
+    nz, ny, nx = shape
+    rng = np.random.default_rng(seed)
+    ngrains = max(3, int(round(nx * ny / 400.0)))
+    seeds2 = np.stack([np.zeros(ngrains), rng.uniform(0, ny, ngrains), rng.uniform(0, nx, ngrains)], 1)
+    lab2 = I._nearest_seed((1, ny, nx), seeds2)[0]
+    solid_of = rng.choice(3, size=ngrains, p=I.LEVER / I.LEVER.sum())
+    sl = torch.from_numpy(solid_of[lab2]).to(dev)
+    phi = torch.zeros((4, nz, ny, nx), dtype=torch.float64, device=dev)
+    for a in range(3):
+        phi[a, :z_front] = (sl == a).to(torch.float64)[None]
+    phi[I.LIQUID, z_front:] = 1.0
+    for _ in range(3):
+        for ax in (2, 3):
+            phi = (phi + torch.roll(phi, 1, dims=ax) + torch.roll(phi, -1, dims=ax)) / 3.0
+        up = torch.cat([phi[:, :1], phi[:, :-1]], dim=1)
+        dn = torch.cat([phi[:, 1:], phi[:, -1:]], dim=1)
+        phi = (up + phi + dn) / 3.0
+        del up, dn
+    mu = torch.zeros((2, nz, ny, nx), dtype=torch.float64, device=dev)
+    return phi.contiguous(), mu
+
+
+def lamellae(phi_slice):
+    """Solid area fractions of an x-y slice (phases 0..2), normalised to the solid total."""
+    s = phi_slice[:3].sum(dim=(1, 2))
+    tot = float(s.sum())
+    return [float(v) / tot for v in s] if tot > 0 else [0.0, 0.0, 0.0]
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--shape", default="2000,400,400", help="nz,ny,nx")
+    ap.add_argument("--steps", type=int, default=20000)
+    ap.add_argument("--check", type=int, default=1000)
+    ap.add_argument("--below", type=int, default=20)
+    ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "config5.jsonl"))
+    args = ap.parse_args()
+    shape = tuple(int(v) for v in args.shape.split(","))
+    nz = shape[0]
+    dev = torch.device("cuda", 0)
+    torch.cuda.set_device(dev)
+    z_front = nz // 4
+    P = I.params_c4("ds", window_check=10, window_frac=0.5)
+    P["T0"] = I.ds_T0(z_front, P["G"])
+    g = pf.PhaseField(shape, P, bc=I.BC_DS, device=0)
+    phi, mu = ic_lamellar_device(shape, 20191117, z_front, dev)
+    g.init_fields(phi, mu)
+    del phi, mu
+    torch.cuda.empty_cache()
+    os.makedirs(os.path.dirname(args.out), exist_ok=True)
+    out = open(args.out, "w")
+    cells = shape[0] * shape[1] * shape[2]
+    lever = [float(v) for v in I.LEVER / I.LEVER.sum()]
+    ok_all = True
+    done = 0
+    t_gpu = 0.0
+    while True:
+        ph, _ = g.download(device=True)
+        H = g.front_height()
+        zs = max(0, H - args.below)
+        fr = lamellae(ph[:, zs])
+        err, mn = g.monitor()
+        st = g.state()
+        present = all(f > 0.0 for f in fr)
+        within = all(abs(f - l) <= 0.1 for f, l in zip(fr, lever))
+        ok = present and within and err <= 1e-14 and mn >= 0.0
+        ok_all &= ok
+        rec = {"step": st["step"], "z_off": st["z_off"], "front_height": H, "slice_z": zs, "solid_fractions": fr,
+               "lever": lever, "all_present": present, "within_0.1": within, "max_sum_err": err, "min_phi": mn,
+               "ok": ok}
+        print(json.dumps(rec), flush=True)
+        out.write(json.dumps(rec) + "\n")
+        out.flush()
+        del ph
+        if done >= args.steps:
+            break
+        n = min(args.check, args.steps - done)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(g.stream)
+        g.step(n)
+        e1.record(g.stream)
+        e1.synchronize()
+        t_gpu += e0.elapsed_time(e1) * 1e-3
+        done += n
+    summ = {"config": "config 5 on one B200: 400x400x2000 DS, moving window, IC-L, C.4", "shape_zyx": list(shape),
+            "steps": done, "gpu_seconds": t_gpu, "mlups": cells * done / t_gpu / 1e6 if t_gpu else None,
+            "all_checks_ok": ok_all}
+    print(json.dumps(summ), flush=True)
+    out.write(json.dumps(summ) + "\n")
+    out.close()
+    g.close()
+    sys.exit(0 if ok_all else 1)
+
+
+if __name__ == "__main__":
+    main()
