@@ -192,6 +192,9 @@ def main():
                     help="weak: config 2/3 (n^3 DS block per GPU); strong: config 4 (fixed 512x512x1024 "
                          "periodic domain, z-slabs)")
     ap.add_argument("--variant", default="jit", choices=["jit", "tuned", "naive"])
+    ap.add_argument("--autotune", type=int, default=2, metavar="PASSES",
+                    help="run pf_autotune (coordinate search over the JIT tuning knobs, timed on this block) with "
+                         "this many passes before the warm-up; 0 = built-in defaults")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     args = ap.parse_args()
@@ -262,6 +265,12 @@ def main():
         g.init_fields(phi_pin, mu_pin)
     stream = g.stream
     cells_local = lshape[0] * lshape[1] * lshape[2]
+    tune_rep = None
+    if args.autotune > 0 and args.variant == "jit":
+        t_at = time.time()
+        rep = g.autotune(passes=args.autotune, reps=5)  # collective: same choice on every rank
+        tune_rep = {"passes": args.autotune, "seconds": round(time.time() - t_at, 1),
+                    "phi": rep["phi"], "mu": rep["mu"], "tried": len(rep["tried"])}
 
     def barrier():
         if dist is not None:
@@ -325,7 +334,7 @@ def main():
                                 f"solidification, moving window (check every 10 steps), IC-L, C.4 parameters"),
                    "global_xyz": [gshape[2], gshape[1], gshape[0]], "procs_xyz": list(procs),
                    "parallelism": f"domain decomposition {procs[0]}x{procs[1]}x{procs[2]}",
-                   "variant": args.variant,
+                   "variant": args.variant, "tuning": g.tuning() if args.variant == "jit" else None,
                    "l2": f"inputs larger than L2 ({(6 * 2) * cells_local * 8 / 1e9:.2f} GB of fields per GPU)"},
         "per_gpu_mlups": value / world,
         "step_roofline": {"R_mlups": R, "F_flop_per_cell": F_STEP, "Q_bytes_per_cell": Q_STEP,
@@ -342,6 +351,7 @@ def main():
                     "share_phi": phi_ms / ms if ms else None,
                     "ghost_ms_total": prof["ghost"][0], "window_ms_total": prof["window"][0]},
         "gpu_launches": launches,
+        "autotune": tune_rep,
         "clocks": clk,
         "state": {"step": st["step"], "z_off": st["z_off"], "max_sum_err": mon[0], "min_phi": mon[1]},
     }

@@ -193,6 +193,64 @@ int pf_set_state(pf_ctx* ctx, const pf_state* s);
  * per process); PF_ECUDA with the NVRTC log if that fails.                 */
 int pf_set_variant(pf_ctx* ctx, int variant);
 
+/* Tuning of the run-time specialised kernels (PF_VARIANT_JIT): the
+ * thread-to-cell mapping (tile shape, z-chunk), the occupancy requested from
+ * the register allocator and schedule transformations of the two sweeps.
+ * The paper's code generator exposes exactly these as tunables -- "an
+ * auto-tuning mechanism can then test and optimize different mappings"
+ * and register-usage transformations tuned "for each kernel"
+ * (P:L808-865).  Every setting computes the same result (the arithmetic per
+ * cell does not depend on it; tests/test_gpu_autotune.py checks bitwise
+ * equality).  Ranges (PF_EINVAL outside them):                              */
+typedef struct {
+  int phi_ty;        /* phi-sweep tile height (width 32): 4, 8, 16                  */
+  int phi_minb;      /* phi-sweep CTAs per SM requested from ptxas: 1..8            */
+  int phi_zc;        /* phi-sweep planes per CTA along z: 4..512                    */
+  int phi_faces6;    /* 1: every thread computes all six faces of its cell (no
+                        barrier); 0: each face once, +x/+y exchanged on chip        */
+  int phi_unroll;    /* phi-sweep z-loop unroll factor: 1..4                        */
+  int phi_prefetch;  /* software prefetch of the own column: 0 off, 1 L2, 2 L1      */
+  int phi_pfd;       /* prefetch distance in planes: 1..4                           */
+  int mu_ty;         /* mu-sweep tile height: 3..8 (tile width 32), 4..8 (width 16) */
+  int mu_tx;         /* mu-sweep tile width: 16 or 32                               */
+  int mu_minb;       /* mu-sweep CTAs per SM requested from ptxas: 1..6             */
+  int mu_zc;         /* mu-sweep planes per CTA along z: 4..512                     */
+  int mu_prefetch;   /* software prefetch of the own column: 0 off, 1 L2, 2 L1      */
+  int mu_pfd;        /* prefetch distance in planes: 2..4                           */
+  int mu_rpf;        /* 1: own cell's L1-missing loads one plane ahead in registers */
+  int mu_halo_l1;    /* 1: halo-ring cells' next-plane lines prefetched into L1     */
+  int mu_fxreg;      /* 1: own -x/-y fluxes taken from registers in the divergence  */
+} pf_tuning;
+
+/* The built-in defaults (the measured best at 256^3 on one B200,
+ * profiles/README.md), each overridable by the PF_* environment variable
+ * of the same knob (PF_PHI_TY, PF_MU_MINB, ...). No device needed.          */
+int pf_tuning_default(pf_tuning* out);
+/* Select the tuning of this context; the specialised kernels are rebuilt on
+ * the next step (cached per process).  PF_EINVAL for a value out of range.  */
+int pf_set_tuning(pf_ctx* ctx, const pf_tuning* t);
+int pf_get_tuning(const pf_ctx* ctx, pf_tuning* out);
+/* Range check of a tuning without a context or device: PF_OK, or PF_EINVAL
+ * with the reason in log[0..logn).                                         */
+int pf_tuning_check(const pf_tuning* t, char* log, int logn);
+
+/* Auto-tuning (S§8(f) NEXT-2): starting from the current tuning, a
+ * coordinate search over the knobs of the kernels in `mask` (PF_PHI: the
+ * phi-sweep, PF_MU: the mu-sweep), at most `passes` sweeps over the knobs.
+ * Per knob, all candidate values are compiled concurrently with NVRTC on
+ * host threads, then each candidate kernel is timed on this context's own
+ * block and fields with CUDA events on the compute stream (median of `reps`
+ * launches after 2 warm-up launches); a candidate replaces the current
+ * setting if it is faster by more than 1 %.  With world > 1 the times are
+ * max-reduced over ranks (NCCL) so that every rank selects the same tuning
+ * (collective).  The timed launches read only the current time level and
+ * write only the scratch level: the state (fields, step, z_off) is
+ * unchanged.  Needs params and fields (PF_ESTATE otherwise) and the JIT
+ * variant.  On return the context uses the best tuning found; `log` (may be
+ * NULL) receives a JSON document with every candidate and its time,
+ * truncated to logn bytes.  Synchronous.                                   */
+int pf_autotune(pf_ctx* ctx, unsigned mask, int passes, int reps, char* log, int logn);
+
 /* Optional per-kernel timing with CUDA events on the compute stream:
  * pf_profile(ctx, 1) resets the counters and enables event timing
  * (pf_profile(ctx, 0) resets and disables it); pf_profile_read() returns the
@@ -209,10 +267,13 @@ int pf_profile_read(pf_ctx* ctx, double ms[4], int64_t launches[4]);
 int pf_nccl_unique_id(unsigned char out[128]);
 
 /* Build check without a device: compile the run-time specialised kernels
- * (PF_VARIANT_JIT) for parameters p, liquid index `liquid` and an n^3 block
- * with NVRTC; optionally write the sm_100a cubin to cubin_path.  Returns the
- * cubin size in bytes, or -1 with the compiler log in log[0..logn).       */
-int pf_jit_compile_only(const pf_params* p, int liquid, int n, const char* cubin_path, char* log, int logn);
+ * (PF_VARIANT_JIT) for parameters p, liquid index `liquid`, an n^3 block and
+ * tuning t (NULL = pf_tuning_default) with NVRTC; optionally write the
+ * sm_100a cubins to cubin_path (mu-sweep) and cubin_path + ".phi" (phi-sweep).
+ * Returns the total cubin size in bytes, or -1 with the compiler log in
+ * log[0..logn).                                                            */
+int pf_jit_compile_only(const pf_params* p, int liquid, int n, const pf_tuning* t, const char* cubin_path, char* log,
+                        int logn);
 
 const char* pf_last_error(const pf_ctx* ctx);
 const char* pf_version(void);

@@ -14,6 +14,7 @@
 
 #include <algorithm>
 #include <string>
+#include <thread>
 #include <vector>
 
 #include "pf_internal.h"
@@ -99,7 +100,9 @@ struct pf_ctx {
   cudaEvent_t ev_phi = nullptr, ev_phix = nullptr, ev_mu = nullptr, ev_mux = nullptr;
   bool mux_pending = false;         // mu exchange in flight on comm_s
   bool overlap = true;
-  JitModule* jit = nullptr;  // specialised kernels for (dp, g); reset by pf_set_params
+  JitKernel* jphi = nullptr;  // specialised sweeps for (dp, g, tune); reset by pf_set_params / pf_set_tuning
+  JitKernel* jmu = nullptr;
+  pf_tuning tune;             // tuning of the specialised sweeps (pf_set_tuning, pf_autotune)
   ncclComm_t comm = nullptr;
   // profiling
   bool prof = false;
@@ -374,6 +377,7 @@ int pf_create(const pf_config* cfg, pf_ctx** out) {
   pf_ctx* ctx = new (std::nothrow) pf_ctx();
   if (!ctx) return PF_ENOMEM;
   ctx->cfg = *cfg;
+  tuning_default(&ctx->tune);
   if (layout_of(cfg, &ctx->lay, ctx->coord) != PF_OK) {
     delete ctx;
     return PF_EINVAL;
@@ -579,7 +583,7 @@ int pf_set_params(pf_ctx* ctx, const pf_params* p) {
   pf::fill_dev_params(*p, L, &ctx->dp);
   ctx->hp = *p;
   ctx->have_params = true;
-  ctx->jit = nullptr;
+  ctx->jphi = ctx->jmu = nullptr;
   return PF_OK;
 }
 
@@ -699,7 +703,7 @@ static int launch_mu(pf_ctx* ctx, const TileSel* ts, dim3 grid, const double* ps
   if (ctx->variant == PF_VARIANT_NAIVE)
     launch_mu_naive(ctx->dp, ctx->g, ps, pd, ms, md, ctx->stream);
   else if (ctx->variant == PF_VARIANT_JIT)
-    CU(jit_launch_mu(ctx->jit, ctx->dp, ts, grid, ps, pd, ms, md, ctx->stream));
+    CU(jit_launch_mu(ctx->jmu, ctx->dp, ts, grid, ps, pd, ms, md, ctx->stream));
   else
     launch_mu_tuned(ctx->dp, ctx->g, ts, grid, ps, pd, ms, md, ctx->stream);
   ctx->nlaunch[1] += 1;
@@ -717,10 +721,11 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
   ctx->dp.Tbase = ctx->hp.T0 + ctx->hp.G * (((double)g.z0 + (double)ctx->z_off) * ctx->hp.dx - ctx->hp.v * t);
   ctx->dp.step = (unsigned long long)ctx->step;  // fluctuation counter [B4]
   cudaEvent_t e0 = nullptr;
-  if (ctx->variant == PF_VARIANT_JIT && !ctx->jit) {
+  if (ctx->variant == PF_VARIANT_JIT && (!ctx->jphi || !ctx->jmu)) {
     std::string err;
-    ctx->jit = jit_get(ctx->dp, g, &err);
-    if (!ctx->jit) return fail(ctx, PF_ECUDA, "run-time specialisation failed: %s", err.c_str());
+    ctx->jphi = jit_get(ctx->dp, g, ctx->tune, JIT_PHI, &err);
+    if (ctx->jphi) ctx->jmu = jit_get(ctx->dp, g, ctx->tune, JIT_MU, &err);
+    if (!ctx->jphi || !ctx->jmu) return fail(ctx, PF_ECUDA, "run-time specialisation failed: %s", err.c_str());
   }
   // overlap: the exchanged dimensions' ghosts travel on the
   // comm stream while the mu-sweep updates the tiles that do not read them
@@ -730,7 +735,7 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
   if (ctx->variant == PF_VARIANT_NAIVE)
     launch_phi_naive(ctx->dp, g, ps, ms, pd, ctx->stream);
   else if (ctx->variant == PF_VARIANT_JIT)
-    CU(jit_launch_phi(ctx->jit, ctx->dp, ps, ms, pd, ctx->stream));
+    CU(jit_launch_phi(ctx->jphi, ctx->dp, ps, ms, pd, ctx->stream));
   else
     launch_phi_tuned(ctx->dp, g, ps, ms, pd, ctx->stream);
   ctx->nlaunch[0] += 1;
@@ -778,9 +783,9 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
     // the mu-sweep reads mu ghosts: the previous mu exchange must be done
     if (int r = join_comm(ctx)) return r;
     // line 3: interior tiles (no phi_dst ghost of an exchanged dimension is read)
-    const int mty = ctx->variant == PF_VARIANT_JIT ? jit_mu_ty_of(ctx->jit) : tuned_mu_ty_default();
-    const int zc = ctx->variant == PF_VARIANT_JIT ? jit_mu_zc_of(ctx->jit) : 0;
-    const int mtx = ctx->variant == PF_VARIANT_JIT ? jit_mu_tx_of(ctx->jit) : 32;
+    const int mty = ctx->variant == PF_VARIANT_JIT ? jit_mu_ty_of(ctx->jmu) : tuned_mu_ty_default();
+    const int zc = ctx->variant == PF_VARIANT_JIT ? jit_mu_zc_of(ctx->jmu) : 0;
+    const int mtx = ctx->variant == PF_VARIANT_JIT ? jit_mu_tx_of(ctx->jmu) : 32;
     const dim3 full = tuned_grid_mu(g, mty, zc, mtx);
     const int nb[3] = {(int)full.x, (int)full.y, (int)full.z};
     TileSel in = {{0, 0, 0}, {0, 0, 0}, {nb[0], nb[1], nb[2]}, 0};
@@ -993,6 +998,232 @@ static int window_maybe(pf_ctx* ctx) {
   if (int r = front_height_impl(ctx, &H)) return r;
   const int thr = (int)floor(ctx->hp.window_frac * (double)ctx->cfg.global[2]);
   if (H > thr) return pf_shift_window(ctx, H - thr);
+  return PF_OK;
+}
+
+// ---------------------------------------------------------------------------
+// tuning and auto-tuning of the specialised sweeps (S§8(f) NEXT-2;
+// P:L797-806 mapping auto-tuning, P:L808-865 per-kernel tuning)
+// ---------------------------------------------------------------------------
+int pf_tuning_default(pf_tuning* out) {
+  if (!out) return PF_EINVAL;
+  tuning_default(out);
+  return PF_OK;
+}
+
+int pf_set_tuning(pf_ctx* ctx, const pf_tuning* t) {
+  if (!ctx || !t) return PF_EINVAL;
+  if (const char* m = tuning_check(*t)) return fail(ctx, PF_EINVAL, "pf_set_tuning: %s", m);
+  ctx->tune = *t;
+  ctx->jphi = ctx->jmu = nullptr;
+  return PF_OK;
+}
+
+int pf_get_tuning(const pf_ctx* ctx, pf_tuning* out) {
+  if (!ctx || !out) return PF_EINVAL;
+  *out = ctx->tune;
+  return PF_OK;
+}
+
+namespace {
+struct TuneKnob {
+  const char* name;
+  int pf_tuning::*f;
+  int which;
+  std::vector<int> dom;
+};
+const std::vector<TuneKnob>& tune_knobs() {
+  static const std::vector<TuneKnob> k = {
+      {"phi_ty", &pf_tuning::phi_ty, JIT_PHI, {4, 8, 16}},
+      {"phi_minb", &pf_tuning::phi_minb, JIT_PHI, {3, 4, 5, 6}},
+      {"phi_zc", &pf_tuning::phi_zc, JIT_PHI, {8, 12, 16, 24, 32}},
+      {"phi_faces6", &pf_tuning::phi_faces6, JIT_PHI, {0, 1}},
+      {"phi_unroll", &pf_tuning::phi_unroll, JIT_PHI, {1, 2, 3}},
+      {"phi_prefetch", &pf_tuning::phi_prefetch, JIT_PHI, {0, 1, 2}},
+      {"phi_pfd", &pf_tuning::phi_pfd, JIT_PHI, {1, 2, 3}},
+      {"mu_ty", &pf_tuning::mu_ty, JIT_MU, {3, 4, 5, 6, 8}},
+      {"mu_tx", &pf_tuning::mu_tx, JIT_MU, {16, 32}},
+      {"mu_minb", &pf_tuning::mu_minb, JIT_MU, {2, 3, 4}},
+      {"mu_zc", &pf_tuning::mu_zc, JIT_MU, {8, 12, 16, 24}},
+      {"mu_prefetch", &pf_tuning::mu_prefetch, JIT_MU, {0, 1, 2}},
+      {"mu_pfd", &pf_tuning::mu_pfd, JIT_MU, {2, 3}},
+      {"mu_rpf", &pf_tuning::mu_rpf, JIT_MU, {0, 1}},
+      {"mu_halo_l1", &pf_tuning::mu_halo_l1, JIT_MU, {0, 1}},
+      {"mu_fxreg", &pf_tuning::mu_fxreg, JIT_MU, {0, 1}},
+  };
+  return k;
+}
+
+std::string tuning_json(const pf_tuning& t) {
+  std::string o = "{";
+  bool first = true;
+  for (const auto& k : tune_knobs()) {
+    char b[64];
+    snprintf(b, sizeof b, "%s\"%s\": %d", first ? "" : ", ", k.name, t.*(k.f));
+    o += b;
+    first = false;
+  }
+  return o + "}";
+}
+}  // namespace
+
+// median launch time (ms) of one specialised sweep on this context's fields;
+// reads only the current level, writes only the scratch level
+static int time_sweep(pf_ctx* ctx, JitKernel* k, int which, int reps, double* out) {
+  const double* ps = ctx->phi[ctx->cur];
+  double* pd = ctx->phi[1 - ctx->cur];
+  const double* ms = ctx->mu[ctx->cur];
+  double* md = ctx->mu[1 - ctx->cur];
+  auto launch = [&]() {
+    return which == JIT_PHI ? jit_launch_phi(k, ctx->dp, ps, ms, pd, ctx->stream)
+                            : jit_launch_mu(k, ctx->dp, nullptr, dim3(), ps, pd, ms, md, ctx->stream);
+  };
+  for (int i = 0; i < 2; ++i) CU(launch());
+  std::vector<cudaEvent_t> ev(reps + 1);
+  for (auto& e : ev) CU(cudaEventCreate(&e));
+  CU(cudaEventRecord(ev[0], ctx->stream));
+  for (int i = 0; i < reps; ++i) {
+    CU(launch());
+    CU(cudaEventRecord(ev[i + 1], ctx->stream));
+  }
+  CU(cudaEventSynchronize(ev[reps]));
+  std::vector<double> t(reps);
+  for (int i = 0; i < reps; ++i) {
+    float v = 0;
+    cudaEventElapsedTime(&v, ev[i], ev[i + 1]);
+    t[i] = v;
+  }
+  for (auto e : ev) cudaEventDestroy(e);
+  std::sort(t.begin(), t.end());
+  *out = t[reps / 2];
+  return PF_OK;
+}
+
+// times of candidate kernels (inf where the build failed), max over ranks
+static int time_candidates(pf_ctx* ctx, const std::vector<pf_tuning>& cands, int which, int reps,
+                           std::vector<double>* ms, std::vector<std::string>* why) {
+  const int nthr = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
+  jit_precompile(ctx->dp, ctx->g, cands, which, nthr);
+  ms->assign(cands.size(), INFINITY);
+  why->assign(cands.size(), "");
+  for (size_t i = 0; i < cands.size(); ++i) {
+    std::string err;
+    JitKernel* k = jit_get(ctx->dp, ctx->g, cands[i], which, &err);
+    if (!k) {
+      (*why)[i] = err.substr(0, 200);
+      continue;
+    }
+    double v = INFINITY;
+    if (int r = time_sweep(ctx, k, which, reps, &v)) {
+      cudaGetLastError();  // e.g. a launch the tile shape cannot fit: not sticky
+      (*why)[i] = "launch failed";
+      (void)r;
+      continue;
+    }
+    (*ms)[i] = v;
+  }
+  if (ctx->comm) {  // every rank takes the same decision: max over ranks
+    double* d = (double*)ctx->red;
+    for (size_t o = 0; o < cands.size(); o += 32) {
+      const size_t n = std::min<size_t>(32, cands.size() - o);
+      CU(cudaMemcpyAsync(d, ms->data() + o, n * sizeof(double), cudaMemcpyHostToDevice, ctx->stream));
+      NC(g_nccl.AllReduce(d, d, n, ncclFloat64, ncclMax, ctx->comm, ctx->stream));
+      CU(cudaMemcpyAsync(ms->data() + o, d, n * sizeof(double), cudaMemcpyDeviceToHost, ctx->stream));
+      CU(cudaStreamSynchronize(ctx->stream));
+    }
+  }
+  return PF_OK;
+}
+
+int pf_autotune(pf_ctx* ctx, unsigned mask, int passes, int reps, char* log, int logn) {
+  if (!ctx) return PF_EINVAL;
+  if (!ctx->have_params || !ctx->have_fields) return fail(ctx, PF_ESTATE, "pf_autotune before pf_set_params/pf_init_fields");
+  if (ctx->variant != PF_VARIANT_JIT) return fail(ctx, PF_ESTATE, "pf_autotune tunes the JIT variant only");
+  if (!(mask & (PF_PHI | PF_MU)) || passes < 1 || reps < 1 || reps > 1000)
+    return fail(ctx, PF_EINVAL, "pf_autotune: mask PF_PHI|PF_MU, passes >= 1, 1 <= reps <= 1000");
+  if (const char* m = tuning_check(ctx->tune)) return fail(ctx, PF_EINVAL, "current tuning invalid: %s", m);
+  if (int r = join_comm(ctx)) return r;
+  CU(cudaStreamSynchronize(ctx->stream));
+  const pf_tuning start = ctx->tune;
+  pf_tuning best = start;
+  std::string cl;  // candidate records
+  std::string kj;  // per-kernel summary
+  for (int which : {JIT_PHI, JIT_MU}) {
+    if (!(mask & (which == JIT_PHI ? PF_PHI : PF_MU))) continue;
+    const char* kname = which == JIT_PHI ? "phi" : "mu";
+    if (which == JIT_MU) {  // the mu-sweep reads phi_dst: one phi-sweep of the best phi kernel first
+      std::string err;
+      JitKernel* kp = jit_get(ctx->dp, ctx->g, best, JIT_PHI, &err);
+      if (!kp) return fail(ctx, PF_ECUDA, "autotune: %s", err.c_str());
+      CU(jit_launch_phi(kp, ctx->dp, ctx->phi[ctx->cur], ctx->mu[ctx->cur], ctx->phi[1 - ctx->cur], ctx->stream));
+      if (int r = fill_ghosts(ctx, ctx->phi[1 - ctx->cur], PF_N, false)) return r;
+    }
+    std::vector<double> t0;
+    std::vector<std::string> w0;
+    if (int r = time_candidates(ctx, {best}, which, reps, &t0, &w0)) return r;
+    if (!std::isfinite(t0[0])) return fail(ctx, PF_ECUDA, "autotune: the current %s kernel failed: %s", kname, w0[0].c_str());
+    const double start_ms = t0[0];
+    double best_ms = start_ms;
+    int ncand = 0;
+    for (int pass = 0; pass < passes; ++pass) {
+      bool improved = false;
+      for (const auto& kn : tune_knobs()) {
+        if (kn.which != which) continue;
+        std::vector<pf_tuning> cands;
+        std::vector<int> vals;
+        for (int v : kn.dom) {
+          if (v == best.*(kn.f)) continue;
+          pf_tuning c = best;
+          c.*(kn.f) = v;
+          // a new tile shape comes with its natural occupancy
+          if (kn.f == &pf_tuning::phi_ty) c.phi_minb = phi_minb_for(c.phi_ty);
+          if (kn.f == &pf_tuning::mu_ty || kn.f == &pf_tuning::mu_tx) c.mu_minb = mu_minb_for(c.mu_ty, c.mu_tx);
+          if (tuning_check(c)) continue;
+          cands.push_back(c);
+          vals.push_back(v);
+        }
+        if (cands.empty()) continue;
+        std::vector<double> tm;
+        std::vector<std::string> why;
+        if (int r = time_candidates(ctx, cands, which, reps, &tm, &why)) return r;
+        int bi = -1;
+        for (size_t i = 0; i < cands.size(); ++i) {
+          char b[512];
+          snprintf(b, sizeof b, "%s{\"kernel\": \"%s\", \"pass\": %d, \"knob\": \"%s\", \"value\": %d, \"ms\": %s, \"error\": \"%s\"}",
+                   cl.empty() ? "" : ",\n  ", kname, pass, kn.name, vals[i],
+                   std::isfinite(tm[i]) ? std::to_string(tm[i]).c_str() : "null", why[i].c_str());
+          cl += b;
+          ++ncand;
+          if (tm[i] < best_ms * 0.99 && (bi < 0 || tm[i] < tm[bi])) bi = (int)i;
+        }
+        if (bi >= 0) {
+          best = cands[bi];
+          best_ms = tm[bi];
+          improved = true;
+        }
+      }
+      if (!improved) break;
+    }
+    char b[256];
+    snprintf(b, sizeof b, "%s\"%s\": {\"start_ms\": %.6f, \"best_ms\": %.6f, \"candidates\": %d}", kj.empty() ? "" : ", ",
+             kname, start_ms, best_ms, ncand);
+    kj += b;
+  }
+  ctx->tune = best;
+  ctx->jphi = ctx->jmu = nullptr;
+  {
+    std::string err;
+    ctx->jphi = jit_get(ctx->dp, ctx->g, best, JIT_PHI, &err);
+    if (ctx->jphi) ctx->jmu = jit_get(ctx->dp, ctx->g, best, JIT_MU, &err);
+    if (!ctx->jphi || !ctx->jmu) return fail(ctx, PF_ECUDA, "autotune: %s", err.c_str());
+  }
+  // the scratch level's ghosts were overwritten: nothing reads them before the next sweep writes it
+  CU(cudaStreamSynchronize(ctx->stream));
+  if (log && logn > 0) {
+    std::string j = "{\"start\": " + tuning_json(start) + ",\n \"best\": " + tuning_json(best) + ",\n " + kj +
+                    ",\n \"reps\": " + std::to_string(reps) + ",\n \"tried\": [\n  " + cl + "]}";
+    snprintf(log, (size_t)logn, "%s", j.c_str());
+  }
   return PF_OK;
 }
 

@@ -7,6 +7,7 @@
 #include <stdint.h>
 
 #include <string>
+#include <vector>
 
 #include "../../include/pf.h"
 #include "pf_dev.cuh"
@@ -58,16 +59,24 @@ void launch_unpack(const Geom& g, int d, int idx, int ncomp, double* f, const do
 void fill_dev_params(const pf_params& p, int liquid, DevParams* out);
 
 // ---- run-time specialisation (NVRTC) -------------------------------------
-struct JitModule;  // compiled sweep kernels for one (geometry, parameters)
-// build (or fetch from the process cache) the specialised kernels; returns
+enum { JIT_PHI = 0, JIT_MU = 1 };
+struct JitKernel;  // one specialised sweep compiled for (parameters, geometry, tuning)
+void tuning_default(pf_tuning* t);            // built-in defaults + PF_* environment overrides
+const char* tuning_check(const pf_tuning& t);  // nullptr if valid, else the reason
+// build (or fetch from the process cache) a specialised kernel; returns
 // nullptr and sets *err on failure
-JitModule* jit_get(const DevParams& P, const Geom& g, std::string* err);
-cudaError_t jit_launch_phi(JitModule* m, const DevParams& P, const double* ps, const double* ms, double* pd,
+JitKernel* jit_get(const DevParams& P, const Geom& g, const pf_tuning& t, int which, std::string* err);
+// compile the kernels of several tunings into the cubin cache, concurrently
+// on up to nthreads host threads (no device needed)
+void jit_precompile(const DevParams& P, const Geom& g, const std::vector<pf_tuning>& ts, int which, int nthreads);
+cudaError_t jit_launch_phi(JitKernel* m, const DevParams& P, const double* ps, const double* ms, double* pd,
                            cudaStream_t s);
-cudaError_t jit_launch_mu(JitModule* m, const DevParams& P, const TileSel* ts, dim3 grid, const double* ps,
+cudaError_t jit_launch_mu(JitKernel* m, const DevParams& P, const TileSel* ts, dim3 grid, const double* ps,
                           const double* pd, const double* ms, double* md, cudaStream_t s);
-int jit_mu_ty_of(const JitModule* m);
-int jit_mu_tx_of(const JitModule* m);
-int jit_mu_zc_of(const JitModule* m);
+int jit_mu_ty_of(const JitKernel* m);
+int jit_mu_tx_of(const JitKernel* m);
+int jit_mu_zc_of(const JitKernel* m);
+int phi_minb_for(int pty);            // natural CTAs per SM of a tile shape
+int mu_minb_for(int mty, int mtx);
 
 }  // namespace pf

@@ -51,6 +51,14 @@ class PFParams(C.Structure):
                 ("xi_amp", C.c_double), ("xi_seed", C.c_uint32)]
 
 
+TUNING_KNOBS = ("phi_ty", "phi_minb", "phi_zc", "phi_faces6", "phi_unroll", "phi_prefetch", "phi_pfd",
+                "mu_ty", "mu_tx", "mu_minb", "mu_zc", "mu_prefetch", "mu_pfd", "mu_rpf", "mu_halo_l1", "mu_fxreg")
+
+
+class PFTuning(C.Structure):
+    _fields_ = [(k, C.c_int) for k in TUNING_KNOBS]
+
+
 class PFState(C.Structure):
     _fields_ = [("step", C.c_int64), ("z_off", C.c_int64)]
 
@@ -58,7 +66,8 @@ class PFState(C.Structure):
 # every symbol include/pf.h declares (checked by tests/test_abi.py)
 ABI_SYMBOLS = ["pf_query_layout", "pf_query_neighbors", "pf_create", "pf_destroy", "pf_set_params", "pf_init_fields", "pf_step",
                "pf_step_phi_only", "pf_halo_exchange", "pf_shift_window", "pf_front_height", "pf_monitor",
-               "pf_download", "pf_get_state", "pf_set_state", "pf_set_variant", "pf_profile", "pf_profile_read",
+               "pf_download", "pf_get_state", "pf_set_state", "pf_set_variant", "pf_tuning_default", "pf_set_tuning",
+               "pf_get_tuning", "pf_tuning_check", "pf_autotune", "pf_profile", "pf_profile_read",
                "pf_nccl_unique_id", "pf_jit_compile_only", "pf_last_error", "pf_version"]
 
 _lib = None
@@ -90,10 +99,15 @@ def load_library(path: str = LIB_PATH):
     L.pf_get_state.argtypes = [vp, C.POINTER(PFState)]
     L.pf_set_state.argtypes = [vp, C.POINTER(PFState)]
     L.pf_set_variant.argtypes = [vp, ip]
+    L.pf_tuning_default.argtypes = [C.POINTER(PFTuning)]
+    L.pf_set_tuning.argtypes = [vp, C.POINTER(PFTuning)]
+    L.pf_get_tuning.argtypes = [vp, C.POINTER(PFTuning)]
+    L.pf_tuning_check.argtypes = [C.POINTER(PFTuning), C.c_char_p, ip]
+    L.pf_autotune.argtypes = [vp, C.c_uint, ip, ip, C.c_char_p, ip]
     L.pf_profile.argtypes = [vp, ip]
     L.pf_profile_read.argtypes = [vp, dp, C.POINTER(C.c_int64)]
     L.pf_nccl_unique_id.argtypes = [C.POINTER(C.c_ubyte)]
-    L.pf_jit_compile_only.argtypes = [C.POINTER(PFParams), ip, ip, C.c_char_p, C.c_char_p, ip]
+    L.pf_jit_compile_only.argtypes = [C.POINTER(PFParams), ip, ip, C.POINTER(PFTuning), C.c_char_p, C.c_char_p, ip]
     L.pf_last_error.argtypes = [vp]
     L.pf_last_error.restype = C.c_char_p
     L.pf_version.restype = C.c_char_p
@@ -103,6 +117,13 @@ def load_library(path: str = LIB_PATH):
 
 class PFError(RuntimeError):
     pass
+
+
+def tuning_default() -> dict:
+    """Built-in tuning of the specialised sweeps (+ PF_* environment overrides)."""
+    t = PFTuning()
+    load_library().pf_tuning_default(C.byref(t))
+    return {k: int(getattr(t, k)) for k in TUNING_KNOBS}
 
 
 def make_params(P: dict) -> PFParams:
@@ -138,12 +159,26 @@ def make_params(P: dict) -> PFParams:
     return p
 
 
-def jit_compile_only(params: dict, n: int = 64, cubin_path: str | None = None) -> int:
-    """Compile the run-time specialised kernels for `params` and an n^3 block
-    without a GPU (NVRTC only); returns the cubin size."""
+def _tuning_struct(tuning: dict) -> PFTuning:
+    t = dict(tuning_default(), **tuning)
+    return PFTuning(*[int(t[k]) for k in TUNING_KNOBS])
+
+
+def tuning_check(tuning: dict) -> str:
+    """pf_tuning_check: "ok" or the reason the tuning is out of range."""
+    log = C.create_string_buffer(256)
+    load_library().pf_tuning_check(C.byref(_tuning_struct(tuning)), log, 256)
+    return log.value.decode()
+
+
+def jit_compile_only(params: dict, n: int = 64, cubin_path: str | None = None, tuning: dict | None = None) -> int:
+    """Compile the run-time specialised kernels for `params`, an n^3 block and
+    `tuning` (None: the default) without a GPU (NVRTC only); returns the
+    total cubin size (mu-sweep cubin at cubin_path, phi-sweep at cubin_path.phi)."""
     p = make_params(params)
     log = C.create_string_buffer(8192)
-    r = load_library().pf_jit_compile_only(C.byref(p), int(params.get("liquid", 3)), int(n),
+    t = C.byref(_tuning_struct(tuning)) if tuning is not None else None
+    r = load_library().pf_jit_compile_only(C.byref(p), int(params.get("liquid", 3)), int(n), t,
                                            (cubin_path or "").encode(), log, 8192)
     if r < 0:
         raise PFError(f"specialised compile failed: {log.value.decode()}")
@@ -347,6 +382,30 @@ class PhaseField:
 
     def set_variant(self, name: str):
         self._check(self.lib.pf_set_variant(self._h, VARIANT[name]), "pf_set_variant")
+
+    def tuning(self) -> dict:
+        t = PFTuning()
+        self._check(self.lib.pf_get_tuning(self._h, C.byref(t)), "pf_get_tuning")
+        return {k: int(getattr(t, k)) for k in TUNING_KNOBS}
+
+    def set_tuning(self, tuning: dict):
+        """Set knobs of the specialised sweeps; unspecified knobs keep their value."""
+        cur = self.tuning()
+        unknown = set(tuning) - set(TUNING_KNOBS)
+        if unknown:
+            raise KeyError(f"unknown tuning knobs {sorted(unknown)}")
+        cur.update({k: int(v) for k, v in tuning.items()})
+        t = PFTuning(*[cur[k] for k in TUNING_KNOBS])
+        self._check(self.lib.pf_set_tuning(self._h, C.byref(t)), "pf_set_tuning")
+
+    def autotune(self, mask: int = PF_PHI | PF_MU, passes: int = 1, reps: int = 7) -> dict:
+        """pf_autotune: coordinate search over the tuning knobs, timed on this
+        block; returns the JSON report (start, best, per-kernel times, every
+        candidate).  The context keeps the best tuning."""
+        import json
+        buf = C.create_string_buffer(1 << 16)
+        self._check(self.lib.pf_autotune(self._h, int(mask), int(passes), int(reps), buf, len(buf)), "pf_autotune")
+        return json.loads(buf.value.decode())
 
     def profile(self, enable: bool = True):
         self._check(self.lib.pf_profile(self._h, int(enable)), "pf_profile")

@@ -62,6 +62,7 @@ int main(void) {
   printf("%zu %zu %zu %zu\n", offsetof(pf_config, stream), offsetof(pf_config, workspace),
          offsetof(pf_params, D), offsetof(pf_params, window_check));
   printf("%zu %zu\n", offsetof(pf_layout, pitch), offsetof(pf_layout, workspace_bytes));
+  printf("%zu %zu\n", sizeof(pf_tuning), offsetof(pf_tuning, mu_ty));
   return 0;
 }
 '''
@@ -73,7 +74,8 @@ int main(void) {
         vals = [int(v) for v in subprocess.check_output([exe], text=True).split()]
     got = [C.sizeof(pf.PFConfig), C.sizeof(pf.PFLayout), C.sizeof(pf.PFParams), C.sizeof(pf.PFState),
            pf.PFConfig.stream.offset, pf.PFConfig.workspace.offset, pf.PFParams.D.offset,
-           pf.PFParams.window_check.offset, pf.PFLayout.pitch.offset, pf.PFLayout.workspace_bytes.offset]
+           pf.PFParams.window_check.offset, pf.PFLayout.pitch.offset, pf.PFLayout.workspace_bytes.offset,
+           C.sizeof(pf.PFTuning), pf.PFTuning.mu_ty.offset]
     assert got == vals
 
 
@@ -96,5 +98,36 @@ def test_specialised_kernels_compile_without_gpu(lib, tmp_path):
     cub = str(tmp_path / "k.cubin")
     assert pf.jit_compile_only(I.params_c4("ds"), n=48, cubin_path=cub) > 0
     out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-sass", cub], capture_output=True, text=True).stdout
-    assert "pf_jit_phi" in out and "pf_jit_mu" in out and "DFMA" in out
+    assert "pf_jit_mu" in out and "DFMA" in out
+    out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-sass", cub + ".phi"], capture_output=True, text=True).stdout
+    assert "pf_jit_phi" in out and "DFMA" in out
     assert pf.jit_compile_only(dict(I.params_stress(), liquid=1), n=17) > 0
+
+
+def test_tuning_defaults_and_range_check(lib):
+    """pf_tuning_default / pf_tuning_check (NEXT-2): the defaults are valid,
+    values outside the documented ranges are rejected with a reason."""
+    from paper_conf_sc_0003hehshhkwnr19_b200 import pf
+    t = pf.tuning_default()
+    assert set(t) == set(pf.TUNING_KNOBS)
+    assert pf.tuning_check(t) == "ok"
+    for bad in ({"phi_ty": 5}, {"mu_ty": 2}, {"mu_tx": 16, "mu_ty": 3}, {"mu_minb": 7}, {"phi_unroll": 0},
+                {"mu_pfd": 1}, {"phi_minb": 8, "phi_ty": 16}, {"mu_rpf": 2}, {"mu_zc": 1000}):
+        msg = pf.tuning_check(dict(t, **bad))
+        assert msg != "ok", bad
+
+
+@pytest.mark.parametrize("knobs", [
+    {"phi_ty": 16, "phi_minb": 1, "phi_faces6": 0, "phi_unroll": 4, "phi_prefetch": 2, "phi_pfd": 3,
+     "mu_ty": 8, "mu_tx": 16, "mu_minb": 4, "mu_rpf": 0, "mu_halo_l1": 0, "mu_fxreg": 0, "mu_prefetch": 0},
+    {"phi_ty": 8, "phi_minb": 2, "phi_zc": 32, "phi_prefetch": 0, "mu_ty": 3, "mu_minb": 5, "mu_zc": 24,
+     "mu_pfd": 3, "mu_prefetch": 2},
+])
+def test_tuned_variants_compile_without_gpu(lib, knobs):
+    """Extreme corners of the auto-tuning space (pf_autotune's knobs) still
+    build with NVRTC for sm_100a."""
+    from paper_conf_sc_0003hehshhkwnr19_b200 import inputs as I
+    from paper_conf_sc_0003hehshhkwnr19_b200 import pf
+    t = dict(pf.tuning_default(), **knobs)
+    assert pf.tuning_check(t) == "ok"
+    assert pf.jit_compile_only(I.params_c4("ds"), n=40, tuning=t) > 0

@@ -1,0 +1,139 @@
+"""Auto-tuning of the specialised sweeps (S§8(f) NEXT-2; "an
+auto-tuning mechanism can then test and optimize different mappings",
+P:L808-865 per-kernel tuning): every tuning computes the same step, the
+tuner leaves the state untouched and keeps the fastest setting.  -m gpu.
+
+The bar is the parity bar of test_gpu_parity.py (<= 1e-12 after one step
+against the oracle) for tuned corners, and bitwise equality between tunings:
+the arithmetic per cell does not depend on the thread-to-cell mapping, the
+occupancy or the schedule transformations (each face flux is evaluated on
+the same two operands whichever thread computes it).
+"""
+import os
+
+import numpy as np
+import pytest
+
+from paper_conf_sc_0003hehshhkwnr19_b200 import inputs as I
+
+pytestmark = pytest.mark.gpu
+
+TOL_1 = 1e-12
+
+# corners of the search space of pf_autotune (tile shapes, occupancy,
+# z-chunks, schedule transformations)
+CORNERS = [
+    {},
+    {"phi_ty": 16, "phi_minb": 1, "phi_faces6": 0, "phi_unroll": 4, "phi_prefetch": 2, "phi_pfd": 3},
+    {"phi_ty": 8, "phi_minb": 2, "phi_zc": 5, "phi_faces6": 0, "phi_prefetch": 0},
+    {"mu_ty": 8, "mu_tx": 16, "mu_minb": 4, "mu_rpf": 0, "mu_halo_l1": 0, "mu_fxreg": 0, "mu_prefetch": 0},
+    {"mu_ty": 3, "mu_minb": 5, "mu_zc": 7, "mu_pfd": 3, "mu_prefetch": 2},
+    {"mu_ty": 6, "mu_minb": 2, "mu_zc": 24, "phi_zc": 32, "phi_unroll": 3},
+]
+
+
+def rel_linf(a, b):
+    return float(np.abs(a - b).max() / max(np.abs(b).max(), 1e-300))
+
+
+@pytest.fixture(scope="module")
+def pfmod():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.fail("GPU test without a CUDA device")
+    from paper_conf_sc_0003hehshhkwnr19_b200 import build, pf
+    build.build()
+    return pf
+
+
+@pytest.fixture(scope="module")
+def omod():
+    from oracle import oracle as O
+    O.build()
+    O.set_threads(min(16, os.cpu_count() or 1))
+    return O
+
+
+def gpu_run(pfmod, shape, P, phi, mu, steps, tuning=None, bc=None):
+    g = pfmod.PhaseField(shape, P, bc=bc)
+    if tuning:
+        g.set_tuning(tuning)
+    g.init_fields(phi, mu)
+    g.step(steps)
+    out = g.download()
+    g.close()
+    return out
+
+
+@pytest.mark.parametrize("pset", ["c4", "stress"])
+def test_tuning_corners_bitwise_and_parity(pfmod, omod, pset):
+    P = I.params_c4("ds") if pset == "c4" else I.params_stress()
+    bc = I.BC_DS if pset == "c4" else None
+    shape = (23, 21, 45)  # ragged in every tile dimension of every corner
+    phi, mu = I.make_ic("L" if pset == "c4" else "R", shape, seed=7)
+    o = omod.Oracle(shape, P, bc)
+    o.init(phi, mu)
+    o.step(1)
+    op, om = o.download()
+    ref3 = None
+    for c in CORNERS:
+        gp, gm = gpu_run(pfmod, shape, P, phi, mu, 1, c, bc)
+        assert rel_linf(gp, op) <= TOL_1 and rel_linf(gm, om) <= TOL_1, c
+        g3 = gpu_run(pfmod, shape, P, phi, mu, 3, c, bc)
+        if ref3 is None:
+            ref3 = g3
+        assert np.array_equal(g3[0], ref3[0]) and np.array_equal(g3[1], ref3[1]), c
+
+
+def test_set_tuning_rejects_out_of_range(pfmod):
+    shape = (8, 8, 32)
+    g = pfmod.PhaseField(shape, I.params_c4())
+    with pytest.raises(pfmod.PFError):
+        g.set_tuning({"mu_ty": 9})
+    with pytest.raises(pfmod.PFError):
+        g.set_tuning({"phi_ty": 16, "phi_minb": 8})
+    g.set_tuning({"mu_ty": 5})
+    assert g.tuning()["mu_ty"] == 5
+
+
+def test_autotune_keeps_state_and_result(pfmod):
+    """pf_autotune on a DS block: state (fields, step, z_off) unchanged, the
+    chosen tuning is valid and reported, and the run continues bitwise as
+    with the default tuning."""
+    P = I.params_c4("ds")
+    shape = (48, 64, 64)
+    phi, mu = I.make_ic("L", shape, seed=3)
+    g = pfmod.PhaseField(shape, P, bc=I.BC_DS)
+    g.init_fields(phi, mu)
+    g.step(2)
+    before = g.download()
+    st = g.state()
+    rep = g.autotune(passes=1, reps=3)
+    assert g.state() == st
+    after = g.download()
+    assert np.array_equal(before[0], after[0]) and np.array_equal(before[1], after[1])
+    assert rep["best"] == g.tuning()
+    assert pfmod.tuning_check(rep["best"]) == "ok"
+    for k in ("phi", "mu"):
+        assert rep[k]["best_ms"] <= rep[k]["start_ms"] and rep[k]["candidates"] > 5
+    assert all((c["ms"] is None) == bool(c["error"]) for c in rep["tried"])
+    assert sum(c["ms"] is not None for c in rep["tried"]) >= 10
+    g.step(3)
+    tuned = g.download()
+    g.close()
+    ref = gpu_run(pfmod, shape, P, phi, mu, 5, None, I.BC_DS)
+    assert np.array_equal(tuned[0], ref[0]) and np.array_equal(tuned[1], ref[1])
+
+
+def test_autotune_requires_fields_and_jit(pfmod):
+    g = pfmod.PhaseField((8, 8, 32), I.params_c4())
+    with pytest.raises(pfmod.PFError):
+        g.autotune()
+    phi, mu = I.make_ic("R", (8, 8, 32), seed=1)
+    g.init_fields(phi, mu)
+    g.set_variant("tuned")
+    with pytest.raises(pfmod.PFError):
+        g.autotune()
+    g.set_variant("jit")
+    rep = g.autotune(mask=pfmod.PF_MU, passes=1, reps=2)
+    assert "mu" in rep and "phi" not in rep
