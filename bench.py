@@ -195,6 +195,7 @@ def main():
     ap.add_argument("--autotune", type=int, default=2, metavar="PASSES",
                     help="run pf_autotune (coordinate search over the JIT tuning knobs, timed on this block) with "
                          "this many passes before the warm-up; 0 = built-in defaults")
+    ap.add_argument("--tuning", default=None, help="JSON dict of pf_tuning knobs set before the auto-tuning")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     args = ap.parse_args()
@@ -266,6 +267,8 @@ def main():
     stream = g.stream
     cells_local = lshape[0] * lshape[1] * lshape[2]
     tune_rep = None
+    if args.tuning and args.variant == "jit":
+        g.set_tuning(json.loads(args.tuning))
     if args.autotune > 0 and args.variant == "jit":
         t_at = time.time()
         rep = g.autotune(passes=args.autotune, reps=5)  # collective: same choice on every rank

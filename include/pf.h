@@ -220,6 +220,10 @@ typedef struct {
   int mu_rpf;        /* 1: own cell's L1-missing loads one plane ahead in registers */
   int mu_halo_l1;    /* 1: halo-ring cells' next-plane lines prefetched into L1     */
   int mu_fxreg;      /* 1: own -x/-y fluxes taken from registers in the divergence  */
+  int mu_qreg;       /* 1: own cell's face-side data kept in registers from the
+                        build (no shared-memory re-read; needs registers)        */
+  int mu_ldhint;     /* L1 policy of the mu-sweep's phi_dst / mu loads: 0 default,
+                        1 evict_first, 2 no_allocate                              */
 } pf_tuning;
 
 /* The built-in defaults (the measured best at 256^3 on one B200,

@@ -1050,6 +1050,8 @@ const std::vector<TuneKnob>& tune_knobs() {
       {"mu_rpf", &pf_tuning::mu_rpf, JIT_MU, {0, 1}},
       {"mu_halo_l1", &pf_tuning::mu_halo_l1, JIT_MU, {0, 1}},
       {"mu_fxreg", &pf_tuning::mu_fxreg, JIT_MU, {0, 1}},
+      {"mu_qreg", &pf_tuning::mu_qreg, JIT_MU, {0, 1}},
+      {"mu_ldhint", &pf_tuning::mu_ldhint, JIT_MU, {0, 1, 2}},
   };
   return k;
 }

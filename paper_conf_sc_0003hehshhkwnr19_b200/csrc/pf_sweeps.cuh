@@ -47,6 +47,24 @@ constexpr int kPhiUnroll = PF_PHI_UNROLL;
 #ifndef PF_PREFETCH_D
 #define PF_PREFETCH_D 2  // planes ahead
 #endif
+#ifndef PF_MU_LDHINT  // L1 policy of the mu-sweep's phi_dst / mu loads: 0 default, 1 evict_first, 2 no_allocate
+#define PF_MU_LDHINT 0
+#endif
+// load of a phi_dst / mu value in the mu-sweep (used by at most the cells of
+// one plane: a hint keeps these lines from evicting the reused phi_src lines)
+__device__ __forceinline__ double ldh(const double* p) {
+#if PF_MU_LDHINT == 1
+  double v;
+  asm("ld.global.nc.L1::evict_first.f64 %0, [%1];" : "=d"(v) : "l"(p));
+  return v;
+#elif PF_MU_LDHINT == 2
+  double v;
+  asm("ld.global.nc.L1::no_allocate.f64 %0, [%1];" : "=d"(v) : "l"(p));
+  return v;
+#else
+  return __ldg(p);
+#endif
+}
 __device__ __forceinline__ void prefetch_line(const void* p) {
 #if PF_PREFETCH == 1
   asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
@@ -317,10 +335,10 @@ __device__ __forceinline__ void build_cell(const GT& g, const double* __restrict
     v[D_CX + a] = wx ? __ldg(f + 1) - __ldg(f - 1) : 0.0;
     v[D_CY + a] = wy ? __ldg(f + g.pitch) - __ldg(f - g.pitch) : 0.0;
     v[D_CZ + a] = wz ? __ldg(f + g.plane) - __ldg(f - g.plane) : 0.0;
-    v[D_DP + a] = __ldg(pd + a * F + c) - v[D_F + a];
+    v[D_DP + a] = ldh(pd + a * F + c) - v[D_F + a];
   }
-  v[D_MU + 0] = __ldg(ms + c);
-  v[D_MU + 1] = __ldg(ms + F + c);
+  v[D_MU + 0] = ldh(ms + c);
+  v[D_MU + 1] = ldh(ms + F + c);
   double2* d = reinterpret_cast<double2*>(D + (size_t)i * D_NV);
 #pragma unroll
   for (int j = 0; j < D_NV / 2; ++j) d[j] = make_double2(v[2 * j], v[2 * j + 1]);
@@ -344,11 +362,11 @@ __device__ __forceinline__ void build_own_carry(const GT& g, const double* __res
     v[D_CX + a] = __ldg(f + 1) - __ldg(f - 1);
     v[D_CY + a] = __ldg(f + g.pitch) - __ldg(f - g.pitch);
     v[D_CZ + a] = wz ? fp - fm[a] : 0.0;
-    v[D_DP + a] = __ldg(pd + a * F + c) - fc[a];
+    v[D_DP + a] = ldh(pd + a * F + c) - fc[a];
     fc[a] = fp;
   }
-  v[D_MU + 0] = __ldg(ms + c);
-  v[D_MU + 1] = __ldg(ms + F + c);
+  v[D_MU + 0] = ldh(ms + c);
+  v[D_MU + 1] = ldh(ms + F + c);
   double2* d = reinterpret_cast<double2*>(D + (size_t)i * D_NV);
 #pragma unroll
   for (int j = 0; j < D_NV / 2; ++j) d[j] = make_double2(v[2 * j], v[2 * j + 1]);
@@ -384,10 +402,10 @@ __device__ __forceinline__ void build_own_rpf(const GT& g, const double* __restr
 #pragma unroll
   for (int a = 0; a < N; ++a) {
     nf[a] = __ldg(ps + a * F + c + 2 * g.plane);
-    nd[a] = __ldg(pd + a * F + c + g.plane);
+    nd[a] = ldh(pd + a * F + c + g.plane);
   }
-  nm[0] = __ldg(ms + c + g.plane);
-  nm[1] = __ldg(ms + F + c + g.plane);
+  nm[0] = ldh(ms + c + g.plane);
+  nm[1] = ldh(ms + F + c + g.plane);
 }
 
 template <bool B>
@@ -490,10 +508,10 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
 #pragma unroll
     for (int s = 0; s < NSOL; ++s) {
       const int a = solid_phase(L, s);
-      Dp.ds[s] = __ldg(pd + a * F + c) - Dp.f[a];
+      Dp.ds[s] = ldh(pd + a * F + c) - Dp.f[a];
     }
-    Dp.m[0] = __ldg(ms + c);
-    Dp.m[1] = __ldg(ms + F + c);
+    Dp.m[0] = ldh(ms + c);
+    Dp.m[1] = ldh(ms + F + c);
   }
   double divxy[M] = {0.0, 0.0}, Fzm[M] = {0.0, 0.0};
 #if PF_MU_ZCARRY
@@ -511,10 +529,10 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
 #pragma unroll
     for (int a = 0; a < N; ++a) {
       rnf[a] = __ldg(ps + a * F + c + g.plane);
-      rnd[a] = __ldg(pd + a * F + c);
+      rnd[a] = ldh(pd + a * F + c);
     }
-    rnm[0] = __ldg(ms + c);
-    rnm[1] = __ldg(ms + F + c);
+    rnm[0] = ldh(ms + c);
+    rnm[1] = ldh(ms + F + c);
   }
 #endif
 
