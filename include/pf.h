@@ -211,6 +211,8 @@ typedef struct {
   int phi_unroll;    /* phi-sweep z-loop unroll factor: 1..4                        */
   int phi_prefetch;  /* software prefetch of the own column: 0 off, 1 L2, 2 L1      */
   int phi_pfd;       /* prefetch distance in planes: 1..4                           */
+  int phi_xghost;    /* 1: the phi-sweep writes phi_dst's x ghost columns itself when
+                        x is periodic inside the block (the ghost fill skips them) */
   int mu_ty;         /* mu-sweep tile height: 3..8 (tile width 32), 4..8 (width 16) */
   int mu_tx;         /* mu-sweep tile width: 16 or 32                               */
   int mu_minb;       /* mu-sweep CTAs per SM requested from ptxas: 1..6             */

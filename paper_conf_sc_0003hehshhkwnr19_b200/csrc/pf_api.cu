@@ -452,6 +452,9 @@ int pf_create(const pf_config* cfg, pf_ctx** out) {
     const char* fe = getenv("PF_FORCE_EXCHANGE");  // debug: periodic self-exchange through pack/unpack
     ctx->force_exchange = fe && fe[0] == '1';
   }
+  // x periodic inside the block: the specialised phi-sweep may write phi_dst's x ghost columns
+  ctx->g.xwrap = (cfg->bc_lo[0] == PF_BC_PERIODIC && !ctx->exchange[0] && !ctx->force_exchange) ? 1 : 0;
+  if (getenv("PF_NO_XWRAP")) ctx->g.xwrap = 0;
   ctx->first_ex = 3;
   for (int d = 0; d < 3; ++d)
     if (ctx->exchange[d] || (ctx->force_exchange && cfg->bc_lo[d] == PF_BC_PERIODIC)) {
@@ -591,11 +594,14 @@ int pf_set_params(pf_ctx* ctx, const pf_params* p) {
 // ghost layers of one field set (Alg. 1 lines 2 / 4): local BCs + halo exchange
 // ---------------------------------------------------------------------------
 // dimensions [d0, d1) of the ordered x -> y -> z ghost fill, on stream `st`
-static int fill_ghost_dims(pf_ctx* ctx, double* f, int ncomp, bool is_mu, int d0, int d1, cudaStream_t st) {
+// x_done: the producing sweep already wrote the x ghost columns (Geom::xwrap)
+static int fill_ghost_dims(pf_ctx* ctx, double* f, int ncomp, bool is_mu, int d0, int d1, cudaStream_t st,
+                           bool x_done = false) {
   const double* dir = is_mu ? ctx->hp.mu_inf : nullptr;
   const bool any_ex = ctx->first_ex < 3;
+  const bool skipx = x_done;
   if (!any_ex && d0 == 0 && d1 == 3) {
-    launch_ghost_fill(ctx->g, ctx->bc_all, f, ncomp, dir, st);
+    launch_ghost_fill(ctx->g, ctx->bc_all, f, ncomp, dir, st, skipx);
     ctx->nlaunch[2] += 1;
     return check_launch(ctx, "ghost_fill");
   }
@@ -603,6 +609,7 @@ static int fill_ghost_dims(pf_ctx* ctx, double* f, int ncomp, bool is_mu, int d0
   for (int d = d0; d < d1; ++d) {
     const bool ex = ctx->exchange[d] || (ctx->force_exchange && ctx->cfg.bc_lo[d] == PF_BC_PERIODIC);
     if (!ex) {
+      if (d == 0 && skipx) continue;
       launch_ghost_stage(ctx->g, d, ctx->cfg.bc_lo[d], ctx->cfg.bc_hi[d], f, ncomp, dir, st);
       ctx->nlaunch[2] += 1;
       if (int r = check_launch(ctx, "ghost_stage")) return r;
@@ -645,8 +652,8 @@ static int fill_ghost_dims(pf_ctx* ctx, double* f, int ncomp, bool is_mu, int d0
   return PF_OK;
 }
 
-static int fill_ghosts(pf_ctx* ctx, double* f, int ncomp, bool is_mu) {
-  return fill_ghost_dims(ctx, f, ncomp, is_mu, 0, 3, ctx->stream);
+static int fill_ghosts(pf_ctx* ctx, double* f, int ncomp, bool is_mu, bool x_done = false) {
+  return fill_ghost_dims(ctx, f, ncomp, is_mu, 0, 3, ctx->stream, x_done);
 }
 
 // make the compute stream wait for an exchange still in flight on comm_s
@@ -730,6 +737,8 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
   // overlap: the exchanged dimensions' ghosts travel on the
   // comm stream while the mu-sweep updates the tiles that do not read them
   const bool ov = ctx->overlap && ctx->first_ex < 3 && ctx->variant != PF_VARIANT_NAIVE && !phi_only;
+  // the specialised phi-sweep writes phi_dst's x ghost columns itself (tuning phi_xghost)
+  const bool phi_x_done = g.xwrap && ctx->variant == PF_VARIANT_JIT && ctx->tune.phi_xghost;
   // Algorithm 1, line 1: phi-sweep (reads no mu ghosts: may overlap the previous mu exchange)
   prof_begin(ctx, 0, &e0);
   if (ctx->variant == PF_VARIANT_NAIVE)
@@ -745,7 +754,7 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
     if (int r = join_comm(ctx)) return r;
     // line 2: phi_dst communication and boundary handling
     prof_begin(ctx, 2, &e0);
-    int r = fill_ghosts(ctx, pd, PF_N, false);
+    int r = fill_ghosts(ctx, pd, PF_N, false, phi_x_done);
     prof_end(ctx, 2, e0);
     if (r) return r;
     if (phi_only) {
@@ -775,7 +784,7 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
     // line 2: local dimensions before the first exchanged one on the compute
     // stream, the rest (exchanges in x -> y -> z order) on the comm stream
     const int fe = ctx->first_ex;
-    if (int r = fill_ghost_dims(ctx, pd, PF_N, false, 0, fe, ctx->stream)) return r;
+    if (int r = fill_ghost_dims(ctx, pd, PF_N, false, 0, fe, ctx->stream, phi_x_done)) return r;
     CU(cudaEventRecord(ctx->ev_phi, ctx->stream));
     CU(cudaStreamWaitEvent(ctx->comm_s, ctx->ev_phi, 0));
     if (int r = fill_ghost_dims(ctx, pd, PF_N, false, fe, 3, ctx->comm_s)) return r;
@@ -1041,6 +1050,7 @@ const std::vector<TuneKnob>& tune_knobs() {
       {"phi_unroll", &pf_tuning::phi_unroll, JIT_PHI, {1, 2, 3}},
       {"phi_prefetch", &pf_tuning::phi_prefetch, JIT_PHI, {0, 1, 2}},
       {"phi_pfd", &pf_tuning::phi_pfd, JIT_PHI, {1, 2, 3}},
+      {"phi_xghost", &pf_tuning::phi_xghost, JIT_PHI, {0, 1}},
       {"mu_ty", &pf_tuning::mu_ty, JIT_MU, {3, 4, 5, 6, 8}},
       {"mu_tx", &pf_tuning::mu_tx, JIT_MU, {16, 32}},
       {"mu_minb", &pf_tuning::mu_minb, JIT_MU, {2, 3, 4}},

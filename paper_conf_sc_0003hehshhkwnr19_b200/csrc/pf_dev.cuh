@@ -25,10 +25,44 @@ struct Geom {
   int z0;  // global z index of local interior plane 0
   i64 pitch, plane, field, xoff;
   int x0, y0;  // global x / y index of local interior cell 0 (fluctuation counters)
+  // x periodic within this block (x not exchanged): the tuned phi-sweep
+  // writes the x ghost columns of phi_dst itself (store_x_ghost) and the
+  // ghost fill skips them (S§8(a) a6: the strided columns are its costly part)
+  int xwrap;
   __host__ __device__ __forceinline__ i64 at(int x, int y, int z) const {
     return (i64)(z + GUARD) * plane + (i64)(y + GUARD) * pitch + xoff + x;
   }
 };
+
+// x ghost columns of phi_dst written by the phi-sweep itself (x periodic
+// inside the block): cell x = nx-1 is the ghost x = -1, cell 0 the ghost
+// x = nx.  With nx % 4 == 0 the whole 32-B sector around the ghost is stored
+// (x = -4..-1, nx..nx+3; the other slots are guard cells no result reads),
+// so that L2 never merges a partial sector with DRAM.
+template <class GT>
+__device__ __forceinline__ void store_x_ghost(const GT& g, double* __restrict__ pd, int x, int y, int z, int a,
+                                              double v) {
+  if (!g.xwrap) return;
+  const bool vec = (g.nx % 4) == 0;
+  if (x == g.nx - 1) {
+    double* q = pd + a * g.field + g.at(vec ? -4 : -1, y, z);
+    if (vec) {
+      reinterpret_cast<double2*>(q)[0] = make_double2(v, v);
+      reinterpret_cast<double2*>(q)[1] = make_double2(v, v);
+    } else {
+      *q = v;
+    }
+  }
+  if (x == 0) {
+    double* q = pd + a * g.field + g.at(g.nx, y, z);
+    if (vec) {
+      reinterpret_cast<double2*>(q)[0] = make_double2(v, v);
+      reinterpret_cast<double2*>(q)[1] = make_double2(v, v);
+    } else {
+      *q = v;
+    }
+  }
+}
 
 // Tile selection of a sweep launch (interior / shell split for overlapping
 // the halo exchange): tile = blockIdx + off; if skip, tiles

@@ -41,7 +41,9 @@ size_t tuned_phi_smem();
 struct BCSpec {
   int kind_lo[3], kind_hi[3];
 };
-void launch_ghost_fill(const Geom& g, const BCSpec& bc, double* f, int ncomp, const double* dirichlet, cudaStream_t s);
+// skip_x: leave the x ghost columns (the sweeps wrap x, Geom::xwrap)
+void launch_ghost_fill(const Geom& g, const BCSpec& bc, double* f, int ncomp, const double* dirichlet, cudaStream_t s,
+                       bool skip_x = false);
 void launch_ghost_stage(const Geom& g, int d, int klo, int khi, double* f, int ncomp, const double* dirichlet,
                         cudaStream_t s);
 void launch_shift(const Geom& g, int k, int liquid, const double* mu_inf, const double* phi_src, const double* mu_src,

@@ -238,7 +238,8 @@ __global__ void k_ghost(GhostArgs A, double* __restrict__ f) {
     if (c < A.ncomp) f[c * g.field + dst] = v[c];
 }
 
-void launch_ghost_fill(const Geom& g, const BCSpec& bc, double* f, int ncomp, const double* dirichlet, cudaStream_t s) {
+void launch_ghost_fill(const Geom& g, const BCSpec& bc, double* f, int ncomp, const double* dirichlet, cudaStream_t s,
+                       bool skip_x) {
   GhostArgs A;
   A.g = g;
   A.bc = bc;
@@ -250,7 +251,8 @@ void launch_ghost_fill(const Geom& g, const BCSpec& bc, double* f, int ncomp, co
   const int64_t n0 = 2 * (int64_t)(g.nx + 2) * (g.ny + 2), n1 = 2 * (int64_t)(g.nx + 2) * g.nz,
                 n2 = 2 * (int64_t)g.ny * g.nz;
   const int64_t mx = n0 > n1 ? (n0 > n2 ? n0 : n2) : (n1 > n2 ? n1 : n2);
-  dim3 grid((unsigned)((mx + 255) / 256), 3);
+  // segment 2 (the x ghost columns) is not needed when the sweeps wrap x
+  dim3 grid((unsigned)((mx + 255) / 256), skip_x ? 2 : 3);
   k_ghost<<<grid, 256, 0, s>>>(A, f);
 }
 

@@ -168,6 +168,8 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, 
 #pragma unroll
       for (int a = 0; a < N; ++a) pd[a * F + c] = out[a];
 #pragma unroll
+      for (int a = 0; a < N; ++a) store_x_ghost(g, pd, x, y, z, a, out[a]);
+#pragma unroll
       for (int a = 0; a < N; ++a) {
         pm[a] = p0[a];
         p0[a] = pp[a];
@@ -273,6 +275,8 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, 
     if (active) {
 #pragma unroll
       for (int a = 0; a < N; ++a) pd[a * F + c] = out[a];
+#pragma unroll
+      for (int a = 0; a < N; ++a) store_x_ghost(g, pd, x, y, z, a, out[a]);
     }
 #pragma unroll
     for (int a = 0; a < N; ++a) {

@@ -66,7 +66,9 @@ size_t tuned_phi_smem() { return 0; }  // static shared memory only
 template <int L, bool TA>
 static void phi_launch(const DevParams& P, const Geom& g, const double* ps, const double* ms, double* pd,
                        cudaStream_t s) {
-  k_phi_tuned<L, TA><<<tuned_grid_phi(g, TY, 0), tuned_block(), 0, s>>>(P, g, ps, ms, pd);
+  Geom g0 = g;
+  g0.xwrap = 0;  // the generic build leaves the x ghost columns to the ghost fill
+  k_phi_tuned<L, TA><<<tuned_grid_phi(g0, TY, 0), tuned_block(), 0, s>>>(P, g0, ps, ms, pd);
 }
 
 void launch_phi_tuned(const DevParams& P, const Geom& g, const double* ps, const double* ms, double* pd,

@@ -119,7 +119,8 @@ def test_tuning_defaults_and_range_check(lib):
 
 @pytest.mark.parametrize("knobs", [
     {"phi_ty": 16, "phi_minb": 1, "phi_faces6": 0, "phi_unroll": 4, "phi_prefetch": 2, "phi_pfd": 3,
-     "mu_ty": 8, "mu_tx": 16, "mu_minb": 4, "mu_rpf": 0, "mu_halo_l1": 0, "mu_fxreg": 0, "mu_prefetch": 0},
+     "mu_ty": 8, "mu_tx": 16, "mu_minb": 4, "mu_rpf": 0, "mu_halo_l1": 0, "mu_fxreg": 0, "mu_prefetch": 0,
+     "phi_xghost": 1, "mu_ldhint": 2, "mu_qreg": 1},
     {"phi_ty": 8, "phi_minb": 2, "phi_zc": 32, "phi_prefetch": 0, "mu_ty": 3, "mu_minb": 5, "mu_zc": 24,
      "mu_pfd": 3, "mu_prefetch": 2},
 ])

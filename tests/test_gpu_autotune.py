@@ -24,11 +24,14 @@ TOL_1 = 1e-12
 # z-chunks, schedule transformations)
 CORNERS = [
     {},
-    {"phi_ty": 16, "phi_minb": 1, "phi_faces6": 0, "phi_unroll": 4, "phi_prefetch": 2, "phi_pfd": 3},
+    {"phi_ty": 16, "phi_minb": 1, "phi_faces6": 0, "phi_unroll": 4, "phi_prefetch": 2, "phi_pfd": 3,
+     "phi_xghost": 1},
     {"phi_ty": 8, "phi_minb": 2, "phi_zc": 5, "phi_faces6": 0, "phi_prefetch": 0},
     {"mu_ty": 8, "mu_tx": 16, "mu_minb": 4, "mu_rpf": 0, "mu_halo_l1": 0, "mu_fxreg": 0, "mu_prefetch": 0},
     {"mu_ty": 3, "mu_minb": 5, "mu_zc": 7, "mu_pfd": 3, "mu_prefetch": 2},
-    {"mu_ty": 6, "mu_minb": 2, "mu_zc": 24, "phi_zc": 32, "phi_unroll": 3},
+    {"mu_ty": 6, "mu_minb": 2, "mu_zc": 24, "phi_zc": 32, "phi_unroll": 3, "phi_xghost": 1},
+    {"mu_ldhint": 1, "mu_qreg": 1, "phi_xghost": 1},
+    {"mu_ldhint": 2, "mu_tx": 16, "mu_ty": 4, "mu_minb": 4},
 ]
 
 
