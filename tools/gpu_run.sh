@@ -1,5 +1,6 @@
 #!/bin/bash
-# One GPU session: micro-benchmarks, GPU tests, short bench, ncu launch list + full capture.
+# One GPU session: GPU tests, smoke, bench (config 2 and config 4, auto-tuned),
+# ncu launch list + full captures of the sweeps in the tuning the bench chose.
 # usage (from the repo root on the GPU box): bash tools/gpu_run.sh [tag]
 TAG=${1:-r01}
 OUT=gpurun_out/$TAG
@@ -7,16 +8,19 @@ mkdir -p $OUT
 nvidia-smi > $OUT/nvidia-smi.txt 2>&1
 python -c "import __graft_entry__ as g; g.build()" > $OUT/build.log 2>&1
 [ -x tools/build/fp64_micro ] && timeout 120 tools/build/fp64_micro > $OUT/fp64_micro.json 2>&1
-timeout 900 python -m pytest tests -m gpu -x -q > $OUT/pytest_gpu.log 2>&1; echo "pytest exit $?" >> $OUT/pytest_gpu.log
+timeout 1200 python -m pytest tests -m gpu -x -q > $OUT/pytest_gpu.log 2>&1; echo "pytest exit $?" >> $OUT/pytest_gpu.log
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $OUT/smoke.log 2>&1
-timeout 600 python bench.py --steps 100 --warmup 5 > $OUT/bench.json 2> $OUT/bench.err
-timeout 600 python bench.py --config strong --steps 20 --warmup 3 --no-cpu-baseline > $OUT/bench_strong.json 2>> $OUT/bench.err
+timeout 900 python bench.py --steps 200 --warmup 10 > $OUT/bench.json 2> $OUT/bench.err
+timeout 900 python bench.py --config strong --steps 20 --warmup 3 --no-cpu-baseline --autotune 1 > $OUT/bench_strong.json 2>> $OUT/bench.err
+# the tuning the bench selected; the profiled runs use it without re-tuning
+TUNE=$(python -c "import json; print(json.dumps(json.load(open('$OUT/bench.json'))['config']['tuning']))" 2>/dev/null || echo '{}')
+echo "$TUNE" > $OUT/tuning.json
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches.csv \
-   python bench.py --steps 10 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_launch.log 2>&1
+   python bench.py --steps 10 --warmup 3 --no-cpu-baseline --no-e2e --autotune 0 --tuning "$TUNE" > $OUT/ncu_launch.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:pf_jit_mu -s 3 -c 1 -o $OUT/prof_mu \
-   python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_mu.log 2>&1
+   python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e --autotune 0 --tuning "$TUNE" > $OUT/ncu_mu.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:pf_jit_phi -s 3 -c 1 -o $OUT/prof_phi \
-   python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_phi.log 2>&1
+   python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e --autotune 0 --tuning "$TUNE" > $OUT/ncu_phi.log 2>&1
 timeout 600 ncu --set full --clock-control none -k regex:k_ghost -s 6 -c 1 -o $OUT/prof_ghost \
-   python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e > $OUT/ncu_ghost.log 2>&1
+   python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e --autotune 0 --tuning "$TUNE" > $OUT/ncu_ghost.log 2>&1
 echo done > $OUT/DONE
