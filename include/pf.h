@@ -211,6 +211,8 @@ typedef struct {
   int phi_unroll;    /* phi-sweep z-loop unroll factor: 1..4                        */
   int phi_prefetch;  /* software prefetch of the own column: 0 off, 1 L2, 2 L1      */
   int phi_pfd;       /* prefetch distance in planes: 1..4                           */
+  int phi_zrec;      /* 1: the -z face flux is recomputed per plane instead of
+                        carried in registers (fewer registers, more fp64 work)   */
   int phi_xghost;    /* 1: the phi-sweep writes phi_dst's x ghost columns itself when
                         x is periodic inside the block (the ghost fill skips them) */
   int mu_ty;         /* mu-sweep tile height: 3..8 (tile width 32), 4..8 (width 16) */
@@ -226,6 +228,8 @@ typedef struct {
                         build (no shared-memory re-read; needs registers)        */
   int mu_ldhint;     /* L1 policy of the mu-sweep's phi_dst / mu loads: 0 default,
                         1 evict_first, 2 no_allocate                              */
+  int mu_hpipe;      /* 1: halo-ring cells' loads for plane k+1 issued at the end of
+                        plane k's face phase (software pipelining)               */
 } pf_tuning;
 
 /* The built-in defaults (the measured best at 256^3 on one B200,

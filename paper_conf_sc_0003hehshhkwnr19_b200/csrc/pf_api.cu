@@ -1050,6 +1050,7 @@ const std::vector<TuneKnob>& tune_knobs() {
       {"phi_unroll", &pf_tuning::phi_unroll, JIT_PHI, {1, 2, 3}},
       {"phi_prefetch", &pf_tuning::phi_prefetch, JIT_PHI, {0, 1, 2}},
       {"phi_pfd", &pf_tuning::phi_pfd, JIT_PHI, {1, 2, 3}},
+      {"phi_zrec", &pf_tuning::phi_zrec, JIT_PHI, {0, 1}},
       {"phi_xghost", &pf_tuning::phi_xghost, JIT_PHI, {0, 1}},
       {"mu_ty", &pf_tuning::mu_ty, JIT_MU, {3, 4, 5, 6, 8}},
       {"mu_tx", &pf_tuning::mu_tx, JIT_MU, {16, 32}},
@@ -1062,6 +1063,7 @@ const std::vector<TuneKnob>& tune_knobs() {
       {"mu_fxreg", &pf_tuning::mu_fxreg, JIT_MU, {0, 1}},
       {"mu_qreg", &pf_tuning::mu_qreg, JIT_MU, {0, 1}},
       {"mu_ldhint", &pf_tuning::mu_ldhint, JIT_MU, {0, 1, 2}},
+      {"mu_hpipe", &pf_tuning::mu_hpipe, JIT_MU, {0, 1}},
   };
   return k;
 }

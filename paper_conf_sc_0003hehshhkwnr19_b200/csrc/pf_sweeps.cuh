@@ -47,6 +47,9 @@ constexpr int kPhiUnroll = PF_PHI_UNROLL;
 #ifndef PF_PREFETCH_D
 #define PF_PREFETCH_D 2  // planes ahead
 #endif
+#ifndef PF_MU_HPIPE  // halo-ring cell's loads for plane k+1 issued at the end of plane k's face phase
+#define PF_MU_HPIPE 0
+#endif
 #ifndef PF_MU_LDHINT  // L1 policy of the mu-sweep's phi_dst / mu loads: 0 default, 1 evict_first, 2 no_allocate
 #define PF_MU_LDHINT 0
 #endif
@@ -348,6 +351,49 @@ __device__ __forceinline__ void build_cell(const GT& g, const double* __restrict
   for (int j = 0; j < D_NV / 2; ++j) d[j] = make_double2(v[2 * j], v[2 * j + 1]);
 }
 
+// halo-ring cell of the mu-sweep, software-pipelined (PF_MU_HPIPE): the raw
+// values of plane k+1 are loaded at the end of plane k's face phase (the
+// loads complete under the barrier and the next own-cell build) and turned
+// into D at plane k+1.  Same arithmetic as build_cell (bitwise equal).
+struct HaloRaw {
+  double f[N], tp[N], tm[N], zp[N], zm[N], d[N], m[M];
+};
+template <class GT>
+__device__ __forceinline__ void halo_load(const GT& g, const double* __restrict__ ps, const double* __restrict__ pd,
+                                          const double* __restrict__ ms, int x, int y, int k, i64 toff, HaloRaw& h) {
+  const i64 F = g.field;
+  const i64 c = g.at(x, y, k);
+#pragma unroll
+  for (int a = 0; a < N; ++a) {
+    const double* f = ps + a * F + c;
+    h.f[a] = __ldg(f);
+    h.tp[a] = __ldg(f + toff);
+    h.tm[a] = __ldg(f - toff);
+    h.zp[a] = __ldg(f + g.plane);
+    h.zm[a] = __ldg(f - g.plane);
+    h.d[a] = ldh(pd + a * F + c);
+  }
+  h.m[0] = ldh(ms + c);
+  h.m[1] = ldh(ms + F + c);
+}
+__device__ __forceinline__ void halo_store(const HaloRaw& h, bool wx, double* __restrict__ D, int i) {
+  double v[D_NV];
+#pragma unroll
+  for (int a = 0; a < N; ++a) {
+    const double t = h.tp[a] - h.tm[a];
+    v[D_F + a] = h.f[a];
+    v[D_CX + a] = wx ? t : 0.0;
+    v[D_CY + a] = wx ? 0.0 : t;
+    v[D_CZ + a] = h.zp[a] - h.zm[a];
+    v[D_DP + a] = h.d[a] - h.f[a];
+  }
+  v[D_MU + 0] = h.m[0];
+  v[D_MU + 1] = h.m[1];
+  double2* d = reinterpret_cast<double2*>(D + (size_t)i * D_NV);
+#pragma unroll
+  for (int j = 0; j < D_NV / 2; ++j) d[j] = make_double2(v[2 * j], v[2 * j + 1]);
+}
+
 // build D of the own cell (x,y,k) into slot i with its z column carried in
 // registers: fc = phi_src(k) (loaded as the +z neighbour one plane earlier),
 // fm = phi_src(k-1); loads phi_src(k+1) into fc for the next plane.
@@ -518,6 +564,11 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
     Dp.m[1] = ldh(ms + F + c);
   }
   double divxy[M] = {0.0, 0.0}, Fzm[M] = {0.0, 0.0};
+#if PF_MU_HPIPE
+  HaloRaw hraw;
+  const i64 htoff = hwx ? 1 : g.pitch;  // the halo cell's tangential direction
+  if (hs >= 0 && z0 < z1) halo_load(g, ps, pd, ms, hgx, hgy, z0, htoff, hraw);
+#endif
 #if PF_MU_ZCARRY
   double fcar[N];  // phi_src(k) of the own cell, carried along z
   {
@@ -573,7 +624,11 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
 #else
     build_cell<NC>(g, ps, pd, ms, xc, yc, k, true, true, !last, D, me);
 #endif
+#if PF_MU_HPIPE
+    if (!last && hs >= 0) halo_store(hraw, hwx, D, hs);
+#else
     if (!last && hs >= 0) build_cell<NC>(g, ps, pd, ms, hgx, hgy, k, hwx, hwy, true, D, hs);
+#endif
     __syncthreads();
     // (b) z-face k-1/2 from registers (plane k-1) and shared memory (plane k)
     FaceSide q;
@@ -679,6 +734,9 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, c
       }
     }
     if constexpr (!last) {
+#if PF_MU_HPIPE
+      if (hs >= 0 && k + 1 < z1) halo_load(g, ps, pd, ms, hgx, hgy, k + 1, htoff, hraw);
+#endif
       __syncthreads();
 #pragma unroll
       for (int i = 0; i < M; ++i)
