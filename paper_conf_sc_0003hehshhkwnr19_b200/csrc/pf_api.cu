@@ -449,8 +449,26 @@ int pf_create(const pf_config* cfg, pf_ctx** out) {
     }
   }
   {
-    const char* fe = getenv("PF_FORCE_EXCHANGE");  // debug: periodic self-exchange through pack/unpack
-    ctx->force_exchange = fe && fe[0] == '1';
+    // debug: periodic self-exchange through pack/unpack ("1": device copies;
+    // "nccl": a 1-rank NCCL communicator, so that the NCCL send/recv and
+    // all-reduce code of world > 1 runs on one GPU)
+    const char* fe = getenv("PF_FORCE_EXCHANGE");
+    const bool fnccl = fe && strcmp(fe, "nccl") == 0;
+    ctx->force_exchange = fe && (fe[0] == '1' || fnccl);
+    if (fnccl && world == 1) {
+      if (!g_nccl.load(&ctx->err)) {
+        *out = ctx;
+        return PF_ENCCL;
+      }
+      ncclUniqueId id;
+      ncclResult_t r = g_nccl.GetUniqueId(&id);
+      if (r == ncclSuccess) r = g_nccl.CommInitRank(&ctx->comm, 1, id, 0);
+      if (r != ncclSuccess) {
+        ctx->err = std::string("1-rank NCCL communicator: ") + g_nccl.GetErrorString(r);
+        *out = ctx;
+        return PF_ENCCL;
+      }
+    }
   }
   // x periodic inside the block: the specialised phi-sweep may write phi_dst's x ghost columns
   ctx->g.xwrap = (cfg->bc_lo[0] == PF_BC_PERIODIC && !ctx->exchange[0] && !ctx->force_exchange) ? 1 : 0;

@@ -215,6 +215,38 @@ def test_forced_exchange_path_bitwise(pfmod, monkeypatch):
     assert np.array_equal(ref[0], got[0]) and np.array_equal(ref[1], got[1])
 
 
+@pytest.mark.parametrize("bc", ["periodic", "ds"])
+def test_nccl_self_exchange_bitwise(pfmod, monkeypatch, bc):
+    """The world > 1 code path on one GPU: PF_FORCE_EXCHANGE=nccl gives the
+    context a 1-rank NCCL communicator, so the halo exchange of every
+    periodic dimension goes through pack -> ncclSend/ncclRecv to itself ->
+    unpack (on the comm stream, overlapped with the interior mu tiles), and
+    the window / monitor reductions through ncclAllReduce.  Bitwise equal to
+    the local ghost fill; window shifts included for the DS case."""
+    if bc == "periodic":
+        P, B, shape = I.params_stress(), None, (40, 20, 70)
+        phi, mu = I.ic_voronoi(shape, seed=8)
+    else:
+        P = I.params_c4("ds", window_check=2, window_frac=0.3)
+        B, shape = I.BC_DS, (24, 20, 40)
+        phi, mu = I.ic_lamellar(shape, seed=3, z_front=10)
+    outs = []
+    for force in ("0", "nccl"):
+        monkeypatch.setenv("PF_FORCE_EXCHANGE", force)
+        g = pfmod.PhaseField(shape, P, bc=B)
+        g.init_fields(phi, mu)
+        g.step(6)
+        rep = g.autotune(mask=pfmod.PF_MU, passes=1, reps=2) if force == "nccl" else None
+        g.step(4)
+        outs.append((g.download(), g.state(), g.monitor(), g.front_height()))
+        g.close()
+    (a, sa, ma, ha), (b, sb, mb, hb) = outs
+    assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
+    assert sa == sb and ha == hb and np.array_equal(ma, mb)
+    if bc == "ds":
+        assert sa["z_off"] > 0  # the window shifted (collective front height)
+
+
 @pytest.mark.parametrize("variant", ["jit", "tuned"])
 def test_overlapped_exchange_bitwise(pfmod, monkeypatch, variant):
     """Interior/shell split of the mu-sweep with the phi exchange on a second
