@@ -100,9 +100,22 @@ struct pf_ctx {
   cudaEvent_t ev_phi = nullptr, ev_phix = nullptr, ev_mu = nullptr, ev_mux = nullptr;
   bool mux_pending = false;         // mu exchange in flight on comm_s
   bool overlap = true;
+  int64_t mu_launches_per_step = 1, ghost_launches_per_step = 0;  // launch accounting of graph replays
   JitKernel* jphi = nullptr;  // specialised sweeps for (dp, g, tune); reset by pf_set_params / pf_set_tuning
   JitKernel* jmu = nullptr;
   pf_tuning tune;             // tuning of the specialised sweeps (pf_set_tuning, pf_autotune)
+  // CUDA-graph steps (S§8(d) D.7): runs of steps between window checks are
+  // captured once per (length, buffer parity) and replayed; the sweeps read
+  // the per-step values (T base, step) from sv_dev, written before each replay
+  bool use_graph = true;
+  cudaStream_t cap_s = nullptr;      // private stream the steps are captured on (the caller's may be legacy)
+  StepVals* sv_dev = nullptr;        // [64] in the workspace
+  const StepVals* cap_sv = nullptr;  // set while capturing one step of a graph
+  struct GraphEntry {
+    int k, cur;
+    cudaGraphExec_t exec;
+  };
+  std::vector<GraphEntry> graphs;
   ncclComm_t comm = nullptr;
   // profiling
   bool prof = false;
@@ -115,6 +128,11 @@ struct pf_ctx {
 };
 
 namespace {
+
+void drop_graphs(pf_ctx* c) {
+  for (auto& e : c->graphs) cudaGraphExecDestroy(e.exec);
+  c->graphs.clear();
+}
 
 int fail(pf_ctx* c, int code, const char* fmt, ...) {
   if (c) {
@@ -178,7 +196,7 @@ int layout_of(const pf_config* cfg, pf_layout* L, int coord[3]) {
   L->field = L->plane * (nz + 2 * GUARD);
   L->phi_bytes = (size_t)PF_N * L->field * sizeof(double) + 256;  // +256: tail slack for vector loads
   L->mu_bytes = (size_t)PF_M * L->field * sizeof(double) + 256;
-  size_t ws = 256;  // reduction scratch
+  size_t ws = 256 + 1024;  // reduction scratch, per-step values of CUDA-graph steps
   Geom g{nx, ny, nz, L->offset[2], L->pitch, L->plane, L->field, L->x_off, L->offset[0], L->offset[1]};
   for (int d = 0; d < 3; ++d) ws += 4 * align256(halo_slab_elems(g, d) * PF_N * sizeof(double));
   L->workspace_bytes = ws;
@@ -415,6 +433,8 @@ int pf_create(const pf_config* cfg, pf_ctx** out) {
   char* w = (char*)cfg->workspace;
   ctx->red = (unsigned long long*)w;
   w += 256;
+  ctx->sv_dev = (StepVals*)w;
+  w += 1024;
   for (int d = 0; d < 3; ++d) {
     const size_t b = align256(halo_slab_elems(ctx->g, d) * PF_N * sizeof(double));
     for (int s = 0; s < 2; ++s) {
@@ -482,7 +502,10 @@ int pf_create(const pf_config* cfg, pf_ctx** out) {
   {  // side stream: halo exchanges (N > 1) and the mu ghost fill (any N)
     const char* ov = getenv("PF_OVERLAP");
     ctx->overlap = !(ov && ov[0] == '0');
+    const char* gr = getenv("PF_GRAPH");
+    ctx->use_graph = !(gr && gr[0] == '0');
     e = cudaStreamCreateWithFlags(&ctx->comm_s, cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&ctx->cap_s, cudaStreamNonBlocking);
     cudaEvent_t* evs[4] = {&ctx->ev_phi, &ctx->ev_phix, &ctx->ev_mu, &ctx->ev_mux};
     for (cudaEvent_t* ev : evs)
       if (e == cudaSuccess) e = cudaEventCreateWithFlags(ev, cudaEventDisableTiming);
@@ -510,11 +533,13 @@ int pf_destroy(pf_ctx* ctx) {
     cudaEventDestroy(o.second.first);
     cudaEventDestroy(o.second.second);
   }
+  drop_graphs(ctx);
   if (ctx->comm) g_nccl.CommDestroy(ctx->comm);
   if (ctx->comm_s) {
     cudaStreamSynchronize(ctx->comm_s);
     cudaStreamDestroy(ctx->comm_s);
   }
+  if (ctx->cap_s) cudaStreamDestroy(ctx->cap_s);
   for (cudaEvent_t ev : {ctx->ev_phi, ctx->ev_phix, ctx->ev_mu, ctx->ev_mux})
     if (ev) cudaEventDestroy(ev);
   if (ctx->pinned) cudaFreeHost(ctx->pinned);
@@ -605,6 +630,7 @@ int pf_set_params(pf_ctx* ctx, const pf_params* p) {
   ctx->hp = *p;
   ctx->have_params = true;
   ctx->jphi = ctx->jmu = nullptr;
+  drop_graphs(ctx);
   return PF_OK;
 }
 
@@ -728,7 +754,7 @@ static int launch_mu(pf_ctx* ctx, const TileSel* ts, dim3 grid, const double* ps
   if (ctx->variant == PF_VARIANT_NAIVE)
     launch_mu_naive(ctx->dp, ctx->g, ps, pd, ms, md, ctx->stream);
   else if (ctx->variant == PF_VARIANT_JIT)
-    CU(jit_launch_mu(ctx->jmu, ctx->dp, ts, grid, ps, pd, ms, md, ctx->stream));
+    CU(jit_launch_mu(ctx->jmu, ctx->dp, ts, grid, ps, pd, ms, md, ctx->stream, ctx->cap_sv));
   else
     launch_mu_tuned(ctx->dp, ctx->g, ts, grid, ps, pd, ms, md, ctx->stream);
   ctx->nlaunch[1] += 1;
@@ -762,7 +788,7 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
   if (ctx->variant == PF_VARIANT_NAIVE)
     launch_phi_naive(ctx->dp, g, ps, ms, pd, ctx->stream);
   else if (ctx->variant == PF_VARIANT_JIT)
-    CU(jit_launch_phi(ctx->jphi, ctx->dp, ps, ms, pd, ctx->stream));
+    CU(jit_launch_phi(ctx->jphi, ctx->dp, ps, ms, pd, ctx->stream, ctx->cap_sv));
   else
     launch_phi_tuned(ctx->dp, g, ps, ms, pd, ctx->stream);
   ctx->nlaunch[0] += 1;
@@ -848,12 +874,112 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
   return PF_OK;
 }
 
+// k consecutive steps (no window check among them) as one CUDA graph:
+// captured on first use for (k, buffer parity), then replayed; the step
+// values (T base of each step, step index) go to sv_dev first (one kernel)
+static int step_graph(pf_ctx* ctx, int k) {
+  if (int r = join_comm(ctx)) return r;
+  const Geom& g = ctx->g;
+  StepBatch b;
+  b.k = k;
+  b.step0 = (unsigned long long)ctx->step;
+  for (int i = 0; i < k; ++i) {  // the host formula of step_impl, step by step [A13]
+    const double t = (double)(ctx->step + i) * ctx->hp.dt;
+    b.Tbase[i] = ctx->hp.T0 + ctx->hp.G * (((double)g.z0 + (double)ctx->z_off) * ctx->hp.dx - ctx->hp.v * t);
+  }
+  launch_set_steps(ctx->sv_dev, b, ctx->stream);
+  ctx->nlaunch[3] += 1;
+  if (int r = check_launch(ctx, "set_steps")) return r;
+  cudaGraphExec_t exec = nullptr;
+  for (auto& e : ctx->graphs)
+    if (e.k == k && e.cur == ctx->cur) exec = e.exec;
+  const int cur0 = ctx->cur;
+  const int64_t step0 = ctx->step;
+  const int64_t nl[4] = {ctx->nlaunch[0], ctx->nlaunch[1], ctx->nlaunch[2], ctx->nlaunch[3]};
+  if (!exec) {
+    // capture on the library's own stream (the caller's may be the legacy
+    // stream, which cannot be captured); the graph is launched on the caller's.
+    // Any failure of the capture falls back to launching the steps directly.
+    const cudaStream_t user = ctx->stream;
+    const auto nl0 = std::vector<int64_t>(ctx->nlaunch, ctx->nlaunch + 4);
+    cudaError_t e = cudaStreamBeginCapture(ctx->cap_s, cudaStreamCaptureModeThreadLocal);
+    int r = e == cudaSuccess ? PF_OK : PF_ECUDA;
+    if (r == PF_OK) {
+      ctx->stream = ctx->cap_s;
+      for (int i = 0; i < k && r == PF_OK; ++i) {
+        ctx->cap_sv = ctx->sv_dev + i;
+        r = step_impl(ctx, false);
+      }
+      ctx->cap_sv = nullptr;
+      if (r == PF_OK) r = join_comm(ctx);
+      ctx->stream = user;
+      cudaGraph_t graph = nullptr;
+      e = cudaStreamEndCapture(ctx->cap_s, &graph);
+      if (r == PF_OK && e == cudaSuccess) e = cudaGraphInstantiate(&exec, graph, 0);
+      if (graph) cudaGraphDestroy(graph);
+      if (e != cudaSuccess) r = PF_ECUDA;
+    }
+    // the capture only recorded the steps: rewind the host state
+    ctx->cur = cur0;
+    ctx->step = step0;
+    ctx->mux_pending = false;
+    if (r != PF_OK) {
+      cudaGetLastError();
+      if (exec) cudaGraphExecDestroy(exec);
+      for (int i = 0; i < 4; ++i) ctx->nlaunch[i] = nl0[i];
+      ctx->use_graph = false;  // this context steps without graphs from now on
+      ctx->err.clear();
+      for (int i = 0; i < k; ++i)
+        if (int r2 = step_impl(ctx, false)) return r2;
+      return PF_OK;
+    }
+    ctx->graphs.push_back({k, cur0, exec});
+  }
+  CU(cudaGraphLaunch(exec, ctx->stream));
+  for (int i = 0; i < k; ++i) {  // what the k steps did to the host state (step_impl)
+    ctx->cur = 1 - ctx->cur;
+    ctx->step += 1;
+  }
+  // launches per category as if the steps had been launched one by one
+  const int64_t per[4] = {ctx->nlaunch[0] - nl[0], ctx->nlaunch[1] - nl[1], ctx->nlaunch[2] - nl[2],
+                          ctx->nlaunch[3] - nl[3]};
+  if (per[0] == 0) {  // replay of a cached graph: count what its capture launched
+    ctx->nlaunch[0] += k;
+    ctx->nlaunch[1] += (int64_t)k * ctx->mu_launches_per_step;
+    ctx->nlaunch[2] += (int64_t)k * ctx->ghost_launches_per_step;
+  } else {
+    ctx->mu_launches_per_step = per[1] / k;
+    ctx->ghost_launches_per_step = per[2] / k;
+  }
+  ctx->mux_pending = false;
+  return PF_OK;
+}
+
 int pf_step(pf_ctx* ctx, int64_t nsteps) {
   if (!ctx) return PF_EINVAL;
   if (!ctx->have_params || !ctx->have_fields) return fail(ctx, PF_ESTATE, "pf_step before pf_set_params/pf_init_fields");
   if (nsteps < 0) return fail(ctx, PF_EINVAL, "nsteps < 0");
-  for (int64_t n = 0; n < nsteps; ++n) {
-    if (int r = step_impl(ctx, false)) return r;
+  const bool graphs = ctx->use_graph && ctx->variant == PF_VARIANT_JIT && !ctx->prof;
+  for (int64_t n = 0; n < nsteps;) {
+    int64_t k = 1;
+    if (graphs) {  // steps up to the next window check (which needs the host), at most 64
+      k = nsteps - n;
+      const int nc = ctx->hp.window_check;
+      if (nc > 0) k = std::min<int64_t>(k, nc - ctx->step % nc);
+      k = std::min<int64_t>(k, 64);
+    }
+    if (k >= 2) {
+      if (ctx->variant == PF_VARIANT_JIT && (!ctx->jphi || !ctx->jmu)) {
+        std::string err;
+        ctx->jphi = jit_get(ctx->dp, ctx->g, ctx->tune, JIT_PHI, &err);
+        if (ctx->jphi) ctx->jmu = jit_get(ctx->dp, ctx->g, ctx->tune, JIT_MU, &err);
+        if (!ctx->jphi || !ctx->jmu) return fail(ctx, PF_ECUDA, "run-time specialisation failed: %s", err.c_str());
+      }
+      if (int r = step_graph(ctx, (int)k)) return r;
+    } else {
+      if (int r = step_impl(ctx, false)) return r;
+    }
+    n += k;
     if (int r = window_maybe(ctx)) return r;
   }
   return join_comm(ctx);
@@ -944,6 +1070,7 @@ int pf_set_variant(pf_ctx* ctx, int variant) {
   if (!ctx || (variant != PF_VARIANT_TUNED && variant != PF_VARIANT_NAIVE && variant != PF_VARIANT_JIT))
     return PF_EINVAL;
   ctx->variant = variant;
+  drop_graphs(ctx);
   return PF_OK;
 }
 
@@ -1043,6 +1170,7 @@ int pf_set_tuning(pf_ctx* ctx, const pf_tuning* t) {
   if (const char* m = tuning_check(*t)) return fail(ctx, PF_EINVAL, "pf_set_tuning: %s", m);
   ctx->tune = *t;
   ctx->jphi = ctx->jmu = nullptr;
+  drop_graphs(ctx);
   return PF_OK;
 }
 
@@ -1243,6 +1371,7 @@ int pf_autotune(pf_ctx* ctx, unsigned mask, int passes, int reps, char* log, int
   }
   ctx->tune = best;
   ctx->jphi = ctx->jmu = nullptr;
+  drop_graphs(ctx);
   {
     std::string err;
     ctx->jphi = jit_get(ctx->dp, ctx->g, best, JIT_PHI, &err);

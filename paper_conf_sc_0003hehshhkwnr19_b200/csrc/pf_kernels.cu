@@ -274,6 +274,16 @@ __global__ void k_shift(Geom g, int k, int L, double mi0, double mi1, const doub
   md[g.field + c] = in ? ms[g.field + sidx] : mi1;
 }
 
+__global__ void k_set_steps(StepVals* dst, StepBatch b) {
+  const int i = threadIdx.x;
+  if (i < b.k) {
+    dst[i].Tbase = b.Tbase[i];
+    dst[i].step = b.step0 + (unsigned long long)i;
+  }
+}
+
+void launch_set_steps(StepVals* dst, const StepBatch& b, cudaStream_t s) { k_set_steps<<<1, 64, 0, s>>>(dst, b); }
+
 void launch_shift(const Geom& g, int k, int liquid, const double* mu_inf, const double* ps, const double* ms,
                   double* pd, double* md, cudaStream_t s) {
   dim3 b(128), gr((g.nx + 127) / 128, g.ny, g.nz);

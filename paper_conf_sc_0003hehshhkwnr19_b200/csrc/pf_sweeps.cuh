@@ -102,8 +102,8 @@ constexpr int MU_TY = PF_MU_TY;
 #ifndef PF_PHI_ZREC
 #define PF_PHI_ZREC 0
 #endif
-template <class PT, class GT, int L, bool TA, int PTY = TY>
-__device__ __forceinline__ void phi_tuned_body(const PT& P, const DevParams& R, const GT& g,
+template <class PT, class GT, int L, bool TA, int PTY = TY, class RT = DevParams>
+__device__ __forceinline__ void phi_tuned_body(const PT& P, const RT& R, const GT& g,
                                                const double* __restrict__ ps, const double* __restrict__ ms,
                                                double* __restrict__ pd) {
 #if PF_PHI_FACES6
@@ -494,8 +494,8 @@ __device__ __forceinline__ void side_from_smem(const double* __restrict__ D, int
   s.m[1] = t.y;
 }
 
-template <class PT, class GT, int L, bool TA, int MTY, int MTX = TX>
-__device__ __forceinline__ void mu_tuned_body(const PT& P, const DevParams& R, const GT& g, const TileSel& ts,
+template <class PT, class GT, int L, bool TA, int MTY, int MTX = TX, class RT = DevParams>
+__device__ __forceinline__ void mu_tuned_body(const PT& P, const RT& R, const GT& g, const TileSel& ts,
                                               const double* __restrict__ ps, const double* __restrict__ pd,
                                               const double* __restrict__ ms, double* __restrict__ md) {
   constexpr int NC = MuTile<MTY, MTX>::NC, HX = MuTile<MTY, MTX>::HX;

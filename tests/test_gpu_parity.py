@@ -247,6 +247,39 @@ def test_nccl_self_exchange_bitwise(pfmod, monkeypatch, bc):
         assert sa["z_off"] > 0  # the window shifted (collective front height)
 
 
+@pytest.mark.parametrize("case", ["ds_window", "stress_xi", "nccl_periodic"])
+def test_graph_steps_bitwise(pfmod, monkeypatch, case):
+    """pf_step replays runs of steps between window checks as CUDA graphs
+    (S§8(d) D.7), the sweeps reading each step's T base and step index from
+    device memory: bitwise equal to launching every step (PF_GRAPH=0) --
+    frozen temperature moving with v t, window shifts, the fluctuation
+    counter (step) and the NCCL exchange inside the captured graph."""
+    if case == "ds_window":
+        P = I.params_c4("ds", window_check=7, window_frac=0.3)
+        B, shape = I.BC_DS, (24, 20, 40)
+        phi, mu = I.ic_lamellar(shape, seed=3, z_front=10)
+    else:
+        P = I.params_stress(xi_amp=0.02, xi_seed=7) if case == "stress_xi" else I.params_stress()
+        B, shape = None, (20, 24, 40)
+        phi, mu = I.ic_voronoi(shape, seed=5)
+    if case == "nccl_periodic":
+        monkeypatch.setenv("PF_FORCE_EXCHANGE", "nccl")
+    outs = []
+    for gr in ("0", "1"):
+        monkeypatch.setenv("PF_GRAPH", gr)
+        g = pfmod.PhaseField(shape, P, bc=B)
+        g.init_fields(phi, mu)
+        for n in (1, 5, 30, 2, 70):  # runs of several lengths: new and cached graphs, both buffer parities
+            g.step(n)
+        outs.append((g.download(), g.state()))
+        g.close()
+    (a, sa), (b, sb) = outs
+    assert sa == sb
+    assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
+    if case == "ds_window":
+        assert sa["z_off"] > 0
+
+
 @pytest.mark.parametrize("variant", ["jit", "tuned"])
 def test_overlapped_exchange_bitwise(pfmod, monkeypatch, variant):
     """Interior/shell split of the mu-sweep with the phi exchange on a second
