@@ -110,15 +110,19 @@ class ClockSampler:
                 "power_w_max": max(power) if power else None}
 
 
-def traffic_per_launch():
-    """dram read+write bytes per mu-sweep launch from the committed ncu --set
-    full summary (profiles/), or None."""
+def ncu_summary(key, kernel="mu_sweep"):
+    """A per-launch figure of the committed ncu --set full summary
+    (profiles/ncu_summary.json; 256^3 launch), or None."""
     p = os.path.join(ROOT, "profiles", "ncu_summary.json")
     try:
-        d = json.load(open(p))
-        return d["mu_sweep"]["dram_bytes_per_launch"]
+        return json.load(open(p))[kernel][key]
     except Exception:
         return None
+
+
+def traffic_per_launch():
+    """dram read+write bytes per mu-sweep launch from the committed ncu summary, or None."""
+    return ncu_summary("dram_bytes_per_launch")
 
 
 def cpu_baseline(P, bc, seconds=12.0, shape=(64, 96, 96), strong=False):
@@ -347,6 +351,11 @@ def main():
                      # the committed ncu capture is of the 256^3 block launch
                      "traffic": traffic_per_launch() if cells_local == 256 ** 3 else None,
                      "flop_per_cell": F_MU, "cells_per_launch": cells_local,
+                     # context: the fp64 work the specialised kernel actually issues (ncu, DADD + DMUL
+                     # + 2 DFMA per cell at 256^3) and the rate it sustains at this launch time
+                     "hw_flop_per_cell": ncu_summary("hw_flop_per_cell"),
+                     "hw_achieved": (ncu_summary("hw_flop_per_cell") * cells_local / (mu_ms / mu_n * 1e-3) / 1e12)
+                     if (mu_n and ncu_summary("hw_flop_per_cell")) else None,
                      "avg_launch_ms": mu_ms / mu_n if mu_n else None,
                      "peak_note": "derived: 148 SMs x 64 FP64 lanes x 2 x 1.965 GHz (DESIGN.md §6)"},
         "kernels": {"phi_sweep_ms": phi_ms / max(phi_n, 1), "mu_sweep_ms": mu_ms / max(mu_n, 1),

@@ -42,6 +42,22 @@ for kern in ("mu", "phi", "ghost"):
     for k in KEYS:
         if k in m:
             lines.append(f"  {k:70s} {m[k][0]} {m[k][1]}")
+    # hardware-counted fp64 work (S§8(d) D.5): DADD + DMUL + 2 DFMA thread
+    # instructions, per interior cell of the launch (256^3 bench block)
+    hw = {}
+    try:
+        cyc = float(m["smsp__cycles_elapsed.avg"][0])
+        tsec = float(m["gpu__time_duration.sum"][0]) * {"us": 1e-6, "ms": 1e-3, "ns": 1e-9}[m["gpu__time_duration.sum"][1]]
+        cells = 256 ** 3
+        for op in ("dadd", "dmul", "dfma"):
+            hw[op] = float(m[f"smsp__sass_thread_inst_executed_op_{op}_pred_on.sum.per_cycle_elapsed"][0]) * cyc / cells
+        hw["flop_per_cell"] = hw["dadd"] + hw["dmul"] + 2 * hw["dfma"]
+        hw["tflops"] = hw["flop_per_cell"] * cells / tsec / 1e12
+        lines += ["", f"  hardware-counted fp64 per cell (256^3 launch): DADD {hw['dadd']:.1f}, DMUL {hw['dmul']:.1f}, "
+                      f"DFMA {hw['dfma']:.1f} -> {hw['flop_per_cell']:.1f} flop/cell, {hw['tflops']:.2f} TFLOP/s "
+                      f"(rsqrt / rcp seeds on MUFU not counted)"]
+    except (KeyError, ValueError):
+        pass
     st = {n.replace("smsp__average_warps_issue_stalled_", "").replace("_per_issue_active.ratio", ""): float(v[i] or 0)
           for i, n in enumerate(h)
           if n.startswith("smsp__average_warps_issue_stalled") and n.endswith("per_issue_active.ratio")}
@@ -90,6 +106,8 @@ for kern in ("mu", "phi", "ghost"):
     wr = float(m["dram__bytes_write.sum"][0]) * {"Gbyte": 1e9, "Mbyte": 1e6, "Kbyte": 1e3, "byte": 1}[m["dram__bytes_write.sum"][1]]
     summary[f"{kern}_sweep"] = {"dram_bytes_per_launch": rd + wr, "dram_read": rd, "dram_write": wr,
                                 "session": os.path.basename(src), "round": tag}
+    if hw:
+        summary[f"{kern}_sweep"].update({"hw_flop_per_cell": hw["flop_per_cell"], "hw_tflops": hw["tflops"]})
 if summary:
     p = os.path.join(dst, "ncu_summary.json")
     old = json.load(open(p)) if os.path.exists(p) else {}
