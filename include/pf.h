@@ -211,6 +211,8 @@ typedef struct {
   int phi_unroll;    /* phi-sweep z-loop unroll factor: 1..4                        */
   int phi_prefetch;  /* software prefetch of the own column: 0 off, 1 L2, 2 L1      */
   int phi_pfd;       /* prefetch distance in planes: 1..4                           */
+  int phi_xsh;       /* 1 (needs phi_faces6): the +x face flux comes from the next
+                        lane by a warp shuffle, 31 cells per 32-lane tile row      */
   int phi_zrec;      /* 1: the -z face flux is recomputed per plane instead of
                         carried in registers (fewer registers, more fp64 work)   */
   int phi_xghost;    /* 1: the phi-sweep writes phi_dst's x ghost columns itself when

@@ -1196,6 +1196,7 @@ const std::vector<TuneKnob>& tune_knobs() {
       {"phi_unroll", &pf_tuning::phi_unroll, JIT_PHI, {1, 2, 3}},
       {"phi_prefetch", &pf_tuning::phi_prefetch, JIT_PHI, {0, 1, 2}},
       {"phi_pfd", &pf_tuning::phi_pfd, JIT_PHI, {1, 2, 3}},
+      {"phi_xsh", &pf_tuning::phi_xsh, JIT_PHI, {0, 1}},
       {"phi_zrec", &pf_tuning::phi_zrec, JIT_PHI, {0, 1}},
       {"phi_xghost", &pf_tuning::phi_xghost, JIT_PHI, {0, 1}},
       {"mu_ty", &pf_tuning::mu_ty, JIT_MU, {3, 4, 5, 6, 8}},

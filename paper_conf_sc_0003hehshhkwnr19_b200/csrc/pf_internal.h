@@ -29,7 +29,7 @@ void launch_mu_tuned(const DevParams& P, const Geom& g, const TileSel* ts, dim3 
 // launch geometry of the tuned kernels (shared with the specialised build)
 dim3 tuned_block();
 dim3 tuned_block_mu(int mty, int mtx = 32);
-dim3 tuned_grid_phi(const Geom& g, int pty, int zc = 0);  // zc <= 0: the built-in z-chunk
+dim3 tuned_grid_phi(const Geom& g, int pty, int zc = 0, int txc = 32);  // zc <= 0: the built-in z-chunk; txc: cells per row
 dim3 tuned_block_phi(int pty);
 dim3 tuned_grid_mu(const Geom& g, int mty, int zc = 0, int mtx = 32);
 size_t tuned_mu_smem(int mty, int mtx = 32);  // mu-sweep tile: mtx x mty

@@ -102,6 +102,12 @@ constexpr int MU_TY = PF_MU_TY;
 #ifndef PF_PHI_ZREC
 #define PF_PHI_ZREC 0
 #endif
+#ifndef PF_PHI_XSH  // six-face sweep, +x face taken from the next lane (31 cells per 32-lane row)
+#define PF_PHI_XSH 0
+#endif
+// cells per tile row of the phi-sweep: with PF_PHI_XSH the last lane of a row
+// only evaluates the -x face that is the +x face of the lane before it
+constexpr int PHI_TXC = PF_PHI_XSH ? TX - 1 : TX;
 template <class PT, class GT, int L, bool TA, int PTY = TY, class RT = DevParams>
 __device__ __forceinline__ void phi_tuned_body(const PT& P, const RT& R, const GT& g,
                                                const double* __restrict__ ps, const double* __restrict__ ms,
@@ -114,8 +120,20 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const RT& R, const G
     // two extra face evaluations per cell (the neighbour values are loaded
     // for the central differences anyway) and saves the flux exchange, the
     // per-plane barrier and the tile-edge faces.
+#if PF_PHI_XSH
+    // lane i holds cell x0 + i; lanes 0..30 update their cells, lane 31 (and
+    // lanes past the row's end, clamped to the ghost x = nx) only supply the
+    // -x face that is the +x face of the lane before them (same operands:
+    // bitwise equal to evaluating it there)
+    const int xr = blockIdx.x * PHI_TXC + threadIdx.x, y = blockIdx.y * PTY + threadIdx.y;
+    if (y >= g.ny || blockIdx.x * PHI_TXC >= g.nx) return;  // whole warps: the shuffles need all lanes
+    const bool act = xr < g.nx && threadIdx.x < PHI_TXC;
+    const int x = min(xr, g.nx);
+#else
     const int x = blockIdx.x * TX + threadIdx.x, y = blockIdx.y * PTY + threadIdx.y;
     if (x >= g.nx || y >= g.ny) return;
+    constexpr bool act = true;
+#endif
     const int z0 = blockIdx.z * ZC_PHI, z1 = min(z0 + ZC_PHI, g.nz);
     const i64 F = g.field, SY = g.pitch, SZ = g.plane;
     i64 c = g.at(x, y, z0);
@@ -150,7 +168,12 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const RT& R, const G
           gd[a][2] = pp[a] - pm[a];
         }
         phi_face(P, xm, p0, Fa);
+#if PF_PHI_XSH
+#pragma unroll
+        for (int a = 0; a < N; ++a) Fb[a] = __shfl_down_sync(0xffffffffu, Fa[a], 1);
+#else
         phi_face(P, p0, xp, Fb);
+#endif
 #pragma unroll
         for (int a = 0; a < N; ++a) divh[a] = Fb[a] - Fa[a];
         phi_face(P, ym, p0, Fa);
@@ -168,10 +191,12 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const RT& R, const G
       double out[N], xi[N];
       if constexpr (ParamShape<PT>::xi) xi_of(P, R.step, x + g.x0, y + g.y0, z + g.z0, xi);
       phi_cell<TA>(P, plane_T(P, R, (double)z), p0, gd, divh, mu0, mu1, xi, out);
+      if (act) {
 #pragma unroll
-      for (int a = 0; a < N; ++a) pd[a * F + c] = out[a];
+        for (int a = 0; a < N; ++a) pd[a * F + c] = out[a];
 #pragma unroll
-      for (int a = 0; a < N; ++a) store_x_ghost(g, pd, x, y, z, a, out[a]);
+        for (int a = 0; a < N; ++a) store_x_ghost(g, pd, x, y, z, a, out[a]);
+      }
 #pragma unroll
       for (int a = 0; a < N; ++a) {
         pm[a] = p0[a];

@@ -48,9 +48,9 @@ __global__ void __launch_bounds__(TX* MU_TY, MU_TY == 4 ? 3 : 16 / MU_TY) k_mu_t
 dim3 tuned_block() { return dim3(TX, TY); }
 dim3 tuned_block_phi(int pty) { return dim3(TX, pty); }
 dim3 tuned_block_mu(int mty, int mtx) { return dim3(mtx, mty); }
-dim3 tuned_grid_phi(const Geom& g, int pty, int zc) {
+dim3 tuned_grid_phi(const Geom& g, int pty, int zc, int txc) {
   if (zc <= 0) zc = ZC_PHI;
-  return dim3((g.nx + TX - 1) / TX, (g.ny + pty - 1) / pty, (g.nz + zc - 1) / zc);
+  return dim3((g.nx + txc - 1) / txc, (g.ny + pty - 1) / pty, (g.nz + zc - 1) / zc);
 }
 dim3 tuned_grid_mu(const Geom& g, int mty, int zc, int mtx) {
   if (zc <= 0) zc = ZC_MU;

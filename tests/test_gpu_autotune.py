@@ -33,6 +33,8 @@ CORNERS = [
     {"mu_ldhint": 1, "mu_qreg": 1, "phi_xghost": 1},
     {"mu_ldhint": 2, "mu_tx": 16, "mu_ty": 4, "mu_minb": 4},
     {"mu_hpipe": 1, "phi_zrec": 1},
+    {"phi_xsh": 1},
+    {"phi_xsh": 1, "phi_ty": 8, "phi_minb": 2, "phi_xghost": 1, "phi_zc": 7},
     {"mu_hpipe": 1, "mu_rpf": 0, "mu_ty": 5, "mu_minb": 3, "phi_zrec": 1, "phi_faces6": 0},
 ]
 

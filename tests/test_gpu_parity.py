@@ -68,10 +68,13 @@ def test_one_step_parity(pfmod, omod, variant, pset, ic):
         assert ep <= TOL_1 and em <= TOL_1, (ep, em)
 
 
-@pytest.mark.parametrize("variant", ["jit", "tuned"])
-@pytest.mark.parametrize("shape", [(1, 1, 1), (3, 5, 7), (17, 9, 33), (8, 8, 130), (40, 70, 65)])
-def test_ragged_and_tiny_shapes(pfmod, omod, shape, variant):
+@pytest.mark.parametrize("variant", ["jit", "tuned", "jit_xsh"])
+@pytest.mark.parametrize("shape", [(1, 1, 1), (3, 5, 7), (17, 9, 33), (8, 8, 130), (40, 70, 65), (5, 6, 62)])
+def test_ragged_and_tiny_shapes(pfmod, omod, shape, variant, monkeypatch):
     P = I.params_stress()
+    if variant == "jit_xsh":  # 31-cell tile rows: ragged at other widths (62 = 2 x 31)
+        monkeypatch.setenv("PF_PHI_XSH", "1")
+        variant = "jit"
     for t, ep, em, *_ in run_pair(pfmod, omod, shape, P, "R", 2, variant=variant):
         assert ep <= TOL_1 and em <= TOL_1, (shape, ep, em)
 
