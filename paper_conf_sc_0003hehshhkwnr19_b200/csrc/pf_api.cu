@@ -105,15 +105,22 @@ struct pf_ctx {
   JitKernel* jmu = nullptr;
   pf_tuning tune;             // tuning of the specialised sweeps (pf_set_tuning, pf_autotune)
   // CUDA-graph steps (S§8(d) D.7): runs of steps between window checks are
-  // captured once per (length, buffer parity) and replayed; the sweeps read
-  // the per-step values (T base, step) from sv_dev, written before each replay
+  // captured once per (length, buffer parity) and replayed; the per-step
+  // values (T base, step) are written to sv_dev before each replay and each
+  // captured step copies its entry into the sweep modules' constant memory
+  bool zero_copy_z = true;  // z exchanges send / receive whole planes in place (PF_ZC_EXCHANGE=0: pack)
   bool use_graph = true;
+  int64_t graph_min_cells = 128 * 128 * 128;  // PF_GRAPH=1: any size, PF_GRAPH=0: never
   cudaStream_t cap_s = nullptr;      // private stream the steps are captured on (the caller's may be legacy)
   StepVals* sv_dev = nullptr;        // [64] in the workspace
   const StepVals* cap_sv = nullptr;  // set while capturing one step of a graph
+  typedef std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>> ProfPair;  // (category, start, end)
+  std::vector<ProfPair> cap_prof;  // timing events recorded as graph nodes during a capture
   struct GraphEntry {
     int k, cur;
     cudaGraphExec_t exec;
+    std::vector<ProfPair> prof;  // per-kernel timing events of the graph (pf_profile on)
+    bool pending = false;        // replayed, times not yet collected
   };
   std::vector<GraphEntry> graphs;
   ncclComm_t comm = nullptr;
@@ -130,8 +137,29 @@ struct pf_ctx {
 namespace {
 
 void drop_graphs(pf_ctx* c) {
-  for (auto& e : c->graphs) cudaGraphExecDestroy(e.exec);
+  for (auto& e : c->graphs) {
+    if (e.pending && !e.prof.empty()) cudaEventSynchronize(e.prof.back().second.second);
+    cudaGraphExecDestroy(e.exec);
+    for (auto& pp : e.prof) {
+      cudaEventDestroy(pp.second.first);
+      cudaEventDestroy(pp.second.second);
+    }
+  }
   c->graphs.clear();
+}
+
+// per-kernel times of the last replay of a graph (its events are reused by
+// the next replay): wait for it and add them up
+void graph_prof_collect(pf_ctx* c, pf_ctx::GraphEntry& e) {
+  if (!e.pending || e.prof.empty()) return;
+  cudaEventSynchronize(e.prof.back().second.second);
+  for (auto& pp : e.prof) {
+    float ms = 0;
+    cudaEventElapsedTime(&ms, pp.second.first, pp.second.second);
+    c->prof_ms[pp.first] += ms;
+    c->prof_n[pp.first] += 1;
+  }
+  e.pending = false;
 }
 
 int fail(pf_ctx* c, int code, const char* fmt, ...) {
@@ -502,8 +530,11 @@ int pf_create(const pf_config* cfg, pf_ctx** out) {
   {  // side stream: halo exchanges (N > 1) and the mu ghost fill (any N)
     const char* ov = getenv("PF_OVERLAP");
     ctx->overlap = !(ov && ov[0] == '0');
+    const char* zc = getenv("PF_ZC_EXCHANGE");
+    ctx->zero_copy_z = !(zc && zc[0] == '0');
     const char* gr = getenv("PF_GRAPH");
     ctx->use_graph = !(gr && gr[0] == '0');
+    if (gr && gr[0] == '1') ctx->graph_min_cells = 0;
     e = cudaStreamCreateWithFlags(&ctx->comm_s, cudaStreamNonBlocking);
     if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&ctx->cap_s, cudaStreamNonBlocking);
     cudaEvent_t* evs[4] = {&ctx->ev_phi, &ctx->ev_phix, &ctx->ev_mu, &ctx->ev_mux};
@@ -663,6 +694,33 @@ static int fill_ghost_dims(pf_ctx* ctx, double* f, int ncomp, bool is_mu, int d0
     const size_t cnt = halo_slab_elems(ctx->g, d) * ncomp;
     const int lo = ctx->nb_lo[d] >= 0 ? ctx->nb_lo[d] : -1;
     const int hi = ctx->nb_hi[d] >= 0 ? ctx->nb_hi[d] : -1;
+    if (d == 2 && ctx->comm && ctx->zero_copy_z) {
+      // z faces are whole padded planes, contiguous per component and already
+      // carrying their x / y ghosts (ordered fill): NCCL sends them straight
+      // from the field and receives straight into the ghost planes -- no
+      // pack / unpack kernels.  Per peer pair the k-th send matches the k-th
+      // recv: per component send (hi, lo), recv (lo, hi).
+      const Geom& g = ctx->g;
+      const size_t pl = (size_t)g.plane;
+      auto plane_ptr = [&](int a, int z) { return f + (size_t)a * g.field + (size_t)(z + GUARD) * pl; };
+      NC(g_nccl.GroupStart());
+      for (int a = 0; a < ncomp; ++a) {
+        if (hi >= 0) NC(g_nccl.Send(plane_ptr(a, n - 1), pl, ncclDouble, hi, ctx->comm, st));
+        if (lo >= 0) NC(g_nccl.Send(plane_ptr(a, 0), pl, ncclDouble, lo, ctx->comm, st));
+      }
+      for (int a = 0; a < ncomp; ++a) {
+        if (lo >= 0) NC(g_nccl.Recv(plane_ptr(a, -1), pl, ncclDouble, lo, ctx->comm, st));
+        if (hi >= 0) NC(g_nccl.Recv(plane_ptr(a, n), pl, ncclDouble, hi, ctx->comm, st));
+      }
+      NC(g_nccl.GroupEnd());
+      if (lo < 0 || hi < 0) {  // physical boundary on one side
+        launch_ghost_stage(ctx->g, d, lo < 0 ? ctx->cfg.bc_lo[d] : -1, hi < 0 ? ctx->cfg.bc_hi[d] : -1, f, ncomp, dir,
+                           st);
+        ctx->nlaunch[2] += 1;
+        if (int r = check_launch(ctx, "ghost_stage")) return r;
+      }
+      continue;
+    }
     if (hi >= 0) launch_pack(ctx->g, d, n - 1, ncomp, f, ctx->sendbuf[d][1], st);
     if (lo >= 0) launch_pack(ctx->g, d, 0, ncomp, f, ctx->sendbuf[d][0], st);
     ctx->nlaunch[2] += (hi >= 0) + (lo >= 0);
@@ -723,12 +781,24 @@ static cudaEvent_t ev_get(pf_ctx* ctx) {
 }
 static void prof_begin(pf_ctx* ctx, int k, cudaEvent_t* a) {
   if (!ctx->prof) return;
+  (void)k;
+  if (ctx->cap_sv) {  // capturing a graph: an event-record node of the graph
+    cudaEventCreate(a);
+    cudaEventRecordWithFlags(*a, ctx->stream, cudaEventRecordExternal);
+    return;
+  }
   *a = ev_get(ctx);
   cudaEventRecord(*a, ctx->stream);
-  (void)k;
 }
 static void prof_end(pf_ctx* ctx, int k, cudaEvent_t a) {
   if (!ctx->prof) return;
+  if (ctx->cap_sv) {
+    cudaEvent_t b = nullptr;
+    cudaEventCreate(&b);
+    cudaEventRecordWithFlags(b, ctx->stream, cudaEventRecordExternal);
+    ctx->cap_prof.push_back({k, {a, b}});
+    return;
+  }
   cudaEvent_t b = ev_get(ctx);
   cudaEventRecord(b, ctx->stream);
   ctx->ev_open.push_back({k, {a, b}});
@@ -888,11 +958,15 @@ static int step_graph(pf_ctx* ctx, int k) {
     b.Tbase[i] = ctx->hp.T0 + ctx->hp.G * (((double)g.z0 + (double)ctx->z_off) * ctx->hp.dx - ctx->hp.v * t);
   }
   launch_set_steps(ctx->sv_dev, b, ctx->stream);
-  ctx->nlaunch[3] += 1;
   if (int r = check_launch(ctx, "set_steps")) return r;
   cudaGraphExec_t exec = nullptr;
+  pf_ctx::GraphEntry* ge = nullptr;
   for (auto& e : ctx->graphs)
-    if (e.k == k && e.cur == ctx->cur) exec = e.exec;
+    if (e.k == k && e.cur == ctx->cur) {
+      exec = e.exec;
+      ge = &e;
+    }
+  if (ge) graph_prof_collect(ctx, *ge);  // its events are about to be re-recorded
   const int cur0 = ctx->cur;
   const int64_t step0 = ctx->step;
   const int64_t nl[4] = {ctx->nlaunch[0], ctx->nlaunch[1], ctx->nlaunch[2], ctx->nlaunch[3]};
@@ -901,7 +975,8 @@ static int step_graph(pf_ctx* ctx, int k) {
     // stream, which cannot be captured); the graph is launched on the caller's.
     // Any failure of the capture falls back to launching the steps directly.
     const cudaStream_t user = ctx->stream;
-    const auto nl0 = std::vector<int64_t>(ctx->nlaunch, ctx->nlaunch + 4);
+    cudaGraph_t graph = nullptr;
+    ctx->cap_prof.clear();
     cudaError_t e = cudaStreamBeginCapture(ctx->cap_s, cudaStreamCaptureModeThreadLocal);
     int r = e == cudaSuccess ? PF_OK : PF_ECUDA;
     if (r == PF_OK) {
@@ -913,7 +988,6 @@ static int step_graph(pf_ctx* ctx, int k) {
       ctx->cap_sv = nullptr;
       if (r == PF_OK) r = join_comm(ctx);
       ctx->stream = user;
-      cudaGraph_t graph = nullptr;
       e = cudaStreamEndCapture(ctx->cap_s, &graph);
       if (r == PF_OK && e == cudaSuccess) e = cudaGraphInstantiate(&exec, graph, 0);
       if (graph) cudaGraphDestroy(graph);
@@ -926,31 +1000,36 @@ static int step_graph(pf_ctx* ctx, int k) {
     if (r != PF_OK) {
       cudaGetLastError();
       if (exec) cudaGraphExecDestroy(exec);
-      for (int i = 0; i < 4; ++i) ctx->nlaunch[i] = nl0[i];
+      for (int i = 0; i < 4; ++i) ctx->nlaunch[i] = nl[i];
+      for (auto& pp : ctx->cap_prof) {
+        cudaEventDestroy(pp.second.first);
+        cudaEventDestroy(pp.second.second);
+      }
+      ctx->cap_prof.clear();
       ctx->use_graph = false;  // this context steps without graphs from now on
       ctx->err.clear();
       for (int i = 0; i < k; ++i)
         if (int r2 = step_impl(ctx, false)) return r2;
       return PF_OK;
     }
-    ctx->graphs.push_back({k, cur0, exec});
+    ctx->graphs.push_back({k, cur0, exec, ctx->cap_prof, false});
+    ctx->cap_prof.clear();
+    ge = &ctx->graphs.back();
+    ctx->mu_launches_per_step = (ctx->nlaunch[1] - nl[1]) / k;
+    ctx->ghost_launches_per_step = (ctx->nlaunch[2] - nl[2]) / k;
+    for (int i = 0; i < 4; ++i) ctx->nlaunch[i] = nl[i];
   }
   CU(cudaGraphLaunch(exec, ctx->stream));
+  ge->pending = !ge->prof.empty();
   for (int i = 0; i < k; ++i) {  // what the k steps did to the host state (step_impl)
     ctx->cur = 1 - ctx->cur;
     ctx->step += 1;
   }
-  // launches per category as if the steps had been launched one by one
-  const int64_t per[4] = {ctx->nlaunch[0] - nl[0], ctx->nlaunch[1] - nl[1], ctx->nlaunch[2] - nl[2],
-                          ctx->nlaunch[3] - nl[3]};
-  if (per[0] == 0) {  // replay of a cached graph: count what its capture launched
-    ctx->nlaunch[0] += k;
-    ctx->nlaunch[1] += (int64_t)k * ctx->mu_launches_per_step;
-    ctx->nlaunch[2] += (int64_t)k * ctx->ghost_launches_per_step;
-  } else {
-    ctx->mu_launches_per_step = per[1] / k;
-    ctx->ghost_launches_per_step = per[2] / k;
-  }
+  // launches per category as if the steps had been launched one by one (+ set_steps)
+  ctx->nlaunch[0] += k;
+  ctx->nlaunch[1] += (int64_t)k * ctx->mu_launches_per_step;
+  ctx->nlaunch[2] += (int64_t)k * ctx->ghost_launches_per_step;
+  ctx->nlaunch[3] += 1;
   ctx->mux_pending = false;
   return PF_OK;
 }
@@ -959,15 +1038,22 @@ int pf_step(pf_ctx* ctx, int64_t nsteps) {
   if (!ctx) return PF_EINVAL;
   if (!ctx->have_params || !ctx->have_fields) return fail(ctx, PF_ESTATE, "pf_step before pf_set_params/pf_init_fields");
   if (nsteps < 0) return fail(ctx, PF_EINVAL, "nsteps < 0");
-  const bool graphs = ctx->use_graph && ctx->variant == PF_VARIANT_JIT && !ctx->prof;
+  // graphs pay from ~128^3 cells per block (tools/graph_probe.py: 32^3 slower,
+  // 64^3 equal, 256^3 -1.3 % per step); smaller blocks launch directly
+  // With pf_profile timing on, steps launch directly unless PF_GRAPH=1 forces
+  // graphs (their per-kernel events are then event nodes collected after each
+  // replay; measured 0.8 % slower per step at 256^3 than direct profiled steps).
+  const bool forced = ctx->graph_min_cells == 0;
+  const bool graphs = ctx->use_graph && ctx->variant == PF_VARIANT_JIT && (!ctx->prof || forced) &&
+                      (int64_t)ctx->g.nx * ctx->g.ny * ctx->g.nz >= ctx->graph_min_cells;
+  // graph runs have one length: the window-check interval (the host decides
+  // shifts between runs), else 8 steps; shorter remainders launch directly, so
+  // a context captures at most two graphs (one per buffer parity)
+  const int nc = ctx->hp.window_check;
+  const int64_t K = nc > 0 ? std::min(nc, 64) : 8;
   for (int64_t n = 0; n < nsteps;) {
     int64_t k = 1;
-    if (graphs) {  // steps up to the next window check (which needs the host), at most 64
-      k = nsteps - n;
-      const int nc = ctx->hp.window_check;
-      if (nc > 0) k = std::min<int64_t>(k, nc - ctx->step % nc);
-      k = std::min<int64_t>(k, 64);
-    }
+    if (graphs && K >= 2 && nsteps - n >= K && (nc <= 0 || (nc <= 64 && ctx->step % nc == 0))) k = K;
     if (k >= 2) {
       if (ctx->variant == PF_VARIANT_JIT && (!ctx->jphi || !ctx->jmu)) {
         std::string err;
@@ -1393,6 +1479,11 @@ int pf_autotune(pf_ctx* ctx, unsigned mask, int passes, int reps, char* log, int
 int pf_profile(pf_ctx* ctx, int enable) {
   if (!ctx) return PF_EINVAL;
   CU(cudaStreamSynchronize(ctx->stream));
+  if ((enable != 0) != ctx->prof) {
+    drop_graphs(ctx);  // graphs are re-captured with (or without) their timing events
+  } else {
+    for (auto& e : ctx->graphs) e.pending = false;  // discard the replays before the reset
+  }
   for (auto& o : ctx->ev_open) {
     ctx->ev_pool.push_back(o.second.first);
     ctx->ev_pool.push_back(o.second.second);
@@ -1410,6 +1501,7 @@ int pf_profile(pf_ctx* ctx, int enable) {
 int pf_profile_read(pf_ctx* ctx, double ms[4], int64_t launches[4]) {
   if (!ctx) return PF_EINVAL;
   CU(cudaStreamSynchronize(ctx->stream));
+  for (auto& e : ctx->graphs) graph_prof_collect(ctx, e);
   for (auto& o : ctx->ev_open) {
     float v = 0;
     cudaEventElapsedTime(&v, o.second.first, o.second.second);

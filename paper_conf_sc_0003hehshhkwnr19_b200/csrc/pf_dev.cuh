@@ -64,29 +64,13 @@ __device__ __forceinline__ void store_x_ghost(const GT& g, double* __restrict__ 
   }
 }
 
-// Per-step values of one step of a captured CUDA graph (pf_step, graph
-// mode): written to device memory by k_set_steps before each graph launch,
-// read by the specialised sweeps instead of the by-value DevParams fields.
+// Per-step values (T base of the frozen temperature, step index) of one step
+// of a captured CUDA graph (pf_step, graph mode); the sweep bodies read
+// R.Tbase and R.step of whatever R they get (DevParams or this).
 struct StepVals {
   double Tbase;
   unsigned long long step;
 };
-struct StepRT {  // what the sweep bodies read of R
-  double Tbase;
-  unsigned long long step;
-};
-template <class DP>
-__device__ __forceinline__ StepRT step_rt(const DP& R, const StepVals* __restrict__ sv) {
-  StepRT r;
-  if (sv) {
-    r.Tbase = __ldg(&sv->Tbase);
-    r.step = __ldg(&sv->step);
-  } else {
-    r.Tbase = R.Tbase;
-    r.step = R.step;
-  }
-  return r;
-}
 
 // Tile selection of a sweep launch (interior / shell split for overlapping
 // the halo exchange): tile = blockIdx + off; if skip, tiles

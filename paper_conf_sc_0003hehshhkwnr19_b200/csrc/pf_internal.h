@@ -71,13 +71,14 @@ JitKernel* jit_get(const DevParams& P, const Geom& g, const pf_tuning& t, int wh
 // compile the kernels of several tunings into the cubin cache, concurrently
 // on up to nthreads host threads (no device needed)
 void jit_precompile(const DevParams& P, const Geom& g, const std::vector<pf_tuning>& ts, int which, int nthreads);
-// sv: per-step values in device memory (CUDA-graph steps) or nullptr (P's)
+// sv == nullptr: per-step values from P (by value); else a CUDA-graph step:
+// they are copied from device memory sv into the module's constant first
 cudaError_t jit_launch_phi(JitKernel* m, const DevParams& P, const double* ps, const double* ms, double* pd,
                            cudaStream_t s, const StepVals* sv = nullptr);
 cudaError_t jit_launch_mu(JitKernel* m, const DevParams& P, const TileSel* ts, dim3 grid, const double* ps,
                           const double* pd, const double* ms, double* md, cudaStream_t s,
                           const StepVals* sv = nullptr);
-// write the per-step values of the k steps of a graph launch (one thread)
+// write the per-step values of the k steps of a graph launch (one block)
 struct StepBatch {
   double Tbase[64];
   unsigned long long step0;

@@ -234,8 +234,10 @@ def test_nccl_self_exchange_bitwise(pfmod, monkeypatch, bc):
         B, shape = I.BC_DS, (24, 20, 40)
         phi, mu = I.ic_lamellar(shape, seed=3, z_front=10)
     outs = []
-    for force in ("0", "nccl"):
+    # z faces go as whole planes in place (zero copy) unless PF_ZC_EXCHANGE=0
+    for force, zc in (("0", "1"), ("nccl", "1"), ("nccl", "0")):
         monkeypatch.setenv("PF_FORCE_EXCHANGE", force)
+        monkeypatch.setenv("PF_ZC_EXCHANGE", zc)
         g = pfmod.PhaseField(shape, P, bc=B)
         g.init_fields(phi, mu)
         g.step(6)
@@ -243,9 +245,10 @@ def test_nccl_self_exchange_bitwise(pfmod, monkeypatch, bc):
         g.step(4)
         outs.append((g.download(), g.state(), g.monitor(), g.front_height()))
         g.close()
-    (a, sa, ma, ha), (b, sb, mb, hb) = outs
-    assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
-    assert sa == sb and ha == hb and np.array_equal(ma, mb)
+    (a, sa, ma, ha) = outs[0]
+    for (b, sb, mb, hb) in outs[1:]:
+        assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
+        assert sa == sb and ha == hb and np.array_equal(ma, mb)
     if bc == "ds":
         assert sa["z_off"] > 0  # the window shifted (collective front height)
 
@@ -281,6 +284,32 @@ def test_graph_steps_bitwise(pfmod, monkeypatch, case):
     assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
     if case == "ds_window":
         assert sa["z_off"] > 0
+
+
+def test_graph_steps_profiled(pfmod, monkeypatch):
+    """pf_profile timing with graph steps: the per-kernel events are event
+    nodes of the captured graph, collected after each replay; launch counts
+    are those of the direct steps."""
+    P = I.params_c4("ds", window_check=5, window_frac=0.5)
+    shape = (24, 20, 40)
+    phi, mu = I.ic_lamellar(shape, seed=3, z_front=6)
+    res = {}
+    for gr in ("0", "1"):
+        monkeypatch.setenv("PF_GRAPH", gr)
+        g = pfmod.PhaseField(shape, P, bc=I.BC_DS)
+        g.init_fields(phi, mu)
+        g.profile(True)
+        g.step(10)
+        g.profile(True)  # reset counters, keep the graphs
+        g.step(20)
+        res[gr] = (g.profile_read(), g.download())
+        g.close()
+    (pa, a), (pb, b) = res["0"], res["1"]
+    assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
+    for k in ("phi_sweep", "mu_sweep"):
+        assert pa[k][1] == pb[k][1] == 20, (k, pa[k], pb[k])
+        assert pb[k][0] > 0.0
+    assert pa["ghost"][1] == pb["ghost"][1]
 
 
 @pytest.mark.parametrize("variant", ["jit", "tuned"])
