@@ -232,6 +232,10 @@ typedef struct {
                         1 evict_first, 2 no_allocate                              */
   int mu_hpipe;      /* 1: halo-ring cells' loads for plane k+1 issued at the end of
                         plane k's face phase (software pipelining)               */
+  int mu_cly;        /* mu-sweep thread-block clusters of 1, 2 or 4 tiles stacked in
+                        y (mu_tx = 32): tiles of a cluster march z in lockstep and
+                        take the sides of a shared tile edge from each other's
+                        shared memory instead of building a y-halo row            */
 } pf_tuning;
 
 /* The built-in defaults (the measured best at 256^3 on one B200,

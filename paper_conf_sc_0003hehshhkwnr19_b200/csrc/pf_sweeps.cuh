@@ -519,7 +519,71 @@ __device__ __forceinline__ void side_from_smem(const double* __restrict__ D, int
   s.m[1] = t.y;
 }
 
-template <class PT, class GT, int L, bool TA, int MTY, int MTX = TX, class RT = DevParams>
+// ---------------------------------------------------------------------------
+// Thread-block clusters stacked along y (PF tuning knob mu_cly = CLY > 1):
+// the CLY tiles of a cluster march z in lockstep (one cluster barrier per
+// barrier of the plane) and read each other's shared memory (DSMEM), so an
+// interior tile edge builds no y-halo row (its sides are the neighbour's own
+// tile row) and its +y edge face flux is the neighbour's -y face flux.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ unsigned cl_rank() {
+  unsigned r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+// shared::cluster address of the same shared-memory object in CTA `rank`
+__device__ __forceinline__ unsigned cl_map(const void* p, unsigned rank) {
+  const unsigned a = (unsigned)__cvta_generic_to_shared(p);
+  unsigned r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(rank));
+  return r;
+}
+__device__ __forceinline__ double2 ld_cl2(unsigned a) {
+  double2 v;
+  asm volatile("ld.shared::cluster.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ double ld_cl(unsigned a) {
+  double v;
+  asm volatile("ld.shared::cluster.f64 %0, [%1];" : "=d"(v) : "r"(a));
+  return v;
+}
+// all threads of all CTAs of the cluster; release/acquire orders the shared
+// memory writes before it with the (remote) reads after it
+__device__ __forceinline__ void cl_sync() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+// side_from_smem of a slot in another CTA's D (a = its shared::cluster address)
+template <int L>
+__device__ __forceinline__ void side_from_cl(unsigned a, int c1, int c2, FaceSide& s) {
+  double2 t;
+#pragma unroll
+  for (int j = 0; j < N / 2; ++j) {
+    t = ld_cl2(a + 8u * (D_F + 2 * j));
+    s.f[2 * j] = t.x;
+    s.f[2 * j + 1] = t.y;
+    t = ld_cl2(a + 8u * (c1 + 2 * j));
+    s.c1[2 * j] = t.x;
+    s.c1[2 * j + 1] = t.y;
+    t = ld_cl2(a + 8u * (c2 + 2 * j));
+    s.c2[2 * j] = t.x;
+    s.c2[2 * j + 1] = t.y;
+  }
+  double dp[N];
+#pragma unroll
+  for (int j = 0; j < N / 2; ++j) {
+    t = ld_cl2(a + 8u * (D_DP + 2 * j));
+    dp[2 * j] = t.x;
+    dp[2 * j + 1] = t.y;
+  }
+#pragma unroll
+  for (int u = 0; u < NSOL; ++u) s.ds[u] = dp[solid_phase(L, u)];
+  t = ld_cl2(a + 8u * D_MU);
+  s.m[0] = t.x;
+  s.m[1] = t.y;
+}
+
+template <class PT, class GT, int L, bool TA, int MTY, int MTX = TX, int CLY = 1, class RT = DevParams>
 __device__ __forceinline__ void mu_tuned_body(const PT& P, const RT& R, const GT& g, const TileSel& ts,
                                               const double* __restrict__ ps, const double* __restrict__ pd,
                                               const double* __restrict__ ms, double* __restrict__ md) {
@@ -555,6 +619,16 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const RT& R, const GT
   else if (th >= 2 * MTY && th < 2 * MTY + MTX) { hx = th - 2 * MTY + 1; hy = 0; hwx = true; }
   else if (th >= 2 * MTY + MTX && th < 2 * MTY + 2 * MTX) { hx = th - 2 * MTY - MTX + 1; hy = MTY + 1; hwx = true; }
   if (hwx || hwy) hs = hidx<MTX>(hx, hy);
+  // cluster mode: the y-halo row of an edge shared with a tile of the same
+  // cluster is that tile's own row (read through DSMEM), not built here
+  constexpr bool CL = CLY > 1;
+  static_assert(!CL || MTX == 32, "cluster mode needs 32-wide tiles");
+  // (the cluster rank and the DSMEM addresses are re-read where used: fewer
+  // live registers across the march)
+  if constexpr (CL) {
+    const unsigned cr = cl_rank();
+    if ((hy == 0 && hwx && cr > 0) || (hy == MTY + 1 && hwx && cr + 1 < (unsigned)CLY)) hs = -1;
+  }
   const int hgx = min(x0 + hx - 1, g.nx), hgy = min(y0 + hy - 1, g.ny);
   // far-edge face of thread t: t < MTX: +y face of the top tile row, column t;
   // MTX <= t < MTX + MTY: +x face of the right tile column, row t - MTX.
@@ -654,7 +728,10 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const RT& R, const GT
 #else
     if (!last && hs >= 0) build_cell<NC>(g, ps, pd, ms, hgx, hgy, k, hwx, hwy, true, D, hs);
 #endif
-    __syncthreads();
+    if constexpr (CL)
+      cl_sync();
+    else
+      __syncthreads();
     // (b) z-face k-1/2 from registers (plane k-1) and shared memory (plane k)
     FaceSide q;
 #if PF_MU_QREG && (PF_MU_RPF || PF_MU_ZCARRY)
@@ -726,7 +803,10 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const RT& R, const GT
       mu_face<L, TA>(P, Tk, p, s, Fx);
 #pragma unroll
       for (int a = 0; a < N; ++a) s.c1[a] = Dp.c1[a];
-      side_from_smem<L, NC>(D, me - HX, D_CX, D_CZ, p);
+      if (CL && w == 0 && cl_rank() > 0)  // the tile below's top row, column `lane`
+        side_from_cl<L>(cl_map(D + (size_t)hidx<MTX>(lane + 1, MTY) * D_NV, cl_rank() - 1), D_CX, D_CZ, p);
+      else
+        side_from_smem<L, NC>(D, me - HX, D_CX, D_CZ, p);
       mu_face<L, TA>(P, Tk, p, s, Fy);
 #pragma unroll
       for (int i = 0; i < M; ++i) {
@@ -734,7 +814,7 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const RT& R, const GT
         fys[(i * (MTY + 1) + w) * MTX + lane] = Fy[i];
       }
       if constexpr (MTX == 32) {  // far tile edges in different warps: compile-time components
-        if (w == 0) {  // +y face of the top tile edge, column `lane`
+        if (w == 0 && !(CL && cl_rank() + 1 < (unsigned)CLY)) {  // +y face of the top tile edge, column `lane`
           double Fe[M];
           side_from_smem<L, NC>(D, hidx<MTX>(lane + 1, MTY), D_CX, D_CZ, p);
           side_from_smem<L, NC>(D, hidx<MTX>(lane + 1, MTY + 1), D_CX, D_CZ, s);
@@ -762,14 +842,24 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const RT& R, const GT
 #if PF_MU_HPIPE
       if (hs >= 0 && k + 1 < z1) halo_load(g, ps, pd, ms, hgx, hgy, k + 1, htoff, hraw);
 #endif
-      __syncthreads();
+      if constexpr (CL)
+        cl_sync();
+      else
+        __syncthreads();
+      // (cluster mode: the top row's +y flux is the -y flux of the tile above)
+      double fyu[M];
+#pragma unroll
+      for (int i = 0; i < M; ++i)
+        fyu[i] = (CL && w == MTY - 1 && cl_rank() + 1 < (unsigned)CLY)  // row 0 of the tile above
+                     ? ld_cl(cl_map(fys + i * (MTY + 1) * MTX + lane, cl_rank() + 1))
+                     : fys[(i * (MTY + 1) + w + 1) * MTX + lane];
 #pragma unroll
       for (int i = 0; i < M; ++i)
 #if PF_MU_FXREG  // own -x / -y fluxes from registers, only the +x / +y ones from shared memory
-        divxy[i] = (fxs[(i * MTY + w) * (MTX + 1) + lane + 1] - Fx[i]) + (fys[(i * (MTY + 1) + w + 1) * MTX + lane] - Fy[i]);
+        divxy[i] = (fxs[(i * MTY + w) * (MTX + 1) + lane + 1] - Fx[i]) + (fyu[i] - Fy[i]);
 #else
         divxy[i] = (fxs[(i * MTY + w) * (MTX + 1) + lane + 1] - fxs[(i * MTY + w) * (MTX + 1) + lane]) +
-                   (fys[(i * (MTY + 1) + w + 1) * MTX + lane] - fys[(i * (MTY + 1) + w) * MTX + lane]);
+                   (fyu[i] - fys[(i * (MTY + 1) + w) * MTX + lane]);
 #endif
     }
   };

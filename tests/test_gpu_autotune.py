@@ -36,6 +36,12 @@ CORNERS = [
     {"phi_xsh": 1},
     {"phi_xsh": 1, "phi_ty": 8, "phi_minb": 2, "phi_xghost": 1, "phi_zc": 7},
     {"mu_hpipe": 1, "mu_rpf": 0, "mu_ty": 5, "mu_minb": 3, "phi_zrec": 1, "phi_faces6": 0},
+    # clusters stacked in y: 6 tiles of 4 rows (the last one ragged) in
+    # clusters of 2; clusters of 4 do not tile them (plain kernels)
+    {"mu_cly": 2},
+    {"mu_cly": 4},
+    {"mu_cly": 2, "mu_ty": 3, "mu_minb": 5},
+    {"mu_cly": 2, "mu_qreg": 1, "mu_fxreg": 0, "mu_hpipe": 1},
 ]
 
 
@@ -144,3 +150,34 @@ def test_autotune_requires_fields_and_jit(pfmod):
     g.set_variant("jit")
     rep = g.autotune(mask=pfmod.PF_MU, passes=1, reps=2)
     assert "mu" in rep and "phi" not in rep
+
+
+@pytest.mark.parametrize("cly", [2, 4])
+def test_cluster_mu_sweep_bitwise(pfmod, omod, monkeypatch, cly):
+    """mu_cly > 1 (tiles of a thread-block cluster take the sides of their
+    shared y edges from each other's shared memory): bitwise equal to the
+    plain mu-sweep on a DS block with window shifts (8 tiles in y, the last
+    one ragged), on a periodic block where the interior / shell launches of
+    the forced exchange fall back to the plain kernels, and <= 1e-12 from the
+    oracle after one step."""
+    P = I.params_c4("ds", window_check=2, window_frac=0.3)
+    shape = (40, 30, 45)
+    phi, mu = I.ic_lamellar(shape, seed=5, z_front=14)
+    o = omod.Oracle(shape, P, I.BC_DS)
+    o.init(phi, mu)
+    o.step(1)
+    op, om = o.download()
+    gp, gm = gpu_run(pfmod, shape, P, phi, mu, 1, {"mu_cly": cly}, I.BC_DS)
+    assert rel_linf(gp, op) <= TOL_1 and rel_linf(gm, om) <= TOL_1
+    ref = gpu_run(pfmod, shape, P, phi, mu, 12, None, I.BC_DS)
+    got = gpu_run(pfmod, shape, P, phi, mu, 12, {"mu_cly": cly}, I.BC_DS)
+    assert np.array_equal(ref[0], got[0]) and np.array_equal(ref[1], got[1])
+    Ps = I.params_stress()
+    shape = (70, 32, 100)
+    phi, mu = I.ic_voronoi(shape, seed=8)
+    outs = []
+    for force, t in (("0", None), ("0", {"mu_cly": cly}), ("1", {"mu_cly": cly})):
+        monkeypatch.setenv("PF_FORCE_EXCHANGE", force)
+        outs.append(gpu_run(pfmod, shape, Ps, phi, mu, 4, t))
+    for o2 in outs[1:]:
+        assert np.array_equal(outs[0][0], o2[0]) and np.array_equal(outs[0][1], o2[1])
