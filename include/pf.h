@@ -236,6 +236,9 @@ typedef struct {
                         y (mu_tx = 32): tiles of a cluster march z in lockstep and
                         take the sides of a shared tile edge from each other's
                         shared memory instead of building a y-halo row            */
+  int mu_rot;        /* 1: the tile rows and their per-plane roles (halo rows, edge
+                        faces) rotated over the CTA's warps by a hash of the tile,
+                        spreading them over the SM sub-partitions (mu_tx = 32)    */
 } pf_tuning;
 
 /* The built-in defaults (the measured best at 256^3 on one B200,

@@ -1298,6 +1298,7 @@ const std::vector<TuneKnob>& tune_knobs() {
       {"mu_ldhint", &pf_tuning::mu_ldhint, JIT_MU, {0, 1, 2}},
       {"mu_hpipe", &pf_tuning::mu_hpipe, JIT_MU, {0, 1}},
       {"mu_cly", &pf_tuning::mu_cly, JIT_MU, {1, 2, 4}},
+      {"mu_rot", &pf_tuning::mu_rot, JIT_MU, {0, 1}},
   };
   return k;
 }

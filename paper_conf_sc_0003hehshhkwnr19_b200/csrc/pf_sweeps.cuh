@@ -50,6 +50,9 @@ constexpr int kPhiUnroll = PF_PHI_UNROLL;
 #ifndef PF_MU_HPIPE  // halo-ring cell's loads for plane k+1 issued at the end of plane k's face phase
 #define PF_MU_HPIPE 0
 #endif
+#ifndef PF_MU_ROT  // mu-sweep: tile rows (and their roles) rotated over the CTA's warps per tile
+#define PF_MU_ROT 0
+#endif
 #ifndef PF_MU_LDHINT  // L1 policy of the mu-sweep's phi_dst / mu loads: 0 default, 1 evict_first, 2 no_allocate
 #define PF_MU_LDHINT 0
 #endif
@@ -598,7 +601,17 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const RT& R, const GT
   double* D = smem;                          // [NC][D_NV] (AoS: LDS.128 per pair)
   double* fxs = D + D_NV * NC;               // [M][MTY][MTX+1]: x-face fluxes, face i = x0 - 1/2 + i
   double* fys = fxs + M * MTY * (MTX + 1);    // [M][MTY+1][MTX]: y-face fluxes
-  const int lane = threadIdx.x, w = threadIdx.y, t = w * MTX + lane;  // lane: x in the tile, w: row
+  // lane: x in the tile, w: row.  With PF_MU_ROT the row of hardware warp
+  // threadIdx.y is rotated by a hash of the tile: warp i of every CTA sits on
+  // SM sub-partition i, and the extra jobs of a plane (halo rows, far-edge
+  // faces) belong to fixed rows, so without rotation the same sub-partitions
+  // would carry them in every CTA
+  int w = threadIdx.y;
+  if (PF_MU_ROT && MTX == 32) {
+    const unsigned bid = (blockIdx.z * gridDim.y + blockIdx.y) * gridDim.x + blockIdx.x;
+    w = (int)((threadIdx.y + ((bid * 0x9E3779B1u) >> 16)) % (unsigned)MTY);
+  }
+  const int lane = threadIdx.x, t = w * MTX + lane;
   const int x0 = tbx * MTX, y0 = tby * MTY;
   const int x = x0 + lane, y = y0 + w;
   const bool active = x < g.nx && y < g.ny;

@@ -42,6 +42,9 @@ CORNERS = [
     {"mu_cly": 4},
     {"mu_cly": 2, "mu_ty": 3, "mu_minb": 5},
     {"mu_cly": 2, "mu_qreg": 1, "mu_fxreg": 0, "mu_hpipe": 1},
+    # tile rows rotated over the warps (plain and cluster kernels)
+    {"mu_rot": 1},
+    {"mu_rot": 1, "mu_ty": 5, "mu_minb": 3, "mu_cly": 2},
 ]
 
 
