@@ -239,6 +239,8 @@ typedef struct {
   int mu_rot;        /* 1: the tile rows and their per-plane roles (halo rows, edge
                         faces) rotated over the CTA's warps by a hash of the tile,
                         spreading them over the SM sub-partitions (mu_tx = 32)    */
+  int mu_rpt;        /* mu-sweep tile rows per thread: 1, or 2 (mu_tx = 32, mu_ty 6
+                        or 8: a 32 x mu_ty tile on 32 x mu_ty/2 threads)          */
 } pf_tuning;
 
 /* The built-in defaults (the measured best at 256^3 on one B200,

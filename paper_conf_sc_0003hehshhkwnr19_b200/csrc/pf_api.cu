@@ -1299,6 +1299,7 @@ const std::vector<TuneKnob>& tune_knobs() {
       {"mu_hpipe", &pf_tuning::mu_hpipe, JIT_MU, {0, 1}},
       {"mu_cly", &pf_tuning::mu_cly, JIT_MU, {1, 2, 4}},
       {"mu_rot", &pf_tuning::mu_rot, JIT_MU, {0, 1}},
+      {"mu_rpt", &pf_tuning::mu_rpt, JIT_MU, {1, 2}},
   };
   return k;
 }
@@ -1426,7 +1427,10 @@ int pf_autotune(pf_ctx* ctx, unsigned mask, int passes, int reps, char* log, int
           c.*(kn.f) = v;
           // a new tile shape comes with its natural occupancy
           if (kn.f == &pf_tuning::phi_ty) c.phi_minb = phi_minb_for(c.phi_ty);
-          if (kn.f == &pf_tuning::mu_ty || kn.f == &pf_tuning::mu_tx) c.mu_minb = mu_minb_for(c.mu_ty, c.mu_tx);
+          // (two rows per thread come with their natural 32 x 8 tile, one row with 32 x 4)
+          if (kn.f == &pf_tuning::mu_rpt) c.mu_ty = v == 2 ? 8 : 4;
+          if (kn.f == &pf_tuning::mu_ty || kn.f == &pf_tuning::mu_tx || kn.f == &pf_tuning::mu_rpt)
+            c.mu_minb = mu_minb_for(c.mu_ty, c.mu_tx, c.mu_rpt);
           if (tuning_check(c)) continue;
           cands.push_back(c);
           vals.push_back(v);

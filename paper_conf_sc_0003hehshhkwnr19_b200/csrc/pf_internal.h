@@ -89,6 +89,6 @@ int jit_mu_ty_of(const JitKernel* m);
 int jit_mu_tx_of(const JitKernel* m);
 int jit_mu_zc_of(const JitKernel* m);
 int phi_minb_for(int pty);            // natural CTAs per SM of a tile shape
-int mu_minb_for(int mty, int mtx);
+int mu_minb_for(int mty, int mtx, int rpt);
 
 }  // namespace pf

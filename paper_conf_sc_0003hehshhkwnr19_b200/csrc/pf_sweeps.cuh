@@ -880,4 +880,248 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const RT& R, const GT
   plane(BoolC<true>{}, z1);
 }
 
+// ===========================================================================
+// mu-sweep with two tile rows per thread (pf_tuning mu_rpt = 2): a CTA of
+// 32 x (MTY/2) threads owns a 32 x MTY tile; thread (lane, w) updates rows
+// 2w and 2w+1.  Per cell this halves the y-halo ring (2 halo rows per MTY
+// rows), the barriers and the far-edge faces, and the y-face between a
+// thread's two rows takes both sides from registers.  Same per-face and
+// per-cell arithmetic as mu_tuned_body, so the two give the same bits.
+// ===========================================================================
+template <class PT, class GT, int L, bool TA, int MTY, class RT = DevParams>
+__device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g, const TileSel& ts,
+                                           const double* __restrict__ ps, const double* __restrict__ pd,
+                                           const double* __restrict__ ms, double* __restrict__ md) {
+  constexpr int MTX = 32, TYT = MTY / 2, NT = MTX * TYT;
+  constexpr int NC = MuTile<MTY, MTX>::NC, HX = MuTile<MTY, MTX>::HX;
+  static_assert(MTY % 2 == 0 && 2 * MTX + 2 * MTY <= NT && TYT >= 2, "mu_rpt = 2 needs an even MTY >= 6");
+  const int tbx = blockIdx.x + ts.off[0], tby = blockIdx.y + ts.off[1], tbz = blockIdx.z + ts.off[2];
+  if (ts.skip && tbx >= ts.lo[0] && tbx < ts.hi[0] && tby >= ts.lo[1] && tby < ts.hi[1] && tbz >= ts.lo[2] &&
+      tbz < ts.hi[2])
+    return;  // interior tile, done by the other launch
+  extern __shared__ double smem[];
+  double* D = smem;
+  double* fxs = D + D_NV * NC;             // [M][MTY][MTX+1]
+  double* fys = fxs + M * MTY * (MTX + 1);  // [M][MTY+1][MTX]
+  const int lane = threadIdx.x, w = threadIdx.y, t = w * MTX + lane;
+  const int x0 = tbx * MTX, y0 = tby * MTY;
+  const int x = x0 + lane;
+  const int z0 = tbz * ZC_MU, z1 = min(z0 + ZC_MU, g.nz);
+  const i64 F = g.field;
+  const int xc = min(x, g.nx);
+  int yc[2], me[2];
+  bool active[2];
+#pragma unroll
+  for (int r = 0; r < 2; ++r) {
+    const int y = y0 + 2 * w + r;
+    active[r] = x < g.nx && y < g.ny;
+    yc[r] = min(y, g.ny);
+    me[r] = hidx<MTX>(lane + 1, 2 * w + r + 1);
+  }
+  // halo ring: the last 2 MTX + 2 MTY threads, x-halo cells first
+  int hx = 0, hy = 0, hs = -1;
+  bool hwx = false, hwy = false;
+  const int th = t - (NT - (2 * MTX + 2 * MTY));
+  if (th >= 0 && th < MTY) { hx = 0; hy = th + 1; hwy = true; }
+  else if (th >= MTY && th < 2 * MTY) { hx = MTX + 1; hy = th - MTY + 1; hwy = true; }
+  else if (th >= 2 * MTY && th < 2 * MTY + MTX) { hx = th - 2 * MTY + 1; hy = 0; hwx = true; }
+  else if (th >= 2 * MTY + MTX && th < 2 * MTY + 2 * MTX) { hx = th - 2 * MTY - MTX + 1; hy = MTY + 1; hwx = true; }
+  if (hwx || hwy) hs = hidx<MTX>(hx, hy);
+  const int hgx = min(x0 + hx - 1, g.nx), hgy = min(y0 + hy - 1, g.ny);
+
+  FaceSide Dp[2];
+  double dpl[2] = {0.0, 0.0};
+#pragma unroll
+  for (int r = 0; r < 2; ++r) {
+    const i64 c = g.at(xc, yc[r], z0 - 1);
+#pragma unroll
+    for (int a = 0; a < N; ++a) {
+      const double* f = ps + a * F + c;
+      Dp[r].f[a] = __ldg(f);
+      Dp[r].c1[a] = __ldg(f + 1) - __ldg(f - 1);
+      Dp[r].c2[a] = __ldg(f + g.pitch) - __ldg(f - g.pitch);
+    }
+#pragma unroll
+    for (int s = 0; s < NSOL; ++s) {
+      const int a = solid_phase(L, s);
+      Dp[r].ds[s] = ldh(pd + a * F + c) - Dp[r].f[a];
+    }
+    Dp[r].m[0] = ldh(ms + c);
+    Dp[r].m[1] = ldh(ms + F + c);
+  }
+  double divxy[2][M] = {{0.0, 0.0}, {0.0, 0.0}}, Fzm[2][M] = {{0.0, 0.0}, {0.0, 0.0}};
+  double fcar[2][N];
+#if PF_MU_RPF
+  double rnf[2][N], rnd[2][N], rnm[2][M];
+#endif
+#pragma unroll
+  for (int r = 0; r < 2; ++r) {
+    const i64 c = g.at(xc, yc[r], z0);
+#pragma unroll
+    for (int a = 0; a < N; ++a) fcar[r][a] = __ldg(ps + a * F + c);
+#if PF_MU_RPF
+#pragma unroll
+    for (int a = 0; a < N; ++a) {
+      rnf[r][a] = __ldg(ps + a * F + c + g.plane);
+      rnd[r][a] = ldh(pd + a * F + c);
+    }
+    rnm[r][0] = ldh(ms + c);
+    rnm[r][1] = ldh(ms + F + c);
+#endif
+  }
+
+  auto plane = [&](auto lastc, const int k) {
+    constexpr bool last = decltype(lastc)::value;
+    if (PF_PREFETCH && k + PF_PREFETCH_D <= z1 + 1) {
+#pragma unroll
+      for (int r = 0; r < 2; ++r) {
+        const i64 cp = g.at(xc, yc[r], k);
+#pragma unroll
+        for (int a = 0; a < N; ++a) {
+          prefetch_line(ps + a * F + cp + PF_PREFETCH_D * g.plane);
+          prefetch_line(pd + a * F + cp + (PF_PREFETCH_D - 1) * g.plane);
+        }
+        prefetch_line(ms + cp + (PF_PREFETCH_D - 1) * g.plane);
+        prefetch_line(ms + F + cp + (PF_PREFETCH_D - 1) * g.plane);
+      }
+    }
+    if (PF_HALO_L1 && !last && hs >= 0) {
+      const i64 ch = g.at(hgx, hgy, k + 1);
+#pragma unroll
+      for (int a = 0; a < N; ++a) {
+        asm volatile("prefetch.global.L1 [%0];" ::"l"(ps + a * F + ch + g.plane));
+        asm volatile("prefetch.global.L1 [%0];" ::"l"(pd + a * F + ch));
+      }
+      asm volatile("prefetch.global.L1 [%0];" ::"l"(ms + ch));
+      asm volatile("prefetch.global.L1 [%0];" ::"l"(ms + F + ch));
+    }
+    // (a) publish D(k) of the two own cells and of the halo ring
+#pragma unroll
+    for (int r = 0; r < 2; ++r) {
+      double vo[D_NV];
+#if PF_MU_RPF
+      build_own_rpf<NC>(g, ps, pd, ms, xc, yc[r], k, !last, Dp[r].f, fcar[r], rnf[r], rnd[r], rnm[r], D, me[r], vo);
+#else
+      build_own_carry<NC>(g, ps, pd, ms, xc, yc[r], k, !last, Dp[r].f, fcar[r], D, me[r], vo);
+#endif
+    }
+    if (!last && hs >= 0) build_cell<NC>(g, ps, pd, ms, hgx, hgy, k, hwx, hwy, true, D, hs);
+    __syncthreads();
+    // (b) z-faces k-1/2 and (c) cell updates of plane k-1
+#pragma unroll
+    for (int r = 0; r < 2; ++r) {
+      FaceSide q;
+      side_from_smem<L, NC>(D, me[r], D_CX, D_CY, q);
+      double Fz[M];
+      mu_face<L, TA>(P, plane_T(P, R, k - 0.5), Dp[r], q, Fz);
+      if (k > z0 && active[r]) {
+        double ph[N], dph[N], out[M];
+        const double divh[M] = {divxy[r][0] + (Fz[0] - Fzm[r][0]), divxy[r][1] + (Fz[1] - Fzm[r][1])};
+#pragma unroll
+        for (int a = 0; a < N; ++a) ph[a] = Dp[r].f[a];
+#pragma unroll
+        for (int s = 0; s < NSOL; ++s) dph[solid_phase(L, s)] = Dp[r].ds[s];
+        dph[L] = dpl[r];
+        mu_cell<TA>(P, plane_T(P, R, (double)(k - 1)), ph, dph, Dp[r].m, divh, out);
+        const i64 c = g.at(xc, yc[r], k - 1);
+        md[c] = out[0];
+        md[F + c] = out[1];
+      }
+      Fzm[r][0] = Fz[0];
+      Fzm[r][1] = Fz[1];
+      Dp[r] = q;
+      dpl[r] = D[(size_t)me[r] * D_NV + D_DP + L];
+    }
+    if constexpr (!last) {
+      // (d) faces of plane k: -x of both rows, -y of the lower row (from
+      // shared memory), the y-face between the two rows (both sides in
+      // registers), + the far tile edges
+      const double Tk = plane_T(P, R, (double)k);
+      double Fx[2][M], Fy[2][M];
+      double cz[2][N];
+#pragma unroll
+      for (int r = 0; r < 2; ++r) {
+        const double2* d = reinterpret_cast<const double2*>(D + (size_t)me[r] * D_NV + D_CZ);
+        const double2 z01 = d[0], z23 = d[1];
+        cz[r][0] = z01.x; cz[r][1] = z01.y; cz[r][2] = z23.x; cz[r][3] = z23.y;
+      }
+      FaceSide p, s;
+#pragma unroll
+      for (int r = 0; r < 2; ++r) {
+#pragma unroll
+        for (int a = 0; a < N; ++a) {
+          s.f[a] = Dp[r].f[a];
+          s.c1[a] = Dp[r].c2[a];
+          s.c2[a] = cz[r][a];
+        }
+#pragma unroll
+        for (int u = 0; u < NSOL; ++u) s.ds[u] = Dp[r].ds[u];
+        s.m[0] = Dp[r].m[0];
+        s.m[1] = Dp[r].m[1];
+        side_from_smem<L, NC>(D, me[r] - 1, D_CY, D_CZ, p);
+        mu_face<L, TA>(P, Tk, p, s, Fx[r]);
+      }
+#pragma unroll
+      for (int r = 0; r < 2; ++r) {
+#pragma unroll
+        for (int a = 0; a < N; ++a) {
+          s.f[a] = Dp[r].f[a];
+          s.c1[a] = Dp[r].c1[a];
+          s.c2[a] = cz[r][a];
+        }
+#pragma unroll
+        for (int u = 0; u < NSOL; ++u) s.ds[u] = Dp[r].ds[u];
+        s.m[0] = Dp[r].m[0];
+        s.m[1] = Dp[r].m[1];
+        if (r == 0) {
+          side_from_smem<L, NC>(D, me[0] - HX, D_CX, D_CZ, p);
+        } else {  // the lower own cell, tangential x / z
+#pragma unroll
+          for (int a = 0; a < N; ++a) {
+            p.f[a] = Dp[0].f[a];
+            p.c1[a] = Dp[0].c1[a];
+            p.c2[a] = cz[0][a];
+          }
+#pragma unroll
+          for (int u = 0; u < NSOL; ++u) p.ds[u] = Dp[0].ds[u];
+          p.m[0] = Dp[0].m[0];
+          p.m[1] = Dp[0].m[1];
+        }
+        mu_face<L, TA>(P, Tk, p, s, Fy[r]);
+      }
+#pragma unroll
+      for (int r = 0; r < 2; ++r)
+#pragma unroll
+        for (int i = 0; i < M; ++i) fxs[(i * MTY + 2 * w + r) * (MTX + 1) + lane] = Fx[r][i];
+#pragma unroll
+      for (int i = 0; i < M; ++i) fys[(i * (MTY + 1) + 2 * w) * MTX + lane] = Fy[0][i];
+      if (w == 0) {  // +y face of the top tile edge, column `lane`
+        double Fe[M];
+        side_from_smem<L, NC>(D, hidx<MTX>(lane + 1, MTY), D_CX, D_CZ, p);
+        side_from_smem<L, NC>(D, hidx<MTX>(lane + 1, MTY + 1), D_CX, D_CZ, s);
+        mu_face<L, TA>(P, Tk, p, s, Fe);
+#pragma unroll
+        for (int i = 0; i < M; ++i) fys[(i * (MTY + 1) + MTY) * MTX + lane] = Fe[i];
+      } else if (w == 1 && lane < MTY) {  // +x face of the right tile edge, row `lane`
+        double Fe[M];
+        side_from_smem<L, NC>(D, hidx<MTX>(MTX, lane + 1), D_CY, D_CZ, p);
+        side_from_smem<L, NC>(D, hidx<MTX>(MTX + 1, lane + 1), D_CY, D_CZ, s);
+        mu_face<L, TA>(P, Tk, p, s, Fe);
+#pragma unroll
+        for (int i = 0; i < M; ++i) fxs[(i * MTY + lane) * (MTX + 1) + MTX] = Fe[i];
+      }
+      __syncthreads();
+#pragma unroll
+      for (int i = 0; i < M; ++i) {
+        // lower row: its +y face is the upper row's -y face (registers)
+        divxy[0][i] = (fxs[(i * MTY + 2 * w) * (MTX + 1) + lane + 1] - Fx[0][i]) + (Fy[1][i] - Fy[0][i]);
+        divxy[1][i] = (fxs[(i * MTY + 2 * w + 1) * (MTX + 1) + lane + 1] - Fx[1][i]) +
+                      (fys[(i * (MTY + 1) + 2 * w + 2) * MTX + lane] - Fy[1][i]);
+      }
+    }
+  };
+  for (int k = z0; k < z1; ++k) plane(BoolC<false>{}, k);
+  plane(BoolC<true>{}, z1);
+}
+
 }  // namespace pf

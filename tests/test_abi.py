@@ -113,7 +113,8 @@ def test_tuning_defaults_and_range_check(lib):
     assert pf.tuning_check(t) == "ok"
     for bad in ({"phi_ty": 5}, {"mu_ty": 2}, {"mu_tx": 16, "mu_ty": 3}, {"mu_minb": 7}, {"phi_unroll": 0},
                 {"mu_pfd": 1}, {"phi_minb": 8, "phi_ty": 16}, {"mu_rpf": 2}, {"mu_zc": 1000},
-                {"mu_cly": 3}, {"mu_cly": 2, "mu_tx": 16, "mu_ty": 4}, {"mu_rot": 2}):
+                {"mu_cly": 3}, {"mu_cly": 2, "mu_tx": 16, "mu_ty": 4}, {"mu_rot": 2}, {"mu_rpt": 3},
+                {"mu_ty": 4}, {"mu_qreg": 1}, {"mu_cly": 2}):
         msg = pf.tuning_check(dict(t, **bad))
         assert msg != "ok", bad
 
@@ -121,11 +122,12 @@ def test_tuning_defaults_and_range_check(lib):
 @pytest.mark.parametrize("knobs", [
     {"phi_ty": 16, "phi_minb": 1, "phi_faces6": 0, "phi_unroll": 4, "phi_prefetch": 2, "phi_pfd": 3,
      "mu_ty": 8, "mu_tx": 16, "mu_minb": 4, "mu_rpf": 0, "mu_halo_l1": 0, "mu_fxreg": 0, "mu_prefetch": 0,
-     "phi_xghost": 1, "mu_ldhint": 2, "mu_qreg": 1},
+     "phi_xghost": 1, "mu_ldhint": 2, "mu_qreg": 1, "mu_rpt": 1},
     {"phi_ty": 8, "phi_minb": 2, "phi_zc": 32, "phi_prefetch": 0, "mu_ty": 3, "mu_minb": 5, "mu_zc": 24,
-     "mu_pfd": 3, "mu_prefetch": 2},
-    {"mu_cly": 4, "mu_rot": 1},
-    {"mu_cly": 2, "mu_ty": 6, "mu_minb": 2, "mu_qreg": 1, "mu_fxreg": 0, "mu_hpipe": 1},
+     "mu_pfd": 3, "mu_prefetch": 2, "mu_rpt": 1},
+    {"mu_cly": 4, "mu_rot": 1, "mu_rpt": 1, "mu_ty": 4, "mu_minb": 3},
+    {"mu_cly": 2, "mu_ty": 6, "mu_minb": 2, "mu_qreg": 1, "mu_fxreg": 0, "mu_hpipe": 1, "mu_rpt": 1},
+    {"mu_rpt": 2, "mu_ty": 6, "mu_minb": 2, "mu_rpf": 0, "mu_prefetch": 2},
 ])
 def test_tuned_variants_compile_without_gpu(lib, knobs):
     """Extreme corners of the auto-tuning space (pf_autotune's knobs) still

@@ -22,29 +22,36 @@ TOL_1 = 1e-12
 
 # corners of the search space of pf_autotune (tile shapes, occupancy,
 # z-chunks, schedule transformations)
+# one tile row per thread on the 32 x 4 tile (the rows-per-thread knob
+# mu_rpt defaults to 2 on a 32 x 8 tile); knobs that need it start from here
+R1 = {"mu_rpt": 1, "mu_ty": 4, "mu_minb": 3}
 CORNERS = [
     {},
     {"phi_ty": 16, "phi_minb": 1, "phi_faces6": 0, "phi_unroll": 4, "phi_prefetch": 2, "phi_pfd": 3,
      "phi_xghost": 1},
     {"phi_ty": 8, "phi_minb": 2, "phi_zc": 5, "phi_faces6": 0, "phi_prefetch": 0},
-    {"mu_ty": 8, "mu_tx": 16, "mu_minb": 4, "mu_rpf": 0, "mu_halo_l1": 0, "mu_fxreg": 0, "mu_prefetch": 0},
-    {"mu_ty": 3, "mu_minb": 5, "mu_zc": 7, "mu_pfd": 3, "mu_prefetch": 2},
+    dict(R1, **{"mu_ty": 8, "mu_tx": 16, "mu_minb": 4, "mu_rpf": 0, "mu_halo_l1": 0, "mu_fxreg": 0, "mu_prefetch": 0}),
+    dict(R1, **{"mu_ty": 3, "mu_minb": 5, "mu_zc": 7, "mu_pfd": 3, "mu_prefetch": 2}),
     {"mu_ty": 6, "mu_minb": 2, "mu_zc": 24, "phi_zc": 32, "phi_unroll": 3, "phi_xghost": 1},
-    {"mu_ldhint": 1, "mu_qreg": 1, "phi_xghost": 1},
-    {"mu_ldhint": 2, "mu_tx": 16, "mu_ty": 4, "mu_minb": 4},
-    {"mu_hpipe": 1, "phi_zrec": 1},
+    dict(R1, **{"mu_ldhint": 1, "mu_qreg": 1, "phi_xghost": 1}),
+    dict(R1, **{"mu_ldhint": 2, "mu_tx": 16, "mu_ty": 4, "mu_minb": 4}),
+    dict(R1, **{"mu_hpipe": 1, "phi_zrec": 1}),
     {"phi_xsh": 1},
     {"phi_xsh": 1, "phi_ty": 8, "phi_minb": 2, "phi_xghost": 1, "phi_zc": 7},
-    {"mu_hpipe": 1, "mu_rpf": 0, "mu_ty": 5, "mu_minb": 3, "phi_zrec": 1, "phi_faces6": 0},
+    dict(R1, **{"mu_hpipe": 1, "mu_rpf": 0, "mu_ty": 5, "mu_minb": 3, "phi_zrec": 1, "phi_faces6": 0}),
     # clusters stacked in y: 6 tiles of 4 rows (the last one ragged) in
     # clusters of 2; clusters of 4 do not tile them (plain kernels)
-    {"mu_cly": 2},
-    {"mu_cly": 4},
-    {"mu_cly": 2, "mu_ty": 3, "mu_minb": 5},
-    {"mu_cly": 2, "mu_qreg": 1, "mu_fxreg": 0, "mu_hpipe": 1},
+    dict(R1, mu_cly=2),
+    dict(R1, mu_cly=4),
+    dict(R1, **{"mu_cly": 2, "mu_ty": 3, "mu_minb": 5}),
+    dict(R1, **{"mu_cly": 2, "mu_qreg": 1, "mu_fxreg": 0, "mu_hpipe": 1}),
     # tile rows rotated over the warps (plain and cluster kernels)
-    {"mu_rot": 1},
-    {"mu_rot": 1, "mu_ty": 5, "mu_minb": 3, "mu_cly": 2},
+    dict(R1, mu_rot=1),
+    dict(R1, **{"mu_rot": 1, "mu_ty": 5, "mu_minb": 3, "mu_cly": 2}),
+    # two tile rows per thread (3 / 4 ragged tiles in y), one row per thread
+    {"mu_rpt": 2, "mu_ty": 8, "mu_minb": 2, "mu_zc": 5, "mu_prefetch": 0, "mu_halo_l1": 0, "mu_ldhint": 1},
+    {"mu_rpt": 2, "mu_ty": 6, "mu_minb": 3, "mu_rpf": 0, "mu_fxreg": 0, "mu_prefetch": 2},
+    R1,
 ]
 
 
@@ -108,7 +115,11 @@ def test_set_tuning_rejects_out_of_range(pfmod):
         g.set_tuning({"mu_ty": 9})
     with pytest.raises(pfmod.PFError):
         g.set_tuning({"phi_ty": 16, "phi_minb": 8})
-    g.set_tuning({"mu_ty": 5})
+    with pytest.raises(pfmod.PFError):
+        g.set_tuning({"mu_ty": 5})  # odd tile height with two rows per thread
+    g.set_tuning({"mu_ty": 6})
+    assert g.tuning()["mu_ty"] == 6
+    g.set_tuning(dict(R1, mu_ty=5))
     assert g.tuning()["mu_ty"] == 5
 
 
@@ -155,14 +166,16 @@ def test_autotune_requires_fields_and_jit(pfmod):
     assert "mu" in rep and "phi" not in rep
 
 
-@pytest.mark.parametrize("cly", [2, 4])
-def test_cluster_mu_sweep_bitwise(pfmod, omod, monkeypatch, cly):
+@pytest.mark.parametrize("knobs", [dict(R1, mu_cly=2), dict(R1, mu_cly=4), R1,
+                                   {"mu_rpt": 2, "mu_ty": 6, "mu_minb": 3}])
+def test_mu_sweep_layouts_bitwise(pfmod, omod, monkeypatch, knobs):
     """mu_cly > 1 (tiles of a thread-block cluster take the sides of their
-    shared y edges from each other's shared memory): bitwise equal to the
-    plain mu-sweep on a DS block with window shifts (8 tiles in y, the last
-    one ragged), on a periodic block where the interior / shell launches of
-    the forced exchange fall back to the plain kernels, and <= 1e-12 from the
-    oracle after one step."""
+    shared y edges from each other's shared memory) and mu_rpt = 2 (two tile
+    rows per thread): bitwise equal to the default mu-sweep on a DS block
+    with window shifts (ragged last tile in y), on a periodic block through
+    the interior / shell launches of the forced exchange (cluster kernels
+    fall back to the plain ones there), and <= 1e-12 from the oracle after
+    one step."""
     P = I.params_c4("ds", window_check=2, window_frac=0.3)
     shape = (40, 30, 45)
     phi, mu = I.ic_lamellar(shape, seed=5, z_front=14)
@@ -170,16 +183,16 @@ def test_cluster_mu_sweep_bitwise(pfmod, omod, monkeypatch, cly):
     o.init(phi, mu)
     o.step(1)
     op, om = o.download()
-    gp, gm = gpu_run(pfmod, shape, P, phi, mu, 1, {"mu_cly": cly}, I.BC_DS)
+    gp, gm = gpu_run(pfmod, shape, P, phi, mu, 1, knobs, I.BC_DS)
     assert rel_linf(gp, op) <= TOL_1 and rel_linf(gm, om) <= TOL_1
     ref = gpu_run(pfmod, shape, P, phi, mu, 12, None, I.BC_DS)
-    got = gpu_run(pfmod, shape, P, phi, mu, 12, {"mu_cly": cly}, I.BC_DS)
+    got = gpu_run(pfmod, shape, P, phi, mu, 12, knobs, I.BC_DS)
     assert np.array_equal(ref[0], got[0]) and np.array_equal(ref[1], got[1])
     Ps = I.params_stress()
     shape = (70, 32, 100)
     phi, mu = I.ic_voronoi(shape, seed=8)
     outs = []
-    for force, t in (("0", None), ("0", {"mu_cly": cly}), ("1", {"mu_cly": cly})):
+    for force, t in (("0", None), ("0", knobs), ("1", knobs)):
         monkeypatch.setenv("PF_FORCE_EXCHANGE", force)
         outs.append(gpu_run(pfmod, shape, Ps, phi, mu, 4, t))
     for o2 in outs[1:]:
