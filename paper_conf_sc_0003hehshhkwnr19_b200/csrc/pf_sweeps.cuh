@@ -996,6 +996,58 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
       asm volatile("prefetch.global.L1 [%0];" ::"l"(ms + F + ch));
     }
     // (a) publish D(k) of the two own cells and of the halo ring
+#if PF_MU_RPF
+    {
+      // as build_own_rpf for both rows; each row's y-neighbour inside the
+      // pair is the other row's carried phi_src(k) (for an active row it is
+      // the value at that address; an inactive row's cd_y is never read)
+      const i64 c0 = g.at(xc, yc[0], k), c1 = g.at(xc, yc[1], k);
+      double v0[D_NV], v1[D_NV];
+#pragma unroll
+      for (int a = 0; a < N; ++a) {
+        const double* f0 = ps + a * F + c0;
+        const double* f1 = ps + a * F + c1;
+        v0[D_F + a] = fcar[0][a];
+        v1[D_F + a] = fcar[1][a];
+        v0[D_CX + a] = __ldg(f0 + 1) - __ldg(f0 - 1);
+        v1[D_CX + a] = __ldg(f1 + 1) - __ldg(f1 - 1);
+        v0[D_CY + a] = fcar[1][a] - __ldg(f0 - g.pitch);
+        v1[D_CY + a] = __ldg(f1 + g.pitch) - fcar[0][a];
+        v0[D_CZ + a] = !last ? rnf[0][a] - Dp[0].f[a] : 0.0;
+        v1[D_CZ + a] = !last ? rnf[1][a] - Dp[1].f[a] : 0.0;
+        v0[D_DP + a] = rnd[0][a] - fcar[0][a];
+        v1[D_DP + a] = rnd[1][a] - fcar[1][a];
+      }
+#pragma unroll
+      for (int a = 0; a < N; ++a) {
+        fcar[0][a] = rnf[0][a];
+        fcar[1][a] = rnf[1][a];
+      }
+      v0[D_MU] = rnm[0][0];
+      v0[D_MU + 1] = rnm[0][1];
+      v1[D_MU] = rnm[1][0];
+      v1[D_MU + 1] = rnm[1][1];
+      double2* d0 = reinterpret_cast<double2*>(D + (size_t)me[0] * D_NV);
+      double2* d1 = reinterpret_cast<double2*>(D + (size_t)me[1] * D_NV);
+#pragma unroll
+      for (int j = 0; j < D_NV / 2; ++j) {
+        d0[j] = make_double2(v0[2 * j], v0[2 * j + 1]);
+        d1[j] = make_double2(v1[2 * j], v1[2 * j + 1]);
+      }
+      // next plane (k + 2 <= nz + 1 and k + 1 <= nz + 1 stay inside the guard ring)
+#pragma unroll
+      for (int r = 0; r < 2; ++r) {
+        const i64 c = r ? c1 : c0;
+#pragma unroll
+        for (int a = 0; a < N; ++a) {
+          rnf[r][a] = __ldg(ps + a * F + c + 2 * g.plane);
+          rnd[r][a] = ldh(pd + a * F + c + g.plane);
+        }
+        rnm[r][0] = ldh(ms + c + g.plane);
+        rnm[r][1] = ldh(ms + F + c + g.plane);
+      }
+    }
+#else
 #pragma unroll
     for (int r = 0; r < 2; ++r) {
       double vo[D_NV];
@@ -1005,6 +1057,7 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
       build_own_carry<NC>(g, ps, pd, ms, xc, yc[r], k, !last, Dp[r].f, fcar[r], D, me[r], vo);
 #endif
     }
+#endif
     if (!last && hs >= 0) build_cell<NC>(g, ps, pd, ms, hgx, hgy, k, hwx, hwy, true, D, hs);
     __syncthreads();
     // (b) z-faces k-1/2 and (c) cell updates of plane k-1
