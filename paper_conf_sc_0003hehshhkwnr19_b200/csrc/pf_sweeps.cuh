@@ -50,6 +50,9 @@ constexpr int kPhiUnroll = PF_PHI_UNROLL;
 #ifndef PF_MU_HPIPE  // halo-ring cell's loads for plane k+1 issued at the end of plane k's face phase
 #define PF_MU_HPIPE 0
 #endif
+#ifndef PF_HALO_D  // planes ahead of the halo-ring L1 prefetch (two-rows-per-thread sweep)
+#define PF_HALO_D 1
+#endif
 #ifndef PF_MU_ROT  // mu-sweep: tile rows (and their roles) rotated over the CTA's warps per tile
 #define PF_MU_ROT 0
 #endif
@@ -985,8 +988,8 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
         prefetch_line(ms + F + cp + (PF_PREFETCH_D - 1) * g.plane);
       }
     }
-    if (PF_HALO_L1 && !last && hs >= 0) {
-      const i64 ch = g.at(hgx, hgy, k + 1);
+    if (PF_HALO_L1 && !last && hs >= 0 && k + PF_HALO_D <= z1) {  // halo lines PF_HALO_D planes ahead
+      const i64 ch = g.at(hgx, hgy, k + PF_HALO_D);
 #pragma unroll
       for (int a = 0; a < N; ++a) {
         asm volatile("prefetch.global.L1 [%0];" ::"l"(ps + a * F + ch + g.plane));
