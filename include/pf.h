@@ -241,6 +241,8 @@ typedef struct {
                         spreading them over the SM sub-partitions (mu_tx = 32)    */
   int mu_rpt;        /* mu-sweep tile rows per thread: 1, or 2 (mu_tx = 32, mu_ty 6
                         or 8: a 32 x mu_ty tile on 32 x mu_ty/2 threads)          */
+  int phi_rpt;       /* phi-sweep tile rows per thread: 1, or 2 (phi_faces6 = 1,
+                        phi_xsh = 0, even phi_ty: 32 x phi_ty/2 threads)           */
 } pf_tuning;
 
 /* The built-in defaults (the measured best at 256^3 on one B200,

@@ -1300,6 +1300,7 @@ const std::vector<TuneKnob>& tune_knobs() {
       {"mu_cly", &pf_tuning::mu_cly, JIT_MU, {1, 2, 4}},
       {"mu_rot", &pf_tuning::mu_rot, JIT_MU, {0, 1}},
       {"mu_rpt", &pf_tuning::mu_rpt, JIT_MU, {1, 2}},
+      {"phi_rpt", &pf_tuning::phi_rpt, JIT_PHI, {1, 2}},
   };
   return k;
 }
@@ -1426,7 +1427,8 @@ int pf_autotune(pf_ctx* ctx, unsigned mask, int passes, int reps, char* log, int
           pf_tuning c = best;
           c.*(kn.f) = v;
           // a new tile shape comes with its natural occupancy
-          if (kn.f == &pf_tuning::phi_ty) c.phi_minb = phi_minb_for(c.phi_ty);
+          if (kn.f == &pf_tuning::phi_rpt) c.phi_ty = v == 2 ? 8 : 4;
+          if (kn.f == &pf_tuning::phi_ty || kn.f == &pf_tuning::phi_rpt) c.phi_minb = phi_minb_for(c.phi_ty, c.phi_rpt);
           // (two rows per thread come with their natural 32 x 8 tile, one row with 32 x 4)
           if (kn.f == &pf_tuning::mu_rpt) c.mu_ty = v == 2 ? 8 : 4;
           if (kn.f == &pf_tuning::mu_ty || kn.f == &pf_tuning::mu_tx || kn.f == &pf_tuning::mu_rpt)

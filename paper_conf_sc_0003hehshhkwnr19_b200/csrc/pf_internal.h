@@ -88,7 +88,7 @@ void launch_set_steps(StepVals* dst, const StepBatch& b, cudaStream_t s);
 int jit_mu_ty_of(const JitKernel* m);
 int jit_mu_tx_of(const JitKernel* m);
 int jit_mu_zc_of(const JitKernel* m);
-int phi_minb_for(int pty);            // natural CTAs per SM of a tile shape
+int phi_minb_for(int pty, int rpt);            // natural CTAs per SM of a tile shape
 int mu_minb_for(int mty, int mtx, int rpt);
 
 }  // namespace pf

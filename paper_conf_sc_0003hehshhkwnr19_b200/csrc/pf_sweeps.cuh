@@ -322,6 +322,122 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const RT& R, const G
 }
 
 // ===========================================================================
+// phi-sweep with two tile rows per thread (pf_tuning phi_rpt = 2; six-face
+// scheme): thread (lane, w) updates rows y = y0 + 2w and y + 1.  The face
+// between the two rows is evaluated once (it is the +y face of the lower and
+// the -y face of the upper row, on the same operands as in the one-row
+// sweep, so the bits are the same), and each row's y-neighbour inside the
+// pair is the other row's phi_src, in registers (no load).
+// ===========================================================================
+template <class PT, class GT, int L, bool TA, int PTY, class RT = DevParams>
+__device__ __forceinline__ void phi_r2_body(const PT& P, const RT& R, const GT& g,
+                                            const double* __restrict__ ps, const double* __restrict__ ms,
+                                            double* __restrict__ pd) {
+  static_assert(PTY % 2 == 0, "phi_rpt = 2 needs an even tile height");
+  const int x = blockIdx.x * TX + threadIdx.x, y = blockIdx.y * PTY + 2 * threadIdx.y;
+  if (x >= g.nx || y >= g.ny) return;
+  const bool act1 = y + 1 < g.ny;  // upper row inside the block (else: the ghost row, not stored)
+  const int z0 = blockIdx.z * ZC_PHI, z1 = min(z0 + ZC_PHI, g.nz);
+  const i64 F = g.field, SY = g.pitch, SZ = g.plane;
+  // upper row's +y neighbour row; clamped to the ghost row when the upper row
+  // is itself the ghost row (its update is not stored)
+  const i64 SYU = act1 ? SY : 0;
+  i64 c = g.at(x, y, z0);
+  double pm[2][N], p0[2][N], Fzm[2][N];
+#pragma unroll
+  for (int a = 0; a < N; ++a) {
+#pragma unroll
+    for (int r = 0; r < 2; ++r) {
+      pm[r][a] = __ldg(ps + a * F + c + r * SY - SZ);
+      p0[r][a] = __ldg(ps + a * F + c + r * SY);
+    }
+  }
+  phi_face(P, pm[0], p0[0], Fzm[0]);
+  phi_face(P, pm[1], p0[1], Fzm[1]);
+#pragma unroll kPhiUnroll
+  for (int z = z0; z < z1; ++z, c += SZ) {
+    if (PF_PREFETCH && z + PF_PREFETCH_D <= z1 + 1) {
+#pragma unroll
+      for (int r = 0; r < 2; ++r) {
+#pragma unroll
+        for (int a = 0; a < N; ++a) prefetch_line(ps + a * F + c + r * SY + PF_PREFETCH_D * SZ);
+        prefetch_line(ms + c + r * SY + PF_PREFETCH_D * SZ);
+        prefetch_line(ms + F + c + r * SY + PF_PREFETCH_D * SZ);
+      }
+    }
+    double pp[2][N], divh[2][N], gd[2][N][3];
+    {
+      double xm[N], xp[N], yo[N], Fa[N], Fb[N], Fym[N], Fmid[N];
+      // lower row: -x, +x, -y (sums in the one-row sweep's order:
+      // divh = ((F+x - F-x) + (F+y - F-y)) + (F+z - F-z))
+#pragma unroll
+      for (int a = 0; a < N; ++a) {
+        const double* f = ps + a * F + c;
+        pp[0][a] = __ldg(f + SZ);
+        xm[a] = __ldg(f - 1);
+        xp[a] = __ldg(f + 1);
+        yo[a] = __ldg(f - SY);
+        gd[0][a][0] = xp[a] - xm[a];
+        gd[0][a][1] = p0[1][a] - yo[a];
+        gd[0][a][2] = pp[0][a] - pm[0][a];
+      }
+      phi_face(P, xm, p0[0], Fa);
+      phi_face(P, p0[0], xp, Fb);
+#pragma unroll
+      for (int a = 0; a < N; ++a) divh[0][a] = Fb[a] - Fa[a];
+      phi_face(P, yo, p0[0], Fym);
+      // the face between the rows: +y of the lower, -y of the upper row
+      phi_face(P, p0[0], p0[1], Fmid);
+#pragma unroll
+      for (int a = 0; a < N; ++a) divh[0][a] += Fmid[a] - Fym[a];
+      // upper row: -x, +x, +y
+#pragma unroll
+      for (int a = 0; a < N; ++a) {
+        const double* f = ps + a * F + c + SY;
+        pp[1][a] = __ldg(f + SZ);
+        xm[a] = __ldg(f - 1);
+        xp[a] = __ldg(f + 1);
+        yo[a] = __ldg(f + SYU);
+        gd[1][a][0] = xp[a] - xm[a];
+        gd[1][a][1] = yo[a] - p0[0][a];
+        gd[1][a][2] = pp[1][a] - pm[1][a];
+      }
+      phi_face(P, xm, p0[1], Fa);
+      phi_face(P, p0[1], xp, Fb);
+#pragma unroll
+      for (int a = 0; a < N; ++a) divh[1][a] = Fb[a] - Fa[a];
+      phi_face(P, p0[1], yo, Fb);
+#pragma unroll
+      for (int a = 0; a < N; ++a) divh[1][a] += Fb[a] - Fmid[a];
+    }
+#pragma unroll
+    for (int r = 0; r < 2; ++r) {
+      double Fzp[N];
+      phi_face(P, p0[r], pp[r], Fzp);
+#pragma unroll
+      for (int a = 0; a < N; ++a) divh[r][a] += Fzp[a] - Fzm[r][a];
+      const i64 cr = c + r * SY;
+      const double mu0 = __ldg(ms + cr), mu1 = __ldg(ms + F + cr);
+      double out[N], xi[N];
+      if constexpr (ParamShape<PT>::xi) xi_of(P, R.step, x + g.x0, y + r + g.y0, z + g.z0, xi);
+      phi_cell<TA>(P, plane_T(P, R, (double)z), p0[r], gd[r], divh[r], mu0, mu1, xi, out);
+      if (r == 0 || act1) {
+#pragma unroll
+        for (int a = 0; a < N; ++a) pd[a * F + cr] = out[a];
+#pragma unroll
+        for (int a = 0; a < N; ++a) store_x_ghost(g, pd, x, y + r, z, a, out[a]);
+      }
+#pragma unroll
+      for (int a = 0; a < N; ++a) {
+        pm[r][a] = p0[r][a];
+        p0[r][a] = pp[r][a];
+        Fzm[r][a] = Fzp[a];
+      }
+    }
+  }
+}
+
+// ===========================================================================
 // mu-sweep (Algorithm 1 line 3): D3C19 of phi_src, D3C7 of phi_dst and mu.
 //
 // Per plane k every cell of the tile and of its 1-cell halo ring publishes

@@ -114,7 +114,8 @@ def test_tuning_defaults_and_range_check(lib):
     for bad in ({"phi_ty": 5}, {"mu_ty": 2}, {"mu_tx": 16, "mu_ty": 3}, {"mu_minb": 7}, {"phi_unroll": 0},
                 {"mu_pfd": 1}, {"phi_minb": 8, "phi_ty": 16}, {"mu_rpf": 2}, {"mu_zc": 1000},
                 {"mu_cly": 3}, {"mu_cly": 2, "mu_tx": 16, "mu_ty": 4}, {"mu_rot": 2}, {"mu_rpt": 3},
-                {"mu_ty": 4}, {"mu_qreg": 1}, {"mu_cly": 2}):
+                {"mu_ty": 4}, {"mu_qreg": 1}, {"mu_cly": 2}, {"phi_rpt": 2, "phi_faces6": 0},
+                {"phi_rpt": 2, "phi_xsh": 1}):
         msg = pf.tuning_check(dict(t, **bad))
         assert msg != "ok", bad
 
@@ -128,6 +129,7 @@ def test_tuning_defaults_and_range_check(lib):
     {"mu_cly": 4, "mu_rot": 1, "mu_rpt": 1, "mu_ty": 4, "mu_minb": 3},
     {"mu_cly": 2, "mu_ty": 6, "mu_minb": 2, "mu_qreg": 1, "mu_fxreg": 0, "mu_hpipe": 1, "mu_rpt": 1},
     {"mu_rpt": 2, "mu_ty": 6, "mu_minb": 2, "mu_rpf": 0, "mu_prefetch": 2},
+    {"phi_rpt": 2, "phi_ty": 16, "phi_minb": 1, "phi_unroll": 2, "phi_xghost": 1},
 ])
 def test_tuned_variants_compile_without_gpu(lib, knobs):
     """Extreme corners of the auto-tuning space (pf_autotune's knobs) still

@@ -52,6 +52,9 @@ CORNERS = [
     {"mu_rpt": 2, "mu_ty": 8, "mu_minb": 2, "mu_zc": 5, "mu_prefetch": 0, "mu_halo_l1": 0, "mu_ldhint": 1},
     {"mu_rpt": 2, "mu_ty": 6, "mu_minb": 3, "mu_rpf": 0, "mu_fxreg": 0, "mu_prefetch": 2},
     R1,
+    # phi-sweep with two rows per thread (21 rows: the last pair's upper row is the ghost row)
+    {"phi_rpt": 2, "phi_ty": 8, "phi_minb": 3},
+    {"phi_rpt": 2, "phi_ty": 4, "phi_minb": 6, "phi_zc": 7, "phi_prefetch": 2, "phi_xghost": 1},
 ]
 
 
