@@ -222,7 +222,7 @@ typedef struct {
   int mu_minb;       /* mu-sweep CTAs per SM requested from ptxas: 1..6             */
   int mu_zc;         /* mu-sweep planes per CTA along z: 4..512                     */
   int mu_prefetch;   /* software prefetch of the own column: 0 off, 1 L2, 2 L1      */
-  int mu_pfd;        /* prefetch distance in planes: 2..4                           */
+  int mu_pfd;        /* prefetch distance in planes: 2..6                           */
   int mu_rpf;        /* 1: own cell's L1-missing loads one plane ahead in registers */
   int mu_halo_l1;    /* 1: halo-ring cells' next-plane lines prefetched into L1     */
   int mu_fxreg;      /* 1: own -x/-y fluxes taken from registers in the divergence  */

@@ -1290,7 +1290,7 @@ const std::vector<TuneKnob>& tune_knobs() {
       {"mu_minb", &pf_tuning::mu_minb, JIT_MU, {2, 3, 4}},
       {"mu_zc", &pf_tuning::mu_zc, JIT_MU, {8, 12, 16, 24}},
       {"mu_prefetch", &pf_tuning::mu_prefetch, JIT_MU, {0, 1, 2}},
-      {"mu_pfd", &pf_tuning::mu_pfd, JIT_MU, {2, 3}},
+      {"mu_pfd", &pf_tuning::mu_pfd, JIT_MU, {2, 3, 4, 6}},
       {"mu_rpf", &pf_tuning::mu_rpf, JIT_MU, {0, 1}},
       {"mu_halo_l1", &pf_tuning::mu_halo_l1, JIT_MU, {0, 1}},
       {"mu_fxreg", &pf_tuning::mu_fxreg, JIT_MU, {0, 1}},
