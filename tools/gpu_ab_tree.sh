@@ -8,7 +8,7 @@ mkdir -p $OUT
 python -c "import __graft_entry__ as g; g.build()" > $OUT/build.log 2>&1
 (cd ab_head && python -c "import __graft_entry__ as g; g.build()" > $OUT/build_head.log 2>&1)
 for i in 1 2 3; do
-  (cd ab_head && timeout 300 python bench.py --steps 100 --warmup 5 --no-cpu-baseline --no-e2e --autotune 0 --tuning '{"mu_pfd": 3}' > $OUT/head_$i.json 2>> $OUT/bench.err)
-  env $2 timeout 300 python bench.py --steps 100 --warmup 5 --no-cpu-baseline --no-e2e --autotune 0 --tuning '{"mu_pfd": 3}' > $OUT/work_$i.json 2>> $OUT/bench.err
+  (cd ab_head && timeout 300 python bench.py --steps 100 --warmup 5 --no-cpu-baseline --no-e2e --autotune 0 > $OUT/head_$i.json 2>> $OUT/bench.err)
+  env $2 timeout 300 python bench.py --steps 100 --warmup 5 --no-cpu-baseline --no-e2e --autotune 0 > $OUT/work_$i.json 2>> $OUT/bench.err
 done
 echo done > $OUT/DONE
