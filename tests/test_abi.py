@@ -115,9 +115,12 @@ def test_tuning_defaults_and_range_check(lib):
                 {"mu_pfd": 1}, {"phi_minb": 8, "phi_ty": 16}, {"mu_rpf": 2}, {"mu_zc": 1000},
                 {"mu_cly": 3}, {"mu_cly": 2, "mu_tx": 16, "mu_ty": 4}, {"mu_rot": 2}, {"mu_rpt": 3},
                 {"mu_ty": 4}, {"mu_qreg": 1}, {"mu_cly": 2}, {"phi_rpt": 2, "phi_faces6": 0},
-                {"phi_rpt": 2, "phi_xsh": 1}):
+                {"phi_rpt": 2, "phi_xsh": 1}, {"mu_ty": 7, "mu_minb": 1}, {"mu_ty": 18, "mu_minb": 1},
+                {"mu_rpt": 1, "mu_ty": 16, "mu_minb": 1}):
         msg = pf.tuning_check(dict(t, **bad))
         assert msg != "ok", bad
+    # taller two-rows tiles are valid (one CTA per SM; measured slower)
+    assert pf.tuning_check(dict(t, mu_ty=16, mu_minb=1)) == "ok"
 
 
 @pytest.mark.parametrize("knobs", [
