@@ -11,6 +11,6 @@ for e in "$@"; do
   i=$((i+1))
   echo "$i: $e" >> $OUT/configs.txt
   if [ "$e" == "-" ]; then e=""; fi
-  env $e timeout 300 python bench.py --steps 100 --warmup 5 --no-cpu-baseline --no-e2e --autotune 0 --tuning '{"mu_pfd": 3}' > $OUT/bench_$i.json 2>> $OUT/bench.err
+  env $e timeout 300 python bench.py --steps 100 --warmup 5 --no-cpu-baseline --no-e2e --autotune 0 --tuning '{}' > $OUT/bench_$i.json 2>> $OUT/bench.err
 done
 echo done > $OUT/DONE
