@@ -170,7 +170,10 @@ def test_autotune_requires_fields_and_jit(pfmod):
 
 
 @pytest.mark.parametrize("knobs", [dict(R1, mu_cly=2), dict(R1, mu_cly=4), R1,
-                                   {"mu_rpt": 2, "mu_ty": 6, "mu_minb": 3}])
+                                   {"mu_rpt": 2, "mu_ty": 6, "mu_minb": 3},
+                                   # taller two-rows tiles, one CTA per SM (ragged in y)
+                                   {"mu_rpt": 2, "mu_ty": 16, "mu_minb": 1},
+                                   {"mu_rpt": 2, "mu_ty": 10, "mu_minb": 1}])
 def test_mu_sweep_layouts_bitwise(pfmod, omod, monkeypatch, knobs):
     """mu_cly > 1 (tiles of a thread-block cluster take the sides of their
     shared y edges from each other's shared memory) and mu_rpt = 2 (two tile
