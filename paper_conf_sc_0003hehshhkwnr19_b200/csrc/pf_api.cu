@@ -1288,7 +1288,7 @@ const std::vector<TuneKnob>& tune_knobs() {
       {"mu_ty", &pf_tuning::mu_ty, JIT_MU, {3, 4, 5, 6, 8}},
       {"mu_tx", &pf_tuning::mu_tx, JIT_MU, {16, 32}},
       {"mu_minb", &pf_tuning::mu_minb, JIT_MU, {2, 3, 4}},
-      {"mu_zc", &pf_tuning::mu_zc, JIT_MU, {8, 12, 16, 24}},
+      {"mu_zc", &pf_tuning::mu_zc, JIT_MU, {8, 12, 16, 22, 24, 32}},
       {"mu_prefetch", &pf_tuning::mu_prefetch, JIT_MU, {0, 1, 2}},
       {"mu_pfd", &pf_tuning::mu_pfd, JIT_MU, {2, 3, 4, 6}},
       {"mu_rpf", &pf_tuning::mu_rpf, JIT_MU, {0, 1}},
