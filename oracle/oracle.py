@@ -17,9 +17,12 @@ import subprocess
 import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-SRC = os.path.join(HERE, "pf_oracle.c")
+# PF_ORACLE_SRC / PF_ORACLE_LIB: an alternate (mutated) copy of the oracle
+# source and where to build it -- used only by the mutation check
+# (tools/oracle_mutations.py, tests/test_oracle_mutations.py).
+SRC = os.environ.get("PF_ORACLE_SRC") or os.path.join(HERE, "pf_oracle.c")
 HDR = os.path.join(HERE, "pf_oracle.h")
-LIB = os.path.join(HERE, "libpf_oracle.so")
+LIB = os.environ.get("PF_ORACLE_LIB") or os.path.join(HERE, "libpf_oracle.so")
 
 MAXN, MAXM = 4, 2
 BC = {"periodic": 0, "neumann": 1, "dirichlet_mu": 2}
@@ -62,7 +65,7 @@ def build(force: bool = False) -> str:
         return LIB
     tmp = LIB + f".tmp{os.getpid()}"
     cmd = ["gcc", "-std=c99", "-O2", "-ffp-contract=off", "-fno-fast-math", "-fopenmp",
-           "-fPIC", "-shared", "-Wall", "-o", tmp, SRC, "-lm"]
+           "-fPIC", "-shared", "-Wall", "-I", HERE, "-o", tmp, SRC, "-lm"]
     subprocess.check_call(cmd)
     os.replace(tmp, LIB)
     return LIB

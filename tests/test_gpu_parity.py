@@ -114,7 +114,8 @@ def test_config1_50_steps(pfmod, omod):
     P = I.params_c4()
     res = run_pair(pfmod, omod, (32, 32, 32), P, "V", 50, chunks=[1, 2, 5, 10, 50])
     for t, ep, em, *_ in res:
-        assert ep <= 1e-11 and em <= 1e-11, (t, ep, em)
+        tol = TOL_1 if t == 1 else 1e-11
+        assert ep <= tol and em <= tol, (t, ep, em)
 
 
 def test_1000_steps(pfmod, omod):
@@ -133,7 +134,37 @@ def test_ds_window_parity(pfmod, omod):
     res = run_pair(pfmod, omod, shape, P, "L", 60, bc=I.BC_DS, chunks=[1, 20, 60], ic_kw={"z_front": 20})
     for t, ep, em, gs, os_ in res:
         assert gs == os_, (gs, os_)
-        assert ep <= 1e-11 and em <= 1e-11, (t, ep, em)
+        tol = TOL_1 if t == 1 else 1e-11
+        assert ep <= tol and em <= tol, (t, ep, em)
+    assert res[-1][3]["z_off"] > 0
+
+
+# DS boundaries with the stress set: mu_inf != 0, so the
+# Dirichlet-mu ghost at z_hi [A15] differs from the interior from step 1 on
+# (IC-R: mu ~ U(-0.1, 0.1)), A1 != 0 and G v != 0 (frozen T with a Q term),
+# window inflow mu = mu_inf [A16].
+@pytest.mark.parametrize("variant", ["jit", "tuned", "naive"])
+@pytest.mark.parametrize("window", [0, 1])
+def test_ds_stress_one_step(pfmod, omod, variant, window):
+    P = I.params_stress(window_check=window, window_frac=0.5)
+    assert np.all(P["mu_inf"] != 0.0)
+    shape = (20, 24, 40)
+    res = run_pair(pfmod, omod, shape, P, "R", 2, bc=I.BC_DS, variant=variant, chunks=[1, 2])
+    for t, ep, em, gs, os_ in res:
+        assert gs == os_, (gs, os_)
+        assert ep <= TOL_1 and em <= TOL_1, (t, ep, em)
+    if window:
+        assert res[0][3]["z_off"] > 0
+
+
+def test_ds_stress_1000_steps(pfmod, omod):
+    P = I.params_stress(window_check=50, window_frac=0.5)
+    shape = (24, 16, 16)
+    res = run_pair(pfmod, omod, shape, P, "V", 1000, bc=I.BC_DS, chunks=[1, 100, 1000])
+    for t, ep, em, gs, os_ in res:
+        assert gs == os_, (gs, os_)
+        tol = TOL_1 if t == 1 else TOL_1000
+        assert ep <= tol and em <= tol, (t, ep, em)
     assert res[-1][3]["z_off"] > 0
 
 

@@ -213,6 +213,122 @@ def test_p6_front_velocity(oracle_mod):
 
 
 # --------------------------------------------------------------------------
+# A5: tau interpolation "computed from local phase-field values and pairwise
+# kinetic coefficients tau_ab".  Whatever the interpolation, a
+# binary a|b interface must move with its own pair's coefficient: the
+# planar-front speed of App. A.3 is v = d_psi / tau_ab, independent of the
+# tau of pairs that are absent.  Three phases with tau_01 = 2 and
+# tau_02 = tau_12 = 1: the weighted mean gives tau = tau_01 exactly in every
+# cell of the 0|1 front; an unweighted mean over all pairs would give 4/3
+# (50 % faster); a max/min over all pairs 2 or 1.
+# --------------------------------------------------------------------------
+def test_a5_tau_binary_front_speed(oracle_mod):
+    eps, dx, dpsi, L = 3.0, 0.5, 0.03, 40.0
+    nx = int(L / dx)
+    tau01 = 2.0
+    dt = 0.04 * dx * dx
+    u = (np.arange(nx) + 0.5) * dx - 12.0
+    p1 = sine_profile(u, eps)
+    phi = np.zeros((3, 1, 1, nx))
+    phi[1, 0, 0], phi[0, 0, 0] = p1, 1.0 - p1
+    P = simple_params(N=3, dx=dx, dt=dt, dpsi=dpsi, tau=1.0)
+    P["tau"][0, 1] = P["tau"][1, 0] = tau01
+    o = oracle_mod.Oracle((1, 1, nx), P, BC_X_NEUMANN)
+    o.init(phi, np.zeros((1, 1, 1, nx)))
+    o.step(int(30 / dt))
+    f1 = front_position(o.download()[0][1, 0, 0], dx)
+    n = int(60 / dt)
+    o.step(n)
+    p, _ = o.download()
+    f2 = front_position(p[1, 0, 0], dx)
+    assert p[2].max() == 0.0  # the third phase never appears (gamma3 = 10 > 32/pi^2)
+    v = (f2 - f1) / (n * dt)
+    assert v / (dpsi / tau01) == pytest.approx(1.0, abs=0.02)
+
+
+def test_a5_tau_limits_in_cells(oracle_mod):
+    """Delta-t linearity (C.8) isolates 1/tau per cell: without projection the
+    phi increment is dt/(tau(phi) eps) R(phi), with R independent of tau.
+    Against the same step with every tau_ab = 1 (tau = 1 exactly):
+      - a cell where exactly two phases a, b are non-zero has tau = tau_ab
+        (the binary-interface limit; to rounding);
+      - every other mixed cell has tau inside [min, max] of the tau_ab of its
+        present pairs (an interpolation of pairwise coefficients);
+      - a pure cell (no pair present; reading A5's 0/0 case) uses the mean of
+        all tau_ab."""
+    shape = (10, 10, 10)
+    P = I.params_stress()
+    phi, mu = I.ic_voronoi(shape, seed=11, nseeds=12, blur=1, noise=0.0)
+    outs = {}
+    for name, tau in (("one", np.ones((4, 4)) - np.eye(4)), ("S", P["tau"])):
+        o = oracle_mod.Oracle(shape, dict(P, tau=tau, projection=0))
+        o.init(phi, mu)
+        o.step_phi_only()
+        outs[name] = o.download()[0] - phi
+    T = P["tau"]
+    present = phi > 0.0
+    npres = present.sum(0)
+    ok2 = okm = okp = 0
+    for z, y, x in np.ndindex(*shape):
+        a_ref, a_s = outs["one"][:, z, y, x], outs["S"][:, z, y, x]
+        k = int(np.argmax(np.abs(a_ref)))
+        if abs(a_ref[k]) < 1e-9:
+            continue
+        tau = a_ref[k] / a_s[k]  # tau(phi) / 1
+        assert np.allclose(a_s * tau, a_ref, rtol=1e-12, atol=1e-15)  # one scalar per cell
+        pr = np.nonzero(present[:, z, y, x])[0]
+        pairs = [T[a, b] for i, a in enumerate(pr) for b in pr[i + 1:]]
+        if npres[z, y, x] == 2:
+            assert tau == pytest.approx(pairs[0], rel=1e-12)
+            ok2 += 1
+        elif npres[z, y, x] > 2:
+            assert min(pairs) * (1 - 1e-12) <= tau <= max(pairs) * (1 + 1e-12)
+            okm += 1
+        else:
+            assert tau == pytest.approx(T[np.triu_indices(4, 1)].mean(), rel=1e-12)
+            okp += 1
+    assert ok2 > 20 and okm > 20 and okp > 20, (ok2, okm, okp)
+
+
+# --------------------------------------------------------------------------
+# A15: Dirichlet mu = mu_inf at z_hi (DS boundaries), Neumann at z_lo.  Pure
+# liquid, uniform mu0 != mu_inf, dT/dt = 0: the mu equation is FTCS diffusion
+# (App. A.4) whose only source is the top face, between the top cell and a
+# ghost holding mu_inf (C.6.6).  One step changes only the top cell:
+#   mu'_top = mu0 + (dt/dx^2) K (mu_inf - mu0),  K = chi_l^{-1} D_l chi_l,
+# and a second step reaches the cell below by the same factor.
+# --------------------------------------------------------------------------
+def test_a15_dirichlet_mu_top(oracle_mod):
+    P = I.params_stress(G=0.0, v=0.0)
+    P["mu_inf"] = np.array([0.03, -0.02])
+    shape = (6, 3, 4)
+    mu0 = np.array([0.01, 0.005])
+    phi = np.zeros((4,) + shape)
+    phi[3] = 1.0
+    mu = np.zeros((2,) + shape) + mu0[:, None, None, None]
+    o = oracle_mod.Oracle(shape, P, I.BC_DS)
+    o.init(phi, mu)
+    o.step(1)
+    p, m = o.download()
+    A = P["A0"][3] + P["A1"][3] * P["T0"]
+    chi = -(A + A.T)
+    K = np.linalg.solve(chi, P["D"][3] @ chi) * P["dt"] / P["dx"] ** 2
+    top = mu0 + K @ (P["mu_inf"] - mu0)
+    assert np.array_equal(p, phi)
+    assert np.array_equal(m[:, :-1], mu[:, :-1])  # Neumann bottom, untouched interior
+    for i in range(2):
+        np.testing.assert_allclose(m[i, -1], top[i], rtol=0, atol=1e-16)
+    o.step(1)
+    _, m2 = o.download()
+    below = mu0 + K @ (top - mu0)
+    top2 = top + K @ (P["mu_inf"] - top) - K @ (top - mu0)
+    for i in range(2):
+        np.testing.assert_allclose(m2[i, -2], below[i], rtol=0, atol=1e-16)
+        np.testing.assert_allclose(m2[i, -1], top2[i], rtol=0, atol=1e-16)
+    assert np.array_equal(m2[:, :-2], mu[:, :-2])
+
+
+# --------------------------------------------------------------------------
 # P7: r_a = delta Psi / delta phi_a of the oracle converges at second order
 # to sympy's variational derivative of eq. 3 (the paper's own route,
 # `func_diff`, P:L490), on smooth periodic fields.
@@ -637,9 +753,9 @@ def test_openmp_bitwise(oracle_mod):
 
 
 def test_window_shift_semantics(oracle_mod):
-    P = I.params_c4("ds", window_check=0)
+    P = I.params_c4("ds", window_check=0, mu_inf=np.array([0.02, -0.01]))
     shape = (16, 6, 8)
-    phi, mu = I.ic_lamellar(shape, seed=3, z_front=10)
+    phi, mu = I.ic_lamellar(shape, seed=3, z_front=10, mu_inf=(0.005, 0.004))
     o = oracle_mod.Oracle(shape, P, I.BC_DS)
     o.init(phi, mu)
     H = o.front_height()
@@ -647,7 +763,8 @@ def test_window_shift_semantics(oracle_mod):
     o.shift_window(3)
     p, m = o.download()
     assert np.array_equal(p[:, :-3], phi[:, 3:]) and np.array_equal(m[:, :-3], mu[:, 3:])
-    assert np.all(p[3, -3:] == 1.0) and np.all(p[:3, -3:] == 0.0) and np.all(m[:, -3:] == 0.0)
+    assert np.all(p[3, -3:] == 1.0) and np.all(p[:3, -3:] == 0.0)
+    assert np.all(m[0, -3:] == 0.02) and np.all(m[1, -3:] == -0.01)  # inflow mu = mu_inf [A16]
     assert o.state()["z_off"] == 3
 
 
