@@ -565,6 +565,7 @@ int pf_destroy(pf_ctx* ctx) {
     cudaEventDestroy(o.second.second);
   }
   drop_graphs(ctx);
+  jit_release(ctx);
   if (ctx->comm) g_nccl.CommDestroy(ctx->comm);
   if (ctx->comm_s) {
     cudaStreamSynchronize(ctx->comm_s);
@@ -604,6 +605,8 @@ int pf_set_params(pf_ctx* ctx, const pf_params* p) {
           return fail(ctx, PF_EINVAL, "gamma3 must be symmetric");
   if (p->window_check < 0 || (p->window_check > 0 && !(p->window_frac > 0 && p->window_frac < 1)))
     return fail(ctx, PF_EINVAL, "window_check >= 0 and 0 < window_frac < 1");
+  if (p->window_check > 0 && ctx->cfg.procs[2] != 1)  // checked here, not at the first shift
+    return fail(ctx, PF_EINVAL, "the moving window needs the growth axis unsplit (procs[2] == 1)");
   if (!(std::isfinite(p->xi_amp) && p->xi_amp >= 0.0))
     return fail(ctx, PF_EINVAL, "xi_amp must be finite and >= 0");
   // T range over the global domain at t = 0 (frozen gradient; window keeps it bounded)
@@ -844,8 +847,8 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
   cudaEvent_t e0 = nullptr;
   if (ctx->variant == PF_VARIANT_JIT && (!ctx->jphi || !ctx->jmu)) {
     std::string err;
-    ctx->jphi = jit_get(ctx->dp, g, ctx->tune, JIT_PHI, &err);
-    if (ctx->jphi) ctx->jmu = jit_get(ctx->dp, g, ctx->tune, JIT_MU, &err);
+    ctx->jphi = jit_get(ctx, ctx->dp, g, ctx->tune, JIT_PHI, &err);
+    if (ctx->jphi) ctx->jmu = jit_get(ctx, ctx->dp, g, ctx->tune, JIT_MU, &err);
     if (!ctx->jphi || !ctx->jmu) return fail(ctx, PF_ECUDA, "run-time specialisation failed: %s", err.c_str());
   }
   // overlap: the exchanged dimensions' ghosts travel on the
@@ -1057,8 +1060,8 @@ int pf_step(pf_ctx* ctx, int64_t nsteps) {
     if (k >= 2) {
       if (ctx->variant == PF_VARIANT_JIT && (!ctx->jphi || !ctx->jmu)) {
         std::string err;
-        ctx->jphi = jit_get(ctx->dp, ctx->g, ctx->tune, JIT_PHI, &err);
-        if (ctx->jphi) ctx->jmu = jit_get(ctx->dp, ctx->g, ctx->tune, JIT_MU, &err);
+        ctx->jphi = jit_get(ctx, ctx->dp, ctx->g, ctx->tune, JIT_PHI, &err);
+        if (ctx->jphi) ctx->jmu = jit_get(ctx, ctx->dp, ctx->g, ctx->tune, JIT_MU, &err);
         if (!ctx->jphi || !ctx->jmu) return fail(ctx, PF_ECUDA, "run-time specialisation failed: %s", err.c_str());
       }
       if (int r = step_graph(ctx, (int)k)) return r;
@@ -1359,7 +1362,7 @@ static int time_candidates(pf_ctx* ctx, const std::vector<pf_tuning>& cands, int
   why->assign(cands.size(), "");
   for (size_t i = 0; i < cands.size(); ++i) {
     std::string err;
-    JitKernel* k = jit_get(ctx->dp, ctx->g, cands[i], which, &err);
+    JitKernel* k = jit_get(ctx, ctx->dp, ctx->g, cands[i], which, &err);
     if (!k) {
       (*why)[i] = err.substr(0, 200);
       continue;
@@ -1404,7 +1407,7 @@ int pf_autotune(pf_ctx* ctx, unsigned mask, int passes, int reps, char* log, int
     const char* kname = which == JIT_PHI ? "phi" : "mu";
     if (which == JIT_MU) {  // the mu-sweep reads phi_dst: one phi-sweep of the best phi kernel first
       std::string err;
-      JitKernel* kp = jit_get(ctx->dp, ctx->g, best, JIT_PHI, &err);
+      JitKernel* kp = jit_get(ctx, ctx->dp, ctx->g, best, JIT_PHI, &err);
       if (!kp) return fail(ctx, PF_ECUDA, "autotune: %s", err.c_str());
       CU(jit_launch_phi(kp, ctx->dp, ctx->phi[ctx->cur], ctx->mu[ctx->cur], ctx->phi[1 - ctx->cur], ctx->stream));
       if (int r = fill_ghosts(ctx, ctx->phi[1 - ctx->cur], PF_N, false)) return r;
@@ -1469,8 +1472,8 @@ int pf_autotune(pf_ctx* ctx, unsigned mask, int passes, int reps, char* log, int
   drop_graphs(ctx);
   {
     std::string err;
-    ctx->jphi = jit_get(ctx->dp, ctx->g, best, JIT_PHI, &err);
-    if (ctx->jphi) ctx->jmu = jit_get(ctx->dp, ctx->g, best, JIT_MU, &err);
+    ctx->jphi = jit_get(ctx, ctx->dp, ctx->g, best, JIT_PHI, &err);
+    if (ctx->jphi) ctx->jmu = jit_get(ctx, ctx->dp, ctx->g, best, JIT_MU, &err);
     if (!ctx->jphi || !ctx->jmu) return fail(ctx, PF_ECUDA, "autotune: %s", err.c_str());
   }
   // the scratch level's ghosts were overwritten: nothing reads them before the next sweep writes it

@@ -67,7 +67,11 @@ void tuning_default(pf_tuning* t);            // built-in defaults + PF_* enviro
 const char* tuning_check(const pf_tuning& t);  // nullptr if valid, else the reason
 // build (or fetch from the process cache) a specialised kernel; returns
 // nullptr and sets *err on failure
-JitKernel* jit_get(const DevParams& P, const Geom& g, const pf_tuning& t, int which, std::string* err);
+// owner: the pf_ctx the loaded module belongs to (one module per context and
+// device; the compiled cubin itself is shared through a per-process cache)
+JitKernel* jit_get(const void* owner, const DevParams& P, const Geom& g, const pf_tuning& t, int which,
+                   std::string* err);
+void jit_release(const void* owner);  // unload every module of `owner` (pf_destroy)
 // compile the kernels of several tunings into the cubin cache, concurrently
 // on up to nthreads host threads (no device needed)
 void jit_precompile(const DevParams& P, const Geom& g, const std::vector<pf_tuning>& ts, int which, int nthreads);

@@ -595,14 +595,17 @@ __device__ __forceinline__ void build_own_rpf(const GT& g, const double* __restr
   double2* d = reinterpret_cast<double2*>(D + (size_t)i * D_NV);
 #pragma unroll
   for (int j = 0; j < D_NV / 2; ++j) d[j] = make_double2(v[2 * j], v[2 * j + 1]);
-  // next plane (k + 2 <= nz + 1 and k + 1 <= nz + 1 stay inside the guard ring)
+  // next plane: only while the march continues (wz == false on the peeled
+  // last plane k = z1, where k + 2 could pass the guard ring)
+  if (wz) {
 #pragma unroll
-  for (int a = 0; a < N; ++a) {
-    nf[a] = __ldg(ps + a * F + c + 2 * g.plane);
-    nd[a] = ldh(pd + a * F + c + g.plane);
+    for (int a = 0; a < N; ++a) {
+      nf[a] = __ldg(ps + a * F + c + 2 * g.plane);
+      nd[a] = ldh(pd + a * F + c + g.plane);
+    }
+    nm[0] = ldh(ms + c + g.plane);
+    nm[1] = ldh(ms + F + c + g.plane);
   }
-  nm[0] = ldh(ms + c + g.plane);
-  nm[1] = ldh(ms + F + c + g.plane);
 }
 
 template <bool B>
@@ -1153,9 +1156,10 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
         d0[j] = make_double2(v0[2 * j], v0[2 * j + 1]);
         d1[j] = make_double2(v1[2 * j], v1[2 * j + 1]);
       }
-      // next plane (k + 2 <= nz + 1 and k + 1 <= nz + 1 stay inside the guard ring)
+      // next plane (not on the peeled last plane k = z1, where k + 2 could
+      // pass the guard ring)
 #pragma unroll
-      for (int r = 0; r < 2; ++r) {
+      for (int r = 0; r < 2 && !last; ++r) {
         const i64 c = r ? c1 : c0;
 #pragma unroll
         for (int a = 0; a < N; ++a) {
