@@ -202,6 +202,7 @@ def main():
     ap.add_argument("--tuning", default=None, help="JSON dict of pf_tuning knobs set before the auto-tuning")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-stress", action="store_true", help="skip the stress-set (general-expression) line")
     args = ap.parse_args()
     assert args.warmup >= 3 or args.impl == "reference" or os.environ.get("PF_BENCH_ALLOW_SHORT"), "W >= 3"
 
@@ -232,9 +233,11 @@ def main():
     else:  # configs 2/3: n^3 DS block per GPU, growth axis z unsplit
         procs = grid_for(world)
         gshape = (n, n * procs[1], n * procs[0])  # (nz, ny, nx)
-        P = I.params_c4("ds", window_check=10, window_frac=0.5)
-        z_front = n // 4
-        P["T0"] = I.ds_T0(z_front, P["G"])
+        # growing front (inputs.DS_BENCH): it starts one plane above the
+        # window threshold, so the first check shifts and the window keeps
+        # following the front (one plane per ~260 steps at 256^3)
+        z_front = n // 2 + 2
+        P = I.params_ds_growth(z_front, window_check=10, window_frac=0.5, **I.DS_BENCH)
         bc = I.BC_DS
     uid = None
     if world > 1:
@@ -311,6 +314,7 @@ def main():
     barrier()
     # ---- timed region (device events on the library's stream) ----
     g.profile(True)
+    zoff0 = g.state()["z_off"]
     n_clk0 = len(clocks.lines)
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
@@ -327,6 +331,27 @@ def main():
     launches = sum(v[1] for v in prof.values())
     mon = g.monitor()
     st = g.state()
+    window = None
+    if not strong:
+        # one window shift by one plane (front-height reduction excluded),
+        # timed on its own after the timed region: the cost of each shift
+        # (the state is re-initialised by the e2e leg)
+        w0, w1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        barrier()
+        w0.record(stream)
+        g.shift_window(1)
+        w1.record(stream)
+        w1.synchronize()
+        shift_ms = max_over_ranks(w0.elapsed_time(w1))
+        window = {"check_every": int(P["window_check"]), "z_off_before": zoff0, "z_off_after": st["z_off"],
+                  "shifts_in_timed_region": st["z_off"] - zoff0,
+                  "check_and_shift_ms_total": prof["window"][0], "check_and_shift_ms_per_step":
+                      prof["window"][0] / args.steps,
+                  "shift_ms": shift_ms,
+                  "pulling_speed_v": P["v"], "gradient_G": P["G"],
+                  "note": "z_off counts planes shifted since init (warm-up included); a shift is an out-of-place "
+                          "copy of both fields plus a ghost fill; the front advances ~1 plane per ~260 steps "
+                          "(profiles/r02_ds_tune.jsonl)"}
 
     total_cells = cells_local * world
     value = total_cells * args.steps / (ms_max * 1e-3) / 1e6  # whole-job MLUP/s
@@ -347,7 +372,8 @@ def main():
         "config": {"workload": ("config 4: fixed 512x512x1024 periodic domain in z-slabs, ternary eutectic "
                                 "N=4/K-1=2, IC-V (256^3 periodic tile), C.4 parameters") if strong else
                                (f"config 2: {n}^3 block per GPU, ternary eutectic N=4/K-1=2, frozen-T directional "
-                                f"solidification, moving window (check every 10 steps), IC-L, C.4 parameters"),
+                                f"solidification (v={P['v']}, G={P['G']}), moving window (check every 10 steps), "
+                                f"IC-L, C.4 parameters"),
                    "global_xyz": [gshape[2], gshape[1], gshape[0]], "procs_xyz": list(procs),
                    "parallelism": f"domain decomposition {procs[0]}x{procs[1]}x{procs[2]}",
                    "variant": args.variant, "tuning": g.tuning() if args.variant == "jit" else None,
@@ -375,6 +401,7 @@ def main():
         "autotune": tune_rep,
         "clocks": clk,
         "state": {"step": st["step"], "z_off": st["z_off"], "max_sum_err": mon[0], "min_phi": mon[1]},
+        "window": window,
     }
     # ---- end-to-end through the public API with host buffers ----
     if not args.no_e2e:
@@ -398,11 +425,39 @@ def main():
                       "h2d_bytes_per_step": bytes_state / args.steps, "d2h_bytes_per_step": bytes_state / args.steps,
                       "note": "one chunk = pf_init_fields from pinned host memory, K steps, pf_download to pinned "
                               "host memory, all inside the timed region"}
+    # ---- general-expression path: the stress parameter set S (unequal gamma,
+    # A1 != 0, non-diagonal chi / D, mu_inf != 0: none of the specialised
+    # simplifications apply), same block, boundaries and IC
+    if world == 1 and not strong and not args.no_stress and args.variant == "jit":
+        g.close()
+        torch.cuda.empty_cache()
+        Ps = I.params_stress(window_check=10, window_frac=0.5)
+        gs = pf.PhaseField(gshape, Ps, bc=bc, device=local_rank)
+        gs.init_fields(phi_pin, mu_pin)
+        gs.profile(True)
+        gs.step(max(args.warmup, 3) + 10)
+        torch.cuda.synchronize()
+        gs.profile(True)
+        s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        nst = max(20, min(args.steps, 100))
+        s0.record(gs.stream)
+        gs.step(nst)
+        s1.record(gs.stream)
+        s1.synchronize()
+        sms = s0.elapsed_time(s1)
+        sp = gs.profile_read()
+        rec["stress_set"] = {
+            "value": cells_local * nst / (sms * 1e-3) / 1e6, "unit": UNIT, "steps": nst, "ms_per_step": sms / nst,
+            "mu_sweep_ms": sp["mu_sweep"][0] / max(sp["mu_sweep"][1], 1),
+            "phi_sweep_ms": sp["phi_sweep"][0] / max(sp["phi_sweep"][1], 1),
+            "frac_of_R": (cells_local * nst / (sms * 1e-3) / 1e6) / R,
+            "note": "parameter set S of SURVEY C.4 (general expressions), same block / BCs / IC, default tuning"}
+        gs.close()
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         rec["cpu_baseline"] = cpu_baseline(P, bc, strong=strong)
     if rank == 0:
         print(json.dumps(rec), flush=True)
-    g.close()
+    g.close()  # (idempotent)
     if dist is not None:
         dist.destroy_process_group()
 

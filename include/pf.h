@@ -76,7 +76,15 @@ typedef struct {
   int bc_lo[3];     /* PF_BC_* of the low side of x, y, z                    */
   int bc_hi[3];     /* PF_BC_* of the high side; periodic must match low     */
   int rank, world;  /* this process' rank, number of ranks (= GPUs)          */
-  unsigned char nccl_uid[128]; /* ncclUniqueId bytes from rank 0 (world > 1) */
+  unsigned char nccl_uid[128]; /* ncclUniqueId bytes from rank 0 (world > 1); or
+                                  "PFLOCAL:<name>" (NUL-terminated): the `world`
+                                  blocks live in this process (e.g. on one GPU),
+                                  each driven by its own host thread, and the
+                                  halo exchange / reductions use an in-process
+                                  transport (device copies ordered by events,
+                                  host barriers per group call) instead of NCCL;
+                                  CUDA-graph steps are off.  Test harness for
+                                  the multi-block path on one device.       */
   int device;       /* CUDA device ordinal                                   */
   void* stream;     /* cudaStream_t borrowed from the caller (0 = legacy)     */
   double* phi[2];   /* caller-owned device buffers, pf_layout.phi_bytes each */
@@ -88,13 +96,19 @@ typedef struct {
   int local[3];           /* this rank's interior extents nx, ny, nz          */
   int offset[3];          /* global index of its first interior cell          */
   int64_t pitch;          /* doubles per padded row (>= x_off + nx + 2)       */
-  int64_t plane;          /* doubles per z-plane = pitch * (ny + 4)           */
-  int64_t field;          /* doubles per component = plane * (nz + 4)         */
+  int64_t plane;          /* z stride in doubles                              */
+  int64_t field;          /* component stride in doubles                      */
   int64_t x_off;          /* row offset of interior x = 0 (128-B aligned)     */
   /* cell (x,y,z) of component c is at c*field + (z+2)*plane + (y+2)*pitch +
-   * x_off + x: one ghost layer (index -1, n) inside a guard ring of 2.      */
-  size_t phi_bytes;       /* one time level of phi: PF_N * field * 8          */
-  size_t mu_bytes;        /* one time level of mu:  PF_M * field * 8          */
+   * x_off + x: one ghost layer (index -1, n) inside a guard ring of 2.
+   * Default, structure of arrays [c][z][y][x]: plane = pitch*(ny+4),
+   * field = plane*(nz+4).  Environment PF_LAYOUT=il at pf_query_layout /
+   * pf_create time: plane-interleaved [z][c][y][x], field = pitch*(ny+4)
+   * (one padded x-y plane), plane = PF_N*field (mu keeps PF_N slots per
+   * z-plane, PF_M of them used).  Only the library addresses the padded buffers;
+   * pf_init_fields / pf_download use the packed interior layout.           */
+  size_t phi_bytes;       /* one time level of phi: ((PF_N-1)*field + (nz+4)*plane)*8 + 256 */
+  size_t mu_bytes;        /* one time level of mu:  ((PF_M-1)*field + (nz+4)*plane)*8 + 256 */
   size_t workspace_bytes; /* tables, pack buffers, reduction scratch          */
 } pf_layout;
 
@@ -177,9 +191,20 @@ int pf_shift_window(pf_ctx* ctx, int k);
  * domain, -1 if there is no solid.  Collective, synchronous. */
 int pf_front_height(pf_ctx* ctx, int* H);
 
-/* Invariant monitors of the current phi: out[0] = max |sum_a phi_a - 1|,
- * out[1] = min_a,cells phi_a (global over ranks).  Collective, synchronous. */
+/* Invariant monitors of the current fields: out[0] = max |sum_a phi_a - 1|
+ * (+inf if any phi or mu value is not finite), out[1] = min_a,cells phi_a
+ * (global over ranks).  Collective, synchronous.                          */
 int pf_monitor(pf_ctx* ctx, double out[2]);
+
+/* Monitors inside pf_step (SURVEY §8(b) PF_ENUMERIC): every > 0 runs
+ * pf_monitor at the end of every run of steps that reaches a multiple of
+ * `every` (a run = one step, or one CUDA-graph replay of up to
+ * window_check steps) and makes pf_step return PF_ENUMERIC -- the state
+ * being the one after that run, pf_last_error naming the step and the
+ * values -- when max|sum phi - 1| > tol, min phi < -tol, or a value is not
+ * finite.  every = 0 (the default) turns them off.  tol >= 0.  Collective
+ * when world > 1 (every rank takes the same decision).                    */
+int pf_set_monitors(pf_ctx* ctx, int every, double tol);
 
 /* Copy the current interior fields to host (where = PF_HOST) or device
  * (PF_DEVICE) memory in the layout above.  Synchronous.                     */

@@ -316,19 +316,26 @@ __device__ __forceinline__ unsigned long long ord_bits(double v) {
   return (b & 0x8000000000000000ull) ? ~b : (b | 0x8000000000000000ull);
 }
 
-__global__ void k_monitor(Geom g, const double* __restrict__ ph, unsigned long long* out) {
+__global__ void k_monitor(Geom g, const double* __restrict__ ph, const double* __restrict__ mu,
+                          unsigned long long* out) {
   const int z = blockIdx.y;
   double e = -1.0, neg = -INFINITY;
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < g.nx * g.ny; i += gridDim.x * blockDim.x) {
     const int y = i / g.nx, x = i - y * g.nx;
     const int64_t c = g.at(x, y, z);
-    double sum = 0.0, mn = INFINITY;
+    double sum = 0.0, mn = INFINITY, fin = 0.0;  // fin: 0 for finite values, NaN otherwise
     for (int a = 0; a < N; ++a) {
       const double v = ph[a * g.field + c];
       sum += v;
       mn = fmin(mn, v);
+      fin += v - v;
     }
-    e = fmax(e, fabs(sum - 1.0));
+    for (int i2 = 0; i2 < M; ++i2) {
+      const double v = mu[i2 * g.field + c];
+      fin += v - v;
+    }
+    const double err = fabs(sum - 1.0);
+    e = fmax(e, (fin == 0.0 && err <= 1e300) ? err : INFINITY);  // non-finite -> +inf (fmax drops NaN)
     neg = fmax(neg, -mn);
   }
   for (int o = 16; o > 0; o >>= 1) {
@@ -351,11 +358,11 @@ __global__ void k_monitor(Geom g, const double* __restrict__ ph, unsigned long l
   }
 }
 
-void launch_monitor(const Geom& g, const double* phi, unsigned long long* out2, cudaStream_t s) {
+void launch_monitor(const Geom& g, const double* phi, const double* mu, unsigned long long* out2, cudaStream_t s) {
   int bx = (g.nx * g.ny + 255) / 256;
   if (bx > 64) bx = 64;
   dim3 gr(bx, g.nz);
-  k_monitor<<<gr, 256, 0, s>>>(g, phi, out2);
+  k_monitor<<<gr, 256, 0, s>>>(g, phi, mu, out2);
 }
 
 // interior <-> packed [comp][z][y][x] copies

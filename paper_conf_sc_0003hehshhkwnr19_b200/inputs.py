@@ -68,6 +68,26 @@ def ds_T0(z_front: int, G: float, dx: float = 1.0) -> float:
     return T_E - G * z_front * dx
 
 
+# Growing DS workload (SURVEY C.4 "tune v and G so the front advances
+# steadily"): pulling speed and gradient measured with
+# tools/ds_tune.py on a 256^3 block (profiles/r02_ds_tune.jsonl): at v = 0.1
+# the front advances ~0.4 planes per 100 steps (the window shifts every
+# ~260 steps); at v = 0.03 it stays within the P16 lever-rule band longer.
+DS_BENCH = {"v": 0.1, "G": 0.02}
+DS_LONG = {"v": 0.03, "G": 0.02}
+
+
+def params_ds_growth(z_front: int, v: float, G: float, **over) -> dict:
+    """C.4 set with the DS boundary conditions, pulling speed v and gradient
+    G; the isotherm is placed so that the initial front is undercooled by
+    v * tau_sl, the steady planar-front undercooling of App. A.3 (v = dpsi/tau
+    with dpsi = T_E - T for the C.4 slopes s = 1), so the front moves from the
+    first step on instead of waiting for the isotherm."""
+    P = params_c4("ds", v=v, G=G, **over)
+    P["T0"] = ds_T0(z_front, G) - v * P["tau"][0, LIQUID]
+    return P
+
+
 def params_stress(seed: int = 20191117, **over) -> dict:
     """SURVEY C.4 stress set S: every entry perturbed by a seeded +-20 %,
     non-diagonal chi_alpha and D_alpha, non-zero A1, G*v != 0, so that every

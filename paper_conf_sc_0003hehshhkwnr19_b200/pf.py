@@ -67,7 +67,7 @@ class PFState(C.Structure):
 # every symbol include/pf.h declares (checked by tests/test_abi.py)
 ABI_SYMBOLS = ["pf_query_layout", "pf_query_neighbors", "pf_create", "pf_destroy", "pf_set_params", "pf_init_fields", "pf_step",
                "pf_step_phi_only", "pf_halo_exchange", "pf_shift_window", "pf_front_height", "pf_monitor",
-               "pf_download", "pf_get_state", "pf_set_state", "pf_set_variant", "pf_tuning_default", "pf_set_tuning",
+               "pf_set_monitors", "pf_download", "pf_get_state", "pf_set_state", "pf_set_variant", "pf_tuning_default", "pf_set_tuning",
                "pf_get_tuning", "pf_tuning_check", "pf_autotune", "pf_profile", "pf_profile_read",
                "pf_nccl_unique_id", "pf_jit_compile_only", "pf_last_error", "pf_version"]
 
@@ -96,6 +96,7 @@ def load_library(path: str = LIB_PATH):
     L.pf_shift_window.argtypes = [vp, ip]
     L.pf_front_height.argtypes = [vp, C.POINTER(ip)]
     L.pf_monitor.argtypes = [vp, dp]
+    L.pf_set_monitors.argtypes = [vp, ip, C.c_double]
     L.pf_download.argtypes = [vp, vp, vp, ip]
     L.pf_get_state.argtypes = [vp, C.POINTER(PFState)]
     L.pf_set_state.argtypes = [vp, C.POINTER(PFState)]
@@ -233,10 +234,14 @@ class PhaseField:
     shape = global (nz, ny, nx); procs = rank grid (px, py, pz); bc = dict
     {"lo": (x, y, z), "hi": (x, y, z)} of "periodic" / "neumann" /
     "dirichlet_mu".  Buffers are torch tensors owned by this object.
+    local_group = name: this block is rank `rank` of a decomposition whose
+    `world` blocks live in this process (each stepped from its own thread);
+    see pf.h (nccl_uid "PFLOCAL:").
     """
 
     def __init__(self, shape, params: dict, bc=None, liquid: int | None = None, procs=(1, 1, 1), rank: int = 0,
-                 world: int = 1, device: int | None = None, nccl_uid: bytes | None = None, stream=None):
+                 world: int = 1, device: int | None = None, nccl_uid: bytes | None = None, stream=None,
+                 local_group: str | None = None):
         import torch
         if not torch.cuda.is_available():
             raise PFError("no CUDA device: the phase-field step has no CPU fallback")
@@ -256,6 +261,8 @@ class PhaseField:
             cfg.bc_lo[d] = BC[bc["lo"][d]]
             cfg.bc_hi[d] = BC[bc["hi"][d]]
         cfg.rank, cfg.world = int(rank), int(world)
+        if local_group is not None:  # in-process transport (pf.h: "PFLOCAL:<name>")
+            nccl_uid = b"PFLOCAL:" + local_group.encode()[:110] + b"\0"
         if nccl_uid is not None:
             for i, b in enumerate(nccl_uid[:128]):
                 cfg.nccl_uid[i] = b
@@ -349,6 +356,11 @@ class PhaseField:
         out = (C.c_double * 2)()
         self._check(self.lib.pf_monitor(self._h, out), "pf_monitor")
         return float(out[0]), float(out[1])
+
+    def set_monitors(self, every: int, tol: float = 1e-12):
+        """pf_set_monitors: pf_step checks the invariants every `every` steps
+        and raises PFError (PF_ENUMERIC) when they trip; 0 = off."""
+        self._check(self.lib.pf_set_monitors(self._h, int(every), float(tol)), "pf_set_monitors")
 
     def download(self, out=None, device: bool = False):
         """Interior fields; numpy by default, torch cuda tensors if device=True,

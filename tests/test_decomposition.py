@@ -35,7 +35,12 @@ def test_blocks_tile_the_domain(shape, procs):
         nx, ny, nz = L.local
         ox, oy, oz = L.offset
         cover[oz:oz + nz, oy:oy + ny, ox:ox + nx] += 1
-        assert L.pitch % 16 == 0 and L.x_off == 16 and L.plane == L.pitch * (ny + 4)
+        assert L.pitch % 16 == 0 and L.x_off == 16
+        # structure of arrays [c][z][y][x] (default); PF_LAYOUT=il:
+        # plane-interleaved [z][c][y][x], component stride = one padded x-y
+        # plane, z stride = 4 of them
+        pxy = L.pitch * (ny + 4)
+        assert (L.field, L.plane) in ((pxy, 4 * pxy), (pxy * (nz + 4), pxy))
     assert np.all(cover == 1)
 
 

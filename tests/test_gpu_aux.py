@@ -1,0 +1,105 @@
+"""Auxiliary subsystems on the GPU (VERDICT r1 "next" 8): the
+PF_ENUMERIC invariant monitors inside pf_step, bitwise checkpoint / resume
+through the public API (pf_download -> pf_init_fields + pf_set_state), and
+compute-sanitizer memcheck / racecheck over every kernel of the library.
+-m gpu.
+"""
+import os
+import shutil
+import subprocess
+import sys
+
+import numpy as np
+import pytest
+
+from paper_conf_sc_0003hehshhkwnr19_b200 import inputs as I
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def pfmod():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.fail("GPU test without a CUDA device")
+    from paper_conf_sc_0003hehshhkwnr19_b200 import build, pf
+    build.build()
+    return pf
+
+
+def test_monitors_trip_on_non_finite(pfmod):
+    """A non-finite mu value spreads through the step (mu enters psi of the
+    phi equation); with the monitors on, pf_step stops with PF_ENUMERIC."""
+    shape = (12, 10, 14)
+    P = I.params_stress()
+    phi, mu = I.ic_voronoi(shape, seed=2)
+    mu[0, 5, 5, 5] = np.nan
+    g = pfmod.PhaseField(shape, P)
+    g.init_fields(phi, mu)
+    g.set_monitors(1, 1e-12)
+    with pytest.raises(pfmod.PFError) as ei:
+        g.step(5)
+    assert "(-6)" in str(ei.value) and "monitor tripped after step 1" in str(ei.value)
+    assert g.state()["step"] == 1
+    err, _ = g.monitor()
+    assert err == np.inf
+
+
+def test_monitors_tolerance_and_off(pfmod):
+    shape = (12, 10, 14)
+    P = I.params_stress()
+    phi, mu = I.ic_random(shape, seed=4)
+    g = pfmod.PhaseField(shape, P)
+    g.init_fields(phi, mu)
+    g.set_monitors(2, 1e-12)
+    g.step(6)  # healthy run: max|sum phi - 1| is a few ulp
+    assert g.state()["step"] == 6
+    g.set_monitors(1, 0.0)  # zero tolerance: the rounding of the projection trips it
+    with pytest.raises(pfmod.PFError):
+        g.step(3)
+    g.set_monitors(0, 0.0)
+    g.step(3)
+
+
+@pytest.mark.parametrize("variant", ["jit", "tuned"])
+def test_resume_bitwise(pfmod, variant):
+    """Checkpoint / resume: the state is (phi, mu, step, z_off); a run resumed
+    from pf_download + pf_init_fields + pf_set_state continues bitwise equal
+    to the uninterrupted run (frozen T, fluctuation counter and moving window
+    all depend on step / z_off)."""
+    P = I.params_stress(window_check=5, window_frac=0.5, xi_amp=0.02, xi_seed=11)
+    shape = (32, 12, 20)
+    phi, mu = I.ic_lamellar(shape, seed=3, z_front=20, mu_inf=tuple(P["mu_inf"]))
+    a = pfmod.PhaseField(shape, P, bc=I.BC_DS)
+    a.set_variant(variant)
+    a.init_fields(phi, mu)
+    a.step(23)
+    ck = a.download()
+    st = a.state()
+    assert st["z_off"] > 0
+    a.step(31)
+    ref = a.download()
+    b = pfmod.PhaseField(shape, P, bc=I.BC_DS)
+    b.set_variant(variant)
+    b.init_fields(*ck)
+    b.set_state(**st)
+    b.step(31)
+    got = b.download()
+    assert b.state() == a.state()
+    assert np.array_equal(got[0], ref[0]) and np.array_equal(got[1], ref[1])
+
+
+@pytest.mark.parametrize("tool", ["memcheck", "racecheck"])
+def test_compute_sanitizer(tool):
+    cs = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
+    if not os.path.exists(cs):
+        pytest.fail("compute-sanitizer not found")
+    variants = ["jit", "tuned", "naive"] if tool == "memcheck" else ["jit", "tuned"]
+    cmd = [cs, "--tool", tool, "--error-exitcode", "1", sys.executable, os.path.join(ROOT, "tools", "sanitize_run.py"),
+           *variants]
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=1500, cwd=ROOT)
+    tail = (r.stdout + r.stderr)[-3000:]
+    assert r.returncode == 0, tail
+    assert "sanitize run ok" in r.stdout, tail
+    assert "ERROR SUMMARY: 0 errors" in (r.stdout + r.stderr) or "RACECHECK SUMMARY: 0 hazards" in (r.stdout + r.stderr), tail

@@ -31,6 +31,26 @@ __global__ void k(double* out, double a, double b) {
   if (s == 12345.678) out[0] = s;
 }
 
+// dependent-chain latency (one warp per SM, ILP 1), cycles per op by clock64
+template <int OP>
+__global__ void k_lat(double* out, long long* cyc, double a, double b) {
+  double x = a + threadIdx.x * 1e-12;
+  const long long t0 = clock64();
+  for (int it = 0; it < ITERS; ++it) {
+    if (OP == 0) x = fma(x, a, b);
+    if (OP == 1) x = x + b;
+    if (OP == 2) x = x * a;
+    if (OP == 3) {
+      double y;
+      asm volatile("rsqrt.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(x));
+      x = y + b;
+    }
+  }
+  const long long t1 = clock64();
+  if (threadIdx.x == 0) cyc[blockIdx.x] = t1 - t0;
+  if (x == 12345.678) out[0] = x;
+}
+
 int main() {
   cudaDeviceProp p;
   cudaGetDeviceProperties(&p, 0);
@@ -75,6 +95,27 @@ int main() {
       double gops = ops / (best * 1e-3) / 1e9;
       printf("  {\"op\": \"%s\", \"blocks_per_sm\": %d, \"ms\": %.4f, \"Gop_per_s\": %.1f, \"op_per_clk_per_sm_at_1965\": %.2f}%s\n",
              names[op], bps, best, gops, gops * 1e9 / (sms * 1.965e9), (op == 6 && bps == 8) ? "" : ",");
+    }
+  }
+  printf("], \"latency_cycles\": [\n");
+  {
+    long long* cyc;
+    cudaMalloc(&cyc, sizeof(long long) * sms);
+    const char* ln[] = {"dfma", "dadd", "dmul", "mufu.rsq64h+dadd"};
+    for (int op = 0; op < 4; ++op) {
+      for (int r = 0; r < 2; ++r) {
+        switch (op) {
+          case 0: k_lat<0><<<sms, 32>>>(out, cyc, 1.0000001, 1e-9); break;
+          case 1: k_lat<1><<<sms, 32>>>(out, cyc, 1.0000001, 1e-9); break;
+          case 2: k_lat<2><<<sms, 32>>>(out, cyc, 1.0000001, 1e-9); break;
+          case 3: k_lat<3><<<sms, 32>>>(out, cyc, 1.0, 1.0); break;
+        }
+        cudaDeviceSynchronize();
+      }
+      long long c = 0;
+      cudaMemcpy(&c, cyc, sizeof c, cudaMemcpyDeviceToHost);
+      printf("  {\"op\": \"%s\", \"cycles_per_dependent_op\": %.2f}%s\n", ln[op], (double)c / ITERS,
+             op == 3 ? "" : ",");
     }
   }
   printf("]}\n");
