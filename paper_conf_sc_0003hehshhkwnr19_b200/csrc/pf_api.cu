@@ -1315,7 +1315,7 @@ int pf_init_fields(pf_ctx* ctx, const double* phi, const double* mu, int where) 
   if (int r = pf_monitor(ctx, mon)) return r;
   if (!(mon[0] <= 1e-12) || !(mon[1] >= 0.0)) {
     ctx->have_fields = false;
-    return fail(ctx, PF_EINVAL, "initial phi off the Gibbs simplex: max|sum-1| = %g, min = %g", mon[0], mon[1]);
+    return fail(ctx, PF_EINVAL, "initial fields off the Gibbs simplex or not finite: max|sum phi - 1| = %g, min phi = %g", mon[0], mon[1]);
   }
   if (int r = pf_halo_exchange(ctx, PF_PHI | PF_MU)) return r;
   CU(cudaStreamSynchronize(ctx->stream));

@@ -29,13 +29,18 @@ def pfmod():
 
 
 def test_monitors_trip_on_non_finite(pfmod):
-    """A non-finite mu value spreads through the step (mu enters psi of the
-    phi equation); with the monitors on, pf_step stops with PF_ENUMERIC."""
+    """pf_init_fields rejects a non-finite field; a finite but huge mu value
+    overflows psi = mu.A mu of the phi equation in the first step, and with
+    the monitors on pf_step stops there with PF_ENUMERIC."""
     shape = (12, 10, 14)
     P = I.params_stress()
     phi, mu = I.ic_voronoi(shape, seed=2)
-    mu[0, 5, 5, 5] = np.nan
     g = pfmod.PhaseField(shape, P)
+    bad = mu.copy()
+    bad[0, 5, 5, 5] = np.nan
+    with pytest.raises(pfmod.PFError):
+        g.init_fields(phi, bad)
+    mu[0, 5, 5, 5] = 1e200
     g.init_fields(phi, mu)
     g.set_monitors(1, 1e-12)
     with pytest.raises(pfmod.PFError) as ei:
