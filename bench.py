@@ -391,8 +391,13 @@ def main():
                      "hw_flop_per_cell": ncu_summary("hw_flop_per_cell"),
                      "hw_achieved": (ncu_summary("hw_flop_per_cell") * cells_local / (mu_ms / mu_n * 1e-3) / 1e12)
                      if (mu_n and ncu_summary("hw_flop_per_cell")) else None,
+                     "hw_frac": ((ncu_summary("hw_flop_per_cell") * cells_local / (mu_ms / mu_n * 1e-3) / 1e12) / peak_tf)
+                     if (mu_n and ncu_summary("hw_flop_per_cell")) else None,
                      "avg_launch_ms": mu_ms / mu_n if mu_n else None,
-                     "peak_note": "derived: 148 SMs x 64 FP64 lanes x 2 x 1.965 GHz (DESIGN.md §6)"},
+                     "peak_note": "derived: 148 SMs x 64 FP64 lanes x 2 x 1.965 GHz (DESIGN.md §6); measured DFMA "
+                                  "36.8 TF/s at 1965 MHz (profiles/r02_fp64_micro.json)",
+                     "frac_note": "frac: Table-1 algorithmic flops (866/cell); hw_frac: fp64 work the specialised "
+                                  "kernel issues (DADD + DMUL + 2 DFMA per cell, ncu)"},
         "kernels": {"phi_sweep_ms": phi_ms / max(phi_n, 1), "mu_sweep_ms": mu_ms / max(mu_n, 1),
                     "phi_sweep_tflops": phi_tf, "share_mu": mu_ms / ms if ms else None,
                     "share_phi": phi_ms / ms if ms else None,
@@ -423,8 +428,10 @@ def main():
         bytes_state = (phi_pin.numel() + mu_pin.numel()) * 8
         rec["e2e"] = {"value": total_cells * args.steps / (ems * 1e-3) / 1e6, "unit": UNIT,
                       "h2d_bytes_per_step": bytes_state / args.steps, "d2h_bytes_per_step": bytes_state / args.steps,
-                      "note": "one chunk = pf_init_fields from pinned host memory, K steps, pf_download to pinned "
-                              "host memory, all inside the timed region"}
+                      "chunk_steps": args.steps,
+                      "note": f"one chunk = pf_init_fields from pinned host memory, {args.steps} steps, pf_download to "
+                              "pinned host memory, all inside the timed region (the copies amortise over the chunk: "
+                              "the value depends on the chunk length)"}
     # ---- general-expression path: the stress parameter set S (unequal gamma,
     # A1 != 0, non-diagonal chi / D, mu_inf != 0: none of the specialised
     # simplifications apply), same block, boundaries and IC

@@ -268,6 +268,11 @@ typedef struct {
                         or 8: a 32 x mu_ty tile on 32 x mu_ty/2 threads)          */
   int phi_rpt;       /* phi-sweep tile rows per thread: 1, or 2 (phi_faces6 = 1,
                         phi_xsh = 0, even phi_ty: 32 x phi_ty/2 threads)           */
+  int mu_pers;       /* 1: full mu-sweep launches are persistent (one CTA per
+                        resident slot, each a balanced contiguous share of the
+                        tile-planes; no partial last wave, one z-march restart per
+                        share instead of one per mu_zc chunk); mu_rpt = 2 only     */
+  int phi_pers;      /* 1: the same for the phi-sweep (phi_faces6 = 1, phi_rpt = 1) */
 } pf_tuning;
 
 /* The built-in defaults (the measured best at 256^3 on one B200,

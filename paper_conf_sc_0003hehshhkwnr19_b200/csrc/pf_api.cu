@@ -1523,6 +1523,8 @@ const std::vector<TuneKnob>& tune_knobs() {
       {"mu_rot", &pf_tuning::mu_rot, JIT_MU, {0, 1}},
       {"mu_rpt", &pf_tuning::mu_rpt, JIT_MU, {1, 2}},
       {"phi_rpt", &pf_tuning::phi_rpt, JIT_PHI, {1, 2}},
+      {"mu_pers", &pf_tuning::mu_pers, JIT_MU, {0, 1}},
+      {"phi_pers", &pf_tuning::phi_pers, JIT_PHI, {0, 1}},
   };
   return k;
 }

@@ -78,7 +78,7 @@ struct StepVals {
 struct TileSel {
   int off[3];
   int lo[3], hi[3];
-  int skip;
+  int skip;  // 1: skip the tiles inside [lo, hi); 2: persistent launch over all tiles (mu_pers)
 };
 
 // Scalars and coefficients of the model.  Passed by value to every kernel

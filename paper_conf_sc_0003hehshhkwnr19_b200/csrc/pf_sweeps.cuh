@@ -108,6 +108,12 @@ constexpr int MU_TY = PF_MU_TY;
 #ifndef PF_PHI_ZREC
 #define PF_PHI_ZREC 0
 #endif
+#ifndef PF_PHI_PERS  // six-face phi-sweep as a persistent launch (balanced tile-plane shares)
+#define PF_PHI_PERS 0
+#endif
+#ifndef PF_MU_PERS  // two-rows mu-sweep: full launches persistent (balanced tile-plane shares)
+#define PF_MU_PERS 0
+#endif
 #ifndef PF_PHI_XSH  // six-face sweep, +x face taken from the next lane (31 cells per 32-lane row)
 #define PF_PHI_XSH 0
 #endif
@@ -119,7 +125,8 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const RT& R, const G
                                                const double* __restrict__ ps, const double* __restrict__ ms,
                                                double* __restrict__ pd) {
 #if PF_PHI_FACES6
-  {
+  // one tile (bx, by) over planes [z0, z1)
+  auto tile = [&](const int bx, const int by, const int z0, const int z1) {
     // The +x / +y face of a cell is the -x / -y face of its neighbour: both
     // threads evaluate phi_face on the same (left, right) operands, so the
     // two values are bitwise equal and the fluxes still telescope.  Costs
@@ -131,16 +138,15 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const RT& R, const G
     // lanes past the row's end, clamped to the ghost x = nx) only supply the
     // -x face that is the +x face of the lane before them (same operands:
     // bitwise equal to evaluating it there)
-    const int xr = blockIdx.x * PHI_TXC + threadIdx.x, y = blockIdx.y * PTY + threadIdx.y;
-    if (y >= g.ny || blockIdx.x * PHI_TXC >= g.nx) return;  // whole warps: the shuffles need all lanes
+    const int xr = bx * PHI_TXC + threadIdx.x, y = by * PTY + threadIdx.y;
+    if (y >= g.ny || bx * PHI_TXC >= g.nx) return;  // whole warps: the shuffles need all lanes
     const bool act = xr < g.nx && threadIdx.x < PHI_TXC;
     const int x = min(xr, g.nx);
 #else
-    const int x = blockIdx.x * TX + threadIdx.x, y = blockIdx.y * PTY + threadIdx.y;
+    const int x = bx * TX + threadIdx.x, y = by * PTY + threadIdx.y;
     if (x >= g.nx || y >= g.ny) return;
     constexpr bool act = true;
 #endif
-    const int z0 = blockIdx.z * ZC_PHI, z1 = min(z0 + ZC_PHI, g.nz);
     const i64 F = g.field, SY = g.pitch, SZ = g.plane;
     i64 c = g.at(x, y, z0);
     double pm[N], p0[N], Fzm[N];
@@ -210,8 +216,39 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const RT& R, const G
         Fzm[a] = Fzp[a];
       }
     }
-    return;
+  };  // tile
+#if PF_PHI_PERS
+  // persistent launch (tuning phi_pers): gridDim.x CTAs, each a balanced
+  // contiguous share of the tile-planes in tile-major order (no partial last
+  // wave; a tile column restarts its z-march ~once instead of once per chunk).
+  // Warps advance independently (no barrier in this sweep): the share's
+  // position is kept per warp in shared memory, not in registers.
+  {
+    __shared__ long long seg[PTY][2];
+    const int ntx = (g.nx + PHI_TXC - 1) / PHI_TXC, nty = (g.ny + PTY - 1) / PTY;
+    volatile long long* vs = seg[threadIdx.y];
+    if (threadIdx.x == 0) {
+      const i64 total = (i64)ntx * nty * g.nz;
+      vs[0] = total * blockIdx.x / gridDim.x;
+      vs[1] = total * (blockIdx.x + 1) / gridDim.x;
+    }
+    __syncwarp();
+    for (;;) {
+      const i64 lo = vs[0], hi = vs[1];
+      if (lo >= hi) break;
+      const i64 tl = lo / g.nz;
+      const int z0 = (int)(lo - tl * g.nz);
+      const int z1 = (int)min((i64)g.nz, (i64)z0 + (hi - lo));
+      tile((int)(tl % ntx), (int)(tl / ntx), z0, z1);
+      __syncwarp();
+      if (threadIdx.x == 0) vs[0] = lo + (z1 - z0);
+      __syncwarp();
+    }
   }
+#else
+  tile(blockIdx.x, blockIdx.y, blockIdx.z * ZC_PHI, min(blockIdx.z * ZC_PHI + ZC_PHI, g.nz));
+#endif
+  return;
 #endif
   __shared__ double fy[2][N][PTY][TX];  // -y face flux of every thread, by plane parity
   __shared__ double ex[2][N][PTY];      // +x flux on the right tile edge
@@ -1017,10 +1054,8 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
   constexpr int MTX = 32, TYT = MTY / 2, NT = MTX * TYT;
   constexpr int NC = MuTile<MTY, MTX>::NC, HX = MuTile<MTY, MTX>::HX;
   static_assert(MTY % 2 == 0 && 2 * MTX + 2 * MTY <= NT && TYT >= 2, "mu_rpt = 2 needs an even MTY >= 6");
-  const int tbx = blockIdx.x + ts.off[0], tby = blockIdx.y + ts.off[1], tbz = blockIdx.z + ts.off[2];
-  if (ts.skip && tbx >= ts.lo[0] && tbx < ts.hi[0] && tby >= ts.lo[1] && tby < ts.hi[1] && tbz >= ts.lo[2] &&
-      tbz < ts.hi[2])
-    return;  // interior tile, done by the other launch
+  // one tile column (tbx, tby) over planes [z0, z1)
+  auto tile = [&](const int tbx, const int tby, const int z0, const int z1) {
   extern __shared__ double smem[];
   double* D = smem;
   double* fxs = D + D_NV * NC;             // [M][MTY][MTX+1]
@@ -1028,7 +1063,6 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
   const int lane = threadIdx.x, w = threadIdx.y, t = w * MTX + lane;
   const int x0 = tbx * MTX, y0 = tby * MTY;
   const int x = x0 + lane;
-  const int z0 = tbz * ZC_MU, z1 = min(z0 + ZC_MU, g.nz);
   const i64 F = g.field;
   const int xc = min(x, g.nx);
   int yc[2], me[2];
@@ -1298,6 +1332,43 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
   };
   for (int k = z0; k < z1; ++k) plane(BoolC<false>{}, k);
   plane(BoolC<true>{}, z1);
+  };  // tile
+#if PF_MU_PERS
+  if (ts.skip == 2) {
+    // persistent launch (tuning mu_pers): gridDim.x CTAs, each a balanced
+    // contiguous share of the tile-planes in tile-major order, so that every
+    // CTA slot of the GPU finishes at the same time (no partial last wave)
+    // and a tile column restarts its z-march ~once instead of once per chunk.
+    // The share's position lives in shared memory (volatile), not in
+    // registers across the tile's march.
+    __shared__ long long seg[2];
+    const int ntx = (g.nx + MTX - 1) / MTX, nty = (g.ny + MTY - 1) / MTY;
+    if (threadIdx.x == 0 && threadIdx.y == 0) {
+      const i64 total = (i64)ntx * nty * g.nz;
+      seg[0] = total * blockIdx.x / gridDim.x;
+      seg[1] = total * (blockIdx.x + 1) / gridDim.x;
+    }
+    __syncthreads();
+    volatile long long* vs = seg;
+    for (;;) {
+      const i64 lo = vs[0], hi = vs[1];
+      if (lo >= hi) break;
+      const i64 tl = lo / g.nz;
+      const int z0 = (int)(lo - tl * g.nz);
+      const int z1 = (int)min((i64)g.nz, (i64)z0 + (hi - lo));
+      tile((int)(tl % ntx), (int)(tl / ntx), z0, z1);
+      __syncthreads();  // every thread has read seg and finished the tile's shared-memory reads
+      if (threadIdx.x == 0 && threadIdx.y == 0) vs[0] = lo + (z1 - z0);
+      __syncthreads();
+    }
+    return;
+  }
+#endif
+  const int tbx = blockIdx.x + ts.off[0], tby = blockIdx.y + ts.off[1], tbz = blockIdx.z + ts.off[2];
+  if (ts.skip && tbx >= ts.lo[0] && tbx < ts.hi[0] && tby >= ts.lo[1] && tby < ts.hi[1] && tbz >= ts.lo[2] &&
+      tbz < ts.hi[2])
+    return;  // interior tile, done by the other launch
+  tile(tbx, tby, tbz * ZC_MU, min(tbz * ZC_MU + ZC_MU, g.nz));
 }
 
 }  // namespace pf
