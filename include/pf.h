@@ -273,6 +273,13 @@ typedef struct {
                         tile-planes; no partial last wave, one z-march restart per
                         share instead of one per mu_zc chunk); mu_rpt = 2 only     */
   int phi_pers;      /* 1: the same for the phi-sweep (phi_faces6 = 1, phi_rpt = 1) */
+  int sched;         /* step schedule (S§7 step 6): 0 = two full sweeps (phi, ghosts,
+                        mu); 1 = z-slab pipeline: per slab of `slab` mu z-chunks the
+                        phi-sweep of the slab (shifted up one plane), its x/y
+                        ghosts, then the mu-sweep of the slab while its phi_dst is
+                        still in L2.  Applies to the JIT variant with no exchanged
+                        dimension and a non-periodic z (DS); otherwise sched 0     */
+  int slab;          /* mu z-chunks per slab of sched = 1 (1..16)                 */
 } pf_tuning;
 
 /* The built-in defaults (the measured best at 256^3 on one B200,

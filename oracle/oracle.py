@@ -46,6 +46,9 @@ class OrParams(C.Structure):
         ("window_frac", C.c_double), ("window_check", C.c_int),
         ("antitrapping", C.c_int), ("projection", C.c_int),
         ("xi_amp", C.c_double), ("xi_seed", C.c_uint),
+        ("aniso", C.c_int),
+        ("aniso_delta", C.c_double * MAXN * MAXN),
+        ("aniso_R", C.c_double * 3 * 3 * MAXN * MAXN),
     ]
 
 
@@ -139,6 +142,11 @@ def make_params(P: dict) -> OrParams:
     p.projection = int(P.get("projection", 1))
     p.xi_amp = float(P.get("xi_amp", 0.0))
     p.xi_seed = int(P.get("xi_seed", 0)) & 0xFFFFFFFF
+    # P2 anisotropy (reading B6): aniso_delta[N][N], aniso_R[N][N][3][3]
+    p.aniso = int(P.get("aniso", 0))
+    if p.aniso:
+        put(p.aniso_delta, P["aniso_delta"], (N, N))
+        put(p.aniso_R, P["aniso_R"], (N, N, 3, 3))
     return p
 
 

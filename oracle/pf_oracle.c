@@ -186,6 +186,29 @@ void oracle_project_simplex(int N, const double* x, double* out) {
 /* phi-sweep  (Algorithm 1 line 1)                              */
 /* ------------------------------------------------------------------------ */
 
+/* Anisotropic gradient energy (P2, reading B6): f(q) = A(R q)^2 |q|^2 with
+ * A(p) = 1 - delta (3 - 4 sum_i p_i^4 / |p|^4).  grad_q f = R^T grad_p f,
+ *   d f / d p_i = 2 A (dA/dp_i) |p|^2 + 2 A^2 p_i,
+ *   dA/dp_i = 16 delta (p_i^3 / |p|^4 - (sum_j p_j^4) p_i / |p|^6);
+ * f -> 0 and grad f -> 0 as q -> 0 (A is bounded): q = 0 gives 0 exactly. */
+static void aniso_grad(const or_params* p, int a, int b, const double q[3], double out[3]) {
+  const double (*R)[3] = p->aniso_R[a][b];
+  const double delta = p->aniso_delta[a][b];
+  double v[3];
+  for (int i = 0; i < 3; ++i) v[i] = R[i][0] * q[0] + R[i][1] * q[1] + R[i][2] * q[2];
+  double n2 = v[0] * v[0] + v[1] * v[1] + v[2] * v[2];
+  if (n2 == 0.0) { out[0] = out[1] = out[2] = 0.0; return; }
+  double s4 = 0.0;
+  for (int i = 0; i < 3; ++i) s4 += v[i] * v[i] * v[i] * v[i];
+  double A = 1.0 - delta * (3.0 - 4.0 * s4 / (n2 * n2));
+  double gp[3];
+  for (int i = 0; i < 3; ++i) {
+    double dA = 16.0 * delta * (v[i] * v[i] * v[i] / (n2 * n2) - s4 * v[i] / (n2 * n2 * n2));
+    gp[i] = 2.0 * A * dA * n2 + 2.0 * A * A * v[i];
+  }
+  for (int j = 0; j < 3; ++j) out[j] = R[0][j] * gp[0] + R[1][j] * gp[1] + R[2][j] * gp[2];
+}
+
 /* Staggered flux of the gradient energy at the face between p and q = p+e_d
  * (eq. 11 "divergence of fluxes"):
  *   (da/d grad phi_a)_d = 2 sum_{b!=a} gamma_ab phib_b (phib_b d_d phi_a - phib_a d_d phi_b)
@@ -203,6 +226,33 @@ static void phi_face_flux(const pf_oracle* o, int x, int y, int z, int d, double
     double vp = rd(o, F_PHI_SRC, b, x, y, z), vq = rd(o, F_PHI_SRC, b, qx, qy, qz);
     pb[b] = 0.5 * (vp + vq);
     dd[b] = (vq - vp) / p->dx;
+  }
+  if (p->aniso) {
+    /* P2 [B6]: j_a = d a / d (grad phi_a), d-component, at the face:
+     * sum_{b != a} gamma_ab (-phib_b) (grad_q f(q_ab))_d with
+     * q_ab = phib_a G_b - phib_b G_a and the whole face gradient G (normal
+     * difference, tangential = mean of the two central differences [A9]). */
+    double G[OR_MAXN][3];
+    for (int b = 0; b < p->N; ++b)
+      for (int e = 0; e < 3; ++e) {
+        if (e == d) { G[b][e] = dd[b]; continue; }
+        int ex = (e == 0), ey = (e == 1), ez = (e == 2);
+        G[b][e] = (rd(o, F_PHI_SRC, b, x + ex, y + ey, z + ez) - rd(o, F_PHI_SRC, b, x - ex, y - ey, z - ez) +
+                   rd(o, F_PHI_SRC, b, qx + ex, qy + ey, qz + ez) - rd(o, F_PHI_SRC, b, qx - ex, qy - ey, qz - ez)) /
+                  (4.0 * p->dx);
+      }
+    for (int a = 0; a < p->N; ++a) {
+      double s = 0.0;
+      for (int b = 0; b < p->N; ++b) {
+        if (b == a) continue;
+        double qv[3], gf[3];
+        for (int e = 0; e < 3; ++e) qv[e] = pb[a] * G[b][e] - pb[b] * G[a][e];
+        aniso_grad(p, a, b, qv, gf);
+        s += p->gamma[a][b] * (-pb[b]) * gf[d];
+      }
+      j[a] = s;
+    }
+    return;
   }
   for (int a = 0; a < p->N; ++a) {
     double s = 0.0;
@@ -243,6 +293,15 @@ static void phi_rhs_cell(const pf_oracle* o, int x, int y, int z, double* r) {
   for (int a = 0; a < N; ++a) {
     /* da/dphi_a = 2 sum_{b!=a} gamma_ab (phi_a g_b - phi_b g_a) . g_b  (eq. 4) */
     double dadphi = 0.0;
+    if (p->aniso) { /* P2 [B6]: sum_{b!=a} gamma_ab grad_q f(q_ab) . g_b, q_ab = phi_a g_b - phi_b g_a */
+      for (int b = 0; b < N; ++b) {
+        if (b == a) continue;
+        double qv[3], gf[3];
+        for (int d = 0; d < 3; ++d) qv[d] = ph[a] * g[b][d] - ph[b] * g[a][d];
+        aniso_grad(p, a, b, qv, gf);
+        dadphi += p->gamma[a][b] * (gf[0] * g[b][0] + gf[1] * g[b][1] + gf[2] * g[b][2]);
+      }
+    } else {
     for (int b = 0; b < N; ++b) {
       if (b == a) continue;
       double dot = 0.0;
@@ -250,6 +309,7 @@ static void phi_rhs_cell(const pf_oracle* o, int x, int y, int z, double* r) {
       dadphi += p->gamma[a][b] * dot;
     }
     dadphi *= 2.0;
+    }
     /* 3. omega'_a = 16/pi^2 sum_{b!=a} gamma_ab phi_b + sum_{b<d; b,d!=a} gamma_abd phi_b phi_d (eq. 5) */
     double om = 0.0;
     for (int b = 0; b < N; ++b)

@@ -52,6 +52,16 @@ typedef struct {
    * the global cell index and the time step; 0 = off (reading A17)        */
   double xi_amp;
   unsigned int xi_seed;
+  /* P2 parameterisation: anisotropic
+   * gradient energy a = sum_{a<b} gamma_ab A_ab(R_ab q_ab)^2 |q_ab|^2 (eq. 4,
+   * P:L382-398), reading B6: cubic A_ab(p) = 1 - delta_ab (3 - 4 sum_i p_i^4
+   * / |p|^4), R_ab orthonormal, both symmetric in (a, b).  The face flux of
+   * eq. 11 then needs the whole face gradient (normal + mean tangential
+   * central differences, as for mu [A9]): a 19-point phi stencil.
+   * aniso = 0: A = 1 (P1, 7-point phi stencil).                          */
+  int aniso;
+  double aniso_delta[OR_MAXN][OR_MAXN];
+  double aniso_R[OR_MAXN][OR_MAXN][3][3];
 } or_params;
 
 typedef struct {

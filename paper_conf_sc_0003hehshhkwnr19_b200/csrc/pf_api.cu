@@ -1035,7 +1035,67 @@ static int launch_mu(pf_ctx* ctx, const TileSel* ts, dim3 grid, const double* ps
   return check_launch(ctx, "mu_sweep");
 }
 
-static int step_impl(pf_ctx* ctx, bool phi_only) {
+// the z-slab schedule of one step (see step_impl); no exchanged dimension
+static int step_slabs(pf_ctx* ctx, const double* ps, double* pd, const double* ms, double* md, bool dry) {
+  const Geom& g = ctx->g;
+  const int zc = jit_mu_zc_of(ctx->jmu), mty = jit_mu_ty_of(ctx->jmu), mtx = jit_mu_tx_of(ctx->jmu);
+  const int H = zc * ctx->tune.slab;
+  const int S = (g.nz + H - 1) / H;
+  const dim3 full = tuned_grid_mu(g, mty, zc, mtx);
+  BCSpec bxy = ctx->bc_all;  // x / y ghosts of a range of planes: z sides left alone
+  bxy.kind_lo[2] = bxy.kind_hi[2] = -1;
+  for (int s = 0; s < S; ++s) {
+    const int zs = s * H, ze = std::min(g.nz, zs + H);
+    const int plo = s == 0 ? 0 : zs + 1, phi_hi = s == S - 1 ? g.nz : ze + 1;
+    cudaEvent_t e0 = nullptr;
+    prof_begin(ctx, 0, &e0);
+    CU(jit_launch_phi(ctx->jphi, ctx->dp, ps, ms, pd, ctx->stream, ctx->cap_sv, plo, phi_hi));
+    ctx->nlaunch[0] += 1;
+    prof_end(ctx, 0, e0);
+    if (int r = check_launch(ctx, "phi_sweep slab")) return r;
+    prof_begin(ctx, 2, &e0);
+    Geom gs = g;
+    gs.nz = phi_hi - plo;
+    launch_ghost_fill(gs, bxy, pd + (size_t)plo * (size_t)g.plane, PF_N, nullptr, ctx->stream);
+    ctx->nlaunch[2] += 1;
+    if (s == 0 || s == S - 1) {  // z ghost planes (whole extended planes: after their x / y ghosts)
+      launch_ghost_stage(g, 2, s == 0 ? ctx->cfg.bc_lo[2] : -1, s == S - 1 ? ctx->cfg.bc_hi[2] : -1, pd, PF_N,
+                         nullptr, ctx->stream);
+      ctx->nlaunch[2] += 1;
+    }
+    prof_end(ctx, 2, e0);
+    if (int r = check_launch(ctx, "ghost slab")) return r;
+    if (s == 0)
+      if (int r = join_comm(ctx)) return r;  // the previous step's mu ghosts
+    const TileSel ts = {{0, 0, zs / zc}, {0, 0, 0}, {0, 0, 0}, 0};
+    prof_begin(ctx, 1, &e0);
+    if (int r = launch_mu(ctx, &ts, dim3(full.x, full.y, (unsigned)((ze - zs + zc - 1) / zc)), ps, pd, ms, md))
+      return r;
+    prof_end(ctx, 1, e0);
+  }
+  // line 4: mu ghosts on the side stream (overlapping the next step's first phi slab)
+  if (ctx->overlap && ctx->comm_s) {
+    CU(cudaEventRecord(ctx->ev_mu, ctx->stream));
+    CU(cudaStreamWaitEvent(ctx->comm_s, ctx->ev_mu, 0));
+    if (int r = fill_ghost_dims(ctx, md, PF_M, true, 0, 3, ctx->comm_s)) return r;
+    CU(cudaEventRecord(ctx->ev_mux, ctx->comm_s));
+    ctx->mux_pending = true;
+  } else {
+    cudaEvent_t e0 = nullptr;
+    prof_begin(ctx, 2, &e0);
+    const int r = fill_ghosts(ctx, md, PF_M, true);
+    prof_end(ctx, 2, e0);
+    if (r) return r;
+  }
+  if (dry) return PF_OK;
+  ctx->cur = 1 - ctx->cur;
+  ctx->step += 1;
+  return PF_OK;
+}
+
+// dry = true: every kernel of the step, writing only the scratch level, no
+// swap (the state is untouched; pf_autotune times step schedules this way)
+static int step_impl(pf_ctx* ctx, bool phi_only, bool dry = false) {
   const Geom& g = ctx->g;
   double* ps = ctx->phi[ctx->cur];
   double* pd = ctx->phi[1 - ctx->cur];
@@ -1057,6 +1117,14 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
   const bool ov = ctx->overlap && ctx->first_ex < 3 && ctx->variant != PF_VARIANT_NAIVE && !phi_only;
   // the specialised phi-sweep writes phi_dst's x ghost columns itself (tuning phi_xghost)
   const bool phi_x_done = g.xwrap && ctx->variant == PF_VARIANT_JIT && ctx->tune.phi_xghost;
+  // z-slab schedule (tuning sched = 1, S§7 step 6 (ii)): per slab of mu
+  // z-chunks, the phi-sweep of the slab's planes (shifted up by one plane, so
+  // that the slab's top neighbour plane is ready), their x/y ghosts, then the
+  // mu-sweep of the slab, which re-reads phi_src / phi_dst while the slab is
+  // still in L2.  Same kernels and arithmetic per cell as the two sweeps.
+  if (ctx->variant == PF_VARIANT_JIT && ctx->tune.sched == 1 && ctx->first_ex == 3 && !phi_only && !phi_x_done &&
+      ctx->cfg.bc_lo[2] != PF_BC_PERIODIC)
+    return step_slabs(ctx, ps, pd, ms, md, dry);
   // Algorithm 1, line 1: phi-sweep (reads no mu ghosts: may overlap the previous mu exchange)
   prof_begin(ctx, 0, &e0);
   if (ctx->variant == PF_VARIANT_NAIVE)
@@ -1143,6 +1211,7 @@ static int step_impl(pf_ctx* ctx, bool phi_only) {
     ctx->mux_pending = true;
   }
   // line 5: swap
+  if (dry) return PF_OK;
   ctx->cur = 1 - ctx->cur;
   ctx->step += 1;
   return PF_OK;
@@ -1574,6 +1643,31 @@ static int time_sweep(pf_ctx* ctx, JitKernel* k, int which, int reps, double* ou
   return PF_OK;
 }
 
+// median time of one dry step (all kernels of a step on the scratch level)
+static int time_steps(pf_ctx* ctx, int reps, double* out) {
+  for (int i = 0; i < 2; ++i)
+    if (int r = step_impl(ctx, false, true)) return r;
+  std::vector<cudaEvent_t> ev(reps + 1);
+  for (auto& e : ev) CU(cudaEventCreate(&e));
+  CU(cudaEventRecord(ev[0], ctx->stream));
+  for (int i = 0; i < reps; ++i) {
+    if (int r = step_impl(ctx, false, true)) return r;
+    if (int r = join_comm(ctx)) return r;
+    CU(cudaEventRecord(ev[i + 1], ctx->stream));
+  }
+  CU(cudaEventSynchronize(ev[reps]));
+  std::vector<double> t(reps);
+  for (int i = 0; i < reps; ++i) {
+    float v = 0;
+    cudaEventElapsedTime(&v, ev[i], ev[i + 1]);
+    t[i] = v;
+  }
+  for (auto e : ev) cudaEventDestroy(e);
+  std::sort(t.begin(), t.end());
+  *out = t[reps / 2];
+  return PF_OK;
+}
+
 // times of candidate kernels (inf where the build failed), max over ranks
 static int time_candidates(pf_ctx* ctx, const std::vector<pf_tuning>& cands, int which, int reps,
                            std::vector<double>* ms, std::vector<std::string>* why) {
@@ -1696,6 +1790,52 @@ int pf_autotune(pf_ctx* ctx, unsigned mask, int passes, int reps, char* log, int
     ctx->jphi = jit_get(ctx, ctx->dp, ctx->g, best, JIT_PHI, &err);
     if (ctx->jphi) ctx->jmu = jit_get(ctx, ctx->dp, ctx->g, best, JIT_MU, &err);
     if (!ctx->jphi || !ctx->jmu) return fail(ctx, PF_ECUDA, "autotune: %s", err.c_str());
+  }
+  // step schedule (S§8(f) NEXT-2 "full vs split vs fused schedules"): two
+  // sweeps vs the z-slab pipeline, timed as whole dry steps (every kernel of
+  // a step, scratch level only, no swap)
+  const bool slab_ok = (mask & PF_PHI) && (mask & PF_MU) && ctx->first_ex == 3 &&
+                       ctx->cfg.bc_lo[2] != PF_BC_PERIODIC && !(ctx->g.xwrap && ctx->tune.phi_xghost);
+  if (slab_ok) {
+    std::vector<pf_tuning> cands;
+    for (int sc : {0, 1})
+      for (int sl : {1, 2, 4}) {
+        if (sc == 0 && sl != 1) continue;
+        pf_tuning c = best;
+        c.sched = sc;
+        c.slab = sc ? sl : best.slab;
+        if (!tuning_check(c)) cands.push_back(c);
+      }
+    std::vector<double> tm(cands.size(), INFINITY);
+    for (size_t i = 0; i < cands.size(); ++i) {
+      ctx->tune = cands[i];
+      double v = INFINITY;
+      if (int r = time_steps(ctx, reps, &v)) return r;
+      tm[i] = v;
+    }
+    if (ctx->collective()) {
+      double* d = (double*)ctx->red;
+      const int n = (int)cands.size();
+      CU(cudaMemcpyAsync(d, tm.data(), n * sizeof(double), cudaMemcpyHostToDevice, ctx->stream));
+      if (int r = allreduce_max(ctx, d, n)) return r;
+      CU(cudaMemcpyAsync(tm.data(), d, n * sizeof(double), cudaMemcpyDeviceToHost, ctx->stream));
+      CU(cudaStreamSynchronize(ctx->stream));
+    }
+    size_t bi = 0;
+    for (size_t i = 0; i < cands.size(); ++i) {
+      if (tm[i] < tm[bi] * 0.99) bi = i;
+      char b[256];
+      snprintf(b, sizeof b, "%s{\"kernel\": \"step\", \"pass\": 0, \"knob\": \"sched/slab\", \"value\": %d, \"ms\": %s, \"error\": \"\"}",
+               cl.empty() ? "" : ",\n  ", cands[i].sched ? cands[i].slab : 0,
+               std::isfinite(tm[i]) ? std::to_string(tm[i]).c_str() : "null");
+      cl += b;
+    }
+    best = cands[bi];
+    ctx->tune = best;
+    char b[256];
+    snprintf(b, sizeof b, ", \"step\": {\"two_sweeps_ms\": %.6f, \"best_ms\": %.6f, \"sched\": %d, \"slab\": %d}", tm[0],
+             tm[bi], best.sched, best.slab);
+    kj += b;
   }
   // the scratch level's ghosts were overwritten: nothing reads them before the next sweep writes it
   CU(cudaStreamSynchronize(ctx->stream));

@@ -78,8 +78,9 @@ void jit_release(const void* owner);  // unload every module of `owner` (pf_dest
 void jit_precompile(const DevParams& P, const Geom& g, const std::vector<pf_tuning>& ts, int which, int nthreads);
 // sv == nullptr: per-step values from P (by value); else a CUDA-graph step:
 // they are copied from device memory sv into the module's constant first
+// [zlo, zhi): a z-slab of planes (the slab schedule); zhi < 0 = all planes
 cudaError_t jit_launch_phi(JitKernel* m, const DevParams& P, const double* ps, const double* ms, double* pd,
-                           cudaStream_t s, const StepVals* sv = nullptr);
+                           cudaStream_t s, const StepVals* sv = nullptr, int zlo = 0, int zhi = -1);
 cudaError_t jit_launch_mu(JitKernel* m, const DevParams& P, const TileSel* ts, dim3 grid, const double* ps,
                           const double* pd, const double* ms, double* md, cudaStream_t s,
                           const StepVals* sv = nullptr);

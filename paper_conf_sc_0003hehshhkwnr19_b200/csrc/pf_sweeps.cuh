@@ -123,7 +123,9 @@ constexpr int PHI_TXC = PF_PHI_XSH ? TX - 1 : TX;
 template <class PT, class GT, int L, bool TA, int PTY = TY, class RT = DevParams>
 __device__ __forceinline__ void phi_tuned_body(const PT& P, const RT& R, const GT& g,
                                                const double* __restrict__ ps, const double* __restrict__ ms,
-                                               double* __restrict__ pd) {
+                                               double* __restrict__ pd, int zlo = 0, int zhi = 1 << 30) {
+  // [zlo, zhi): planes of this launch (the z-slab schedule, tuning sched = 1;
+  // the six-face one-row sweep only); the grid's z-chunks start at zlo
 #if PF_PHI_FACES6
   // one tile (bx, by) over planes [z0, z1)
   auto tile = [&](const int bx, const int by, const int z0, const int z1) {
@@ -246,7 +248,7 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const RT& R, const G
     }
   }
 #else
-  tile(blockIdx.x, blockIdx.y, blockIdx.z * ZC_PHI, min(blockIdx.z * ZC_PHI + ZC_PHI, g.nz));
+  tile(blockIdx.x, blockIdx.y, zlo + blockIdx.z * ZC_PHI, min(zlo + (int)blockIdx.z * ZC_PHI + ZC_PHI, min(zhi, g.nz)));
 #endif
   return;
 #endif
@@ -369,7 +371,7 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const RT& R, const G
 template <class PT, class GT, int L, bool TA, int PTY, class RT = DevParams>
 __device__ __forceinline__ void phi_r2_body(const PT& P, const RT& R, const GT& g,
                                             const double* __restrict__ ps, const double* __restrict__ ms,
-                                            double* __restrict__ pd) {
+                                            double* __restrict__ pd, int = 0, int = 0) {  // (full launches only)
   static_assert(PTY % 2 == 0, "phi_rpt = 2 needs an even tile height");
   const int x = blockIdx.x * TX + threadIdx.x, y = blockIdx.y * PTY + 2 * threadIdx.y;
   if (x >= g.nx || y >= g.ny) return;

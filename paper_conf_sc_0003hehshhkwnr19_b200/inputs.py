@@ -140,6 +140,96 @@ def params_stress(seed: int = 20191117, **over) -> dict:
     return P
 
 
+def rot(axis: str, deg: float) -> np.ndarray:
+    """Rotation matrix about a coordinate axis (data for the P2 grain orientations)."""
+    c, s = np.cos(np.radians(deg)), np.sin(np.radians(deg))
+    i, j = {"x": (1, 2), "y": (2, 0), "z": (0, 1)}[axis]
+    R = np.eye(3)
+    R[i, i], R[i, j], R[j, i], R[j, j] = c, -s, s, c
+    return R
+
+
+def params_p2(**over) -> dict:
+    """P2 parameterisation: 3 phases (two
+    solid grains of one phase with different orientations + liquid), 2
+    components (one chemical potential), anisotropic gradient energy
+    (reading B6: cubic A_ab(R_ab q) with strength delta on the solid-liquid
+    pairs, the grains rotated against each other, as in Fig. 4 right:
+    dendrites of different orientations).  Synthetic, nondimensional."""
+    N, M, L = 3, 1, 2
+    gamma = np.ones((N, N)) - np.eye(N)
+    gamma3 = np.zeros((N, N, N))
+    for a, b, d in ((0, 1, 2), (0, 2, 1), (1, 0, 2), (1, 2, 0), (2, 0, 1), (2, 1, 0)):
+        gamma3[a, b, d] = 10.0
+    tau = np.full((N, N), 2.0)
+    tau[L, :] = tau[:, L] = 1.0
+    np.fill_diagonal(tau, 0.0)
+    chi = np.array([[[0.5]], [[0.5]], [[1.0]]])
+    A0 = -0.5 * chi
+    c0 = np.array([0.02, 0.02, 0.17])  # Al-rich solid, Cu-enriched liquid (binary Al-Cu-like)
+    b = 0.1
+    B0 = -c0[:, None].copy()
+    B1 = np.zeros((N, M))
+    B0[L, 0] = -c0[L] + b * T_E
+    B1[L, 0] = -b
+    s = np.array([1.0, 1.0, 0.0])
+    D = np.array([[[0.01]], [[0.01]], [[1.0]]])
+    delta = np.zeros((N, N))
+    delta[0, L] = delta[L, 0] = delta[1, L] = delta[L, 1] = 0.05
+    R = np.zeros((N, N, 3, 3))
+    Rg = [np.eye(3), rot("y", 30.0) @ rot("z", 20.0)]
+    for a in range(N):
+        for bb in range(N):
+            R[a, bb] = np.eye(3)
+    for g in (0, 1):
+        R[g, L] = R[L, g] = Rg[g]
+    P = dict(N=N, M=M, liquid=L, dx=1.0, dt=0.03, eps=3.0, gamma=gamma, gamma3=gamma3, tau=tau,
+             A0=A0, A1=np.zeros((N, M, M)), B0=B0, B1=B1, C0=-s * T_E, C1=s.copy(), D=D,
+             T0=0.99, G=0.0, v=0.0, mu_inf=np.zeros(M), window_frac=0.5, window_check=0,
+             antitrapping=1, projection=1, aniso=1, aniso_delta=delta, aniso_R=R)
+    P.update(over)
+    return P
+
+
+def params_p2_stress(seed: int = 20191118, **over) -> dict:
+    """P2 stress set (parity only): every pair anisotropic with its own
+    strength and a seeded random rotation, unequal gamma / tau, A1 != 0,
+    G v != 0, mu_inf != 0."""
+    rng = np.random.default_rng(seed)
+    P = params_p2()
+    N = 3
+
+    def pert(x, rel=0.2):
+        return x * (1.0 + rel * rng.uniform(-1.0, 1.0, size=np.shape(x)))
+
+    g = pert(P["gamma"])
+    P["gamma"] = np.triu(g, 1) + np.triu(g, 1).T
+    t = pert(P["tau"])
+    P["tau"] = np.triu(t, 1) + np.triu(t, 1).T
+    d = rng.uniform(0.02, 0.08, size=(N, N))
+    P["aniso_delta"] = np.triu(d, 1) + np.triu(d, 1).T
+    R = np.zeros((N, N, 3, 3))
+    for a in range(N):
+        for b in range(a, N):
+            Q, _ = np.linalg.qr(rng.normal(size=(3, 3)))
+            Q *= np.sign(np.linalg.det(Q))
+            R[a, b] = R[b, a] = Q
+    P["aniso_R"] = R
+    P["A1"] = 0.1 * P["A0"] * rng.uniform(0.2, 1.0, size=(N, 1, 1))
+    P["B0"] = pert(P["B0"])
+    P["B1"] = 0.05 * rng.uniform(-1.0, 1.0, size=(N, 1))
+    P["C0"] = pert(P["C0"]) + 0.01 * rng.uniform(-1, 1, size=N)
+    P["C1"] = pert(P["C1"]) + 0.01 * rng.uniform(-1, 1, size=N)
+    P["D"] = pert(P["D"])
+    P["G"] = 2e-3
+    P["v"] = 5e-3
+    P["T0"] = 0.98
+    P["mu_inf"] = np.array([0.007])
+    P["dt"] = 0.025
+    P.update(over)
+    return P
+
+
 # ---------------------------------------------------------------------------
 # Initial conditions (SURVEY C.5).  Arrays are [component][z][y][x], float64.
 # ---------------------------------------------------------------------------

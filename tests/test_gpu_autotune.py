@@ -206,3 +206,48 @@ def test_mu_sweep_layouts_bitwise(pfmod, omod, monkeypatch, knobs):
         outs.append(gpu_run(pfmod, shape, Ps, phi, mu, 4, t))
     for o2 in outs[1:]:
         assert np.array_equal(outs[0][0], o2[0]) and np.array_equal(outs[0][1], o2[1])
+
+
+# Step schedules (tuning sched / slab; S§7 step 6 (ii), NEXT-2): the z-slab
+# pipeline launches the same kernels on slabs of planes (phi shifted up one
+# plane, x / y ghosts per slab, z ghosts at the ends), so it must give the
+# same bits as the two full sweeps -- DS boundaries (non-periodic z), window
+# shifts, ragged z extents, mu z-chunks that do not divide nz.
+@pytest.mark.parametrize("slab,mu_zc,shape", [(1, 5, (23, 14, 40)), (2, 4, (37, 9, 33)), (4, 6, (30, 16, 64)),
+                                              (16, 22, (21, 8, 32))])
+def test_slab_schedule_bitwise(pfmod, omod, slab, mu_zc, shape):
+    P = I.params_stress(window_check=4, window_frac=0.5)
+    phi, mu = I.ic_lamellar(shape, seed=7, z_front=shape[0] // 2 + 2, mu_inf=tuple(P["mu_inf"]))
+    outs = []
+    for t in ({"sched": 0, "mu_zc": mu_zc}, {"sched": 1, "slab": slab, "mu_zc": mu_zc}):
+        g = pfmod.PhaseField(shape, P, bc=I.BC_DS)
+        g.set_tuning(t)
+        g.init_fields(phi, mu)
+        g.step(9)
+        outs.append((g.download(), g.state()))
+        g.close()
+    (p0, m0), s0 = outs[0]
+    (p1, m1), s1 = outs[1]
+    assert s0 == s1 and s0["z_off"] > 0
+    assert np.array_equal(p0, p1) and np.array_equal(m0, m1)
+    o = omod.Oracle(shape, P, I.BC_DS)
+    o.init(phi, mu)
+    o.step(9)
+    op, om = o.download()
+    assert np.abs(p1 - op).max() / np.abs(op).max() <= 1e-11 and np.abs(m1 - om).max() / np.abs(om).max() <= 1e-11
+
+
+def test_autotune_step_schedule(pfmod):
+    """pf_autotune times the step schedules as dry steps (state untouched) and
+    reports the choice."""
+    shape = (48, 32, 64)
+    P = I.params_c4("ds", window_check=0)
+    phi, mu = I.ic_lamellar(shape, seed=3)
+    g = pfmod.PhaseField(shape, P, bc=I.BC_DS)
+    g.init_fields(phi, mu)
+    before = g.download()
+    rep = g.autotune(passes=1, reps=3)
+    after = g.download()
+    assert np.array_equal(before[0], after[0]) and np.array_equal(before[1], after[1])
+    assert "step" in rep and rep["step"]["sched"] in (0, 1)
+    assert any(c["kernel"] == "step" for c in rep["tried"])

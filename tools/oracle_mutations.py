@@ -75,6 +75,18 @@ MUTANTS = [
     ("} else if (bc == OR_BC_DIRICHLET_MU && is_mu) {", "} else if (bc == OR_BC_DIRICHLET_MU && !is_mu) {",
      ["test_a15_dirichlet_mu_top"]),
     ("int src_neu = side ? n[d] - 1 : 0;", "int src_neu = side ? n[d] - 2 : 1;", ["test_mobility_face_interpolation"]),
+    # reading B6 (P2 anisotropy)
+    ("for (int j = 0; j < 3; ++j) out[j] = R[0][j] * gp[0] + R[1][j] * gp[1] + R[2][j] * gp[2];",
+     "for (int j = 0; j < 3; ++j) out[j] = R[j][0] * gp[0] + R[j][1] * gp[1] + R[j][2] * gp[2];",
+     ["tests/test_oracle_p2.py::test_p2_lattice_rotation_covariance"]),
+    ("gp[i] = 2.0 * A * dA * n2 + 2.0 * A * A * v[i];", "gp[i] = 2.0 * A * A * v[i];",
+     ["tests/test_oracle_p2.py::test_p2_sympy_variational_derivative"]),
+    ("double A = 1.0 - delta * (3.0 - 4.0 * s4 / (n2 * n2));", "double A = 1.0 + delta * (3.0 - 4.0 * s4 / (n2 * n2));",
+     ["tests/test_oracle_p2.py::test_p2_planar_profile_width"]),
+    ("s += p->gamma[a][b] * (-pb[b]) * gf[d];", "s += p->gamma[a][b] * (-pb[a]) * gf[d];",
+     ["tests/test_oracle_p2.py::test_p2_sympy_variational_derivative"]),
+    ("if (e == d) { G[b][e] = dd[b]; continue; }", "if (1) { G[b][e] = e == d ? dd[b] : 0.0; continue; }",
+     ["tests/test_oracle_p2.py::test_p2_sympy_variational_derivative", "tests/test_oracle_p2.py::test_p2_table1_footprint"]),
     # reading A16: window inflow
     ("mu[idx(o, i, x, y, z)] = z + k < nz ? mu[idx(o, i, x, y, z + k)] : o->p.mu_inf[i];",
      "mu[idx(o, i, x, y, z)] = z + k < nz ? mu[idx(o, i, x, y, z + k)] : 0.0;", ["test_window_shift_semantics"]),
@@ -92,7 +104,8 @@ def run_mutant(i: int, full: bool = False, timeout: float = 600.0):
         open(src, "w").write(orig.replace(a, b, 1))
         env = dict(os.environ, PF_ORACLE_SRC=src, PF_ORACLE_LIB=os.path.join(td, "libpf_oracle.so"),
                    OMP_NUM_THREADS="1")
-        sel = [PINS] if (full or catch is None) else [f"{PINS}::{t}" for t in catch]
+        sel = ([PINS, "tests/test_oracle_p2.py"] if (full or catch is None)
+               else [t if "::" in t else f"{PINS}::{t}" for t in catch])
         r = subprocess.run([sys.executable, "-m", "pytest", *sel, "-q", "-x", "-p", "no:cacheprovider"],
                            capture_output=True, text=True, cwd=ROOT, env=env, timeout=timeout)
     fails = [ln.split()[1] for ln in r.stdout.splitlines() if ln.startswith("FAILED")]
