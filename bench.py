@@ -34,6 +34,10 @@ F_PHI = 66 + 124 + 202 + 282 + 9          # phi-split: adds + muls + divs = 683
 F_MU = 256 + 389 + 75 + 90 + 17 + 21 + 18  # mu-split: adds + muls + divs + sqrts + rsqrts = 866
 F_STEP = F_PHI + F_MU                      # 1549
 Q_STEP = 96                                # bytes/cell: read phi, mu; write phi, mu (fp64)
+# P2 (Table 1, P2 split columns): phi 364+368 adds, 792+557 muls, 18+14 divs;
+# mu 142+26 adds, 248+46 muls, 6+9 divs, 3 sqrts, 12 rsqrts
+F_STEP_P2 = (364 + 368 + 792 + 557 + 18 + 14) + (142 + 26 + 248 + 46 + 6 + 9 + 3 + 12)  # 2605
+Q_STEP_P2 = 2 * (3 + 1) * 8                # read + write phi (3) and mu (1)
 # fp64 peak derived from unit counts and clocks: 148 SMs x 64
 # FP64 FMA lanes x 2 flop x 1.965 GHz (clocks.max.sm)
 SMS, FP64_LANES, SM_MAX_GHZ = 148, 64, 1.965
@@ -203,6 +207,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-stress", action="store_true", help="skip the stress-set (general-expression) line")
+    ap.add_argument("--no-p2", action="store_true", help="skip the P2 (NEXT-4) line")
     args = ap.parse_args()
     assert args.warmup >= 3 or args.impl == "reference" or os.environ.get("PF_BENCH_ALLOW_SHORT"), "W >= 3"
 
@@ -460,6 +465,35 @@ def main():
             "frac_of_R": (cells_local * nst / (sms * 1e-3) / 1e6) / R,
             "note": "parameter set S of SURVEY C.4 (general expressions), same block / BCs / IC, default tuning"}
         gs.close()
+    # ---- P2 parameterisation: 3 phases,
+    # 1 mu, anisotropic phi (pf_p2.cu), n^3 periodic block, IC-V
+    if world == 1 and not strong and not args.no_p2:
+        torch.cuda.empty_cache()
+        P2 = I.params_p2()
+        g2 = pf.PhaseField((n, n, n), P2, device=local_rank)
+        ph2, mu2 = I.ic_voronoi((n, n, n), seed=20191117, N=3, M=1)
+        g2.init_fields(ph2, mu2)
+        g2.profile(True)
+        g2.step(3)
+        torch.cuda.synchronize()
+        g2.profile(True)
+        n2 = max(10, min(args.steps, 40))
+        s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s0.record(g2.stream)
+        g2.step(n2)
+        s1.record(g2.stream)
+        s1.synchronize()
+        ms2 = s0.elapsed_time(s1)
+        pr2 = g2.profile_read()
+        val2 = n ** 3 * n2 / (ms2 * 1e-3) / 1e6
+        R2 = min(peak_tf * 1e12 / F_STEP_P2, hbm * 1e9 / Q_STEP_P2) / 1e6
+        rec["p2"] = {"value": val2, "unit": UNIT, "steps": n2, "ms_per_step": ms2 / n2,
+                     "phi_sweep_ms": pr2["phi_sweep"][0] / max(pr2["phi_sweep"][1], 1),
+                     "mu_sweep_ms": pr2["mu_sweep"][0] / max(pr2["mu_sweep"][1], 1),
+                     "R_mlups": R2, "frac_of_R": val2 / R2, "F_flop_per_cell": F_STEP_P2,
+                     "workload": f"P2: {n}^3 periodic block, 3 phases / 1 mu, anisotropic gamma (reading B6), IC-V",
+                     "note": "first B200 version: one thread per cell, every face evaluated by both cells"}
+        g2.close()
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         rec["cpu_baseline"] = cpu_baseline(P, bc, strong=strong)
     if rank == 0:

@@ -133,6 +133,17 @@ typedef struct {
    * xi_amp = 0: off (reading A17).  xi_amp >= 0 and finite.                  */
   double xi_amp;
   uint32_t xi_seed;
+  /* P2 parameterisation (n_phases = 3, n_mu = 1 in pf_config; SURVEY §8(f)
+   * NEXT-4): the leading 3 x 3 / 3 x 1 blocks of the arrays
+   * above are used, and the gradient energy of eq. 4 is anisotropic,
+   * a = sum_{a<b} gamma_ab A_ab(R_ab q_ab)^2 |q_ab|^2 with the cubic
+   * A(p) = 1 - delta_ab (3 - 4 sum_i p_i^4 / |p|^4) of reading B6
+   * (aniso = 1; 0: A = 1).  aniso_delta symmetric, >= 0 and < 1/5 (A > 0);
+   * aniso_R[a][b] orthonormal 3 x 3, row-major, R_ab = R_ba.  The P2 path
+   * has no fluctuation term (xi_amp = 0).  Ignored for P1.               */
+  int aniso;
+  double aniso_delta[PF_N][PF_N];
+  double aniso_R[PF_N][PF_N][3][3];
 } pf_params;
 
 typedef struct {

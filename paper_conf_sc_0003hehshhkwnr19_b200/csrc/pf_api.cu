@@ -13,6 +13,7 @@
 #include <string.h>
 
 #include <algorithm>
+#include <array>
 #include <condition_variable>
 #include <deque>
 #include <map>
@@ -191,6 +192,10 @@ struct pf_ctx {
   std::vector<GraphEntry> graphs;
   ncclComm_t comm = nullptr;
   std::shared_ptr<LocalGroup> lg;  // in-process transport instead of NCCL (world > 1, "PFLOCAL:")
+  // P2 parameterisation (3 phases, 1 mu, anisotropic phi; pf_p2.cu)
+  bool p2 = false;
+  int nph = PF_N, nmu = PF_M;
+  std::vector<unsigned char> p2par;
   bool collective() const { return comm != nullptr || lg != nullptr; }
   // profiling
   bool prof = false;
@@ -392,8 +397,9 @@ int layout_of(const pf_config* cfg, pf_layout* L, int coord[3]) {
     L->field = pxy * (nz + 2 * GUARD);
   }
   const int64_t zspan = L->plane * (nz + 2 * GUARD);
-  L->phi_bytes = (size_t)((PF_N - 1) * L->field + zspan) * sizeof(double) + 256;  // +256: tail slack for vector loads
-  L->mu_bytes = (size_t)((PF_M - 1) * L->field + zspan) * sizeof(double) + 256;
+  const int nph = cfg->n_phases == 3 ? 3 : PF_N, nmu = cfg->n_phases == 3 ? 1 : PF_M;  // P2: 3 phases, 1 mu
+  L->phi_bytes = (size_t)((nph - 1) * L->field + zspan) * sizeof(double) + 256;  // +256: tail slack for vector loads
+  L->mu_bytes = (size_t)((nmu - 1) * L->field + zspan) * sizeof(double) + 256;
   size_t ws = 256 + 1024;  // reduction scratch, per-step values of CUDA-graph steps
   Geom g{nx, ny, nz, L->offset[2], L->pitch, L->plane, L->field, L->x_off, L->offset[0], L->offset[1]};
   for (int d = 0; d < 3; ++d) ws += 4 * align256(halo_slab_elems(g, d) * PF_N * sizeof(double));
@@ -589,10 +595,16 @@ int pf_query_neighbors(const pf_config* cfg, int nb_lo[3], int nb_hi[3]) {
 int pf_create(const pf_config* cfg, pf_ctx** out) {
   if (!cfg || !out) return PF_EINVAL;
   *out = nullptr;
-  if (cfg->n_phases != PF_N || cfg->n_mu != PF_M || cfg->liquid < 0 || cfg->liquid >= PF_N) return PF_EINVAL;
+  // P1 (4 phases, 2 mu) or P2 (3 phases, 1 mu)
+  const bool is_p2 = cfg->n_phases == 3 && cfg->n_mu == 1;
+  if (!((cfg->n_phases == PF_N && cfg->n_mu == PF_M) || is_p2) || cfg->liquid < 0 || cfg->liquid >= cfg->n_phases)
+    return PF_EINVAL;
   pf_ctx* ctx = new (std::nothrow) pf_ctx();
   if (!ctx) return PF_ENOMEM;
   ctx->cfg = *cfg;
+  ctx->p2 = is_p2;
+  ctx->nph = is_p2 ? 3 : PF_N;
+  ctx->nmu = is_p2 ? 1 : PF_M;
   tuning_default(&ctx->tune);
   if (layout_of(cfg, &ctx->lay, ctx->coord) != PF_OK) {
     delete ctx;
@@ -779,8 +791,99 @@ int pf_destroy(pf_ctx* ctx) {
 }
 
 // ---------------------------------------------------------------------------
+// P2 parameters (3 phases, 1 mu, anisotropic phi): validation, explicit
+// stability bound, parameter block of pf_p2.cu
+static int set_params_p2(pf_ctx* ctx, const pf_params* p) {
+  const int L = ctx->cfg.liquid;
+  auto finite = [](double v) { return isfinite(v); };
+  const double* raw = (const double*)p;
+  for (size_t i = 0; i < offsetof(pf_params, window_check) / sizeof(double); ++i)
+    if (!finite(raw[i])) return fail(ctx, PF_EINVAL, "non-finite parameter at offset %zu", i);
+  if (!(p->dx > 0 && p->dt > 0 && p->eps > 0)) return fail(ctx, PF_EINVAL, "dx, dt, eps must be > 0");
+  if (p->xi_amp != 0.0) return fail(ctx, PF_EINVAL, "the P2 path has no fluctuation term (xi_amp = 0)");
+  double gmax = 0, tmin = INFINITY, dmax = 0;
+  for (int a = 0; a < 3; ++a)
+    for (int b = 0; b < 3; ++b) {
+      if (p->gamma[a][b] != p->gamma[b][a] || p->tau[a][b] != p->tau[b][a])
+        return fail(ctx, PF_EINVAL, "gamma and tau must be symmetric");
+      if (a == b) continue;
+      if (!(p->gamma[a][b] > 0 && p->tau[a][b] > 0)) return fail(ctx, PF_EINVAL, "gamma_ab, tau_ab must be > 0");
+      gmax = std::max(gmax, p->gamma[a][b]);
+      tmin = std::min(tmin, p->tau[a][b]);
+      if (p->aniso) {
+        const double d = p->aniso_delta[a][b];
+        if (!(d >= 0.0 && d < 0.2 && finite(d)) || d != p->aniso_delta[b][a])
+          return fail(ctx, PF_EINVAL, "aniso_delta symmetric, 0 <= delta < 1/5");
+        dmax = std::max(dmax, d);
+        for (int i = 0; i < 3; ++i)
+          for (int j = 0; j < 3; ++j) {
+            double s = 0.0;
+            for (int k = 0; k < 3; ++k) s += p->aniso_R[a][b][i][k] * p->aniso_R[a][b][j][k];
+            if (!(fabs(s - (i == j ? 1.0 : 0.0)) < 1e-12) || p->aniso_R[a][b][i][j] != p->aniso_R[b][a][i][j])
+              return fail(ctx, PF_EINVAL, "aniso_R[%d][%d] must be orthonormal and R_ab = R_ba", a, b);
+          }
+      }
+    }
+  double dmx = 0.0;
+  const double Tlo = p->T0 - fabs(p->G) * (ctx->cfg.global[2] + 2) * p->dx, Thi = p->T0 + fabs(p->G) * (ctx->cfg.global[2] + 2) * p->dx;
+  for (int a = 0; a < 3; ++a)
+    for (double T : {Tlo, Thi}) {
+      const double chi = -2.0 * (p->A0[a][0][0] + p->A1[a][0][0] * T);
+      if (!(chi > 0)) return fail(ctx, PF_EINVAL, "A_%d(T=%g) must be < 0 (dc/dmu > 0)", a, T);
+      dmx = std::max(dmx, p->D[a][0][0]);
+      if (!(p->D[a][0][0] >= 0)) return fail(ctx, PF_EINVAL, "D_%d must be >= 0", a);
+    }
+  // phi: the gradient coefficient grows by up to (1 + delta)^2 and the
+  // derivative terms of A; mu (M = 1): D_eff = sum_a g_a D_a chi_a / sum_a
+  // h_a chi_a, sampled over the simplex (vertices, edge midpoints,
+  // barycentre, 1000 seeded points) at the extreme temperatures
+  const double dt_phi = tmin * p->dx * p->dx / (12.0 * gmax * (1.0 + dmax) * (1.0 + dmax) * (1.0 + 8.0 * dmax));
+  std::vector<std::array<double, 3>> pts = {{1, 0, 0}, {0, 1, 0}, {0, 0, 1}, {0.5, 0.5, 0}, {0.5, 0, 0.5},
+                                            {0, 0.5, 0.5}, {1.0 / 3, 1.0 / 3, 1.0 / 3}};
+  uint64_t sd = 20191117ull;
+  for (int i = 0; i < 1000; ++i) {
+    std::array<double, 3> v;
+    double sum = 0;
+    for (int a = 0; a < 3; ++a) {
+      sd = sd * 6364136223846793005ull + 1442695040888963407ull;
+      v[a] = -log(((sd >> 11) + 0.5) * (1.0 / 9007199254740992.0));
+      sum += v[a];
+    }
+    for (int a = 0; a < 3; ++a) v[a] /= sum;
+    pts.push_back(v);
+  }
+  double deff = 0.0;
+  for (const auto& v : pts)
+    for (double T : {Tlo, Thi}) {
+      double num = 0.0, den = 0.0;
+      for (int a = 0; a < 3; ++a) {
+        const double chi = -2.0 * (p->A0[a][0][0] + p->A1[a][0][0] * T);
+        num += v[a] * p->D[a][0][0] * chi;
+        den += v[a] * v[a] * (3.0 - 2.0 * v[a]) * chi;
+      }
+      deff = std::max(deff, num / den);
+    }
+  (void)dmx;
+  const double dt_mu = deff > 0 ? p->dx * p->dx / (6.0 * deff) : INFINITY;
+  if (p->dt > dt_phi || p->dt > dt_mu)
+    return fail(ctx, PF_EINVAL, "dt = %g exceeds the explicit stability bound min(%g [phi], %g [mu])", p->dt, dt_phi,
+                dt_mu);
+  if (p->window_check < 0 || (p->window_check > 0 && !(p->window_frac > 0 && p->window_frac < 1)))
+    return fail(ctx, PF_EINVAL, "window_check >= 0 and 0 < window_frac < 1");
+  if (p->window_check > 0 && ctx->cfg.procs[2] != 1)
+    return fail(ctx, PF_EINVAL, "the moving window needs the growth axis unsplit (procs[2] == 1)");
+  ctx->p2par.assign(p2_params_size(), 0);
+  p2_fill_params(*p, L, ctx->p2par.data());
+  ctx->hp = *p;
+  ctx->have_params = true;
+  ctx->jphi = ctx->jmu = nullptr;
+  drop_graphs(ctx);
+  return PF_OK;
+}
+
 int pf_set_params(pf_ctx* ctx, const pf_params* p) {
   if (!ctx || !p) return PF_EINVAL;
+  if (ctx->p2) return set_params_p2(ctx, p);
   const int L = ctx->cfg.liquid;
   auto finite = [](double v) { return isfinite(v); };
   const double* raw = (const double*)p;
@@ -1056,10 +1159,10 @@ static int step_slabs(pf_ctx* ctx, const double* ps, double* pd, const double* m
     prof_begin(ctx, 2, &e0);
     Geom gs = g;
     gs.nz = phi_hi - plo;
-    launch_ghost_fill(gs, bxy, pd + (size_t)plo * (size_t)g.plane, PF_N, nullptr, ctx->stream);
+    launch_ghost_fill(gs, bxy, pd + (size_t)plo * (size_t)g.plane, ctx->nph, nullptr, ctx->stream);
     ctx->nlaunch[2] += 1;
     if (s == 0 || s == S - 1) {  // z ghost planes (whole extended planes: after their x / y ghosts)
-      launch_ghost_stage(g, 2, s == 0 ? ctx->cfg.bc_lo[2] : -1, s == S - 1 ? ctx->cfg.bc_hi[2] : -1, pd, PF_N,
+      launch_ghost_stage(g, 2, s == 0 ? ctx->cfg.bc_lo[2] : -1, s == S - 1 ? ctx->cfg.bc_hi[2] : -1, pd, ctx->nph,
                          nullptr, ctx->stream);
       ctx->nlaunch[2] += 1;
     }
@@ -1077,13 +1180,13 @@ static int step_slabs(pf_ctx* ctx, const double* ps, double* pd, const double* m
   if (ctx->overlap && ctx->comm_s) {
     CU(cudaEventRecord(ctx->ev_mu, ctx->stream));
     CU(cudaStreamWaitEvent(ctx->comm_s, ctx->ev_mu, 0));
-    if (int r = fill_ghost_dims(ctx, md, PF_M, true, 0, 3, ctx->comm_s)) return r;
+    if (int r = fill_ghost_dims(ctx, md, ctx->nmu, true, 0, 3, ctx->comm_s)) return r;
     CU(cudaEventRecord(ctx->ev_mux, ctx->comm_s));
     ctx->mux_pending = true;
   } else {
     cudaEvent_t e0 = nullptr;
     prof_begin(ctx, 2, &e0);
-    const int r = fill_ghosts(ctx, md, PF_M, true);
+    const int r = fill_ghosts(ctx, md, ctx->nmu, true);
     prof_end(ctx, 2, e0);
     if (r) return r;
   }
@@ -1104,6 +1207,37 @@ static int step_impl(pf_ctx* ctx, bool phi_only, bool dry = false) {
   // frozen temperature of this step: T(k) = T0 + G ((k + z0 + z_off) dx - v t_n), t_n = step dt  [A13]
   const double t = (double)ctx->step * ctx->hp.dt;
   ctx->dp.Tbase = ctx->hp.T0 + ctx->hp.G * (((double)g.z0 + (double)ctx->z_off) * ctx->hp.dx - ctx->hp.v * t);
+  if (ctx->p2) {
+    // P2 (pf_p2.cu): phi-sweep, phi ghosts, mu-sweep, mu ghosts, swap (Algorithm 1)
+    if (int r = join_comm(ctx)) return r;
+    cudaEvent_t e0 = nullptr;
+    prof_begin(ctx, 0, &e0);
+    p2_launch_phi(ctx->p2par.data(), ctx->dp.Tbase, g, ps, ms, pd, ctx->stream);
+    ctx->nlaunch[0] += 1;
+    prof_end(ctx, 0, e0);
+    if (int r = check_launch(ctx, "p2 phi_sweep")) return r;
+    prof_begin(ctx, 2, &e0);
+    int r = fill_ghosts(ctx, pd, ctx->nph, false);
+    prof_end(ctx, 2, e0);
+    if (r) return r;
+    if (phi_only) {
+      CU(cudaMemcpyAsync(md, ms, ctx->lay.mu_bytes - 256, cudaMemcpyDeviceToDevice, ctx->stream));
+    } else {
+      prof_begin(ctx, 1, &e0);
+      p2_launch_mu(ctx->p2par.data(), ctx->dp.Tbase, g, ps, pd, ms, md, ctx->stream);
+      ctx->nlaunch[1] += 1;
+      prof_end(ctx, 1, e0);
+      if (int r2 = check_launch(ctx, "p2 mu_sweep")) return r2;
+      prof_begin(ctx, 2, &e0);
+      r = fill_ghosts(ctx, md, ctx->nmu, true);
+      prof_end(ctx, 2, e0);
+      if (r) return r;
+    }
+    if (dry) return PF_OK;
+    ctx->cur = 1 - ctx->cur;
+    ctx->step += 1;
+    return PF_OK;
+  }
   ctx->dp.step = (unsigned long long)ctx->step;  // fluctuation counter [B4]
   cudaEvent_t e0 = nullptr;
   if (ctx->variant == PF_VARIANT_JIT && (!ctx->jphi || !ctx->jmu)) {
@@ -1140,7 +1274,7 @@ static int step_impl(pf_ctx* ctx, bool phi_only, bool dry = false) {
     if (int r = join_comm(ctx)) return r;
     // line 2: phi_dst communication and boundary handling
     prof_begin(ctx, 2, &e0);
-    int r = fill_ghosts(ctx, pd, PF_N, false, phi_x_done);
+    int r = fill_ghosts(ctx, pd, ctx->nph, false, phi_x_done);
     prof_end(ctx, 2, e0);
     if (r) return r;
     if (phi_only) {
@@ -1156,12 +1290,12 @@ static int step_impl(pf_ctx* ctx, bool phi_only, bool dry = false) {
       if (ctx->overlap && ctx->comm_s) {
         CU(cudaEventRecord(ctx->ev_mu, ctx->stream));
         CU(cudaStreamWaitEvent(ctx->comm_s, ctx->ev_mu, 0));
-        if (int r2 = fill_ghost_dims(ctx, md, PF_M, true, 0, 3, ctx->comm_s)) return r2;
+        if (int r2 = fill_ghost_dims(ctx, md, ctx->nmu, true, 0, 3, ctx->comm_s)) return r2;
         CU(cudaEventRecord(ctx->ev_mux, ctx->comm_s));
         ctx->mux_pending = true;
       } else {
         prof_begin(ctx, 2, &e0);
-        r = fill_ghosts(ctx, md, PF_M, true);
+        r = fill_ghosts(ctx, md, ctx->nmu, true);
         prof_end(ctx, 2, e0);
         if (r) return r;
       }
@@ -1170,10 +1304,10 @@ static int step_impl(pf_ctx* ctx, bool phi_only, bool dry = false) {
     // line 2: local dimensions before the first exchanged one on the compute
     // stream, the rest (exchanges in x -> y -> z order) on the comm stream
     const int fe = ctx->first_ex;
-    if (int r = fill_ghost_dims(ctx, pd, PF_N, false, 0, fe, ctx->stream, phi_x_done)) return r;
+    if (int r = fill_ghost_dims(ctx, pd, ctx->nph, false, 0, fe, ctx->stream, phi_x_done)) return r;
     CU(cudaEventRecord(ctx->ev_phi, ctx->stream));
     CU(cudaStreamWaitEvent(ctx->comm_s, ctx->ev_phi, 0));
-    if (int r = fill_ghost_dims(ctx, pd, PF_N, false, fe, 3, ctx->comm_s)) return r;
+    if (int r = fill_ghost_dims(ctx, pd, ctx->nph, false, fe, 3, ctx->comm_s)) return r;
     CU(cudaEventRecord(ctx->ev_phix, ctx->comm_s));
     // the mu-sweep reads mu ghosts: the previous mu exchange must be done
     if (int r = join_comm(ctx)) return r;
@@ -1203,10 +1337,10 @@ static int step_impl(pf_ctx* ctx, bool phi_only, bool dry = false) {
     if (int r = launch_mu(ctx, &sh, full, ps, pd, ms, md)) return r;
     prof_end(ctx, 1, e0);
     // line 4: mu ghosts; the exchange overlaps the next phi-sweep
-    if (int r = fill_ghost_dims(ctx, md, PF_M, true, 0, fe, ctx->stream)) return r;
+    if (int r = fill_ghost_dims(ctx, md, ctx->nmu, true, 0, fe, ctx->stream)) return r;
     CU(cudaEventRecord(ctx->ev_mu, ctx->stream));
     CU(cudaStreamWaitEvent(ctx->comm_s, ctx->ev_mu, 0));
-    if (int r = fill_ghost_dims(ctx, md, PF_M, true, fe, 3, ctx->comm_s)) return r;
+    if (int r = fill_ghost_dims(ctx, md, ctx->nmu, true, fe, 3, ctx->comm_s)) return r;
     CU(cudaEventRecord(ctx->ev_mux, ctx->comm_s));
     ctx->mux_pending = true;
   }
@@ -1317,7 +1451,7 @@ int pf_step(pf_ctx* ctx, int64_t nsteps) {
   // graphs (their per-kernel events are then event nodes collected after each
   // replay; measured 0.8 % slower per step at 256^3 than direct profiled steps).
   const bool forced = ctx->graph_min_cells == 0;
-  const bool graphs = ctx->use_graph && ctx->variant == PF_VARIANT_JIT && (!ctx->prof || forced) &&
+  const bool graphs = ctx->use_graph && !ctx->p2 && ctx->variant == PF_VARIANT_JIT && (!ctx->prof || forced) &&
                       (int64_t)ctx->g.nx * ctx->g.ny * ctx->g.nz >= ctx->graph_min_cells;
   // graph runs have one length: the window-check interval (the host decides
   // shifts between runs), else 8 steps; shorter remainders launch directly, so
@@ -1356,9 +1490,9 @@ int pf_halo_exchange(pf_ctx* ctx, unsigned mask) {
   if (!ctx->have_params) return fail(ctx, PF_ESTATE, "pf_halo_exchange before pf_set_params");
   if (int r = join_comm(ctx)) return r;
   if (mask & PF_PHI)
-    if (int r = fill_ghosts(ctx, ctx->phi[ctx->cur], PF_N, false)) return r;
+    if (int r = fill_ghosts(ctx, ctx->phi[ctx->cur], ctx->nph, false)) return r;
   if (mask & PF_MU)
-    if (int r = fill_ghosts(ctx, ctx->mu[ctx->cur], PF_M, true)) return r;
+    if (int r = fill_ghosts(ctx, ctx->mu[ctx->cur], ctx->nmu, true)) return r;
   return PF_OK;
 }
 
@@ -1371,10 +1505,10 @@ int pf_init_fields(pf_ctx* ctx, const double* phi, const double* mu, int where) 
   const cudaMemcpyKind kind = where == PF_HOST ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
   ctx->cur = 0;
   // stage the packed arrays in the (scratch) second time level, then scatter
-  CU(cudaMemcpyAsync(ctx->phi[1], phi, cells * PF_N * sizeof(double), kind, ctx->stream));
-  CU(cudaMemcpyAsync(ctx->mu[1], mu, cells * PF_M * sizeof(double), kind, ctx->stream));
-  launch_copy_interior(g, PF_N, ctx->phi[1], ctx->phi[0], 0, ctx->stream);
-  launch_copy_interior(g, PF_M, ctx->mu[1], ctx->mu[0], 0, ctx->stream);
+  CU(cudaMemcpyAsync(ctx->phi[1], phi, cells * ctx->nph * sizeof(double), kind, ctx->stream));
+  CU(cudaMemcpyAsync(ctx->mu[1], mu, cells * ctx->nmu * sizeof(double), kind, ctx->stream));
+  launch_copy_interior(g, ctx->nph, ctx->phi[1], ctx->phi[0], 0, ctx->stream);
+  launch_copy_interior(g, ctx->nmu, ctx->mu[1], ctx->mu[0], 0, ctx->stream);
   if (int r = check_launch(ctx, "init copy")) return r;
   ctx->step = 0;
   ctx->z_off = 0;
@@ -1399,14 +1533,14 @@ int pf_download(pf_ctx* ctx, double* phi, double* mu, int where) {
   const cudaMemcpyKind kind = where == PF_HOST ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice;
   // pack into the scratch time level, then copy out
   if (phi) {
-    launch_copy_interior(g, PF_N, ctx->phi[ctx->cur], ctx->phi[1 - ctx->cur], 1, ctx->stream);
+    launch_copy_interior(g, ctx->nph, ctx->phi[ctx->cur], ctx->phi[1 - ctx->cur], 1, ctx->stream);
     if (int r = check_launch(ctx, "download copy")) return r;
-    CU(cudaMemcpyAsync(phi, ctx->phi[1 - ctx->cur], cells * PF_N * sizeof(double), kind, ctx->stream));
+    CU(cudaMemcpyAsync(phi, ctx->phi[1 - ctx->cur], cells * ctx->nph * sizeof(double), kind, ctx->stream));
   }
   if (mu) {
-    launch_copy_interior(g, PF_M, ctx->mu[ctx->cur], ctx->mu[1 - ctx->cur], 1, ctx->stream);
+    launch_copy_interior(g, ctx->nmu, ctx->mu[ctx->cur], ctx->mu[1 - ctx->cur], 1, ctx->stream);
     if (int r = check_launch(ctx, "download copy")) return r;
-    CU(cudaMemcpyAsync(mu, ctx->mu[1 - ctx->cur], cells * PF_M * sizeof(double), kind, ctx->stream));
+    CU(cudaMemcpyAsync(mu, ctx->mu[1 - ctx->cur], cells * ctx->nmu * sizeof(double), kind, ctx->stream));
   }
   CU(cudaStreamSynchronize(ctx->stream));
   return PF_OK;
@@ -1483,7 +1617,7 @@ int pf_monitor(pf_ctx* ctx, double out[2]) {
   if (!ctx || !out) return PF_EINVAL;
   if (!ctx->have_fields) return fail(ctx, PF_ESTATE, "no fields");
   CU(cudaMemsetAsync(ctx->red, 0, 16, ctx->stream));
-  launch_monitor(ctx->g, ctx->phi[ctx->cur], ctx->mu[ctx->cur], ctx->red, ctx->stream);
+  launch_monitor(ctx->g, ctx->nph, ctx->nmu, ctx->phi[ctx->cur], ctx->mu[ctx->cur], ctx->red, ctx->stream);
   if (int r = check_launch(ctx, "monitor")) return r;
   if (int r = allreduce_max_u64(ctx, ctx->red, 2)) return r;
   CU(cudaMemcpyAsync(ctx->pinned, ctx->red, 16, cudaMemcpyDeviceToHost, ctx->stream));
@@ -1512,7 +1646,7 @@ int pf_shift_window(pf_ctx* ctx, int k) {
   if (int r = join_comm(ctx)) return r;
   cudaEvent_t e0 = nullptr;
   prof_begin(ctx, 3, &e0);
-  launch_shift(ctx->g, k, ctx->cfg.liquid, ctx->hp.mu_inf, ctx->phi[ctx->cur], ctx->mu[ctx->cur],
+  launch_shift(ctx->g, k, ctx->cfg.liquid, ctx->nph, ctx->nmu, ctx->hp.mu_inf, ctx->phi[ctx->cur], ctx->mu[ctx->cur],
                ctx->phi[1 - ctx->cur], ctx->mu[1 - ctx->cur], ctx->stream);
   ctx->nlaunch[3] += 1;
   prof_end(ctx, 3, e0);
@@ -1707,7 +1841,7 @@ static int time_candidates(pf_ctx* ctx, const std::vector<pf_tuning>& cands, int
 int pf_autotune(pf_ctx* ctx, unsigned mask, int passes, int reps, char* log, int logn) {
   if (!ctx) return PF_EINVAL;
   if (!ctx->have_params || !ctx->have_fields) return fail(ctx, PF_ESTATE, "pf_autotune before pf_set_params/pf_init_fields");
-  if (ctx->variant != PF_VARIANT_JIT) return fail(ctx, PF_ESTATE, "pf_autotune tunes the JIT variant only");
+  if (ctx->variant != PF_VARIANT_JIT || ctx->p2) return fail(ctx, PF_ESTATE, "pf_autotune tunes the JIT variant of P1 only");
   if (!(mask & (PF_PHI | PF_MU)) || passes < 1 || reps < 1 || reps > 1000)
     return fail(ctx, PF_EINVAL, "pf_autotune: mask PF_PHI|PF_MU, passes >= 1, 1 <= reps <= 1000");
   if (const char* m = tuning_check(ctx->tune)) return fail(ctx, PF_EINVAL, "current tuning invalid: %s", m);
@@ -1725,7 +1859,7 @@ int pf_autotune(pf_ctx* ctx, unsigned mask, int passes, int reps, char* log, int
       JitKernel* kp = jit_get(ctx, ctx->dp, ctx->g, best, JIT_PHI, &err);
       if (!kp) return fail(ctx, PF_ECUDA, "autotune: %s", err.c_str());
       CU(jit_launch_phi(kp, ctx->dp, ctx->phi[ctx->cur], ctx->mu[ctx->cur], ctx->phi[1 - ctx->cur], ctx->stream));
-      if (int r = fill_ghosts(ctx, ctx->phi[1 - ctx->cur], PF_N, false)) return r;
+      if (int r = fill_ghosts(ctx, ctx->phi[1 - ctx->cur], ctx->nph, false)) return r;
     }
     std::vector<double> t0;
     std::vector<std::string> w0;

@@ -46,10 +46,11 @@ void launch_ghost_fill(const Geom& g, const BCSpec& bc, double* f, int ncomp, co
                        bool skip_x = false);
 void launch_ghost_stage(const Geom& g, int d, int klo, int khi, double* f, int ncomp, const double* dirichlet,
                         cudaStream_t s);
-void launch_shift(const Geom& g, int k, int liquid, const double* mu_inf, const double* phi_src, const double* mu_src,
-                  double* phi_dst, double* mu_dst, cudaStream_t s);
+void launch_shift(const Geom& g, int k, int liquid, int nph, int nmu, const double* mu_inf, const double* phi_src,
+                  const double* mu_src, double* phi_dst, double* mu_dst, cudaStream_t s);
 void launch_front_height(const Geom& g, int liquid, const double* phi, int* out, cudaStream_t s);
-void launch_monitor(const Geom& g, const double* phi, const double* mu, unsigned long long* out2, cudaStream_t s);
+void launch_monitor(const Geom& g, int nph, int nmu, const double* phi, const double* mu, unsigned long long* out2,
+                    cudaStream_t s);
 void launch_copy_interior(const Geom& g, int ncomp, const double* src, double* dst, int to_packed, cudaStream_t s);
 // face pack/unpack for the ordered x -> y -> z halo exchange along dimension
 // d: slab at index idx of dimension d, extended (ghosted) ranges for the
@@ -59,7 +60,15 @@ void launch_pack(const Geom& g, int d, int idx, int ncomp, const double* f, doub
 void launch_unpack(const Geom& g, int d, int idx, int ncomp, double* f, const double* buf, cudaStream_t s);
 
 void fill_dev_params(const pf_params& p, int liquid, DevParams* out);
-bool plane_interleaved();  // field layout: [z][c][y][x] (default) or [c][z][y][x] (PF_LAYOUT=soa)
+bool plane_interleaved();  // field layout: [c][z][y][x] (default) or [z][c][y][x] (PF_LAYOUT=il)
+
+// ---- P2 parameterisation (pf_p2.cu): 3 phases, 1 mu, anisotropic phi ----
+size_t p2_params_size();                                                // bytes of the opaque parameter block
+void p2_fill_params(const pf_params& p, int liquid, void* out);          // host values -> parameter block
+void p2_launch_phi(const void* P, double Tbase, const Geom& g, const double* ps, const double* ms, double* pd,
+                   cudaStream_t s);
+void p2_launch_mu(const void* P, double Tbase, const Geom& g, const double* ps, const double* pd, const double* ms,
+                  double* md, cudaStream_t s);
 
 // ---- run-time specialisation (NVRTC) -------------------------------------
 enum { JIT_PHI = 0, JIT_MU = 1 };

@@ -260,7 +260,7 @@ void launch_ghost_fill(const Geom& g, const BCSpec& bc, double* f, int ncomp, co
 // Moving window [A16]: dst(z) = src(z + k) for z + k < nz, else inflow
 // (phi = e_l, mu = mu_inf).  Out-of-place; the caller swaps.
 // ---------------------------------------------------------------------------
-__global__ void k_shift(Geom g, int k, int L, double mi0, double mi1, const double* __restrict__ ps,
+__global__ void k_shift(Geom g, int k, int L, int nph, int nmu, double mi0, double mi1, const double* __restrict__ ps,
                         const double* __restrict__ ms, double* __restrict__ pd, double* __restrict__ md) {
   const int x = blockIdx.x * blockDim.x + threadIdx.x;
   const int y = blockIdx.y;
@@ -269,9 +269,9 @@ __global__ void k_shift(Geom g, int k, int L, double mi0, double mi1, const doub
   const int64_t c = g.at(x, y, z);
   const bool in = z + k < g.nz;
   const int64_t sidx = in ? g.at(x, y, z + k) : 0;
-  for (int a = 0; a < N; ++a) pd[a * g.field + c] = in ? ps[a * g.field + sidx] : (a == L ? 1.0 : 0.0);
+  for (int a = 0; a < nph; ++a) pd[a * g.field + c] = in ? ps[a * g.field + sidx] : (a == L ? 1.0 : 0.0);
   md[c] = in ? ms[sidx] : mi0;
-  md[g.field + c] = in ? ms[g.field + sidx] : mi1;
+  if (nmu > 1) md[g.field + c] = in ? ms[g.field + sidx] : mi1;
 }
 
 __global__ void k_set_steps(StepVals* dst, StepBatch b) {
@@ -284,10 +284,10 @@ __global__ void k_set_steps(StepVals* dst, StepBatch b) {
 
 void launch_set_steps(StepVals* dst, const StepBatch& b, cudaStream_t s) { k_set_steps<<<1, 64, 0, s>>>(dst, b); }
 
-void launch_shift(const Geom& g, int k, int liquid, const double* mu_inf, const double* ps, const double* ms,
-                  double* pd, double* md, cudaStream_t s) {
+void launch_shift(const Geom& g, int k, int liquid, int nph, int nmu, const double* mu_inf, const double* ps,
+                  const double* ms, double* pd, double* md, cudaStream_t s) {
   dim3 b(128), gr((g.nx + 127) / 128, g.ny, g.nz);
-  k_shift<<<gr, b, 0, s>>>(g, k, liquid, mu_inf[0], mu_inf[1], ps, ms, pd, md);
+  k_shift<<<gr, b, 0, s>>>(g, k, liquid, nph, nmu, mu_inf[0], nmu > 1 ? mu_inf[1] : 0.0, ps, ms, pd, md);
 }
 
 // front height: max z with phi_l < 1/2 (deterministic integer max).  One
@@ -316,7 +316,7 @@ __device__ __forceinline__ unsigned long long ord_bits(double v) {
   return (b & 0x8000000000000000ull) ? ~b : (b | 0x8000000000000000ull);
 }
 
-__global__ void k_monitor(Geom g, const double* __restrict__ ph, const double* __restrict__ mu,
+__global__ void k_monitor(Geom g, int nph, int nmu, const double* __restrict__ ph, const double* __restrict__ mu,
                           unsigned long long* out) {
   const int z = blockIdx.y;
   double e = -1.0, neg = -INFINITY;
@@ -324,13 +324,13 @@ __global__ void k_monitor(Geom g, const double* __restrict__ ph, const double* _
     const int y = i / g.nx, x = i - y * g.nx;
     const int64_t c = g.at(x, y, z);
     double sum = 0.0, mn = INFINITY, fin = 0.0;  // fin: 0 for finite values, NaN otherwise
-    for (int a = 0; a < N; ++a) {
+    for (int a = 0; a < nph; ++a) {
       const double v = ph[a * g.field + c];
       sum += v;
       mn = fmin(mn, v);
       fin += v - v;
     }
-    for (int i2 = 0; i2 < M; ++i2) {
+    for (int i2 = 0; i2 < nmu; ++i2) {
       const double v = mu[i2 * g.field + c];
       fin += v - v;
     }
@@ -358,11 +358,12 @@ __global__ void k_monitor(Geom g, const double* __restrict__ ph, const double* _
   }
 }
 
-void launch_monitor(const Geom& g, const double* phi, const double* mu, unsigned long long* out2, cudaStream_t s) {
+void launch_monitor(const Geom& g, int nph, int nmu, const double* phi, const double* mu, unsigned long long* out2,
+                    cudaStream_t s) {
   int bx = (g.nx * g.ny + 255) / 256;
   if (bx > 64) bx = 64;
   dim3 gr(bx, g.nz);
-  k_monitor<<<gr, 256, 0, s>>>(g, phi, mu, out2);
+  k_monitor<<<gr, 256, 0, s>>>(g, nph, nmu, phi, mu, out2);
 }
 
 // interior <-> packed [comp][z][y][x] copies

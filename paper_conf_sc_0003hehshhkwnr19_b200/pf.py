@@ -48,7 +48,9 @@ class PFParams(C.Structure):
                 ("D", C.c_double * M * M * N),
                 ("T0", C.c_double), ("G", C.c_double), ("v", C.c_double),
                 ("mu_inf", C.c_double * M), ("window_frac", C.c_double), ("window_check", C.c_int),
-                ("xi_amp", C.c_double), ("xi_seed", C.c_uint32)]
+                ("xi_amp", C.c_double), ("xi_seed", C.c_uint32),
+                ("aniso", C.c_int), ("aniso_delta", C.c_double * N * N),
+                ("aniso_R", C.c_double * 3 * 3 * N * N)]
 
 
 TUNING_KNOBS = ("phi_ty", "phi_minb", "phi_zc", "phi_faces6", "phi_unroll", "phi_prefetch", "phi_pfd", "phi_xsh", "phi_zrec", "phi_xghost",
@@ -130,7 +132,8 @@ def tuning_default() -> dict:
 
 def make_params(P: dict) -> PFParams:
     p = PFParams()
-    assert int(P["N"]) == N and int(P["M"]) == M, "the CUDA path is specialised to N = 4, M = 2"
+    n, m = int(P["N"]), int(P["M"])
+    assert (n, m) in ((N, M), (3, 1)), "the CUDA path runs P1 (N = 4, M = 2) or P2 (N = 3, M = 1)"
 
     def put(dst, arr, shape):
         arr = np.asarray(arr, dtype=np.float64)
@@ -142,18 +145,22 @@ def make_params(P: dict) -> PFParams:
             o[ix[-1]] = float(arr[ix])
 
     p.dx, p.dt, p.eps = float(P["dx"]), float(P["dt"]), float(P["eps"])
-    put(p.gamma, P["gamma"], (N, N))
-    put(p.gamma3, P["gamma3"], (N, N, N))
-    put(p.tau, P["tau"], (N, N))
-    put(p.A0, P["A0"], (N, M, M))
-    put(p.A1, P["A1"], (N, M, M))
-    put(p.B0, P["B0"], (N, M))
-    put(p.B1, P["B1"], (N, M))
-    put(p.C0, P["C0"], (N,))
-    put(p.C1, P["C1"], (N,))
-    put(p.D, P["D"], (N, M, M))
+    put(p.gamma, P["gamma"], (n, n))
+    put(p.gamma3, P["gamma3"], (n, n, n))
+    put(p.tau, P["tau"], (n, n))
+    put(p.A0, P["A0"], (n, m, m))
+    put(p.A1, P["A1"], (n, m, m))
+    put(p.B0, P["B0"], (n, m))
+    put(p.B1, P["B1"], (n, m))
+    put(p.C0, P["C0"], (n,))
+    put(p.C1, P["C1"], (n,))
+    put(p.D, P["D"], (n, m, m))
     p.T0, p.G, p.v = float(P["T0"]), float(P["G"]), float(P["v"])
-    put(p.mu_inf, P["mu_inf"], (M,))
+    put(p.mu_inf, P["mu_inf"], (m,))
+    p.aniso = int(P.get("aniso", 0))
+    if p.aniso:
+        put(p.aniso_delta, P["aniso_delta"], (n, n))
+        put(p.aniso_R, P["aniso_R"], (n, n, 3, 3))
     p.window_frac = float(P.get("window_frac", 0.5))
     p.window_check = int(P.get("window_check", 0))
     p.xi_amp = float(P.get("xi_amp", 0.0))
@@ -254,7 +261,8 @@ class PhaseField:
         bc = bc or {"lo": ("periodic",) * 3, "hi": ("periodic",) * 3}
         cfg = PFConfig()
         liquid = int(params.get("liquid", 3)) if liquid is None else int(liquid)
-        cfg.n_phases, cfg.n_mu, cfg.liquid = N, M, liquid
+        self.N, self.M = int(params.get("N", N)), int(params.get("M", M))
+        cfg.n_phases, cfg.n_mu, cfg.liquid = self.N, self.M, liquid
         for d, n in enumerate((nx, ny, nz)):
             cfg.global_[d] = n
             cfg.procs[d] = int(procs[d])
@@ -331,7 +339,8 @@ class PhaseField:
             where = PF_HOST
             pp, mp = phi.ctypes.data, mu.ctypes.data
             keep = (phi, mu)
-        assert tuple(phi.shape) == (N,) + self.local and tuple(mu.shape) == (M,) + self.local, (phi.shape, self.local)
+        assert tuple(phi.shape) == (self.N,) + self.local and tuple(mu.shape) == (self.M,) + self.local, (
+            phi.shape, self.local)
         self._check(self.lib.pf_init_fields(self._h, C.c_void_p(pp), C.c_void_p(mp), where), "pf_init_fields")
         del keep
 
@@ -373,13 +382,13 @@ class PhaseField:
                         "pf_download")
             return phi, mu
         if device:
-            phi = torch.empty((N,) + self.local, dtype=torch.float64, device=self.device)
-            mu = torch.empty((M,) + self.local, dtype=torch.float64, device=self.device)
+            phi = torch.empty((self.N,) + self.local, dtype=torch.float64, device=self.device)
+            mu = torch.empty((self.M,) + self.local, dtype=torch.float64, device=self.device)
             self._check(self.lib.pf_download(self._h, C.c_void_p(phi.data_ptr()), C.c_void_p(mu.data_ptr()),
                                              PF_DEVICE), "pf_download")
             return phi, mu
-        phi = np.empty((N,) + self.local)
-        mu = np.empty((M,) + self.local)
+        phi = np.empty((self.N,) + self.local)
+        mu = np.empty((self.M,) + self.local)
         self._check(self.lib.pf_download(self._h, C.c_void_p(phi.ctypes.data), C.c_void_p(mu.ctypes.data), PF_HOST),
                     "pf_download")
         return phi, mu

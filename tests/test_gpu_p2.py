@@ -1,0 +1,100 @@
+"""GPU parity of the P2 parameterisation (SURVEY §8(f) NEXT-4, P:L1199-1213;
+pf_p2.cu): 3 phases, 1 chemical potential, anisotropic gradient energy
+(reading B6), against the oracle on the same seeded inputs.  Bar as for P1
+(north_star): relative L-inf <= 1e-12 after one step, <= 1e-9 after 1000.
+-m gpu.
+"""
+import os
+
+import numpy as np
+import pytest
+
+from paper_conf_sc_0003hehshhkwnr19_b200 import inputs as I
+
+pytestmark = pytest.mark.gpu
+
+
+def rel_linf(a, b):
+    return float(np.abs(a - b).max() / max(np.abs(b).max(), 1e-300))
+
+
+@pytest.fixture(scope="module")
+def pfmod():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.fail("GPU test without a CUDA device")
+    from paper_conf_sc_0003hehshhkwnr19_b200 import build, pf
+    build.build()
+    return pf
+
+
+@pytest.fixture(scope="module")
+def omod():
+    from oracle import oracle as O
+    O.build()
+    O.set_threads(min(16, os.cpu_count() or 1))
+    return O
+
+
+def run_pair(pfmod, omod, shape, P, phi, mu, chunks, bc=None):
+    g = pfmod.PhaseField(shape, P, bc=bc)
+    g.init_fields(phi, mu)
+    o = omod.Oracle(shape, P, bc)
+    o.init(phi, mu)
+    out, done = [], 0
+    for t in chunks:
+        g.step(t - done)
+        o.step(t - done)
+        done = t
+        gp, gm = g.download()
+        op, om = o.download()
+        out.append((t, rel_linf(gp, op), rel_linf(gm, om), g.state(), o.state()))
+    g.close()
+    return out
+
+
+@pytest.mark.parametrize("pset", ["p2", "p2_stress", "p2_iso"])
+@pytest.mark.parametrize("ic", ["R", "V"])
+def test_p2_one_step_parity(pfmod, omod, pset, ic):
+    P = {"p2": I.params_p2(), "p2_stress": I.params_p2_stress(), "p2_iso": I.params_p2(aniso=0)}[pset]
+    shape = (18, 21, 37)
+    phi, mu = I.make_ic(ic, shape, seed=11, N=3, M=1)
+    for t, ep, em, *_ in run_pair(pfmod, omod, shape, P, phi, mu, [1, 2]):
+        assert ep <= 1e-12 and em <= 1e-12, (t, ep, em)
+
+
+def test_p2_ds_window_parity(pfmod, omod):
+    """DS boundaries (Dirichlet mu_inf != 0 at z_hi), frozen T with G v != 0,
+    window shifts."""
+    P = I.params_p2_stress(window_check=5, window_frac=0.5, v=0.05)
+    shape = (32, 12, 20)
+    phi, mu = I.ic_voronoi(shape, seed=5, N=3, M=1)
+    res = run_pair(pfmod, omod, shape, P, phi, mu, [1, 40], bc=I.BC_DS)
+    for t, ep, em, gs, os_ in res:
+        assert gs == os_
+        tol = 1e-12 if t == 1 else 1e-11
+        assert ep <= tol and em <= tol, (t, ep, em)
+    assert res[-1][3]["z_off"] > 0
+
+
+def test_p2_1000_steps(pfmod, omod):
+    P = I.params_p2_stress()
+    shape = (16, 16, 16)
+    phi, mu = I.ic_voronoi(shape, seed=6, N=3, M=1)
+    for t, ep, em, *_ in run_pair(pfmod, omod, shape, P, phi, mu, [1, 100, 1000]):
+        tol = 1e-12 if t == 1 else 1e-9
+        assert ep <= tol and em <= tol, (t, ep, em)
+
+
+def test_p2_invariants_and_monitor(pfmod):
+    P = I.params_p2()
+    shape = (24, 24, 24)
+    phi, mu = I.ic_voronoi(shape, seed=2, N=3, M=1)
+    g = pfmod.PhaseField(shape, P)
+    g.init_fields(phi, mu)
+    g.set_monitors(5, 1e-13)
+    g.step(50)
+    err, mn = g.monitor()
+    assert err <= 8 * 2.2e-16 and mn >= 0.0
+    p, _ = g.download()
+    assert p.shape == (3,) + shape
