@@ -1741,7 +1741,10 @@ std::string tuning_json(const pf_tuning& t) {
     o += b;
     first = false;
   }
-  return o + "}";
+  // the step schedule (timed as whole dry steps, not a per-kernel knob)
+  char b[64];
+  snprintf(b, sizeof b, ", \"sched\": %d, \"slab\": %d", t.sched, t.slab);
+  return o + b + "}";
 }
 }  // namespace
 

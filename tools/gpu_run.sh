@@ -1,26 +1,28 @@
 #!/bin/bash
-# One GPU session: GPU tests, smoke, bench (config 2 and config 4, auto-tuned),
-# ncu launch list + full captures of the sweeps in the tuning the bench chose.
-# usage (from the repo root on the GPU box): bash tools/gpu_run.sh [tag]
-TAG=${1:-r01}
+# One GPU session: GPU tests, smoke, bench (config 2 and config 4), ncu launch
+# list + full captures of the sweeps (P1 mu / phi, P2 phi), config 5.
+# usage (from the repo root on the GPU box): bash tools/gpu_run.sh [tag] [skip_config5]
+TAG=${1:-r02}
 OUT=gpurun_out/$TAG
 mkdir -p $OUT
 nvidia-smi > $OUT/nvidia-smi.txt 2>&1
 python -c "import __graft_entry__ as g; g.build()" > $OUT/build.log 2>&1
-[ -x tools/build/fp64_micro ] && timeout 120 tools/build/fp64_micro > $OUT/fp64_micro.json 2>&1
-timeout 1200 python -m pytest tests -m gpu -x -q > $OUT/pytest_gpu.log 2>&1; echo "pytest exit $?" >> $OUT/pytest_gpu.log
+timeout 2400 python -m pytest tests -m gpu -q > $OUT/pytest_gpu.log 2>&1; echo "pytest exit $?" >> $OUT/pytest_gpu.log
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $OUT/smoke.log 2>&1
 timeout 900 python bench.py --steps 200 --warmup 10 > $OUT/bench.json 2> $OUT/bench.err
 timeout 900 python bench.py --config strong --steps 20 --warmup 3 --no-cpu-baseline --autotune 1 > $OUT/bench_strong.json 2>> $OUT/bench.err
-# the tuning the bench selected; the profiled runs use it without re-tuning
 TUNE=$(python -c "import json; print(json.dumps(json.load(open('$OUT/bench.json'))['config']['tuning']))" 2>/dev/null || echo '{}')
 echo "$TUNE" > $OUT/tuning.json
+export PF_BENCH_ALLOW_SHORT=1
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches.csv \
-   python bench.py --steps 10 --warmup 3 --no-cpu-baseline --no-e2e --autotune 0 --tuning "$TUNE" > $OUT/ncu_launch.log 2>&1
+   python bench.py --steps 10 --warmup 3 --no-cpu-baseline --no-e2e --no-stress --no-p2 --autotune 0 --tuning "$TUNE" > $OUT/ncu_launch.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:pf_jit_mu -s 3 -c 1 -o $OUT/prof_mu \
-   python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e --autotune 0 --tuning "$TUNE" > $OUT/ncu_mu.log 2>&1
+   python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e --no-stress --no-p2 --autotune 0 --tuning "$TUNE" > $OUT/ncu_mu.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:pf_jit_phi -s 3 -c 1 -o $OUT/prof_phi \
-   python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e --autotune 0 --tuning "$TUNE" > $OUT/ncu_phi.log 2>&1
-timeout 600 ncu --set full --clock-control none -k regex:k_ghost -s 6 -c 1 -o $OUT/prof_ghost \
-   python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e --autotune 0 --tuning "$TUNE" > $OUT/ncu_ghost.log 2>&1
+   python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e --no-stress --no-p2 --autotune 0 --tuning "$TUNE" > $OUT/ncu_phi.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_phi -s 1 -c 1 -o $OUT/prof_p2phi \
+   python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e --no-stress --autotune 0 --tuning "$TUNE" > $OUT/ncu_p2phi.log 2>&1
+if [ -z "$2" ]; then
+  timeout 1500 python tools/config5.py --out $OUT/config5.jsonl > $OUT/config5.log 2>&1
+fi
 echo done > $OUT/DONE
