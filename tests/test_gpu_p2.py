@@ -53,9 +53,13 @@ def run_pair(pfmod, omod, shape, P, phi, mu, chunks, bc=None):
     return out
 
 
+@pytest.mark.parametrize("naive", [0, 1])
 @pytest.mark.parametrize("pset", ["p2", "p2_stress", "p2_iso"])
 @pytest.mark.parametrize("ic", ["R", "V"])
-def test_p2_one_step_parity(pfmod, omod, pset, ic):
+def test_p2_one_step_parity(pfmod, omod, pset, ic, naive, monkeypatch):
+    """z-marching sweeps (default; every face once, ragged tiles and
+    z-chunks at this shape) and the one-thread-per-cell kernels."""
+    monkeypatch.setenv("PF_P2_NAIVE", str(naive))
     P = {"p2": I.params_p2(), "p2_stress": I.params_p2_stress(), "p2_iso": I.params_p2(aniso=0)}[pset]
     shape = (18, 21, 37)
     phi, mu = I.make_ic(ic, shape, seed=11, N=3, M=1)
@@ -84,6 +88,24 @@ def test_p2_1000_steps(pfmod, omod):
     for t, ep, em, *_ in run_pair(pfmod, omod, shape, P, phi, mu, [1, 100, 1000]):
         tol = 1e-12 if t == 1 else 1e-9
         assert ep <= tol and em <= tol, (t, ep, em)
+
+
+def test_p2_liquid_index_not_hardcoded(pfmod, omod):
+    """Any phase may be the liquid (compile-time L of the mu kernels)."""
+    P = I.params_p2_stress()
+    perm = [2, 1, 0]  # phase 0 plays the liquid
+    Q = dict(P, liquid=0)
+    for key in ("A0", "A1", "B0", "B1", "C0", "C1", "D"):
+        Q[key] = P[key][perm]
+    Q["gamma"] = P["gamma"][np.ix_(perm, perm)]
+    Q["tau"] = P["tau"][np.ix_(perm, perm)]
+    Q["gamma3"] = P["gamma3"][np.ix_(perm, perm, perm)]
+    Q["aniso_delta"] = P["aniso_delta"][np.ix_(perm, perm)]
+    Q["aniso_R"] = P["aniso_R"][np.ix_(perm, perm)]
+    shape = (10, 12, 14)
+    phi, mu = I.ic_voronoi(shape, seed=9, N=3, M=1)
+    for t, ep, em, *_ in run_pair(pfmod, omod, shape, Q, phi, mu, [2]):
+        assert ep <= 1e-12 and em <= 1e-12, (t, ep, em)
 
 
 def test_p2_invariants_and_monitor(pfmod):
