@@ -291,6 +291,10 @@ typedef struct {
                         still in L2.  Applies to the JIT variant with no exchanged
                         dimension and a non-periodic z (DS); otherwise sched 0     */
   int slab;          /* mu z-chunks per slab of sched = 1 (1..16)                 */
+  int mu_tmem;       /* 1: the two-rows mu-sweep keeps the carried side of plane
+                        k-1 in tensor memory (tcgen05.st / ld, 68 columns per
+                        thread) instead of registers, and re-reads the own
+                        sides of the x / y faces from shared memory             */
 } pf_tuning;
 
 /* The built-in defaults (the measured best at 256^3 on one B200,

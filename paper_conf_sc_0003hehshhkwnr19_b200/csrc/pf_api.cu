@@ -1728,6 +1728,7 @@ const std::vector<TuneKnob>& tune_knobs() {
       {"phi_rpt", &pf_tuning::phi_rpt, JIT_PHI, {1, 2}},
       {"mu_pers", &pf_tuning::mu_pers, JIT_MU, {0, 1}},
       {"phi_pers", &pf_tuning::phi_pers, JIT_PHI, {0, 1}},
+      {"mu_tmem", &pf_tuning::mu_tmem, JIT_MU, {0, 1}},
   };
   return k;
 }

@@ -111,6 +111,9 @@ constexpr int MU_TY = PF_MU_TY;
 #ifndef PF_PHI_PERS  // six-face phi-sweep as a persistent launch (balanced tile-plane shares)
 #define PF_PHI_PERS 0
 #endif
+#ifndef PF_MU_TMEM  // two-rows mu-sweep: the carried side of plane k-1 in tensor memory (TMEM), not registers
+#define PF_MU_TMEM 0
+#endif
 #ifndef PF_MU_PERS  // two-rows mu-sweep: full launches persistent (balanced tile-plane shares)
 #define PF_MU_PERS 0
 #endif
@@ -1041,6 +1044,45 @@ __device__ __forceinline__ void mu_tuned_body(const PT& P, const RT& R, const GT
   plane(BoolC<true>{}, z1);
 }
 
+
+#if PF_MU_TMEM
+// ---------------------------------------------------------------------------
+// Tensor memory (TMEM, 256 KB per SM, tcgen05.*) as per-thread scratch from
+// SIMT code: the 17 doubles of a face side (f, c1, c2, ds, m) as 34 columns
+// of the thread's TMEM lane (a warp accesses the 32 lanes of its quarter).
+// tools/tmem_probe.cu measured the round trip on a B200.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ void tm_st_side(unsigned ta, const FaceSide& s) {
+  unsigned u[34];
+  double v[17];
+#pragma unroll
+  for (int a = 0; a < N; ++a) { v[a] = s.f[a]; v[4 + a] = s.c1[a]; v[8 + a] = s.c2[a]; }
+#pragma unroll
+  for (int t = 0; t < NSOL; ++t) v[12 + t] = s.ds[t];
+  v[15] = s.m[0];
+  v[16] = s.m[1];
+#pragma unroll
+  for (int i = 0; i < 17; ++i) { u[2 * i] = (unsigned)__double2loint(v[i]); u[2 * i + 1] = (unsigned)__double2hiint(v[i]); }
+  asm volatile("tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, %15, %16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, %28, %29, %30, %31, %32};\n" ::"r"(ta), "r"(u[0]), "r"(u[1]), "r"(u[2]), "r"(u[3]), "r"(u[4]), "r"(u[5]), "r"(u[6]), "r"(u[7]), "r"(u[8]), "r"(u[9]), "r"(u[10]), "r"(u[11]), "r"(u[12]), "r"(u[13]), "r"(u[14]), "r"(u[15]), "r"(u[16]), "r"(u[17]), "r"(u[18]), "r"(u[19]), "r"(u[20]), "r"(u[21]), "r"(u[22]), "r"(u[23]), "r"(u[24]), "r"(u[25]), "r"(u[26]), "r"(u[27]), "r"(u[28]), "r"(u[29]), "r"(u[30]), "r"(u[31]) : "memory");
+  asm volatile("tcgen05.st.sync.aligned.32x32b.x2.b32 [%0], {%1, %2};\n" ::"r"(ta + 32u), "r"(u[32]), "r"(u[33]) : "memory");
+}
+__device__ __forceinline__ void tm_ld_side(unsigned ta, FaceSide& s) {
+  unsigned u[34];
+  asm volatile("tcgen05.wait::st.sync.aligned;\n" ::: "memory");
+  asm volatile("tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, %15, %16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, %28, %29, %30, %31}, [%32];\n" : "=r"(u[0]), "=r"(u[1]), "=r"(u[2]), "=r"(u[3]), "=r"(u[4]), "=r"(u[5]), "=r"(u[6]), "=r"(u[7]), "=r"(u[8]), "=r"(u[9]), "=r"(u[10]), "=r"(u[11]), "=r"(u[12]), "=r"(u[13]), "=r"(u[14]), "=r"(u[15]), "=r"(u[16]), "=r"(u[17]), "=r"(u[18]), "=r"(u[19]), "=r"(u[20]), "=r"(u[21]), "=r"(u[22]), "=r"(u[23]), "=r"(u[24]), "=r"(u[25]), "=r"(u[26]), "=r"(u[27]), "=r"(u[28]), "=r"(u[29]), "=r"(u[30]), "=r"(u[31]) : "r"(ta) : "memory");
+  asm volatile("tcgen05.ld.sync.aligned.32x32b.x2.b32 {%0, %1}, [%2];\n" : "=r"(u[32]), "=r"(u[33]) : "r"(ta + 32u) : "memory");
+  asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
+  double v[17];
+#pragma unroll
+  for (int i = 0; i < 17; ++i) v[i] = __hiloint2double((int)u[2 * i + 1], (int)u[2 * i]);
+#pragma unroll
+  for (int a = 0; a < N; ++a) { s.f[a] = v[a]; s.c1[a] = v[4 + a]; s.c2[a] = v[8 + a]; }
+#pragma unroll
+  for (int t = 0; t < NSOL; ++t) s.ds[t] = v[12 + t];
+  s.m[0] = v[15];
+  s.m[1] = v[16];
+}
+#endif
 // ===========================================================================
 // mu-sweep with two tile rows per thread (pf_tuning mu_rpt = 2): a CTA of
 // 32 x (MTY/2) threads owns a 32 x MTY tile; thread (lane, w) updates rows
@@ -1107,6 +1149,28 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
     Dp[r].m[0] = ldh(ms + c);
     Dp[r].m[1] = ldh(ms + F + c);
   }
+#if PF_MU_TMEM
+  // the carried side of plane k-1 lives in TMEM between planes (68 columns
+  // of this thread's lane: row r at column 34 r); only its phi_src (the z
+  // central difference of the build) stays in registers
+  __shared__ unsigned tm_base;
+  if (w == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 128;\n" ::"r"(
+                     (unsigned)__cvta_generic_to_shared(&tm_base)));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;\n");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;\n" ::: "memory");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
+  const unsigned tm = tm_base + ((unsigned)(32 * (w & 3)) << 16);
+  double fprev[2][N];
+#pragma unroll
+  for (int r = 0; r < 2; ++r) {
+    tm_st_side(tm + 34u * r, Dp[r]);
+#pragma unroll
+    for (int a = 0; a < N; ++a) fprev[r][a] = Dp[r].f[a];
+  }
+#endif
   double divxy[2][M] = {{0.0, 0.0}, {0.0, 0.0}}, Fzm[2][M] = {{0.0, 0.0}, {0.0, 0.0}};
   double fcar[2][N];
 #if PF_MU_RPF
@@ -1171,8 +1235,13 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
         v1[D_CX + a] = __ldg(f1 + 1) - __ldg(f1 - 1);
         v0[D_CY + a] = fcar[1][a] - __ldg(f0 - g.pitch);
         v1[D_CY + a] = __ldg(f1 + g.pitch) - fcar[0][a];
+#if PF_MU_TMEM
+        v0[D_CZ + a] = !last ? rnf[0][a] - fprev[0][a] : 0.0;
+        v1[D_CZ + a] = !last ? rnf[1][a] - fprev[1][a] : 0.0;
+#else
         v0[D_CZ + a] = !last ? rnf[0][a] - Dp[0].f[a] : 0.0;
         v1[D_CZ + a] = !last ? rnf[1][a] - Dp[1].f[a] : 0.0;
+#endif
         v0[D_DP + a] = rnd[0][a] - fcar[0][a];
         v1[D_DP + a] = rnd[1][a] - fcar[1][a];
       }
@@ -1212,6 +1281,8 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
       double vo[D_NV];
 #if PF_MU_RPF
       build_own_rpf<NC>(g, ps, pd, ms, xc, yc[r], k, !last, Dp[r].f, fcar[r], rnf[r], rnd[r], rnm[r], D, me[r], vo);
+#elif PF_MU_TMEM
+      build_own_carry<NC>(g, ps, pd, ms, xc, yc[r], k, !last, fprev[r], fcar[r], D, me[r], vo);
 #else
       build_own_carry<NC>(g, ps, pd, ms, xc, yc[r], k, !last, Dp[r].f, fcar[r], D, me[r], vo);
 #endif
@@ -1224,6 +1295,9 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
     for (int r = 0; r < 2; ++r) {
       FaceSide q;
       side_from_smem<L, NC>(D, me[r], D_CX, D_CY, q);
+#if PF_MU_TMEM
+      tm_ld_side(tm + 34u * r, Dp[r]);
+#endif
       double Fz[M];
       mu_face<L, TA>(P, plane_T(P, R, k - 0.5), Dp[r], q, Fz);
       if (k > z0 && active[r]) {
@@ -1241,7 +1315,15 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
       }
       Fzm[r][0] = Fz[0];
       Fzm[r][1] = Fz[1];
+#if PF_MU_TMEM
+      if constexpr (!last) {
+        tm_st_side(tm + 34u * r, q);
+#pragma unroll
+        for (int a = 0; a < N; ++a) fprev[r][a] = q.f[a];
+      }
+#else
       Dp[r] = q;
+#endif
       dpl[r] = D[(size_t)me[r] * D_NV + D_DP + L];
     }
     if constexpr (!last) {
@@ -1258,6 +1340,22 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
         cz[r][0] = z01.x; cz[r][1] = z01.y; cz[r][2] = z23.x; cz[r][3] = z23.y;
       }
       FaceSide p, s;
+#if PF_MU_TMEM
+      // own sides from shared memory (the carried copy is in TMEM)
+      (void)cz;
+#pragma unroll
+      for (int r = 0; r < 2; ++r) {
+        side_from_smem<L, NC>(D, me[r], D_CY, D_CZ, s);
+        side_from_smem<L, NC>(D, me[r] - 1, D_CY, D_CZ, p);
+        mu_face<L, TA>(P, Tk, p, s, Fx[r]);
+      }
+#pragma unroll
+      for (int r = 0; r < 2; ++r) {
+        side_from_smem<L, NC>(D, me[r], D_CX, D_CZ, s);
+        side_from_smem<L, NC>(D, r == 0 ? me[0] - HX : me[0], D_CX, D_CZ, p);
+        mu_face<L, TA>(P, Tk, p, s, Fy[r]);
+      }
+#else
 #pragma unroll
       for (int r = 0; r < 2; ++r) {
 #pragma unroll
@@ -1301,6 +1399,7 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
         }
         mu_face<L, TA>(P, Tk, p, s, Fy[r]);
       }
+#endif
 #pragma unroll
       for (int r = 0; r < 2; ++r)
 #pragma unroll
@@ -1334,6 +1433,12 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
   };
   for (int k = z0; k < z1; ++k) plane(BoolC<false>{}, k);
   plane(BoolC<true>{}, z1);
+#if PF_MU_TMEM
+  asm volatile("tcgen05.wait::st.sync.aligned;\n" ::: "memory");
+  asm volatile("tcgen05.fence::before_thread_sync;\n" ::: "memory");
+  __syncthreads();
+  if (w == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;\n" ::"r"(tm_base));
+#endif
   };  // tile
 #if PF_MU_PERS
   if (ts.skip == 2) {

@@ -55,6 +55,9 @@ CORNERS = [
     # phi-sweep with two rows per thread (21 rows: the last pair's upper row is the ghost row)
     {"phi_rpt": 2, "phi_ty": 8, "phi_minb": 3},
     {"phi_rpt": 2, "phi_ty": 4, "phi_minb": 6, "phi_zc": 7, "phi_prefetch": 2, "phi_xghost": 1},
+    # the carried side of the two-rows mu-sweep in tensor memory (TMEM)
+    {"mu_tmem": 1, "mu_rpf": 0, "mu_minb": 3},
+    {"mu_tmem": 1, "mu_zc": 7, "mu_ty": 6, "mu_minb": 3},
     # persistent launches: balanced tile-plane shares, segments crossing tile columns
     {"mu_pers": 1, "phi_pers": 1},
     {"mu_pers": 1, "mu_ty": 6, "mu_minb": 3, "phi_pers": 1, "phi_ty": 8, "phi_minb": 2, "phi_xsh": 1},
