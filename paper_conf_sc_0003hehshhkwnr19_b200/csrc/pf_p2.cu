@@ -426,8 +426,6 @@ __global__ void __launch_bounds__(TXP * TYP) k_mu_march(Params P, Geom g, const 
 // ---------------------------------------------------------------------------
 // host side
 // ---------------------------------------------------------------------------
-static p2::Params g_dummy;  // (size reference for the binding)
-
 void p2_fill_params(const pf_params& p, int liquid, void* out) {
   p2::Params& P = *reinterpret_cast<p2::Params*>(out);
   P = p2::Params{};
@@ -469,7 +467,7 @@ void p2_fill_params(const pf_params& p, int liquid, void* out) {
   P.aniso = p.aniso ? 1 : 0;
   P.mu_inf = p.mu_inf[0];
 }
-size_t p2_params_size() { return sizeof(g_dummy); }
+size_t p2_params_size() { return sizeof(p2::Params); }
 
 // PF_P2_NAIVE=1: the one-thread-per-cell kernels (every face twice)
 static bool p2_naive() {

@@ -194,12 +194,14 @@ def jit_compile_only(params: dict, n: int = 64, cubin_path: str | None = None, t
     return r
 
 
-def make_config(shape, bc=None, liquid: int = 3, procs=(1, 1, 1), rank: int = 0, world: int = 1) -> PFConfig:
-    """pf_config for a global (nz, ny, nx) domain (no buffers bound)."""
+def make_config(shape, bc=None, liquid: int = 3, procs=(1, 1, 1), rank: int = 0, world: int = 1,
+                n_phases: int = N, n_mu: int = M) -> PFConfig:
+    """pf_config for a global (nz, ny, nx) domain (no buffers bound); P1
+    (4 phases, 2 mu) or P2 (3 phases, 1 mu)."""
     nz, ny, nx = shape
     bc = bc or {"lo": ("periodic",) * 3, "hi": ("periodic",) * 3}
     cfg = PFConfig()
-    cfg.n_phases, cfg.n_mu, cfg.liquid = N, M, int(liquid)
+    cfg.n_phases, cfg.n_mu, cfg.liquid = int(n_phases), int(n_mu), int(liquid)
     for d, n in enumerate((nx, ny, nz)):
         cfg.global_[d] = n
         cfg.procs[d] = int(procs[d])
@@ -209,10 +211,12 @@ def make_config(shape, bc=None, liquid: int = 3, procs=(1, 1, 1), rank: int = 0,
     return cfg
 
 
-def query_layout(shape, procs=(1, 1, 1), rank: int = 0, world: int = 1, bc=None) -> PFLayout:
+def query_layout(shape, procs=(1, 1, 1), rank: int = 0, world: int = 1, bc=None, n_phases: int = N,
+                 n_mu: int = M) -> PFLayout:
     """Host-only block layout of `rank` (no GPU needed)."""
     lay = PFLayout()
-    r = load_library().pf_query_layout(C.byref(make_config(shape, bc, 3, procs, rank, world)), C.byref(lay))
+    cfg = make_config(shape, bc, n_phases - 1, procs, rank, world, n_phases, n_mu)
+    r = load_library().pf_query_layout(C.byref(cfg), C.byref(lay))
     if r != PF_OK:
         raise PFError(f"pf_query_layout failed ({r})")
     return lay

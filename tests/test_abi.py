@@ -142,3 +142,21 @@ def test_tuned_variants_compile_without_gpu(lib, knobs):
     t = dict(pf.tuning_default(), **knobs)
     assert pf.tuning_check(t) == "ok"
     assert pf.jit_compile_only(I.params_c4("ds"), n=40, tuning=t) > 0
+
+
+def test_p2_layout_and_params_struct():
+    """P2 (NEXT-4) through the same ABI: 3 phase and 1 mu components per
+    buffer; pf_params carries the anisotropy (aniso, aniso_delta, aniso_R)."""
+    from paper_conf_sc_0003hehshhkwnr19_b200 import build, inputs as I, pf
+    build.build()
+    L1 = pf.query_layout((20, 24, 40))
+    L2 = pf.query_layout((20, 24, 40), n_phases=3, n_mu=1)
+    assert (L1.pitch, L1.plane, L1.field) == (L2.pitch, L2.plane, L2.field)
+    assert L2.phi_bytes == 3 * L2.field * 8 + 256 and L2.mu_bytes == L2.field * 8 + 256
+    assert L1.phi_bytes == 4 * L1.field * 8 + 256 and L1.mu_bytes == 2 * L1.field * 8 + 256
+    p = pf.make_params(I.params_p2_stress())
+    P = I.params_p2_stress()
+    assert p.aniso == 1
+    assert abs(p.aniso_R[0][2][1][0] - P["aniso_R"][0, 2, 1, 0]) == 0.0
+    assert p.aniso_delta[1][2] == P["aniso_delta"][1, 2]
+    assert p.A0[2][0][0] == P["A0"][2, 0, 0] and p.D[1][0][0] == P["D"][1, 0, 0]
