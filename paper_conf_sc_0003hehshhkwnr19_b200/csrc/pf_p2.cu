@@ -33,6 +33,7 @@ struct Params {
   double delta[N3][N3];
   double R[N3][N3][9];  // R_ab row-major
   int liquid, aniso;
+  int prefetch;  // z-marching sweeps: own column's lines P2_PD planes ahead into L2 (PF_P2_PREFETCH, default 1)
   double mu_inf;
 };
 
@@ -338,8 +339,14 @@ __global__ void __launch_bounds__(256) k_mu(Params P, Geom g, const double* __re
 // ---------------------------------------------------------------------------
 constexpr int TXP = 32, TYP = 4, ZCP = 16;
 
-template <int K, class FaceF, class CellF>
-__device__ __forceinline__ void march(const Geom& g, FaceF face, CellF cell) {
+
+__device__ __forceinline__ void pf_l2(const double* p) { asm volatile("prefetch.global.L2 [%0];" ::"l"(p)); }
+
+// own column's lines of the fields a sweep reads, PD planes ahead, into L2
+constexpr int P2_PD = 3;
+
+template <int K, class FaceF, class CellF, class PrefF>
+__device__ __forceinline__ void march(const Geom& g, bool prefetch, FaceF face, CellF cell, PrefF pref) {
   __shared__ double fy[2][K][TYP][TXP];  // -y face flux of every thread
   __shared__ double ex[2][K][TYP];       // +x flux on the right tile edge
   __shared__ double ey[2][K][TXP];       // +y flux on the top tile edge
@@ -359,6 +366,7 @@ __device__ __forceinline__ void march(const Geom& g, FaceF face, CellF cell) {
   for (int z = z0; z < z1; ++z) {
     const int b = z & 1;
     const i64 c = g.at(xc, yc, z);
+    if (prefetch && z + P2_PD <= z1) pref(c + P2_PD * g.plane);
     double Fx[K], Fy[K], Fzp[K];
     face(c - 1, 0, z, Fx);
     face(c - g.pitch, 1, z, Fy);
@@ -391,34 +399,49 @@ __device__ __forceinline__ void march(const Geom& g, FaceF face, CellF cell) {
   }
 }
 
-__global__ void __launch_bounds__(TXP * TYP) k_phi_march(Params P, Geom g, const double* __restrict__ ps,
+// MB: CTAs per SM the kernel is compiled for (register cap 65536 / (128 MB))
+template <int MB>
+__global__ void __launch_bounds__(TXP * TYP, MB) k_phi_march(Params P, Geom g, const double* __restrict__ ps,
                                                          const double* __restrict__ ms, double* __restrict__ pd) {
   const i64 F = g.field;
   const i64 st[3] = {1, g.pitch, g.plane};
   march<N3>(
-      g, [&](i64 c, int d, int, double* j) { phi_face(P, ps, F, c, d, st, j); },
+      g, P.prefetch != 0, [&](i64 c, int d, int, double* j) { phi_face(P, ps, F, c, d, st, j); },
       [&](i64 c, int z, const double* dv) {
         double div[N3];
 #pragma unroll
         for (int a = 0; a < N3; ++a) div[a] = dv[a] * P.inv_dx;
         phi_cell(P, g, ps, ms, pd, c, z, div);
+      },
+      [&](i64 cp) {
+#pragma unroll
+        for (int a = 0; a < N3; ++a) pf_l2(ps + a * F + cp);
+        pf_l2(ms + cp);
       });
 }
 
-template <int L>
-__global__ void __launch_bounds__(TXP * TYP) k_mu_march(Params P, Geom g, const double* __restrict__ ps,
+template <int L, int MB>
+__global__ void __launch_bounds__(TXP * TYP, MB) k_mu_march(Params P, Geom g, const double* __restrict__ ps,
                                                         const double* __restrict__ pd, const double* __restrict__ ms,
                                                         double* __restrict__ md) {
   const i64 F = g.field;
   const i64 st[3] = {1, g.pitch, g.plane};
   march<1>(
-      g,
+      g, P.prefetch != 0,
       [&](i64 c, int d, int z, double* f) {
         // T at the face: plane z for x / y faces, z + 1/2 for the face z | z+1 [A13]
         const double Tf = fma(P.Tdz, d == 2 ? z + 0.5 : (double)z, P.Tbase);
         f[0] = mu_face<L>(P, ps, pd, ms, F, c, d, st, Tf);
       },
-      [&](i64 c, int z, const double* dv) { mu_cell(P, g, ps, pd, ms, md, c, z, dv[0] * P.inv_dx); });
+      [&](i64 c, int z, const double* dv) { mu_cell(P, g, ps, pd, ms, md, c, z, dv[0] * P.inv_dx); },
+      [&](i64 cp) {
+#pragma unroll
+        for (int a = 0; a < N3; ++a) {
+          pf_l2(ps + a * F + cp);
+          pf_l2(pd + a * F + cp);
+        }
+        pf_l2(ms + cp);
+      });
 }
 
 }  // namespace p2
@@ -466,8 +489,18 @@ void p2_fill_params(const pf_params& p, int liquid, void* out) {
   P.liquid = liquid;
   P.aniso = p.aniso ? 1 : 0;
   P.mu_inf = p.mu_inf[0];
+  const char* e = getenv("PF_P2_PREFETCH");
+  P.prefetch = e ? atoi(e) : 1;
 }
 size_t p2_params_size() { return sizeof(p2::Params); }
+
+// CTAs per SM the z-marching kernels are compiled for: 4 (128 registers, a
+// 24-64 B spill) by default -- 7.08 vs 6.25 GLUP/s at 256^3 for 3 (168
+// registers, no spill), same-box A/B (profiles/r02_ab_p2.json); PF_P2_MINB=3
+static int p2_minb() {
+  const char* e = getenv("PF_P2_MINB");
+  return e && atoi(e) == 3 ? 3 : 4;
+}
 
 // PF_P2_NAIVE=1: the one-thread-per-cell kernels (every face twice)
 static bool p2_naive() {
@@ -486,7 +519,10 @@ void p2_launch_phi(const void* Pv, double Tbase, const Geom& g, const double* ps
   }
   dim3 b(p2::TXP, p2::TYP), gr((g.nx + p2::TXP - 1) / p2::TXP, (g.ny + p2::TYP - 1) / p2::TYP,
                                (g.nz + p2::ZCP - 1) / p2::ZCP);
-  p2::k_phi_march<<<gr, b, 0, s>>>(P, g, ps, ms, pd);
+  if (p2_minb() == 4)
+    p2::k_phi_march<4><<<gr, b, 0, s>>>(P, g, ps, ms, pd);
+  else
+    p2::k_phi_march<3><<<gr, b, 0, s>>>(P, g, ps, ms, pd);
 }
 
 void p2_launch_mu(const void* Pv, double Tbase, const Geom& g, const double* ps, const double* pd, const double* ms,
@@ -504,11 +540,15 @@ void p2_launch_mu(const void* Pv, double Tbase, const Geom& g, const double* ps,
   }
   dim3 b(p2::TXP, p2::TYP), gr((g.nx + p2::TXP - 1) / p2::TXP, (g.ny + p2::TYP - 1) / p2::TYP,
                                (g.nz + p2::ZCP - 1) / p2::ZCP);
+#define PF_P2_MU(LL)                                                        \
+  (p2_minb() == 4 ? (p2::k_mu_march<LL, 4><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md)) \
+                  : (p2::k_mu_march<LL, 3><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md)))
   switch (P.liquid) {  // the liquid index as a compile-time constant (register-resident face arrays)
-    case 0: p2::k_mu_march<0><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md); break;
-    case 1: p2::k_mu_march<1><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md); break;
-    default: p2::k_mu_march<2><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md); break;
+    case 0: PF_P2_MU(0); break;
+    case 1: PF_P2_MU(1); break;
+    default: PF_P2_MU(2); break;
   }
+#undef PF_P2_MU
 }
 
 }  // namespace pf
