@@ -25,8 +25,19 @@
 #include <vector>
 
 #include "pf_internal.h"
+#include <nvtx3/nvToolsExt.h>  // header-only NVTX3: ranges for nsys / ncu timelines (no cost without a tool)
 
 using namespace pf;
+
+namespace {
+// scoped NVTX range on the host thread around the enqueue of one phase of a
+// step (phi-sweep, ghosts / exchange, mu-sweep, window); with a profiler
+// attached the ranges line up with the kernels they enqueue
+struct NvtxRange {
+  explicit NvtxRange(const char* m) { nvtxRangePushA(m); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
+}  // namespace
 
 
 // ---------------------------------------------------------------------------
@@ -977,6 +988,7 @@ int pf_set_params(pf_ctx* ctx, const pf_params* p) {
 // x_done: the producing sweep already wrote the x ghost columns (Geom::xwrap)
 static int fill_ghost_dims(pf_ctx* ctx, double* f, int ncomp, bool is_mu, int d0, int d1, cudaStream_t st,
                            bool x_done = false) {
+  NvtxRange nr(is_mu ? "pf mu ghosts / exchange" : "pf phi ghosts / exchange");
   const double* dir = is_mu ? ctx->hp.mu_inf : nullptr;
   const bool any_ex = ctx->first_ex < 3;
   const bool skipx = x_done;
@@ -1260,6 +1272,7 @@ static int step_impl(pf_ctx* ctx, bool phi_only, bool dry = false) {
       ctx->cfg.bc_lo[2] != PF_BC_PERIODIC)
     return step_slabs(ctx, ps, pd, ms, md, dry);
   // Algorithm 1, line 1: phi-sweep (reads no mu ghosts: may overlap the previous mu exchange)
+  NvtxRange nr_step("pf step: phi-sweep, phi ghosts, mu-sweep, mu ghosts");
   prof_begin(ctx, 0, &e0);
   if (ctx->variant == PF_VARIANT_NAIVE)
     launch_phi_naive(ctx->dp, g, ps, ms, pd, ctx->stream);
@@ -1443,6 +1456,7 @@ static int step_graph(pf_ctx* ctx, int k) {
 
 int pf_step(pf_ctx* ctx, int64_t nsteps) {
   if (!ctx) return PF_EINVAL;
+  NvtxRange nr("pf_step");
   if (!ctx->have_params || !ctx->have_fields) return fail(ctx, PF_ESTATE, "pf_step before pf_set_params/pf_init_fields");
   if (nsteps < 0) return fail(ctx, PF_EINVAL, "nsteps < 0");
   // graphs pay from ~128^3 cells per block (tools/graph_probe.py: 32^3 slower,
@@ -1657,6 +1671,7 @@ int pf_shift_window(pf_ctx* ctx, int k) {
 }
 
 static int window_maybe(pf_ctx* ctx) {
+  NvtxRange nr("pf window check");
   const int nc = ctx->hp.window_check;
   if (nc <= 0 || ctx->step % nc != 0) return PF_OK;
   int H = -1;
