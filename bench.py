@@ -199,7 +199,7 @@ def main():
     ap.add_argument("--config", default="weak", choices=["weak", "strong"],
                     help="weak: config 2/3 (n^3 DS block per GPU); strong: config 4 (fixed 512x512x1024 "
                          "periodic domain, z-slabs)")
-    ap.add_argument("--variant", default="jit", choices=["jit", "tuned", "naive"])
+    ap.add_argument("--variant", default="jit", choices=["jit", "tuned", "naive", "split"])
     ap.add_argument("--autotune", type=int, default=2, metavar="PASSES",
                     help="run pf_autotune (coordinate search over the JIT tuning knobs, timed on this block) with "
                          "this many passes before the warm-up; 0 = built-in defaults")
@@ -283,9 +283,12 @@ def main():
         g.set_tuning(json.loads(args.tuning))
     if args.autotune > 0 and args.variant == "jit":
         t_at = time.time()
-        rep = g.autotune(passes=args.autotune, reps=5)  # collective: same choice on every rank
+        # collective: same choice on every rank; with the kernel-variant ablation
+        # (full / split / fused, NEXT-2) on the single-GPU weak workload
+        rep = g.autotune(passes=args.autotune, reps=5, variants=(world == 1 and not strong))
         tune_rep = {"passes": args.autotune, "seconds": round(time.time() - t_at, 1),
-                    "phi": rep["phi"], "mu": rep["mu"], "tried": len(rep["tried"])}
+                    "phi": rep["phi"], "mu": rep["mu"], "step": rep.get("step"), "variants": rep.get("variants"),
+                    "tried": len(rep["tried"])}
 
     def barrier():
         if dist is not None:

@@ -64,6 +64,14 @@ extern "C" {
 #define PF_VARIANT_JIT 2   /* default: the tuned kernels specialised at run time
                               (NVRTC) with the parameters and the block
                               geometry as compile-time constants */
+#define PF_VARIANT_SPLIT 3 /* the paper's "split" kernels: a
+                              staggered kernel stores every face flux in a
+                              global array (12 doubles per cell for phi, 6 for
+                              mu), a cell kernel reads them back; bitwise equal
+                              to PF_VARIANT_NAIVE ("full").  The staggered
+                              array (12 x field doubles, 1.9 GB at 256^3) is
+                              allocated by the library on first use and freed
+                              by pf_destroy -- the one buffer it owns.     */
 
 typedef struct pf_ctx pf_ctx;
 
@@ -323,7 +331,16 @@ int pf_tuning_check(const pf_tuning* t, char* log, int logn);
  * unchanged.  Needs params and fields (PF_ESTATE otherwise) and the JIT
  * variant.  On return the context uses the best tuning found; `log` (may be
  * NULL) receives a JSON document with every candidate and its time,
- * truncated to logn bytes.  Synchronous.                                   */
+ * truncated to logn bytes.  Synchronous.
+ * Step level (mask has PF_PHI and PF_MU): the step schedules (two sweeps vs
+ * the z-slab pipeline, tuning sched / slab) are timed as whole dry steps
+ * (every kernel of a step, scratch level only, no swap) and the faster is
+ * kept; with PF_AUTOTUNE_VARIANTS in `mask` the "full" (PF_VARIANT_NAIVE)
+ * and "split" (PF_VARIANT_SPLIT, which allocates its staggered array) kernel
+ * variants are timed the same way and reported ("variants" in the log); the
+ * context keeps PF_VARIANT_JIT unless one of them is faster (S§8(f) NEXT-2:
+ * full vs split vs fused).                                      */
+#define PF_AUTOTUNE_VARIANTS 4u
 int pf_autotune(pf_ctx* ctx, unsigned mask, int passes, int reps, char* log, int logn);
 
 /* Optional per-kernel timing with CUDA events on the compute stream:

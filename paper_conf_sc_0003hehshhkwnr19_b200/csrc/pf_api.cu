@@ -206,6 +206,7 @@ struct pf_ctx {
   // P2 parameterisation (3 phases, 1 mu, anisotropic phi; pf_p2.cu)
   bool p2 = false;
   int nph = PF_N, nmu = PF_M;
+  double* stag = nullptr;  // PF_VARIANT_SPLIT: staggered face fluxes (library-owned, freed by pf_destroy)
   std::vector<unsigned char> p2par;
   bool collective() const { return comm != nullptr || lg != nullptr; }
   // profiling
@@ -781,6 +782,7 @@ int pf_destroy(pf_ctx* ctx) {
   }
   drop_graphs(ctx);
   jit_release(ctx);
+  if (ctx->stag) cudaFree(ctx->stag);
   if (ctx->comm) g_nccl.CommDestroy(ctx->comm);
   if (ctx->lg) {
     std::lock_guard<std::mutex> lk(ctx->lg->m);
@@ -1142,6 +1144,8 @@ static int launch_mu(pf_ctx* ctx, const TileSel* ts, dim3 grid, const double* ps
                      const double* ms, double* md) {
   if (ctx->variant == PF_VARIANT_NAIVE)
     launch_mu_naive(ctx->dp, ctx->g, ps, pd, ms, md, ctx->stream);
+  else if (ctx->variant == PF_VARIANT_SPLIT)
+    launch_mu_split(ctx->dp, ctx->g, ps, pd, ms, ctx->stag, md, ctx->stream);
   else if (ctx->variant == PF_VARIANT_JIT)
     CU(jit_launch_mu(ctx->jmu, ctx->dp, ts, grid, ps, pd, ms, md, ctx->stream, ctx->cap_sv));
   else
@@ -1260,7 +1264,11 @@ static int step_impl(pf_ctx* ctx, bool phi_only, bool dry = false) {
   }
   // overlap: the exchanged dimensions' ghosts travel on the
   // comm stream while the mu-sweep updates the tiles that do not read them
-  const bool ov = ctx->overlap && ctx->first_ex < 3 && ctx->variant != PF_VARIANT_NAIVE && !phi_only;
+  const bool ov = ctx->overlap && ctx->first_ex < 3 && ctx->variant != PF_VARIANT_NAIVE &&
+                  ctx->variant != PF_VARIANT_SPLIT && !phi_only;
+  if (ctx->variant == PF_VARIANT_SPLIT && !ctx->stag) {  // the staggered array of the split kernels
+    CU(cudaMalloc(&ctx->stag, 12 * (size_t)g.field * sizeof(double) + 256));
+  }
   // the specialised phi-sweep writes phi_dst's x ghost columns itself (tuning phi_xghost)
   const bool phi_x_done = g.xwrap && ctx->variant == PF_VARIANT_JIT && ctx->tune.phi_xghost;
   // z-slab schedule (tuning sched = 1, S§7 step 6 (ii)): per slab of mu
@@ -1276,6 +1284,8 @@ static int step_impl(pf_ctx* ctx, bool phi_only, bool dry = false) {
   prof_begin(ctx, 0, &e0);
   if (ctx->variant == PF_VARIANT_NAIVE)
     launch_phi_naive(ctx->dp, g, ps, ms, pd, ctx->stream);
+  else if (ctx->variant == PF_VARIANT_SPLIT)
+    launch_phi_split(ctx->dp, g, ps, ms, ctx->stag, pd, ctx->stream);
   else if (ctx->variant == PF_VARIANT_JIT)
     CU(jit_launch_phi(ctx->jphi, ctx->dp, ps, ms, pd, ctx->stream, ctx->cap_sv));
   else
@@ -1575,7 +1585,8 @@ int pf_set_state(pf_ctx* ctx, const pf_state* s) {
 }
 
 int pf_set_variant(pf_ctx* ctx, int variant) {
-  if (!ctx || (variant != PF_VARIANT_TUNED && variant != PF_VARIANT_NAIVE && variant != PF_VARIANT_JIT))
+  if (!ctx || (variant != PF_VARIANT_TUNED && variant != PF_VARIANT_NAIVE && variant != PF_VARIANT_JIT &&
+               variant != PF_VARIANT_SPLIT))
     return PF_EINVAL;
   ctx->variant = variant;
   drop_graphs(ctx);
@@ -1989,6 +2000,33 @@ int pf_autotune(pf_ctx* ctx, unsigned mask, int passes, int reps, char* log, int
     snprintf(b, sizeof b, ", \"step\": {\"two_sweeps_ms\": %.6f, \"best_ms\": %.6f, \"sched\": %d, \"slab\": %d}", tm[0],
              tm[bi], best.sched, best.slab);
     kj += b;
+    if (mask & PF_AUTOTUNE_VARIANTS) {
+      // kernel variants of the paper: full (every face flux
+      // evaluated by both cells) and split (staggered fluxes through a global
+      // array) against the fused on-chip JIT sweeps, as whole dry steps
+      double tj = tm[bi], tv[2] = {INFINITY, INFINITY};
+      const int vs[2] = {PF_VARIANT_NAIVE, PF_VARIANT_SPLIT};
+      for (int i = 0; i < 2; ++i) {
+        ctx->variant = vs[i];
+        if (int r = time_steps(ctx, reps, &tv[i])) {
+          ctx->variant = PF_VARIANT_JIT;
+          return r;
+        }
+      }
+      if (ctx->collective()) {
+        double* d = (double*)ctx->red;
+        CU(cudaMemcpyAsync(d, tv, 2 * sizeof(double), cudaMemcpyHostToDevice, ctx->stream));
+        if (int r = allreduce_max(ctx, d, 2)) return r;
+        CU(cudaMemcpyAsync(tv, d, 2 * sizeof(double), cudaMemcpyDeviceToHost, ctx->stream));
+        CU(cudaStreamSynchronize(ctx->stream));
+      }
+      ctx->variant = PF_VARIANT_JIT;
+      if (tv[0] < tj * 0.99 || tv[1] < tj * 0.99) ctx->variant = tv[0] < tv[1] ? vs[0] : vs[1];
+      snprintf(b, sizeof b,
+               ", \"variants\": {\"fused_jit_ms\": %.6f, \"full_ms\": %.6f, \"split_ms\": %.6f, \"chosen\": %d}", tj,
+               tv[0], tv[1], ctx->variant);
+      kj += b;
+    }
   }
   // the scratch level's ghosts were overwritten: nothing reads them before the next sweep writes it
   CU(cudaStreamSynchronize(ctx->stream));

@@ -23,6 +23,11 @@ void launch_mu_naive(const DevParams& P, const Geom& g, const double* ps, const 
                      double* md, cudaStream_t s);
 void launch_phi_tuned(const DevParams& P, const Geom& g, const double* ps, const double* ms, double* pd,
                       cudaStream_t s);
+// split variant: staggered fluxes through the global array J (12 x g.field doubles)
+void launch_phi_split(const DevParams& P, const Geom& g, const double* ps, const double* ms, double* J, double* pd,
+                      cudaStream_t s);
+void launch_mu_split(const DevParams& P, const Geom& g, const double* ps, const double* pd, const double* ms,
+                     double* J, double* md, cudaStream_t s);
 // ts == nullptr: all tiles (grid ignored); else the selected tiles of `grid`
 void launch_mu_tuned(const DevParams& P, const Geom& g, const TileSel* ts, dim3 grid, const double* ps,
                      const double* pd, const double* ms, double* md, cudaStream_t s);

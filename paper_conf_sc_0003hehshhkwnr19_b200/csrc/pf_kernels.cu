@@ -148,6 +148,138 @@ void launch_mu_naive(const DevParams& P, const Geom& g, const double* ps, const 
 }
 
 // ---------------------------------------------------------------------------
+// Split kernels (the paper's "split" variant; Table 1 "partial"):
+// a staggered kernel evaluates each face flux once and stores it in a global
+// array J[d][comp] (the flux of the face c - e_d / 2, for cells c in
+// [0, n] per axis), a cell kernel reads the six fluxes of its cell back.  The
+// face and cell arithmetic is the naive kernels', in the same order, so the
+// results are bitwise equal to PF_VARIANT_NAIVE.
+// ---------------------------------------------------------------------------
+template <int L, bool TA>
+__global__ void __launch_bounds__(256) k_phi_stag(DevParams P, Geom g, const double* __restrict__ ps,
+                                                  double* __restrict__ J) {
+  const int x = blockIdx.x * blockDim.x + threadIdx.x;
+  const int y = blockIdx.y * blockDim.y + threadIdx.y;
+  const int z = blockIdx.z * blockDim.z + threadIdx.z;
+  if (x > g.nx || y > g.ny || z > g.nz) return;
+  const int64_t c = g.at(x, y, z), F = g.field;
+  double q[N];
+#pragma unroll
+  for (int a = 0; a < N; ++a) q[a] = __ldg(ps + a * F + c);
+#pragma unroll
+  for (int d = 0; d < 3; ++d) {
+    const int64_t st = d == 0 ? 1 : (d == 1 ? g.pitch : g.plane);
+    double p[N], j[N];
+#pragma unroll
+    for (int a = 0; a < N; ++a) p[a] = __ldg(ps + a * F + c - st);
+    phi_face(P, p, q, j);
+#pragma unroll
+    for (int a = 0; a < N; ++a) J[(d * N + a) * F + c] = j[a];
+  }
+}
+
+template <int L, bool TA>
+__global__ void __launch_bounds__(256) k_phi_cellsplit(DevParams P, Geom g, const double* __restrict__ ps,
+                                                       const double* __restrict__ ms, const double* __restrict__ J,
+                                                       double* __restrict__ pd) {
+  const int x = blockIdx.x * blockDim.x + threadIdx.x;
+  const int y = blockIdx.y * blockDim.y + threadIdx.y;
+  const int z = blockIdx.z * blockDim.z + threadIdx.z;
+  if (x >= g.nx || y >= g.ny || z >= g.nz) return;
+  const int64_t c = g.at(x, y, z), F = g.field;
+  double ph[N], gd[N][3], divh[N] = {0.0, 0.0, 0.0, 0.0};
+#pragma unroll
+  for (int a = 0; a < N; ++a) ph[a] = __ldg(ps + a * F + c);
+#pragma unroll
+  for (int d = 0; d < 3; ++d) {
+    const int64_t st = d == 0 ? 1 : (d == 1 ? g.pitch : g.plane);
+#pragma unroll
+    for (int a = 0; a < N; ++a) {
+      gd[a][d] = __ldg(ps + a * F + c + st) - __ldg(ps + a * F + c - st);
+      divh[a] += __ldg(J + (d * N + a) * F + c + st) - __ldg(J + (d * N + a) * F + c);
+    }
+  }
+  const double mu0 = __ldg(ms + c), mu1 = __ldg(ms + F + c);
+  double out[N], xi[N];
+  xi_of(P, P.step, x + g.x0, y + g.y0, z + g.z0, xi);
+  phi_cell<TA>(P, plane_T(P, P, (double)z), ph, gd, divh, mu0, mu1, xi, out);
+#pragma unroll
+  for (int a = 0; a < N; ++a) pd[a * F + c] = out[a];
+}
+
+template <int L, bool TA>
+__global__ void __launch_bounds__(256) k_mu_stag(DevParams P, Geom g, const double* __restrict__ ps,
+                                                 const double* __restrict__ pd, const double* __restrict__ ms,
+                                                 double* __restrict__ J) {
+  const int x = blockIdx.x * blockDim.x + threadIdx.x;
+  const int y = blockIdx.y * blockDim.y + threadIdx.y;
+  const int z = blockIdx.z * blockDim.z + threadIdx.z;
+  if (x > g.nx || y > g.ny || z > g.nz) return;
+  const int64_t c = g.at(x, y, z), F = g.field;
+  const double Tc = plane_T(P, P, (double)z);
+#pragma unroll 1
+  for (int d = 0; d < 3; ++d) {
+    const int64_t sn = d == 0 ? 1 : (d == 1 ? g.pitch : g.plane);
+    const int64_t s1 = d == 0 ? g.pitch : 1;
+    const int64_t s2 = d == 2 ? g.pitch : g.plane;
+    const double Tm = d == 2 ? plane_T(P, P, z - 0.5) : Tc;
+    FaceSide sm, s0;
+    load_side<L>(ps, pd, ms, F, c - sn, s1, s2, sm);
+    load_side<L>(ps, pd, ms, F, c, s1, s2, s0);
+    double Fm[M];
+    mu_face<L, TA>(P, Tm, sm, s0, Fm);
+#pragma unroll
+    for (int i = 0; i < M; ++i) J[(d * M + i) * F + c] = Fm[i];
+  }
+}
+
+template <int L, bool TA>
+__global__ void __launch_bounds__(256) k_mu_cellsplit(DevParams P, Geom g, const double* __restrict__ ps,
+                                                      const double* __restrict__ pd, const double* __restrict__ ms,
+                                                      const double* __restrict__ J, double* __restrict__ md) {
+  const int x = blockIdx.x * blockDim.x + threadIdx.x;
+  const int y = blockIdx.y * blockDim.y + threadIdx.y;
+  const int z = blockIdx.z * blockDim.z + threadIdx.z;
+  if (x >= g.nx || y >= g.ny || z >= g.nz) return;
+  const int64_t c = g.at(x, y, z), F = g.field;
+  const double Tc = plane_T(P, P, (double)z);
+  double divh[M] = {0.0, 0.0};
+#pragma unroll
+  for (int d = 0; d < 3; ++d) {
+    const int64_t sn = d == 0 ? 1 : (d == 1 ? g.pitch : g.plane);
+#pragma unroll
+    for (int i = 0; i < M; ++i) divh[i] += __ldg(J + (d * M + i) * F + c + sn) - __ldg(J + (d * M + i) * F + c);
+  }
+  double ph[N], dph[N], mu[M], out[M];
+#pragma unroll
+  for (int a = 0; a < N; ++a) {
+    ph[a] = __ldg(ps + a * F + c);
+    dph[a] = __ldg(pd + a * F + c) - ph[a];
+  }
+#pragma unroll
+  for (int i = 0; i < M; ++i) mu[i] = __ldg(ms + i * F + c);
+  mu_cell<TA>(P, Tc, ph, dph, mu, divh, out);
+#pragma unroll
+  for (int i = 0; i < M; ++i) md[i * F + c] = out[i];
+}
+
+void launch_phi_split(const DevParams& P, const Geom& g, const double* ps, const double* ms, double* J, double* pd,
+                      cudaStream_t s) {
+  dim3 b(32, 4, 2), gs((g.nx + 1 + 31) / 32, (g.ny + 1 + 3) / 4, (g.nz + 1 + 1) / 2),
+      gc((g.nx + 31) / 32, (g.ny + 3) / 4, (g.nz + 1) / 2);
+  PF_DISPATCH(P.liquid, P.TA, (k_phi_stag<LL, TT><<<gs, b, 0, s>>>(P, g, ps, J)));
+  PF_DISPATCH(P.liquid, P.TA, (k_phi_cellsplit<LL, TT><<<gc, b, 0, s>>>(P, g, ps, ms, J, pd)));
+}
+
+void launch_mu_split(const DevParams& P, const Geom& g, const double* ps, const double* pd, const double* ms,
+                     double* J, double* md, cudaStream_t s) {
+  dim3 b(32, 4, 2), gs((g.nx + 1 + 31) / 32, (g.ny + 1 + 3) / 4, (g.nz + 1 + 1) / 2),
+      gc((g.nx + 31) / 32, (g.ny + 3) / 4, (g.nz + 1) / 2);
+  PF_DISPATCH(P.liquid, P.TA, (k_mu_stag<LL, TT><<<gs, b, 0, s>>>(P, g, ps, pd, ms, J)));
+  PF_DISPATCH(P.liquid, P.TA, (k_mu_cellsplit<LL, TT><<<gc, b, 0, s>>>(P, g, ps, pd, ms, J, md)));
+}
+
+// ---------------------------------------------------------------------------
 // Ghost layers (Alg. 1 lines 2 and 4, "communication and boundary handling").
 // Every ghost cell is written from interior values by a per-axis index map,
 // which equals the ordered x -> y -> z fill (edges and corners consistent,

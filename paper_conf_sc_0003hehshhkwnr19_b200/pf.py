@@ -20,7 +20,7 @@ PF_OK, PF_EINVAL, PF_ENOMEM, PF_ECUDA, PF_ENCCL, PF_ESTATE, PF_ENUMERIC = 0, -1,
 BC = {"periodic": 0, "neumann": 1, "dirichlet_mu": 2}
 PF_HOST, PF_DEVICE = 0, 1
 PF_PHI, PF_MU = 1, 2
-VARIANT = {"tuned": 0, "naive": 1, "jit": 2}
+VARIANT = {"tuned": 0, "naive": 1, "jit": 2, "split": 3}
 N, M = 4, 2
 
 
@@ -424,12 +424,14 @@ class PhaseField:
         t = PFTuning(*[cur[k] for k in TUNING_KNOBS])
         self._check(self.lib.pf_set_tuning(self._h, C.byref(t)), "pf_set_tuning")
 
-    def autotune(self, mask: int = PF_PHI | PF_MU, passes: int = 1, reps: int = 7) -> dict:
+    def autotune(self, mask: int = PF_PHI | PF_MU, passes: int = 1, reps: int = 7, variants: bool = False) -> dict:
         """pf_autotune: coordinate search over the tuning knobs, timed on this
         block; returns the JSON report (start, best, per-kernel times, every
         candidate).  The context keeps the best tuning."""
         import json
         buf = C.create_string_buffer(1 << 16)
+        if variants:  # PF_AUTOTUNE_VARIANTS: also time the full and split variants (S§8(f) NEXT-2)
+            mask |= 4
         self._check(self.lib.pf_autotune(self._h, int(mask), int(passes), int(reps), buf, len(buf)), "pf_autotune")
         return json.loads(buf.value.decode())
 

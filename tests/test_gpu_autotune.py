@@ -249,8 +249,10 @@ def test_autotune_step_schedule(pfmod):
     g = pfmod.PhaseField(shape, P, bc=I.BC_DS)
     g.init_fields(phi, mu)
     before = g.download()
-    rep = g.autotune(passes=1, reps=3)
+    rep = g.autotune(passes=1, reps=3, variants=True)
     after = g.download()
     assert np.array_equal(before[0], after[0]) and np.array_equal(before[1], after[1])
     assert "step" in rep and rep["step"]["sched"] in (0, 1)
+    v = rep["variants"]
+    assert v["chosen"] == 2 and v["fused_jit_ms"] < v["full_ms"] and v["fused_jit_ms"] < v["split_ms"], v
     assert any(c["kernel"] == "step" for c in rep["tried"])

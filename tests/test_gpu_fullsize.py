@@ -36,13 +36,16 @@ def omod():
     return O
 
 
+ZF = NFULL // 2 + 2  # bench.py: the growing front starts two planes above the window threshold
+
+
 @pytest.fixture(scope="module")
 def bench_case(pfmod):
-    """The bench.py workload: 256^3, DS BCs, C.4 'ds' parameters, IC-L."""
+    """The bench.py workload: 256^3, DS BCs, C.4 parameters with the growing
+    front (inputs.DS_BENCH), IC-L."""
     n = NFULL
-    P = I.params_c4("ds", window_check=10, window_frac=0.5)
-    P["T0"] = I.ds_T0(n // 4, P["G"])
-    phi, mu = I.ic_lamellar((n, n, n), seed=20191117, z_front=n // 4)
+    P = I.params_ds_growth(ZF, window_check=10, window_frac=0.5, **I.DS_BENCH)
+    phi, mu = I.ic_lamellar((n, n, n), seed=20191117, z_front=ZF)
     g = pfmod.PhaseField((n, n, n), P, bc=I.BC_DS)
     g.init_fields(phi, mu)
     g.step(1)
@@ -60,7 +63,7 @@ def test_sampled_cells_match_oracle(omod, bench_case):
     n = NFULL
     rng = np.random.default_rng(20191117)
     # samples: random interior, around the front, and at the z boundaries
-    zs = list(rng.integers(2, n - 2, 120)) + list(rng.integers(n // 4 - 8, n // 4 + 8, 60)) + [0, 1, 2, n - 3, n - 2, n - 1]
+    zs = list(rng.integers(2, n - 2, 120)) + list(rng.integers(ZF - 8, ZF + 8, 60)) + [0, 1, 2, n - 3, n - 2, n - 1]
     ys = rng.integers(0, n, len(zs))
     xs = rng.integers(0, n, len(zs))
     Pq = dict(P, window_check=0)
@@ -125,3 +128,37 @@ def test_fullsize_periodic_translation(pfmod):
     h.step(20)
     b = h.download()
     assert np.array_equal(roll(a[0]), b[0]) and np.array_equal(roll(a[1]), b[1])
+
+
+def test_p2_fullsize_sampled_cells(pfmod, omod):
+    """P2 (NEXT-4) in the configuration bench.py times: 256^3 periodic,
+    params_p2, IC-V; one step on the GPU, sampled cells against the oracle on
+    5^3 periodic sub-blocks (the 19-point phi stencil still has radius 1,
+    so a step reads radius 2)."""
+    n = NFULL
+    P = I.params_p2()
+    phi, mu = I.ic_voronoi((n, n, n), seed=20191117, N=3, M=1)
+    g = pfmod.PhaseField((n, n, n), P)
+    g.init_fields(phi, mu)
+    g.step(1)
+    gp, gm = g.download()
+    g.close()
+    assert np.abs(gp.sum(0) - 1.0).max() <= 8 * 2.2e-16 and gp.min() >= 0.0
+    rng = np.random.default_rng(7)
+    # samples in interfaces (where every term is active) and anywhere
+    mixed = np.argwhere(phi.max(0) < 0.99)
+    pick = mixed[rng.integers(0, len(mixed), 120)]
+    anyc = rng.integers(0, n, (40, 3))
+    errp = errm = 0.0
+    scale_p, scale_m = np.abs(gp).max(), np.abs(gm).max()
+    for z, y, x in list(pick) + list(anyc):
+        zr, yr, xr = np.arange(z - 2, z + 3) % n, np.arange(y - 2, y + 3), np.arange(x - 2, x + 3)
+        sp = _sub_block(phi, zr, yr, xr).copy()
+        sm = _sub_block(mu, zr, yr, xr).copy()
+        o = omod.Oracle((5, 5, 5), P)
+        o.init(sp, sm)
+        o.step(1)
+        op, om = o.download()
+        errp = max(errp, np.abs(op[:, 2, 2, 2] - gp[:, z, y, x]).max())
+        errm = max(errm, np.abs(om[:, 2, 2, 2] - gm[:, z, y, x]).max())
+    assert errp / scale_p <= 1e-12 and errm / scale_m <= 1e-12, (errp / scale_p, errm / scale_m)

@@ -58,7 +58,7 @@ def run_pair(pfmod, omod, shape, P, ic, steps, bc=None, seed=20191117, variant="
     return out
 
 
-@pytest.mark.parametrize("variant", ["jit", "tuned", "naive"])
+@pytest.mark.parametrize("variant", ["jit", "tuned", "naive", "split"])
 @pytest.mark.parametrize("pset", ["c4", "stress"])
 @pytest.mark.parametrize("ic", ["R", "V", "L"])
 def test_one_step_parity(pfmod, omod, variant, pset, ic):
@@ -143,7 +143,7 @@ def test_ds_window_parity(pfmod, omod):
 # Dirichlet-mu ghost at z_hi [A15] differs from the interior from step 1 on
 # (IC-R: mu ~ U(-0.1, 0.1)), A1 != 0 and G v != 0 (frozen T with a Q term),
 # window inflow mu = mu_inf [A16].
-@pytest.mark.parametrize("variant", ["jit", "tuned", "naive"])
+@pytest.mark.parametrize("variant", ["jit", "tuned", "naive", "split"])
 @pytest.mark.parametrize("window", [0, 1])
 def test_ds_stress_one_step(pfmod, omod, variant, window):
     P = I.params_stress(window_check=window, window_frac=0.5)
@@ -427,3 +427,22 @@ def test_e2e_pinned_roundtrip(pfmod):
     om = torch.empty_like(tm).pin_memory()
     g.download(out=(op, om))
     assert np.array_equal(op.numpy(), phi) and np.array_equal(om.numpy(), mu)
+
+
+def test_split_variant_bitwise_equals_full(pfmod):
+    """The split kernels (staggered fluxes through a global array, the
+    paper's "split" variant) evaluate the same face and cell arithmetic in
+    the same order as the full (naive) kernels: bitwise equal, DS + window."""
+    P = I.params_stress(window_check=4, window_frac=0.5, xi_amp=0.02, xi_seed=5)
+    shape = (24, 18, 37)
+    phi, mu = I.ic_lamellar(shape, seed=4, z_front=14, mu_inf=tuple(P["mu_inf"]))
+    outs = []
+    for v in ("naive", "split"):
+        g = pfmod.PhaseField(shape, P, bc=I.BC_DS)
+        g.set_variant(v)
+        g.init_fields(phi, mu)
+        g.step(12)
+        outs.append((g.download(), g.state()))
+        g.close()
+    assert outs[0][1] == outs[1][1] and outs[0][1]["z_off"] > 0
+    assert np.array_equal(outs[0][0][0], outs[1][0][0]) and np.array_equal(outs[0][0][1], outs[1][0][1])
