@@ -273,7 +273,8 @@ typedef struct {
   int mu_qreg;       /* 1: own cell's face-side data kept in registers from the
                         build (no shared-memory re-read; needs registers)        */
   int mu_ldhint;     /* L1 policy of the mu-sweep's phi_dst / mu loads: 0 default,
-                        1 evict_first, 2 no_allocate                              */
+                        1 evict_first, 2 no_allocate, 3 no_allocate and the
+                        two-rows sweep's own phi_src(k+2) loads evict_last        */
   int mu_hpipe;      /* 1: halo-ring cells' loads for plane k+1 issued at the end of
                         plane k's face phase (software pipelining)               */
   int mu_cly;        /* mu-sweep thread-block clusters of 1, 2 or 4 tiles stacked in
@@ -303,6 +304,15 @@ typedef struct {
                         k-1 in tensor memory (tcgen05.st / ld, 68 columns per
                         thread) instead of registers, and re-reads the own
                         sides of the x / y faces from shared memory             */
+  int mu_hcar;       /* 1: the two-rows mu-sweep carries the phi_src z column of
+                        its halo ring in shared memory (a 3-plane ring): a halo
+                        cell loads phi_src(k+1), the solids' phi_dst and mu per
+                        plane (9 loads, not 26) and takes its tangential / z
+                        differences from the ring; mu_rpt = 2, mu_hpipe = 0   */
+  int mu_xshfl;      /* 1: the two-rows mu-sweep takes the x-neighbours' phi_src
+                        of its own cells from the neighbour lanes' carried
+                        values (warp shuffles; lanes 0 / 31 load the halo
+                        column) instead of two L1 loads; mu_rpt = 2, mu_rpf = 1 */
 } pf_tuning;
 
 /* The built-in defaults (the measured best at 256^3 on one B200,

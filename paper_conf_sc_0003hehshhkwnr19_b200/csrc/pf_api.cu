@@ -1746,7 +1746,7 @@ const std::vector<TuneKnob>& tune_knobs() {
       {"mu_halo_l1", &pf_tuning::mu_halo_l1, JIT_MU, {0, 1}},
       {"mu_fxreg", &pf_tuning::mu_fxreg, JIT_MU, {0, 1}},
       {"mu_qreg", &pf_tuning::mu_qreg, JIT_MU, {0, 1}},
-      {"mu_ldhint", &pf_tuning::mu_ldhint, JIT_MU, {0, 1, 2}},
+      {"mu_ldhint", &pf_tuning::mu_ldhint, JIT_MU, {0, 1, 2, 3}},
       {"mu_hpipe", &pf_tuning::mu_hpipe, JIT_MU, {0, 1}},
       {"mu_cly", &pf_tuning::mu_cly, JIT_MU, {1, 2, 4}},
       {"mu_rot", &pf_tuning::mu_rot, JIT_MU, {0, 1}},
@@ -1755,6 +1755,8 @@ const std::vector<TuneKnob>& tune_knobs() {
       {"mu_pers", &pf_tuning::mu_pers, JIT_MU, {0, 1}},
       {"phi_pers", &pf_tuning::phi_pers, JIT_PHI, {0, 1}},
       {"mu_tmem", &pf_tuning::mu_tmem, JIT_MU, {0, 1}},
+      {"mu_hcar", &pf_tuning::mu_hcar, JIT_MU, {0, 1}},
+      {"mu_xshfl", &pf_tuning::mu_xshfl, JIT_MU, {0, 1}},
   };
   return k;
 }

@@ -56,8 +56,8 @@ constexpr int kPhiUnroll = PF_PHI_UNROLL;
 #ifndef PF_MU_ROT  // mu-sweep: tile rows (and their roles) rotated over the CTA's warps per tile
 #define PF_MU_ROT 0
 #endif
-#ifndef PF_MU_LDHINT  // L1 policy of the mu-sweep's phi_dst / mu loads: 0 default, 1 evict_first, 2 no_allocate
-#define PF_MU_LDHINT 0
+#ifndef PF_MU_LDHINT  // L1 policy of the mu-sweep's phi_dst / mu loads: 0 default, 1 evict_first, 2 no_allocate,
+#define PF_MU_LDHINT 0  // 3 no_allocate + the two-rows sweep's own phi_src(k+2) lines evict_last
 #endif
 // load of a phi_dst / mu value in the mu-sweep (used by at most the cells of
 // one plane: a hint keeps these lines from evicting the reused phi_src lines)
@@ -66,9 +66,19 @@ __device__ __forceinline__ double ldh(const double* p) {
   double v;
   asm("ld.global.nc.L1::evict_first.f64 %0, [%1];" : "=d"(v) : "l"(p));
   return v;
-#elif PF_MU_LDHINT == 2
+#elif PF_MU_LDHINT >= 2
   double v;
   asm("ld.global.nc.L1::no_allocate.f64 %0, [%1];" : "=d"(v) : "l"(p));
+  return v;
+#else
+  return __ldg(p);
+#endif
+}
+// load of an own phi_src line that the x / y differences re-read two planes later
+__device__ __forceinline__ double ldkeep(const double* p) {
+#if PF_MU_LDHINT == 3
+  double v;
+  asm("ld.global.nc.L1::evict_last.f64 %0, [%1];" : "=d"(v) : "l"(p));
   return v;
 #else
   return __ldg(p);
@@ -113,6 +123,12 @@ constexpr int MU_TY = PF_MU_TY;
 #endif
 #ifndef PF_MU_TMEM  // two-rows mu-sweep: the carried side of plane k-1 in tensor memory (TMEM), not registers
 #define PF_MU_TMEM 0
+#endif
+#ifndef PF_MU_HCAR  // two-rows mu-sweep: the halo ring's phi_src z column carried in shared memory
+#define PF_MU_HCAR 0
+#endif
+#ifndef PF_MU_XSHFL  // two-rows mu-sweep: own cd_x from the lane neighbours' carried phi_src (shuffles)
+#define PF_MU_XSHFL 0
 #endif
 #ifndef PF_MU_PERS  // two-rows mu-sweep: full launches persistent (balanced tile-plane shares)
 #define PF_MU_PERS 0
@@ -1128,6 +1144,43 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
   else if (th >= 2 * MTY + MTX && th < 2 * MTY + 2 * MTX) { hx = th - 2 * MTY - MTX + 1; hy = MTY + 1; hwx = true; }
   if (hwx || hwy) hs = hidx<MTX>(hx, hy);
   const int hgx = min(x0 + hx - 1, g.nx), hgy = min(y0 + hy - 1, g.ny);
+#if PF_MU_HCAR
+  // halo ring with its phi_src z column carried in shared memory (tuning
+  // mu_hcar): ring cell ci holds phi_src of planes k-1, k, k+1 in slots
+  // (k+2)%3, k%3, (k+1)%3, so a halo cell loads per plane only phi_src(k+1),
+  // the solids' phi_dst and mu (9 loads instead of 26; the 2 x MTY column
+  // cells are 16 lines per warp load).  Its tangential and z differences
+  // come from the ring: the same operands, so the same bits as build_cell.
+  // Ring order: left column (hy = 0..MTY+1), right column, bottom row
+  // (hx = 1..MTX), top row; the 4 corners are carried by threads 0..3.
+  constexpr int RC = 2 * (MTY + 2) + 2 * MTX;
+  static_assert(NT - 2 * MTX - 2 * MTY >= 4, "mu_hcar: four free threads carry the ring corners");
+  __shared__ __align__(16) double fring[3][N][RC];  // phase-major: a warp's ring reads are contiguous
+  auto ridx = [](int rx, int ry) {
+    return rx == 0 ? ry : rx == MTX + 1 ? MTY + 2 + ry : 2 * (MTY + 2) + (ry == 0 ? 0 : MTX) + rx - 1;
+  };
+  int ci = -1, tpi = 0, tmi = 0;
+  i64 cring = 0;
+  if (hs >= 0) {
+    ci = ridx(hx, hy);
+    tpi = hwx ? ridx(hx + 1, hy) : ridx(hx, hy + 1);
+    tmi = hwx ? ridx(hx - 1, hy) : ridx(hx, hy - 1);
+    cring = g.at(hgx, hgy, 0);
+  } else if (t < 4) {
+    const int chx = (t & 1) ? MTX + 1 : 0, chy = (t & 2) ? MTY + 1 : 0;
+    ci = ridx(chx, chy);
+    cring = g.at(min(x0 + chx - 1, g.nx), min(y0 + chy - 1, g.ny), 0);
+  }
+  if (ci >= 0) {
+    const double* f = ps + cring + (i64)(z0 - 1) * g.plane;
+#pragma unroll
+    for (int a = 0; a < N; ++a) {
+      fring[(z0 + 2) % 3][a][ci] = __ldg(f + a * F);
+      fring[z0 % 3][a][ci] = __ldg(f + a * F + g.plane);
+    }
+  }
+  __syncthreads();
+#endif
 
   FaceSide Dp[2];
   double dpl[2] = {0.0, 0.0};
@@ -1231,8 +1284,22 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
         const double* f1 = ps + a * F + c1;
         v0[D_F + a] = fcar[0][a];
         v1[D_F + a] = fcar[1][a];
+#if PF_MU_XSHFL
+        {
+          // phi_src(k) of the x-neighbours is the neighbour lane's carried
+          // value; lanes 0 / 31 load the halo column's (the same operands)
+          const bool edge = lane == 0 || lane == MTX - 1;
+          const int eo = lane == 0 ? -1 : 1;
+          const double e0 = edge ? __ldg(f0 + eo) : 0.0, e1 = edge ? __ldg(f1 + eo) : 0.0;
+          const double u0 = __shfl_up_sync(0xffffffffu, fcar[0][a], 1), d0 = __shfl_down_sync(0xffffffffu, fcar[0][a], 1);
+          const double u1 = __shfl_up_sync(0xffffffffu, fcar[1][a], 1), d1 = __shfl_down_sync(0xffffffffu, fcar[1][a], 1);
+          v0[D_CX + a] = (lane == MTX - 1 ? e0 : d0) - (lane == 0 ? e0 : u0);
+          v1[D_CX + a] = (lane == MTX - 1 ? e1 : d1) - (lane == 0 ? e1 : u1);
+        }
+#else
         v0[D_CX + a] = __ldg(f0 + 1) - __ldg(f0 - 1);
         v1[D_CX + a] = __ldg(f1 + 1) - __ldg(f1 - 1);
+#endif
         v0[D_CY + a] = fcar[1][a] - __ldg(f0 - g.pitch);
         v1[D_CY + a] = __ldg(f1 + g.pitch) - fcar[0][a];
 #if PF_MU_TMEM
@@ -1268,7 +1335,7 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
         const i64 c = r ? c1 : c0;
 #pragma unroll
         for (int a = 0; a < N; ++a) {
-          rnf[r][a] = __ldg(ps + a * F + c + 2 * g.plane);
+          rnf[r][a] = ldkeep(ps + a * F + c + 2 * g.plane);
           rnd[r][a] = ldh(pd + a * F + c + g.plane);
         }
         rnm[r][0] = ldh(ms + c + g.plane);
@@ -1288,7 +1355,41 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
 #endif
     }
 #endif
+#if PF_MU_HCAR
+    if (!last && ci >= 0) {
+      const i64 c = cring + (i64)k * g.plane;
+      const int sm = (k + 2) % 3, s0 = k % 3, sp = (k + 1) % 3;
+      double fn[N];
+#pragma unroll
+      for (int a = 0; a < N; ++a) fn[a] = __ldg(ps + a * F + c + g.plane);
+      if (hs >= 0) {
+        double v[D_NV];
+#pragma unroll
+        for (int a = 0; a < N; ++a) {
+          const double tt = fring[s0][a][tpi] - fring[s0][a][tmi];
+          v[D_F + a] = fring[s0][a][ci];
+          v[D_CX + a] = hwx ? tt : 0.0;
+          v[D_CY + a] = hwx ? 0.0 : tt;
+          v[D_CZ + a] = fn[a] - fring[sm][a][ci];
+          v[D_DP + a] = 0.0;  // the liquid's dphi of a halo cell is never read
+        }
+#pragma unroll
+        for (int u = 0; u < NSOL; ++u) {
+          const int a = solid_phase(L, u);
+          v[D_DP + a] = ldh(pd + a * F + c) - v[D_F + a];
+        }
+        v[D_MU + 0] = ldh(ms + c);
+        v[D_MU + 1] = ldh(ms + F + c);
+        double2* d = reinterpret_cast<double2*>(D + (size_t)hs * D_NV);
+#pragma unroll
+        for (int j = 0; j < D_NV / 2; ++j) d[j] = make_double2(v[2 * j], v[2 * j + 1]);
+      }
+#pragma unroll
+      for (int a = 0; a < N; ++a) fring[sp][a][ci] = fn[a];
+    }
+#else
     if (!last && hs >= 0) build_cell<NC>(g, ps, pd, ms, hgx, hgy, k, hwx, hwy, true, D, hs);
+#endif
     __syncthreads();
     // (b) z-faces k-1/2 and (c) cell updates of plane k-1
 #pragma unroll

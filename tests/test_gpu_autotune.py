@@ -61,6 +61,15 @@ CORNERS = [
     # persistent launches: balanced tile-plane shares, segments crossing tile columns
     {"mu_pers": 1, "phi_pers": 1},
     {"mu_pers": 1, "mu_ty": 6, "mu_minb": 3, "phi_pers": 1, "phi_ty": 8, "phi_minb": 2, "phi_xsh": 1},
+    # the halo ring's z column carried in shared memory (alone, ragged
+    # chunks, with persistent shares and with the TMEM side)
+    {"mu_hcar": 1},
+    {"mu_hcar": 1, "mu_zc": 7, "mu_ty": 6, "mu_minb": 3, "mu_rpf": 0},
+    {"mu_hcar": 1, "mu_pers": 1, "mu_ty": 10, "mu_minb": 2},
+    {"mu_hcar": 1, "mu_tmem": 1, "mu_halo_l1": 0},
+    # own cd_x by warp shuffles, L1 policies
+    {"mu_xshfl": 1},
+    {"mu_xshfl": 1, "mu_hcar": 1, "mu_ldhint": 3, "mu_ty": 6, "mu_minb": 3, "mu_zc": 5},
 ]
 
 
@@ -126,6 +135,8 @@ def test_set_tuning_rejects_out_of_range(pfmod):
         g.set_tuning({"phi_ty": 16, "phi_minb": 8})
     with pytest.raises(pfmod.PFError):
         g.set_tuning({"mu_ty": 5})  # odd tile height with two rows per thread
+    with pytest.raises(pfmod.PFError):
+        g.set_tuning({"mu_hcar": 1, "mu_hpipe": 1})
     g.set_tuning({"mu_ty": 6})
     assert g.tuning()["mu_ty"] == 6
     g.set_tuning(dict(R1, mu_ty=5))

@@ -100,10 +100,12 @@ def test_compute_sanitizer(tool):
     cs = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
     if not os.path.exists(cs):
         pytest.fail("compute-sanitizer not found")
-    variants = ["jit", "tuned", "naive"] if tool == "memcheck" else ["jit", "tuned"]
+    # memcheck: every kernel family (tools/sanitize_run.py); racecheck: the
+    # kernels that share tiles through shared / tensor memory
+    variants = [] if tool == "memcheck" else ["jit", "tuned", "split", "tunings", "p2"]
     cmd = [cs, "--tool", tool, "--error-exitcode", "1", sys.executable, os.path.join(ROOT, "tools", "sanitize_run.py"),
            *variants]
-    r = subprocess.run(cmd, capture_output=True, text=True, timeout=1500, cwd=ROOT)
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=2400, cwd=ROOT)
     tail = (r.stdout + r.stderr)[-3000:]
     assert r.returncode == 0, tail
     assert "sanitize run ok" in r.stdout, tail
