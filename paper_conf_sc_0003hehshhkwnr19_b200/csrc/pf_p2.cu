@@ -34,6 +34,7 @@ struct Params {
   double R[N3][N3][9];  // R_ab row-major
   int liquid, aniso;
   int prefetch;  // z-marching sweeps: own column's lines P2_PD planes ahead into L2 (PF_P2_PREFETCH, default 1)
+  int side_pd;   // side-staged mu-sweep: L2 prefetch distance in planes, 0 = off (PF_P2_SIDE_PD, default 2)
   double mu_inf;
 };
 
@@ -70,7 +71,8 @@ __device__ __forceinline__ void aniso_grad(const Params& P, int a, int b, const 
   // below 1e-280 the approximate reciprocal of n2^2 would flush to zero:
   // scale p by 2^300 (exact); A is homogeneous of degree 0 and grad_p f of
   // degree 1, so the result is scaled back by 2^-300
-  const double sc = n2 < 1e-280 ? 0x1p300 : 1.0;
+  const bool tiny = n2 < 1e-280;
+  const double sc = tiny ? 0x1p300 : 1.0, two_sc = tiny ? 0x1p-299 : 2.0;  // two_sc = 2 / sc (exact)
 #pragma unroll
   for (int i = 0; i < 3; ++i) v[i] *= sc;
   n2 *= sc * sc;
@@ -84,7 +86,7 @@ __device__ __forceinline__ void aniso_grad(const Params& P, int a, int b, const 
 #pragma unroll
   for (int i = 0; i < 3; ++i) {
     const double dAn2 = 16.0 * delta * v[i] * fma(v[i] * v[i], i2, -s4 * i4);
-    gp[i] = (2.0 / sc) * A * fma(A, v[i], dAn2);
+    gp[i] = two_sc * A * fma(A, v[i], dAn2);
   }
 #pragma unroll
   for (int j = 0; j < 3; ++j) out[j] = fma(R[j], gp[0], fma(R[3 + j], gp[1], R[6 + j] * gp[2]));
@@ -238,7 +240,37 @@ __global__ void __launch_bounds__(256) k_phi(Params P, Geom g, const double* __r
   phi_cell(P, g, ps, ms, pd, c, z, div);
 }
 
-// mu flux F = M grad mu - J_at at the face p | p+e_d (eqs. 8-10) [A7-A11], M = 1
+// mu flux F = M grad mu - J_at at a face in direction d (eqs. 8-10)
+// [A7-A11], M = 1, from the face operands: pb = mean phi, G = face gradient
+// (normal difference, means of the tangential central differences), dtp =
+// mean d_t phi, mb / dmu = mean / normal difference of mu
+template <int L>
+__device__ __forceinline__ double mu_flux(const Params& P, int d, const double (&pb)[N3], const double (&G)[N3][3],
+                                          const double (&dtp)[N3], double mb, double dmu, double Tf) {
+  // eq. 9: M = sum_a g(pb_a) D_a chi_a(T_f), chi_a = -2 A_a, g(x) = x [A4, A7]
+  double Mf = 0.0;
+#pragma unroll
+  for (int a = 0; a < N3; ++a) Mf = fma(pb[a] * P.D[a], -2.0 * fma(P.A1[a], Tf, P.A0[a]), Mf);
+  double Fl = Mf * dmu;
+  // eq. 10: J_at = (pi eps/4) sum_{s != l} g_s h_l / sqrt(phi_s phi_l) d_t phi_s (n_s . n_l)(c_l - c_s) n_s,d
+  const double nl2 = fma(G[L][0], G[L][0], fma(G[L][1], G[L][1], G[L][2] * G[L][2]));
+  const double cl = fma(-2.0 * fma(P.A1[L], Tf, P.A0[L]), mb, -fma(P.B1[L], Tf, P.B0[L]));
+#pragma unroll
+  for (int a = 0; a < N3; ++a) {
+    if (a == L) continue;
+    const double na2 = fma(G[a][0], G[a][0], fma(G[a][1], G[a][1], G[a][2] * G[a][2]));
+    if (!(pb[a] > 0.0 && pb[L] > 0.0 && na2 > 0.0 && nl2 > 0.0)) continue;  // [A11] exact-zero guards
+    // g h_l / sqrt(pb_a pb_l) (n_a . n_l) n_a,d = pb_a h_l (G_a . G_l) G_a,d / sqrt(pb_a pb_l nl2 na2^2):
+    // one reciprocal square root per solid (as the P1 mu_face)
+    const double dot = fma(G[a][0], G[L][0], fma(G[a][1], G[L][1], G[a][2] * G[L][2]));
+    const double w = P.at_c * h_of(pb[L]) * dtp[a] * pb[a] * rsqrt_nr(pb[a] * pb[L] * nl2 * na2 * na2);
+    const double ca = fma(-2.0 * fma(P.A1[a], Tf, P.A0[a]), mb, -fma(P.B1[a], Tf, P.B0[a]));
+    Fl -= w * (cl - ca) * (dot * G[a][d]);
+  }
+  return Fl;
+}
+
+// mu flux at the face p | p+e_d with its operands loaded from global memory
 template <int L>
 __device__ __forceinline__ double mu_face(const Params& P, const double* __restrict__ ps,
                                           const double* __restrict__ pd, const double* __restrict__ ms, i64 F, i64 c,
@@ -263,48 +295,36 @@ __device__ __forceinline__ double mu_face(const Params& P, const double* __restr
     dtp[a] = ((__ldg(pd + a * F + c) - vp) + (__ldg(pd + a * F + c + sn) - vq)) * (0.5 * P.inv_dt);
   }
   const double mp = __ldg(ms + c), mq = __ldg(ms + c + sn);
-  const double mb = 0.5 * (mp + mq), dmu = (mq - mp) * P.inv_dx;
-  // eq. 9: M = sum_a g(pb_a) D_a chi_a(T_f), chi_a = -2 A_a, g(x) = x [A4, A7]
-  double Mf = 0.0;
-#pragma unroll
-  for (int a = 0; a < N3; ++a) Mf = fma(pb[a] * P.D[a], -2.0 * fma(P.A1[a], Tf, P.A0[a]), Mf);
-  double Fl = Mf * dmu;
-  // eq. 10: J_at = (pi eps/4) sum_{s != l} g_s h_l / sqrt(phi_s phi_l) d_t phi_s (n_s . n_l)(c_l - c_s) n_s,d
-  const double nl2 = fma(G[L][0], G[L][0], fma(G[L][1], G[L][1], G[L][2] * G[L][2]));
-  const double cl = fma(-2.0 * fma(P.A1[L], Tf, P.A0[L]), mb, -fma(P.B1[L], Tf, P.B0[L]));
-#pragma unroll
-  for (int a = 0; a < N3; ++a) {
-    if (a == L) continue;
-    const double na2 = fma(G[a][0], G[a][0], fma(G[a][1], G[a][1], G[a][2] * G[a][2]));
-    if (!(pb[a] > 0.0 && pb[L] > 0.0 && na2 > 0.0 && nl2 > 0.0)) continue;  // [A11] exact-zero guards
-    // g h_l / sqrt(pb_a pb_l) (n_a . n_l) n_a,d = pb_a h_l (G_a . G_l) G_a,d / sqrt(pb_a pb_l nl2 na2^2):
-    // one reciprocal square root per solid (as the P1 mu_face)
-    const double dot = fma(G[a][0], G[L][0], fma(G[a][1], G[L][1], G[a][2] * G[L][2]));
-    const double w = P.at_c * h_of(pb[L]) * dtp[a] * pb[a] * rsqrt_nr(pb[a] * pb[L] * nl2 * na2 * na2);
-    const double ca = fma(-2.0 * fma(P.A1[a], Tf, P.A0[a]), mb, -fma(P.B1[a], Tf, P.B0[a]));
-    Fl -= w * (cl - ca) * (dot * G[a][d]);
-  }
-  return Fl;
+  return mu_flux<L>(P, d, pb, G, dtp, 0.5 * (mp + mq), (mq - mp) * P.inv_dx, Tf);
 }
 
 // mu cell update (C.1 S4 steps 2-3, eq. 8) of cell c at plane z given div
+// from mu, phi and dphi = phi_dst - phi_src of the cell
+__device__ __forceinline__ double mu_cell_v(const Params& P, int z, double mu, const double (&ph)[N3],
+                                            const double (&dph)[N3], double div) {
+  const double T = fma(P.Tdz, (double)z, P.Tbase);
+  double chi = 0.0, S = 0.0, Q = 0.0;
+#pragma unroll
+  for (int a = 0; a < N3; ++a) {
+    const double A = fma(P.A1[a], T, P.A0[a]), B = fma(P.B1[a], T, P.B0[a]);
+    const double h = h_of(ph[a]);
+    chi = fma(h, -2.0 * A, chi);                                            // chi = sum h_a chi_a
+    S = fma(fma(-2.0 * A, mu, -B) * dh_of(ph[a]), dph[a] * P.inv_dt, S);  // sum c_a h'_a d_t phi_a [A12]
+    Q = fma(h, fma(-2.0 * P.A1[a], mu, -P.B1[a]) * P.dTdt, Q);              // sum h_a dc_a/dT d_t T
+  }
+  return fma(P.dt * rcp_nr(chi), div - S - Q, mu);
+}
 __device__ __forceinline__ void mu_cell(const Params& P, const Geom& g, const double* __restrict__ ps,
                                         const double* __restrict__ pd, const double* __restrict__ ms,
                                         double* __restrict__ md, i64 c, int z, double div) {
   const i64 F = g.field;
-  const double T = fma(P.Tdz, (double)z, P.Tbase);
-  const double mu = __ldg(ms + c);
-  double chi = 0.0, S = 0.0, Q = 0.0;
+  double ph[N3], dph[N3];
 #pragma unroll
   for (int a = 0; a < N3; ++a) {
-    const double ph = __ldg(ps + a * F + c), phn = __ldg(pd + a * F + c);
-    const double A = fma(P.A1[a], T, P.A0[a]), B = fma(P.B1[a], T, P.B0[a]);
-    const double h = h_of(ph);
-    chi = fma(h, -2.0 * A, chi);                                            // chi = sum h_a chi_a
-    S = fma(fma(-2.0 * A, mu, -B) * dh_of(ph), (phn - ph) * P.inv_dt, S);  // sum c_a h'_a d_t phi_a [A12]
-    Q = fma(h, fma(-2.0 * P.A1[a], mu, -P.B1[a]) * P.dTdt, Q);              // sum h_a dc_a/dT d_t T
+    ph[a] = __ldg(ps + a * F + c);
+    dph[a] = __ldg(pd + a * F + c) - ph[a];
   }
-  md[c] = fma(P.dt * rcp_nr(chi), div - S - Q, mu);
+  md[c] = mu_cell_v(P, z, __ldg(ms + c), ph, dph, div);
 }
 
 template <int L>
@@ -444,6 +464,207 @@ __global__ void __launch_bounds__(TXP * TYP, MB) k_mu_march(Params P, Geom g, co
       });
 }
 
+// ---------------------------------------------------------------------------
+// mu-sweep with the face operands staged in shared memory (default; the
+// z-marching k_mu_march above with PF_P2_MU=march).  A CTA of 32 x TYS
+// threads owns a 32 x TYS column tile and marches a z-chunk; per plane k
+// every cell of the tile and of its one-cell halo ring publishes its side
+//   S = (phi, cd_x, cd_y, cd_z, dphi = phi_dst - phi_src, mu)
+// to shared memory once (an own cell loads 14 values, its z column carried
+// in registers; a halo cell 19), the -x / -y faces of plane k read both
+// sides from there, the z-face k-1 | k pairs the own side of plane k-1
+// (registers) with that of plane k, and the cell update of plane k-1 follows
+// it (one-plane lag, as the P1 mu-sweep).  The faces' operands are the same
+// differences as mu_face's loads, through the same mu_flux: same bits.
+// ---------------------------------------------------------------------------
+constexpr int TYS = 8, ZCS = 16;
+constexpr int SHX = TXP + 2, SNC = SHX * (TYS + 2);  // halo-tile cells
+// shared side layout, component-major [SV][SNC] (a warp's reads are contiguous)
+constexpr int S_F = 0, S_CX = 3, S_CY = 6, S_CZ = 9, S_DP = 12, S_MU = 15, SV = 16;
+__device__ __forceinline__ int sidx(int hx, int hy) { return hy * SHX + hx; }
+
+struct Side {
+  double f[N3], c1[N3], c2[N3], dp[N3], m;  // c1 / c2: central differences along the two tangential axes
+};
+__device__ __forceinline__ void side_ld(const double (*S)[SNC], int i, int o1, int o2, Side& s) {
+#pragma unroll
+  for (int a = 0; a < N3; ++a) {
+    s.f[a] = S[S_F + a][i];
+    s.c1[a] = S[o1 + a][i];
+    s.c2[a] = S[o2 + a][i];
+    s.dp[a] = S[S_DP + a][i];
+  }
+  s.m = S[S_MU][i];
+}
+// flux at the face p | q in direction d (tangential axes in ascending order in c1, c2)
+template <int L>
+__device__ __forceinline__ double mu_face_side(const Params& P, int d, const Side& p, const Side& q, double Tf) {
+  double pb[N3], G[N3][3], dtp[N3];
+#pragma unroll
+  for (int a = 0; a < N3; ++a) {
+    pb[a] = 0.5 * (p.f[a] + q.f[a]);
+    const double gn = (q.f[a] - p.f[a]) * P.inv_dx;
+    const double t1 = (p.c1[a] + q.c1[a]) * (0.25 * P.inv_dx), t2 = (p.c2[a] + q.c2[a]) * (0.25 * P.inv_dx);
+    G[a][0] = d == 0 ? gn : t1;
+    G[a][1] = d == 1 ? gn : (d == 0 ? t1 : t2);
+    G[a][2] = d == 2 ? gn : t2;
+    dtp[a] = (p.dp[a] + q.dp[a]) * (0.5 * P.inv_dt);
+  }
+  return mu_flux<L>(P, d, pb, G, dtp, 0.5 * (p.m + q.m), (q.m - p.m) * P.inv_dx, Tf);
+}
+
+template <int L>
+__global__ void __launch_bounds__(TXP * TYS, 2) k_mu_side(Params P, Geom g, const double* __restrict__ ps,
+                                                         const double* __restrict__ pd,
+                                                         const double* __restrict__ ms, double* __restrict__ md) {
+  __shared__ double S[SV][SNC];
+  __shared__ double fxs[TYS][TXP + 1];  // -x flux of every cell, +x of the right tile edge at TXP
+  __shared__ double fys[TYS + 1][TXP];  // -y flux of every cell, +y of the top tile edge at TYS
+  const i64 F = g.field;
+  const int lane = threadIdx.x, w = threadIdx.y, t = w * TXP + lane;
+  constexpr int NT = TXP * TYS;
+  const int x0 = blockIdx.x * TXP, y0 = blockIdx.y * TYS;
+  const int x = x0 + lane, y = y0 + w;
+  const bool active = x < g.nx && y < g.ny;
+  const int xc = min(x, g.nx), yc = min(y, g.ny);
+  const int me = sidx(lane + 1, w + 1);
+  const int z0 = blockIdx.z * ZCS, z1 = min(z0 + ZCS, g.nz);
+  // halo ring: the last 2 TXP + 2 TYS threads, one cell each (columns first)
+  const int th = t - (NT - 2 * TXP - 2 * TYS);
+  int hx = 0, hy = 0;
+  bool hcol = false;
+  if (th >= 0 && th < 2 * TYS) {
+    hcol = true;
+    hx = th < TYS ? 0 : TXP + 1;
+    hy = (th < TYS ? th : th - TYS) + 1;
+  } else if (th >= 2 * TYS) {
+    const int r = th - 2 * TYS;
+    hx = (r < TXP ? r : r - TXP) + 1;
+    hy = r < TXP ? 0 : TYS + 1;
+  }
+  const int hs = th >= 0 ? sidx(hx, hy) : -1;
+  const i64 hoff = th >= 0 ? g.at(min(x0 + hx - 1, g.nx), min(y0 + hy - 1, g.ny), 0) : 0;
+  const i64 htan = hcol ? g.pitch : 1;  // the halo cell's in-plane tangential axis (y for columns, x for rows)
+  const i64 coff = g.at(xc, yc, 0);
+
+  // own side of plane z0 - 1 (z-face operands: f, cd_x, cd_y, dphi, mu) and the carried phi column
+  Side Sp;
+  double fc[N3], fm[N3];
+  const bool pfl = (lane & 15) == 0 || th >= 0;  // one L2 prefetch per 128-B line of the own rows; halo cells
+  const i64 pfo = th >= 0 ? hoff : coff;
+  {
+    const i64 c = coff + (i64)(z0 - 1) * g.plane;
+#pragma unroll
+    for (int a = 0; a < N3; ++a) {
+      const double* f = ps + a * F + c;
+      Sp.f[a] = __ldg(f);
+      Sp.c1[a] = __ldg(f + 1) - __ldg(f - 1);
+      Sp.c2[a] = __ldg(f + g.pitch) - __ldg(f - g.pitch);
+      Sp.dp[a] = __ldg(pd + a * F + c) - Sp.f[a];
+      fm[a] = Sp.f[a];
+      fc[a] = __ldg(f + g.plane);
+    }
+    Sp.m = __ldg(ms + c);
+  }
+  double divxy = 0.0, Fzm = 0.0;
+  for (int k = z0; k <= z1; ++k) {
+    const bool last = k == z1;
+    const i64 c = coff + (i64)k * g.plane;
+    if (P.side_pd && pfl && k + P.side_pd <= z1) {
+      const i64 cp = pfo + (i64)(k + P.side_pd) * g.plane;
+#pragma unroll
+      for (int a = 0; a < N3; ++a) {
+        pf_l2(ps + a * F + cp);
+        pf_l2(pd + a * F + cp);
+      }
+      pf_l2(ms + cp);
+    }
+    // (a) publish the sides of plane k
+    Side Q;  // own side, tangential (x, y) for the z-face
+    double cz[N3];
+#pragma unroll
+    for (int a = 0; a < N3; ++a) {
+      const double* f = ps + a * F + c;
+      const double fp = !last ? __ldg(f + g.plane) : 0.0;
+      Q.f[a] = fc[a];
+      Q.c1[a] = __ldg(f + 1) - __ldg(f - 1);
+      Q.c2[a] = __ldg(f + g.pitch) - __ldg(f - g.pitch);
+      cz[a] = !last ? fp - fm[a] : 0.0;
+      Q.dp[a] = __ldg(pd + a * F + c) - fc[a];
+      fm[a] = fc[a];
+      fc[a] = fp;
+    }
+    Q.m = __ldg(ms + c);
+    if (!last) {
+#pragma unroll
+      for (int a = 0; a < N3; ++a) {
+        S[S_F + a][me] = Q.f[a];
+        S[S_CX + a][me] = Q.c1[a];
+        S[S_CY + a][me] = Q.c2[a];
+        S[S_CZ + a][me] = cz[a];
+        S[S_DP + a][me] = Q.dp[a];
+      }
+      S[S_MU][me] = Q.m;
+      if (hs >= 0) {
+        const i64 ch = hoff + (i64)k * g.plane;
+#pragma unroll
+        for (int a = 0; a < N3; ++a) {
+          const double* f = ps + a * F + ch;
+          const double v = __ldg(f), tt = __ldg(f + htan) - __ldg(f - htan);
+          S[S_F + a][hs] = v;
+          S[S_CX + a][hs] = hcol ? 0.0 : tt;
+          S[S_CY + a][hs] = hcol ? tt : 0.0;
+          S[S_CZ + a][hs] = __ldg(f + g.plane) - __ldg(f - g.plane);
+          S[S_DP + a][hs] = __ldg(pd + a * F + ch) - v;
+        }
+        S[S_MU][hs] = __ldg(ms + ch);
+      }
+    }
+    __syncthreads();
+    // (b) z-face k-1 | k and (c) the cell update of plane k-1
+    const double Fz = mu_face_side<L>(P, 2, Sp, Q, fma(P.Tdz, (k - 1) + 0.5, P.Tbase));
+    if (k > z0 && active) {
+      const double div = divxy + (Fz - Fzm);
+      md[c - g.plane] = mu_cell_v(P, k - 1, Sp.m, Sp.f, Sp.dp, div * P.inv_dx);
+    }
+    Fzm = Fz;
+    if (last) break;
+    // (d) x / y faces of plane k: -x and -y of every cell, + the far tile edges
+    const double Tk = fma(P.Tdz, (double)k, P.Tbase);
+    Side p, q;
+#pragma unroll
+    for (int a = 0; a < N3; ++a) {
+      q.f[a] = Q.f[a];
+      q.c1[a] = Q.c2[a];  // tangential y, z
+      q.c2[a] = cz[a];
+      q.dp[a] = Q.dp[a];
+    }
+    q.m = Q.m;
+    side_ld(S, me - 1, S_CY, S_CZ, p);
+    const double Fx = mu_face_side<L>(P, 0, p, q, Tk);
+#pragma unroll
+    for (int a = 0; a < N3; ++a) q.c1[a] = Q.c1[a];  // tangential x, z
+    side_ld(S, me - SHX, S_CX, S_CZ, p);
+    const double Fy = mu_face_side<L>(P, 1, p, q, Tk);
+    fxs[w][lane] = Fx;
+    fys[w][lane] = Fy;
+    if (w == 0 && lane < TYS) {  // +x face of the right tile edge, row `lane`
+      side_ld(S, sidx(TXP, lane + 1), S_CY, S_CZ, p);
+      side_ld(S, sidx(TXP + 1, lane + 1), S_CY, S_CZ, q);
+      fxs[lane][TXP] = mu_face_side<L>(P, 0, p, q, Tk);
+    } else if (w == 1) {  // +y face of the top tile edge, column `lane`
+      side_ld(S, sidx(lane + 1, TYS), S_CX, S_CZ, p);
+      side_ld(S, sidx(lane + 1, TYS + 1), S_CX, S_CZ, q);
+      fys[TYS][lane] = mu_face_side<L>(P, 1, p, q, Tk);
+    }
+    __syncthreads();
+    divxy = (fxs[w][lane + 1] - Fx) + (fys[w + 1][lane] - Fy);
+#pragma unroll
+    for (int a = 0; a < N3; ++a) Sp.f[a] = Q.f[a], Sp.c1[a] = Q.c1[a], Sp.c2[a] = Q.c2[a], Sp.dp[a] = Q.dp[a];
+    Sp.m = Q.m;
+  }
+}
+
 }  // namespace p2
 
 // ---------------------------------------------------------------------------
@@ -491,6 +712,8 @@ void p2_fill_params(const pf_params& p, int liquid, void* out) {
   P.mu_inf = p.mu_inf[0];
   const char* e = getenv("PF_P2_PREFETCH");
   P.prefetch = e ? atoi(e) : 1;
+  const char* e2 = getenv("PF_P2_SIDE_PD");
+  P.side_pd = e2 ? atoi(e2) : 2;
 }
 size_t p2_params_size() { return sizeof(p2::Params); }
 
@@ -500,6 +723,12 @@ size_t p2_params_size() { return sizeof(p2::Params); }
 static int p2_minb() {
   const char* e = getenv("PF_P2_MINB");
   return e && atoi(e) == 3 ? 3 : 4;
+}
+
+// PF_P2_MU=march: the z-marching mu kernel instead of the side-staged one
+static bool p2_mu_march() {
+  const char* e = getenv("PF_P2_MU");
+  return e && e[0] == 'm';
 }
 
 // PF_P2_NAIVE=1: the one-thread-per-cell kernels (every face twice)
@@ -535,6 +764,16 @@ void p2_launch_mu(const void* Pv, double Tbase, const Geom& g, const double* ps,
       case 0: p2::k_mu<0><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md); break;
       case 1: p2::k_mu<1><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md); break;
       default: p2::k_mu<2><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md); break;
+    }
+    return;
+  }
+  if (!p2_mu_march()) {
+    dim3 b(p2::TXP, p2::TYS), gr((g.nx + p2::TXP - 1) / p2::TXP, (g.ny + p2::TYS - 1) / p2::TYS,
+                                 (g.nz + p2::ZCS - 1) / p2::ZCS);
+    switch (P.liquid) {
+      case 0: p2::k_mu_side<0><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md); break;
+      case 1: p2::k_mu_side<1><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md); break;
+      default: p2::k_mu_side<2><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md); break;
     }
     return;
   }

@@ -7,7 +7,8 @@ term) stepped with
   * specialised tunings that select other kernel bodies: persistent
     phi / mu CTAs, the TMEM-carried side of the two-rows mu-sweep, one row
     per thread, cluster kernels, and the z-slab step schedule,
-  * the P2 kernels (z-marching and one-thread-per-cell),
+  * the P2 kernels (z-marching phi, side-staged and z-marching mu,
+    one-thread-per-cell),
   * a 2 x 2 x 1 multi-block run over the in-process transport (pack /
     unpack kernels, zero-copy z planes, interior / shell overlap).
 
@@ -58,8 +59,9 @@ def p2_runs():
     outs = []
     P = I.params_p2_stress(window_check=2, window_frac=0.5, v=0.05)
     phi, mu = I.ic_voronoi((20, 12, 33), seed=5, N=3, M=1)
-    for naive in ("0", "1"):
+    for naive, mu in (("0", "side"), ("0", "march"), ("1", "side")):
         os.environ["PF_P2_NAIVE"] = naive
+        os.environ["PF_P2_MU"] = mu
         g = pf.PhaseField((20, 12, 33), P, bc=I.BC_DS)
         g.init_fields(phi, mu)
         g.step(3)
@@ -67,6 +69,7 @@ def p2_runs():
         outs.append(g.download())
         g.close()
     os.environ.pop("PF_P2_NAIVE", None)
+    os.environ.pop("PF_P2_MU", None)
     return outs
 
 
@@ -122,9 +125,9 @@ def main():
         assert close(o, outs[0]), "variants / tunings disagree"
     n += len(outs)
     if "p2" in groups:
-        a, b = p2_runs()
-        assert close(a, b), "P2 march / naive disagree"
-        n += 2
+        a, b, c = p2_runs()
+        assert close(a, b) and close(a, c), "P2 kernels disagree"
+        n += 3
     if "multiblock" in groups:
         multiblock_run()
         n += 1
