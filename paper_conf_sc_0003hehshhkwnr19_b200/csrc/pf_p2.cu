@@ -9,9 +9,12 @@
 // makes phi the heavy kernel of P2 (Table 1: 3968 normalised FLOPs,
 // P:L1234-1243).  The mu equation (eqs. 8-10) is the P1 one with M = 1.
 //
-// Default: z-marching sweeps, every face flux evaluated once (below);
-// PF_P2_NAIVE=1: one thread per cell, every face evaluated by both of its
-// cells (the paper's "full" kernels).  Written from the paper;
+// Default: side-staged z-marching sweeps (k_phi_side, k_mu_side: every face
+// flux evaluated once, both sides of a face from shared memory);
+// PF_P2_PHI=march / PF_P2_MU=march: z-marching sweeps that load the face
+// operands from global memory (k_phi_march, k_mu_march); PF_P2_NAIVE=1: one
+// thread per cell, every face evaluated by both of its cells (the paper's
+// "full" kernels).  Written from the paper;
 // parity against the oracle in tests/test_gpu_p2.py.
 // Independent of oracle/ (no shared code).
 #include <math.h>
@@ -92,28 +95,11 @@ __device__ __forceinline__ void aniso_grad(const Params& P, int a, int b, const 
   for (int j = 0; j < 3; ++j) out[j] = fma(R[j], gp[0], fma(R[3 + j], gp[1], R[6 + j] * gp[2]));
 }
 
-// staggered phi flux (d-component of d a / d grad phi_a) at the face p | p+e_d;
-// f = phi_src, c = cell offset of p, st[d] = stride of axis d
-__device__ __forceinline__ void phi_face(const Params& P, const double* __restrict__ f, i64 F, i64 c, int d,
-                                         const i64 st[3], double j[N3]) {
-  const i64 sn = st[d];
-  double pb[N3], G[N3][3];
-#pragma unroll
-  for (int b = 0; b < N3; ++b) {
-    const double vp = __ldg(f + b * F + c), vq = __ldg(f + b * F + c + sn);
-    pb[b] = 0.5 * (vp + vq);
-#pragma unroll
-    for (int e = 0; e < 3; ++e) {
-      if (e == d) {
-        G[b][e] = (vq - vp) * P.inv_dx;
-      } else {
-        const i64 t = st[e];
-        G[b][e] = ((__ldg(f + b * F + c + t) - __ldg(f + b * F + c - t)) +
-                   (__ldg(f + b * F + c + sn + t) - __ldg(f + b * F + c + sn - t))) *
-                  (0.25 * P.inv_dx);
-      }
-    }
-  }
+// staggered phi flux (d-component of d a / d grad phi_a) at a face in
+// direction d from its operands: pb = mean phi, G = face gradient (normal
+// difference, means of the tangential central differences)
+__device__ __forceinline__ void phi_flux(const Params& P, int d, const double (&pb)[N3], const double (&G)[N3][3],
+                                         double j[N3]) {
 #pragma unroll
   for (int a = 0; a < N3; ++a) j[a] = 0.0;
   if (!P.aniso) {  // isotropic (A = 1): 2 sum_b gamma_ab pb_b (pb_b G_a,d - pb_a G_b,d)
@@ -138,6 +124,31 @@ __device__ __forceinline__ void phi_face(const Params& P, const double* __restri
     }
 }
 
+// phi flux at the face p | p+e_d with its operands loaded from global memory;
+// f = phi_src, c = cell offset of p, st[d] = stride of axis d
+__device__ __forceinline__ void phi_face(const Params& P, const double* __restrict__ f, i64 F, i64 c, int d,
+                                         const i64 st[3], double j[N3]) {
+  const i64 sn = st[d];
+  double pb[N3], G[N3][3];
+#pragma unroll
+  for (int b = 0; b < N3; ++b) {
+    const double vp = __ldg(f + b * F + c), vq = __ldg(f + b * F + c + sn);
+    pb[b] = 0.5 * (vp + vq);
+#pragma unroll
+    for (int e = 0; e < 3; ++e) {
+      if (e == d) {
+        G[b][e] = (vq - vp) * P.inv_dx;
+      } else {
+        const i64 t = st[e];
+        G[b][e] = ((__ldg(f + b * F + c + t) - __ldg(f + b * F + c - t)) +
+                   (__ldg(f + b * F + c + sn + t) - __ldg(f + b * F + c + sn - t))) *
+                  (0.25 * P.inv_dx);
+      }
+    }
+  }
+  phi_flux(P, d, pb, G, j);
+}
+
 __device__ __forceinline__ void project3(double x[N3]) {
   double u0 = x[0], u1 = x[1], u2 = x[2], t;
   if (u1 > u0) { t = u0; u0 = u1; u1 = t; }
@@ -151,23 +162,17 @@ __device__ __forceinline__ void project3(double x[N3]) {
   for (int a = 0; a < N3; ++a) x[a] = fmax(x[a] - th, 0.0);
 }
 
-// phi cell update (C.1 S2 steps 2-8) of cell c at plane z, given the flux
-// divergence div (eq. 11)
-__device__ __forceinline__ void phi_cell(const Params& P, const Geom& g, const double* __restrict__ ps,
-                                         const double* __restrict__ ms, double* __restrict__ pd, i64 c, int z,
-                                         const double div[N3]) {
-  const i64 F = g.field;
-  const i64 st[3] = {1, g.pitch, g.plane};
-  double ph[N3], gd[N3][3];
-#pragma unroll
-  for (int a = 0; a < N3; ++a) ph[a] = __ldg(ps + a * F + c);
+// phi cell update (C.1 S2 steps 2-8) at plane z from its operands: phi,
+// the raw central differences cd[b][d] = phi_b(+e_d) - phi_b(-e_d), mu and
+// the flux divergence div (eq. 11); out = phi_dst
+__device__ __forceinline__ void phi_cell_v(const Params& P, int z, const double (&ph)[N3], const double (&cd)[N3][3],
+                                           double mu, const double (&div)[N3], double (&out)[N3]) {
   // 2. cell-centred gradients (central differences) [A10]
+  double gd[N3][3];
 #pragma unroll
   for (int b = 0; b < N3; ++b)
 #pragma unroll
-    for (int d = 0; d < 3; ++d)
-      gd[b][d] = (__ldg(ps + b * F + c + st[d]) - __ldg(ps + b * F + c - st[d])) * (0.5 * P.inv_dx);
-  const double mu = __ldg(ms + c);
+    for (int d = 0; d < 3; ++d) gd[b][d] = cd[b][d] * (0.5 * P.inv_dx);
   const double T = fma(P.Tdz, (double)z, P.Tbase);
   // da/dphi_a = sum_{b != a} gamma_ab grad_q f(q_ab) . g_b,  q_ab = phi_a g_b - phi_b g_a
   double dad[N3] = {0.0, 0.0, 0.0};
@@ -211,10 +216,24 @@ __device__ __forceinline__ void phi_cell(const Params& P, const Geom& g, const d
     }
   const double f = den != 0.0 ? P.dt_over_eps * (den * rcp_nr(num)) : P.dt_over_eps * P.inv_tau_mean;
   const double rbar = (r[0] + r[1] + r[2]) * (1.0 / 3.0);
-  double out[N3];
 #pragma unroll
   for (int a = 0; a < N3; ++a) out[a] = fma(f, rbar - r[a], ph[a]);
   project3(out);
+}
+// phi cell update of cell c at plane z with its operands loaded from global memory
+__device__ __forceinline__ void phi_cell(const Params& P, const Geom& g, const double* __restrict__ ps,
+                                         const double* __restrict__ ms, double* __restrict__ pd, i64 c, int z,
+                                         const double (&div)[N3]) {
+  const i64 F = g.field;
+  const i64 st[3] = {1, g.pitch, g.plane};
+  double ph[N3], cd[N3][3], out[N3];
+#pragma unroll
+  for (int a = 0; a < N3; ++a) ph[a] = __ldg(ps + a * F + c);
+#pragma unroll
+  for (int b = 0; b < N3; ++b)
+#pragma unroll
+    for (int d = 0; d < 3; ++d) cd[b][d] = __ldg(ps + b * F + c + st[d]) - __ldg(ps + b * F + c - st[d]);
+  phi_cell_v(P, z, ph, cd, __ldg(ms + c), div, out);
 #pragma unroll
   for (int a = 0; a < N3; ++a) pd[a * F + c] = out[a];
 }
@@ -665,6 +684,205 @@ __global__ void __launch_bounds__(TXP * TYS, 2) k_mu_side(Params P, Geom g, cons
   }
 }
 
+// ---------------------------------------------------------------------------
+// phi-sweep with the face operands staged in shared memory (default;
+// k_phi_march with PF_P2_PHI=march): the scheme of k_mu_side with
+// the side (phi, cd_x, cd_y, cd_z) and three fluxes per face; the cell update
+// takes phi, the central differences and mu of the own cell from registers.
+// ---------------------------------------------------------------------------
+constexpr int P_F = 0, P_CX = 3, P_CY = 6, P_CZ = 9, PV = 12;
+struct PSide {
+  double f[N3], c1[N3], c2[N3];
+};
+__device__ __forceinline__ void pside_ld(const double (*S)[SNC], int i, int o1, int o2, PSide& s) {
+#pragma unroll
+  for (int a = 0; a < N3; ++a) {
+    s.f[a] = S[P_F + a][i];
+    s.c1[a] = S[o1 + a][i];
+    s.c2[a] = S[o2 + a][i];
+  }
+}
+__device__ __forceinline__ void phi_face_side(const Params& P, int d, const PSide& p, const PSide& q, double j[N3]) {
+  double pb[N3], G[N3][3];
+#pragma unroll
+  for (int a = 0; a < N3; ++a) {
+    pb[a] = 0.5 * (p.f[a] + q.f[a]);
+    const double gn = (q.f[a] - p.f[a]) * P.inv_dx;
+    const double t1 = (p.c1[a] + q.c1[a]) * (0.25 * P.inv_dx), t2 = (p.c2[a] + q.c2[a]) * (0.25 * P.inv_dx);
+    G[a][0] = d == 0 ? gn : t1;
+    G[a][1] = d == 1 ? gn : (d == 0 ? t1 : t2);
+    G[a][2] = d == 2 ? gn : t2;
+  }
+  phi_flux(P, d, pb, G, j);
+}
+
+__global__ void __launch_bounds__(TXP * TYS, 2) k_phi_side(Params P, Geom g, const double* __restrict__ ps,
+                                                          const double* __restrict__ ms, double* __restrict__ pd) {
+  __shared__ double S[PV][SNC];
+  __shared__ double fxs[N3][TYS][TXP + 1];
+  __shared__ double fys[N3][TYS + 1][TXP];
+  const i64 F = g.field;
+  const int lane = threadIdx.x, w = threadIdx.y, t = w * TXP + lane;
+  constexpr int NT = TXP * TYS;
+  const int x0 = blockIdx.x * TXP, y0 = blockIdx.y * TYS;
+  const int x = x0 + lane, y = y0 + w;
+  const bool active = x < g.nx && y < g.ny;
+  const int xc = min(x, g.nx), yc = min(y, g.ny);
+  const int me = sidx(lane + 1, w + 1);
+  const int z0 = blockIdx.z * ZCS, z1 = min(z0 + ZCS, g.nz);
+  const int th = t - (NT - 2 * TXP - 2 * TYS);
+  int hx = 0, hy = 0;
+  bool hcol = false;
+  if (th >= 0 && th < 2 * TYS) {
+    hcol = true;
+    hx = th < TYS ? 0 : TXP + 1;
+    hy = (th < TYS ? th : th - TYS) + 1;
+  } else if (th >= 2 * TYS) {
+    const int r = th - 2 * TYS;
+    hx = (r < TXP ? r : r - TXP) + 1;
+    hy = r < TXP ? 0 : TYS + 1;
+  }
+  const int hs = th >= 0 ? sidx(hx, hy) : -1;
+  const i64 hoff = th >= 0 ? g.at(min(x0 + hx - 1, g.nx), min(y0 + hy - 1, g.ny), 0) : 0;
+  const i64 htan = hcol ? g.pitch : 1;
+  const i64 coff = g.at(xc, yc, 0);
+  const bool pfl = (lane & 15) == 0 || th >= 0;
+  const i64 pfo = th >= 0 ? hoff : coff;
+
+  // own side of plane z0 - 1 (f, cd_x, cd_y, cd_z: z-face and cell operands), mu, carried phi column
+  double Sf[N3], Sx[N3], Sy[N3], Sz[N3], Smu;
+  double fc[N3], fm[N3];
+  {
+    const i64 c = coff + (i64)(z0 - 1) * g.plane;
+#pragma unroll
+    for (int a = 0; a < N3; ++a) {
+      const double* f = ps + a * F + c;
+      Sf[a] = __ldg(f);
+      Sx[a] = __ldg(f + 1) - __ldg(f - 1);
+      Sy[a] = __ldg(f + g.pitch) - __ldg(f - g.pitch);
+      Sz[a] = 0.0;  // (plane z0 - 1 is never updated here)
+      fm[a] = Sf[a];
+      fc[a] = __ldg(f + g.plane);
+    }
+    Smu = 0.0;
+  }
+  double divxy[N3] = {0.0, 0.0, 0.0}, Fzm[N3] = {0.0, 0.0, 0.0};
+  for (int k = z0; k <= z1; ++k) {
+    const bool last = k == z1;
+    const i64 c = coff + (i64)k * g.plane;
+    if (P.side_pd && pfl && k + P.side_pd <= z1) {
+      const i64 cp = pfo + (i64)(k + P.side_pd) * g.plane;
+#pragma unroll
+      for (int a = 0; a < N3; ++a) pf_l2(ps + a * F + cp);
+      pf_l2(ms + cp);
+    }
+    // (a) publish the sides of plane k
+    double Qf[N3], Qx[N3], Qy[N3], Qz[N3];
+#pragma unroll
+    for (int a = 0; a < N3; ++a) {
+      const double* f = ps + a * F + c;
+      const double fp = !last ? __ldg(f + g.plane) : 0.0;
+      Qf[a] = fc[a];
+      Qx[a] = __ldg(f + 1) - __ldg(f - 1);
+      Qy[a] = __ldg(f + g.pitch) - __ldg(f - g.pitch);
+      Qz[a] = !last ? fp - fm[a] : 0.0;
+      fm[a] = fc[a];
+      fc[a] = fp;
+    }
+    if (!last) {
+#pragma unroll
+      for (int a = 0; a < N3; ++a) {
+        S[P_F + a][me] = Qf[a];
+        S[P_CX + a][me] = Qx[a];
+        S[P_CY + a][me] = Qy[a];
+        S[P_CZ + a][me] = Qz[a];
+      }
+      if (hs >= 0) {
+        const i64 ch = hoff + (i64)k * g.plane;
+#pragma unroll
+        for (int a = 0; a < N3; ++a) {
+          const double* f = ps + a * F + ch;
+          const double tt = __ldg(f + htan) - __ldg(f - htan);
+          S[P_F + a][hs] = __ldg(f);
+          S[P_CX + a][hs] = hcol ? 0.0 : tt;
+          S[P_CY + a][hs] = hcol ? tt : 0.0;
+          S[P_CZ + a][hs] = __ldg(f + g.plane) - __ldg(f - g.plane);
+        }
+      }
+    }
+    __syncthreads();
+    // (b) z-face k-1 | k and (c) the cell update of plane k-1
+    double Fz[N3];
+    {
+      PSide p, q;
+#pragma unroll
+      for (int a = 0; a < N3; ++a) {
+        p.f[a] = Sf[a], p.c1[a] = Sx[a], p.c2[a] = Sy[a];
+        q.f[a] = Qf[a], q.c1[a] = Qx[a], q.c2[a] = Qy[a];
+      }
+      phi_face_side(P, 2, p, q, Fz);
+    }
+    if (k > z0 && active) {
+      double div[N3], cd[N3][3], out[N3];
+#pragma unroll
+      for (int a = 0; a < N3; ++a) {
+        div[a] = (divxy[a] + (Fz[a] - Fzm[a])) * P.inv_dx;
+        cd[a][0] = Sx[a], cd[a][1] = Sy[a], cd[a][2] = Sz[a];
+      }
+      phi_cell_v(P, k - 1, Sf, cd, Smu, div, out);
+      const i64 cm = c - g.plane;
+#pragma unroll
+      for (int a = 0; a < N3; ++a) pd[a * F + cm] = out[a];
+    }
+#pragma unroll
+    for (int a = 0; a < N3; ++a) Fzm[a] = Fz[a];
+    if (last) break;
+    // (d) x / y faces of plane k
+    double Fx[N3], Fy[N3];
+    {
+      PSide p, q;
+#pragma unroll
+      for (int a = 0; a < N3; ++a) q.f[a] = Qf[a], q.c1[a] = Qy[a], q.c2[a] = Qz[a];
+      pside_ld(S, me - 1, P_CY, P_CZ, p);
+      phi_face_side(P, 0, p, q, Fx);
+#pragma unroll
+      for (int a = 0; a < N3; ++a) q.c1[a] = Qx[a];
+      pside_ld(S, me - SHX, P_CX, P_CZ, p);
+      phi_face_side(P, 1, p, q, Fy);
+    }
+#pragma unroll
+    for (int a = 0; a < N3; ++a) {
+      fxs[a][w][lane] = Fx[a];
+      fys[a][w][lane] = Fy[a];
+    }
+    if (w == 0 && lane < TYS) {
+      PSide p, q;
+      double Fe[N3];
+      pside_ld(S, sidx(TXP, lane + 1), P_CY, P_CZ, p);
+      pside_ld(S, sidx(TXP + 1, lane + 1), P_CY, P_CZ, q);
+      phi_face_side(P, 0, p, q, Fe);
+#pragma unroll
+      for (int a = 0; a < N3; ++a) fxs[a][lane][TXP] = Fe[a];
+    } else if (w == 1) {
+      PSide p, q;
+      double Fe[N3];
+      pside_ld(S, sidx(lane + 1, TYS), P_CX, P_CZ, p);
+      pside_ld(S, sidx(lane + 1, TYS + 1), P_CX, P_CZ, q);
+      phi_face_side(P, 1, p, q, Fe);
+#pragma unroll
+      for (int a = 0; a < N3; ++a) fys[a][TYS][lane] = Fe[a];
+    }
+    const double mk = __ldg(ms + c);  // mu of the own cell (plane k), for its update one plane later
+    __syncthreads();
+#pragma unroll
+    for (int a = 0; a < N3; ++a) {
+      divxy[a] = (fxs[a][w][lane + 1] - Fx[a]) + (fys[a][w + 1][lane] - Fy[a]);
+      Sf[a] = Qf[a], Sx[a] = Qx[a], Sy[a] = Qy[a], Sz[a] = Qz[a];
+    }
+    Smu = mk;
+  }
+}
+
 }  // namespace p2
 
 // ---------------------------------------------------------------------------
@@ -725,6 +943,13 @@ static int p2_minb() {
   return e && atoi(e) == 3 ? 3 : 4;
 }
 
+// PF_P2_PHI=march: the z-marching phi kernel instead of the side-staged one
+// (side 1.215 vs march 1.318 ms at 256^3, profiles/r02_ab_p2.json)
+static bool p2_phi_side() {
+  const char* e = getenv("PF_P2_PHI");
+  return !(e && e[0] == 'm');
+}
+
 // PF_P2_MU=march: the z-marching mu kernel instead of the side-staged one
 static bool p2_mu_march() {
   const char* e = getenv("PF_P2_MU");
@@ -744,6 +969,12 @@ void p2_launch_phi(const void* Pv, double Tbase, const Geom& g, const double* ps
   if (p2_naive()) {
     dim3 b(32, 4, 2), gr((g.nx + 31) / 32, (g.ny + 3) / 4, (g.nz + 1) / 2);
     p2::k_phi<<<gr, b, 0, s>>>(P, g, ps, ms, pd);
+    return;
+  }
+  if (p2_phi_side()) {
+    dim3 b(p2::TXP, p2::TYS), gr((g.nx + p2::TXP - 1) / p2::TXP, (g.ny + p2::TYS - 1) / p2::TYS,
+                                 (g.nz + p2::ZCS - 1) / p2::ZCS);
+    p2::k_phi_side<<<gr, b, 0, s>>>(P, g, ps, ms, pd);
     return;
   }
   dim3 b(p2::TXP, p2::TYP), gr((g.nx + p2::TXP - 1) / p2::TXP, (g.ny + p2::TYP - 1) / p2::TYP,

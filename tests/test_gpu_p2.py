@@ -53,14 +53,15 @@ def run_pair(pfmod, omod, shape, P, phi, mu, chunks, bc=None):
     return out
 
 
-@pytest.mark.parametrize("kern", ["default", "mu_march", "naive"])
+@pytest.mark.parametrize("kern", ["default", "mu_march", "phi_march", "naive"])
 @pytest.mark.parametrize("pset", ["p2", "p2_stress", "p2_iso"])
 @pytest.mark.parametrize("ic", ["R", "V"])
 def test_p2_one_step_parity(pfmod, omod, pset, ic, kern, monkeypatch):
-    """Default kernels (z-marching phi, side-staged mu; every face once,
-    ragged tiles and z-chunks at this shape), the z-marching mu kernel, and
-    the one-thread-per-cell kernels."""
+    """Default kernels (side-staged phi and mu; every face once, ragged tiles
+    and z-chunks at this shape), the z-marching mu and phi kernels, and the
+    one-thread-per-cell kernels."""
     monkeypatch.setenv("PF_P2_NAIVE", "1" if kern == "naive" else "0")
+    monkeypatch.setenv("PF_P2_PHI", "march" if kern == "phi_march" else "side")
     monkeypatch.setenv("PF_P2_MU", "march" if kern == "mu_march" else "side")
     P = {"p2": I.params_p2(), "p2_stress": I.params_p2_stress(), "p2_iso": I.params_p2(aniso=0)}[pset]
     shape = (18, 21, 37)

@@ -59,9 +59,10 @@ def p2_runs():
     outs = []
     P = I.params_p2_stress(window_check=2, window_frac=0.5, v=0.05)
     phi, mu = I.ic_voronoi((20, 12, 33), seed=5, N=3, M=1)
-    for naive, mu in (("0", "side"), ("0", "march"), ("1", "side")):
+    for naive, mu, phi in (("0", "side", "side"), ("0", "march", "march"), ("1", "side", "side")):
         os.environ["PF_P2_NAIVE"] = naive
         os.environ["PF_P2_MU"] = mu
+        os.environ["PF_P2_PHI"] = phi
         g = pf.PhaseField((20, 12, 33), P, bc=I.BC_DS)
         g.init_fields(phi, mu)
         g.step(3)
@@ -70,6 +71,7 @@ def p2_runs():
         g.close()
     os.environ.pop("PF_P2_NAIVE", None)
     os.environ.pop("PF_P2_MU", None)
+    os.environ.pop("PF_P2_PHI", None)
     return outs
 
 
