@@ -311,7 +311,9 @@ def main():
     g.step(args.warmup)
     barrier()
     t_wait = time.time()
-    while len(clocks.lines) < 2 and time.time() - t_wait < 3.0:
+    # step until the sampler has two clock lines; the decision is a max over
+    # ranks, so every rank steps (and exchanges halos) the same number of times
+    while max_over_ranks(1.0 if (len(clocks.lines) < 2 and time.time() - t_wait < 3.0) else 0.0) > 0:
         g.step(1)
         torch.cuda.synchronize()
     # realign with the window checks (pf_step runs graphs of window_check
