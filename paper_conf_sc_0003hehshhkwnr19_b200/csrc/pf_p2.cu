@@ -18,6 +18,7 @@
 // parity against the oracle in tests/test_gpu_p2.py.
 // Independent of oracle/ (no shared code).
 #include <math.h>
+#include <string.h>
 
 #include "pf_internal.h"
 
@@ -496,16 +497,17 @@ __global__ void __launch_bounds__(TXP * TYP, MB) k_mu_march(Params P, Geom g, co
 // it (one-plane lag, as the P1 mu-sweep).  The faces' operands are the same
 // differences as mu_face's loads, through the same mu_flux: same bits.
 // ---------------------------------------------------------------------------
-constexpr int TYS = 8, ZCS = 16;
-constexpr int SHX = TXP + 2, SNC = SHX * (TYS + 2);  // halo-tile cells
-// shared side layout, component-major [SV][SNC] (a warp's reads are contiguous)
+constexpr int TYS = 8, ZCS = 16;  // default tile height (PF_P2_SIDE selects others)
+constexpr int SHX = TXP + 2;       // halo-tile row length (a tile of height TY has SHX (TY + 2) cells)
+// shared side layout, component-major [SV][SN] (a warp's reads are contiguous)
 constexpr int S_F = 0, S_CX = 3, S_CY = 6, S_CZ = 9, S_DP = 12, S_MU = 15, SV = 16;
 __device__ __forceinline__ int sidx(int hx, int hy) { return hy * SHX + hx; }
 
 struct Side {
   double f[N3], c1[N3], c2[N3], dp[N3], m;  // c1 / c2: central differences along the two tangential axes
 };
-__device__ __forceinline__ void side_ld(const double (*S)[SNC], int i, int o1, int o2, Side& s) {
+template <int SN>
+__device__ __forceinline__ void side_ld(const double (*S)[SN], int i, int o1, int o2, Side& s) {
 #pragma unroll
   for (int a = 0; a < N3; ++a) {
     s.f[a] = S[S_F + a][i];
@@ -532,34 +534,35 @@ __device__ __forceinline__ double mu_face_side(const Params& P, int d, const Sid
   return mu_flux<L>(P, d, pb, G, dtp, 0.5 * (p.m + q.m), (q.m - p.m) * P.inv_dx, Tf);
 }
 
-template <int L>
-__global__ void __launch_bounds__(TXP * TYS, 2) k_mu_side(Params P, Geom g, const double* __restrict__ ps,
+template <int L, int TY, int MB>
+__global__ void __launch_bounds__(TXP * TY, MB) k_mu_side(Params P, Geom g, const double* __restrict__ ps,
                                                          const double* __restrict__ pd,
                                                          const double* __restrict__ ms, double* __restrict__ md) {
-  __shared__ double S[SV][SNC];
-  __shared__ double fxs[TYS][TXP + 1];  // -x flux of every cell, +x of the right tile edge at TXP
-  __shared__ double fys[TYS + 1][TXP];  // -y flux of every cell, +y of the top tile edge at TYS
+  constexpr int SN = SHX * (TY + 2);
+  __shared__ double S[SV][SN];
+  __shared__ double fxs[TY][TXP + 1];  // -x flux of every cell, +x of the right tile edge at TXP
+  __shared__ double fys[TY + 1][TXP];  // -y flux of every cell, +y of the top tile edge at TY
   const i64 F = g.field;
   const int lane = threadIdx.x, w = threadIdx.y, t = w * TXP + lane;
-  constexpr int NT = TXP * TYS;
-  const int x0 = blockIdx.x * TXP, y0 = blockIdx.y * TYS;
+  constexpr int NT = TXP * TY;
+  const int x0 = blockIdx.x * TXP, y0 = blockIdx.y * TY;
   const int x = x0 + lane, y = y0 + w;
   const bool active = x < g.nx && y < g.ny;
   const int xc = min(x, g.nx), yc = min(y, g.ny);
   const int me = sidx(lane + 1, w + 1);
   const int z0 = blockIdx.z * ZCS, z1 = min(z0 + ZCS, g.nz);
-  // halo ring: the last 2 TXP + 2 TYS threads, one cell each (columns first)
-  const int th = t - (NT - 2 * TXP - 2 * TYS);
+  // halo ring: the last 2 TXP + 2 TY threads, one cell each (columns first)
+  const int th = t - (NT - 2 * TXP - 2 * TY);
   int hx = 0, hy = 0;
   bool hcol = false;
-  if (th >= 0 && th < 2 * TYS) {
+  if (th >= 0 && th < 2 * TY) {
     hcol = true;
-    hx = th < TYS ? 0 : TXP + 1;
-    hy = (th < TYS ? th : th - TYS) + 1;
-  } else if (th >= 2 * TYS) {
-    const int r = th - 2 * TYS;
+    hx = th < TY ? 0 : TXP + 1;
+    hy = (th < TY ? th : th - TY) + 1;
+  } else if (th >= 2 * TY) {
+    const int r = th - 2 * TY;
     hx = (r < TXP ? r : r - TXP) + 1;
-    hy = r < TXP ? 0 : TYS + 1;
+    hy = r < TXP ? 0 : TY + 1;
   }
   const int hs = th >= 0 ? sidx(hx, hy) : -1;
   const i64 hoff = th >= 0 ? g.at(min(x0 + hx - 1, g.nx), min(y0 + hy - 1, g.ny), 0) : 0;
@@ -667,14 +670,14 @@ __global__ void __launch_bounds__(TXP * TYS, 2) k_mu_side(Params P, Geom g, cons
     const double Fy = mu_face_side<L>(P, 1, p, q, Tk);
     fxs[w][lane] = Fx;
     fys[w][lane] = Fy;
-    if (w == 0 && lane < TYS) {  // +x face of the right tile edge, row `lane`
+    if (w == 0 && lane < TY) {  // +x face of the right tile edge, row `lane`
       side_ld(S, sidx(TXP, lane + 1), S_CY, S_CZ, p);
       side_ld(S, sidx(TXP + 1, lane + 1), S_CY, S_CZ, q);
       fxs[lane][TXP] = mu_face_side<L>(P, 0, p, q, Tk);
     } else if (w == 1) {  // +y face of the top tile edge, column `lane`
-      side_ld(S, sidx(lane + 1, TYS), S_CX, S_CZ, p);
-      side_ld(S, sidx(lane + 1, TYS + 1), S_CX, S_CZ, q);
-      fys[TYS][lane] = mu_face_side<L>(P, 1, p, q, Tk);
+      side_ld(S, sidx(lane + 1, TY), S_CX, S_CZ, p);
+      side_ld(S, sidx(lane + 1, TY + 1), S_CX, S_CZ, q);
+      fys[TY][lane] = mu_face_side<L>(P, 1, p, q, Tk);
     }
     __syncthreads();
     divxy = (fxs[w][lane + 1] - Fx) + (fys[w + 1][lane] - Fy);
@@ -694,7 +697,8 @@ constexpr int P_F = 0, P_CX = 3, P_CY = 6, P_CZ = 9, PV = 12;
 struct PSide {
   double f[N3], c1[N3], c2[N3];
 };
-__device__ __forceinline__ void pside_ld(const double (*S)[SNC], int i, int o1, int o2, PSide& s) {
+template <int SN>
+__device__ __forceinline__ void pside_ld(const double (*S)[SN], int i, int o1, int o2, PSide& s) {
 #pragma unroll
   for (int a = 0; a < N3; ++a) {
     s.f[a] = S[P_F + a][i];
@@ -716,31 +720,33 @@ __device__ __forceinline__ void phi_face_side(const Params& P, int d, const PSid
   phi_flux(P, d, pb, G, j);
 }
 
-__global__ void __launch_bounds__(TXP * TYS, 2) k_phi_side(Params P, Geom g, const double* __restrict__ ps,
+template <int TY, int MB>
+__global__ void __launch_bounds__(TXP * TY, MB) k_phi_side(Params P, Geom g, const double* __restrict__ ps,
                                                           const double* __restrict__ ms, double* __restrict__ pd) {
-  __shared__ double S[PV][SNC];
-  __shared__ double fxs[N3][TYS][TXP + 1];
-  __shared__ double fys[N3][TYS + 1][TXP];
+  constexpr int SN = SHX * (TY + 2);
+  __shared__ double S[PV][SN];
+  __shared__ double fxs[N3][TY][TXP + 1];
+  __shared__ double fys[N3][TY + 1][TXP];
   const i64 F = g.field;
   const int lane = threadIdx.x, w = threadIdx.y, t = w * TXP + lane;
-  constexpr int NT = TXP * TYS;
-  const int x0 = blockIdx.x * TXP, y0 = blockIdx.y * TYS;
+  constexpr int NT = TXP * TY;
+  const int x0 = blockIdx.x * TXP, y0 = blockIdx.y * TY;
   const int x = x0 + lane, y = y0 + w;
   const bool active = x < g.nx && y < g.ny;
   const int xc = min(x, g.nx), yc = min(y, g.ny);
   const int me = sidx(lane + 1, w + 1);
   const int z0 = blockIdx.z * ZCS, z1 = min(z0 + ZCS, g.nz);
-  const int th = t - (NT - 2 * TXP - 2 * TYS);
+  const int th = t - (NT - 2 * TXP - 2 * TY);
   int hx = 0, hy = 0;
   bool hcol = false;
-  if (th >= 0 && th < 2 * TYS) {
+  if (th >= 0 && th < 2 * TY) {
     hcol = true;
-    hx = th < TYS ? 0 : TXP + 1;
-    hy = (th < TYS ? th : th - TYS) + 1;
-  } else if (th >= 2 * TYS) {
-    const int r = th - 2 * TYS;
+    hx = th < TY ? 0 : TXP + 1;
+    hy = (th < TY ? th : th - TY) + 1;
+  } else if (th >= 2 * TY) {
+    const int r = th - 2 * TY;
     hx = (r < TXP ? r : r - TXP) + 1;
-    hy = r < TXP ? 0 : TYS + 1;
+    hy = r < TXP ? 0 : TY + 1;
   }
   const int hs = th >= 0 ? sidx(hx, hy) : -1;
   const i64 hoff = th >= 0 ? g.at(min(x0 + hx - 1, g.nx), min(y0 + hy - 1, g.ny), 0) : 0;
@@ -855,7 +861,7 @@ __global__ void __launch_bounds__(TXP * TYS, 2) k_phi_side(Params P, Geom g, con
       fxs[a][w][lane] = Fx[a];
       fys[a][w][lane] = Fy[a];
     }
-    if (w == 0 && lane < TYS) {
+    if (w == 0 && lane < TY) {
       PSide p, q;
       double Fe[N3];
       pside_ld(S, sidx(TXP, lane + 1), P_CY, P_CZ, p);
@@ -866,11 +872,11 @@ __global__ void __launch_bounds__(TXP * TYS, 2) k_phi_side(Params P, Geom g, con
     } else if (w == 1) {
       PSide p, q;
       double Fe[N3];
-      pside_ld(S, sidx(lane + 1, TYS), P_CX, P_CZ, p);
-      pside_ld(S, sidx(lane + 1, TYS + 1), P_CX, P_CZ, q);
+      pside_ld(S, sidx(lane + 1, TY), P_CX, P_CZ, p);
+      pside_ld(S, sidx(lane + 1, TY + 1), P_CX, P_CZ, q);
       phi_face_side(P, 1, p, q, Fe);
 #pragma unroll
-      for (int a = 0; a < N3; ++a) fys[a][TYS][lane] = Fe[a];
+      for (int a = 0; a < N3; ++a) fys[a][TY][lane] = Fe[a];
     }
     const double mk = __ldg(ms + c);  // mu of the own cell (plane k), for its update one plane later
     __syncthreads();
@@ -943,6 +949,19 @@ static int p2_minb() {
   return e && atoi(e) == 3 ? 3 : 4;
 }
 
+// tile height x CTAs per SM of the side-staged kernels, "8x2", "8x1", "4x3"
+// or "4x4": PF_P2_SIDE (phi, default 8x2: 32 x 8 tiles, 2 CTAs/SM at 128
+// registers) and PF_P2_SIDE_MU (mu, default 4x4: 32 x 4 tiles, 4 CTAs/SM);
+// measured at 256^3 (profiles/r02_ab_p2.json): phi 1.215 / 2.004 / 1.374 /
+// 1.251 ms, mu 0.739 / 1.050 / 0.816 / 0.692 ms
+static const char* p2_side_cfg(bool mu) {
+  const char* e = getenv(mu ? "PF_P2_SIDE_MU" : "PF_P2_SIDE");
+  if (e && (!strcmp(e, "8x2") || !strcmp(e, "8x1") || !strcmp(e, "4x3") || !strcmp(e, "4x4"))) return e;
+  return mu ? "4x4" : "8x2";
+}
+static int p2_side_ty(bool mu) { return p2_side_cfg(mu)[0] - '0'; }
+static int p2_side_mb(bool mu) { return p2_side_cfg(mu)[2] - '0'; }
+
 // PF_P2_PHI=march: the z-marching phi kernel instead of the side-staged one
 // (side 1.215 vs march 1.318 ms at 256^3, profiles/r02_ab_p2.json)
 static bool p2_phi_side() {
@@ -972,9 +991,16 @@ void p2_launch_phi(const void* Pv, double Tbase, const Geom& g, const double* ps
     return;
   }
   if (p2_phi_side()) {
-    dim3 b(p2::TXP, p2::TYS), gr((g.nx + p2::TXP - 1) / p2::TXP, (g.ny + p2::TYS - 1) / p2::TYS,
-                                 (g.nz + p2::ZCS - 1) / p2::ZCS);
-    p2::k_phi_side<<<gr, b, 0, s>>>(P, g, ps, ms, pd);
+    const int ty = p2_side_ty(false), mb = p2_side_mb(false);
+    dim3 b(p2::TXP, ty), gr((g.nx + p2::TXP - 1) / p2::TXP, (g.ny + ty - 1) / ty, (g.nz + p2::ZCS - 1) / p2::ZCS);
+    if (ty == 4 && mb == 3)
+      p2::k_phi_side<4, 3><<<gr, b, 0, s>>>(P, g, ps, ms, pd);
+    else if (ty == 4)
+      p2::k_phi_side<4, 4><<<gr, b, 0, s>>>(P, g, ps, ms, pd);
+    else if (mb == 1)
+      p2::k_phi_side<8, 1><<<gr, b, 0, s>>>(P, g, ps, ms, pd);
+    else
+      p2::k_phi_side<8, 2><<<gr, b, 0, s>>>(P, g, ps, ms, pd);
     return;
   }
   dim3 b(p2::TXP, p2::TYP), gr((g.nx + p2::TXP - 1) / p2::TXP, (g.ny + p2::TYP - 1) / p2::TYP,
@@ -999,13 +1025,19 @@ void p2_launch_mu(const void* Pv, double Tbase, const Geom& g, const double* ps,
     return;
   }
   if (!p2_mu_march()) {
-    dim3 b(p2::TXP, p2::TYS), gr((g.nx + p2::TXP - 1) / p2::TXP, (g.ny + p2::TYS - 1) / p2::TYS,
-                                 (g.nz + p2::ZCS - 1) / p2::ZCS);
+    const int ty = p2_side_ty(true), mb = p2_side_mb(true);
+    dim3 b(p2::TXP, ty), gr((g.nx + p2::TXP - 1) / p2::TXP, (g.ny + ty - 1) / ty, (g.nz + p2::ZCS - 1) / p2::ZCS);
+#define PF_P2_MUS(LL)                                                                         \
+  (ty == 4 && mb == 3 ? (p2::k_mu_side<LL, 4, 3><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md))     \
+   : ty == 4          ? (p2::k_mu_side<LL, 4, 4><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md))     \
+   : mb == 1          ? (p2::k_mu_side<LL, 8, 1><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md))     \
+                      : (p2::k_mu_side<LL, 8, 2><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md)))
     switch (P.liquid) {
-      case 0: p2::k_mu_side<0><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md); break;
-      case 1: p2::k_mu_side<1><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md); break;
-      default: p2::k_mu_side<2><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md); break;
+      case 0: PF_P2_MUS(0); break;
+      case 1: PF_P2_MUS(1); break;
+      default: PF_P2_MUS(2); break;
     }
+#undef PF_P2_MUS
     return;
   }
   dim3 b(p2::TXP, p2::TYP), gr((g.nx + p2::TXP - 1) / p2::TXP, (g.ny + p2::TYP - 1) / p2::TYP,

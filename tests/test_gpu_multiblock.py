@@ -140,3 +140,24 @@ def test_ds_window_blocks_bitwise(pfmod, procs):
     assert st1["z_off"] > 0
     assert all(s == st1 for s in states)
     assert np.array_equal(bp, sp) and np.array_equal(bm, sm)
+
+
+@pytest.mark.parametrize("case", ["x2_periodic", "xyz_2x2x2", "ds_xy2x2"])
+def test_p2_blocks_bitwise(pfmod, case):
+    """The P2 parameterisation (pf_p2.cu, 3 phases / 1 mu, anisotropic phi)
+    over the same transport: blocks equal one block bitwise (periodic x,
+    x-y-z split, and DS with window shifts)."""
+    if case == "ds_xy2x2":
+        P = I.params_p2_stress(window_check=5, window_frac=0.5, v=0.05)
+        shape, procs, bc = (32, 12, 40), (2, 2, 1), I.BC_DS
+    else:
+        P = dict(I.params_p2_stress(), G=0.0, v=0.0)
+        shape, procs, _, _, _ = CASES[case]
+        bc = I.BC_PERIODIC
+    phi, mu = I.ic_voronoi(shape, seed=13, N=3, M=1)
+    (sp, sm), st1 = run_single(pfmod, shape, P, bc, phi, mu, 20, "jit")
+    (bp, bm), states, _ = run_blocks(pfmod, shape, P, bc, phi, mu, 20, procs, "jit", chunks=2)
+    assert all(s == st1 for s in states)
+    if case == "ds_xy2x2":
+        assert st1["z_off"] > 0
+    assert np.array_equal(bp, sp) and np.array_equal(bm, sm), (np.abs(bp - sp).max(), np.abs(bm - sm).max())

@@ -123,3 +123,23 @@ def test_p2_invariants_and_monitor(pfmod):
     assert err <= 8 * 2.2e-16 and mn >= 0.0
     p, _ = g.download()
     assert p.shape == (3,) + shape
+
+
+@pytest.mark.parametrize("cfg", ["8x2", "8x1", "4x3", "4x4"])
+def test_p2_side_tilings_bitwise(pfmod, monkeypatch, cfg):
+    """The side-staged kernels' other tile heights / occupancies (PF_P2_SIDE)
+    give the default's bits: each face flux is computed from the same two
+    sides whichever thread evaluates it."""
+    P = I.params_p2_stress()
+    shape = (18, 21, 37)
+    phi, mu = I.ic_voronoi(shape, seed=11, N=3, M=1)
+    outs = []
+    for c in ("default", cfg):
+        monkeypatch.setenv("PF_P2_SIDE", c)
+        monkeypatch.setenv("PF_P2_SIDE_MU", c)
+        g = pfmod.PhaseField(shape, P)
+        g.init_fields(phi, mu)
+        g.step(3)
+        outs.append(g.download())
+        g.close()
+    assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
