@@ -497,7 +497,7 @@ def main():
                      "mu_sweep_ms": pr2["mu_sweep"][0] / max(pr2["mu_sweep"][1], 1),
                      "R_mlups": R2, "frac_of_R": val2 / R2, "F_flop_per_cell": F_STEP_P2,
                      "workload": f"P2: {n}^3 periodic block, 3 phases / 1 mu, anisotropic gamma (reading B6), IC-V",
-                     "note": "P2 sweeps (pf_p2.cu k_phi_side / k_mu_side): z-marching 32x8 tiles, each face flux once with both sides from shared memory, 2 CTAs/SM, L2 prefetch 2 planes ahead"}
+                     "note": "P2 sweeps (pf_p2.cu k_phi_side / k_mu_side): z-marching tiles (phi 32x8 at 2 CTAs/SM, mu 32x4 at 4), each face flux once with both sides from shared memory, L2 prefetch 2 planes ahead"}
         g2.close()
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         rec["cpu_baseline"] = cpu_baseline(P, bc, strong=strong)

@@ -1,6 +1,6 @@
 #!/bin/bash
 # One GPU session: GPU tests, smoke, bench (config 2 and config 4), ncu launch
-# list + full captures of the sweeps (P1 mu / phi, P2 phi), config 5.
+# list + full captures of the sweeps (P1 mu / phi, P2 phi / mu), config 5.
 # usage (from the repo root on the GPU box): bash tools/gpu_run.sh [tag] [skip_config5]
 TAG=${1:-r02}
 OUT=gpurun_out/$TAG
@@ -20,8 +20,10 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:pf_j
    python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e --no-stress --no-p2 --autotune 0 --tuning "$TUNE" > $OUT/ncu_mu.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:pf_jit_phi -s 3 -c 1 -o $OUT/prof_phi \
    python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e --no-stress --no-p2 --autotune 0 --tuning "$TUNE" > $OUT/ncu_phi.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_phi -s 1 -c 1 -o $OUT/prof_p2phi \
-   python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-e2e --no-stress --autotune 0 --tuning "$TUNE" > $OUT/ncu_p2phi.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_phi_side -s 2 -c 1 -o $OUT/prof_p2phi \
+   python tools/p2_run.py 256 4 > $OUT/ncu_p2phi.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_mu_side -s 2 -c 1 -o $OUT/prof_p2mu \
+   python tools/p2_run.py 256 4 > $OUT/ncu_p2mu.log 2>&1
 if [ -z "$2" ]; then
   timeout 1500 python tools/config5.py --out $OUT/config5.jsonl > $OUT/config5.log 2>&1
 fi

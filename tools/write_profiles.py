@@ -30,7 +30,7 @@ KEYS = ["gpu__time_duration.sum", "launch__registers_per_thread", "launch__occup
         "lts__t_sector_hit_rate.pct", "smsp__inst_executed.sum", "smsp__sass_inst_executed_op_global_ld.sum",
         "smsp__sass_inst_executed_op_shared_ld.sum", "smsp__sass_inst_executed_op_local_ld.sum"]
 summary = {}
-for kern in ("mu", "phi", "ghost", "p2phi"):
+for kern in ("mu", "phi", "ghost", "p2phi", "p2mu"):
     rep = os.path.join(src, f"prof_{kern}.ncu-rep")
     if not os.path.exists(rep):
         continue
