@@ -59,10 +59,10 @@ def p2_runs():
     outs = []
     P = I.params_p2_stress(window_check=2, window_frac=0.5, v=0.05)
     phi, mu = I.ic_voronoi((20, 12, 33), seed=5, N=3, M=1)
-    for naive, mu, phi in (("0", "side", "side"), ("0", "march", "march"), ("1", "side", "side")):
+    for naive, kmu, kphi in (("0", "side", "side"), ("0", "march", "march"), ("1", "side", "side")):
         os.environ["PF_P2_NAIVE"] = naive
-        os.environ["PF_P2_MU"] = mu
-        os.environ["PF_P2_PHI"] = phi
+        os.environ["PF_P2_MU"] = kmu
+        os.environ["PF_P2_PHI"] = kphi
         g = pf.PhaseField((20, 12, 33), P, bc=I.BC_DS)
         g.init_fields(phi, mu)
         g.step(3)
