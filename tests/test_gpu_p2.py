@@ -143,3 +143,27 @@ def test_p2_side_tilings_bitwise(pfmod, monkeypatch, cfg):
         outs.append(g.download())
         g.close()
     assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
+
+
+@pytest.mark.parametrize("shape", [(1, 1, 1), (3, 5, 7), (5, 6, 62), (40, 70, 65)])
+def test_p2_ragged_and_tiny_shapes(pfmod, omod, shape):
+    P = I.params_p2_stress()
+    phi, mu = I.ic_random(shape, seed=3, N=3, M=1)
+    for t, ep, em, *_ in run_pair(pfmod, omod, shape, P, phi, mu, [2]):
+        assert ep <= 1e-12 and em <= 1e-12, (shape, ep, em)
+
+
+@pytest.mark.parametrize("pure", [2, 0])
+def test_p2_pure_phase_fields(pfmod, omod, pure):
+    """One phase everywhere (the liquid, or grain 0) with a random mu: the
+    anisotropy sees q = 0 on every pair (grad f(0) = 0, the 0-branch of
+    aniso_grad) and the anti-trapping guards fire on every face."""
+    P = I.params_p2_stress()
+    shape = (9, 14, 37)
+    rng = np.random.default_rng(6)
+    phi = np.zeros((3,) + shape)
+    phi[pure] = 1.0
+    mu = rng.uniform(-0.2, 0.2, size=(1,) + shape)
+    res = run_pair(pfmod, omod, shape, P, phi, mu, [3])
+    t, ep, em, *_ = res[-1]
+    assert ep <= 1e-12 and em <= 1e-12, (ep, em)

@@ -446,3 +446,30 @@ def test_split_variant_bitwise_equals_full(pfmod):
         g.close()
     assert outs[0][1] == outs[1][1] and outs[0][1]["z_off"] > 0
     assert np.array_equal(outs[0][0][0], outs[1][0][0]) and np.array_equal(outs[0][0][1], outs[1][0][1])
+
+
+@pytest.mark.parametrize("variant", ["jit", "tuned", "naive", "split"])
+@pytest.mark.parametrize("pure", [3, 0])
+def test_pure_phase_fields(pfmod, omod, variant, pure):
+    """Degenerate fields: one phase everywhere (the liquid, or solid 0) with a
+    random mu.  Every gradient term and the anti-trapping current vanish
+    (the exact-zero guards [A11]); phi feels only the obstacle and driving
+    forces at the simplex corner, which the projection absorbs, and mu
+    evolves by diffusion alone -- as in the oracle."""
+    P = I.params_stress()
+    shape = (9, 14, 37)
+    rng = np.random.default_rng(5)
+    phi = np.zeros((4,) + shape)
+    phi[pure] = 1.0
+    mu = rng.uniform(-0.2, 0.2, size=(2,) + shape)
+    g = pfmod.PhaseField(shape, P)
+    g.set_variant(variant)
+    g.init_fields(phi, mu)
+    o = omod.Oracle(shape, P)
+    o.init(phi, mu)
+    g.step(3)
+    o.step(3)
+    gp, gm = g.download()
+    op, om = o.download()
+    assert rel_linf(gp, op) <= TOL_1 and rel_linf(gm, om) <= TOL_1
+    assert np.abs(gp.sum(axis=0) - 1.0).max() <= 8 * 2.2e-16 and gp.min() >= 0.0
