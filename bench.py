@@ -486,6 +486,12 @@ def main():
         g2 = pf.PhaseField((n, n, n), P2, device=local_rank)
         ph2, mu2 = I.ic_voronoi((n, n, n), seed=20191117, N=3, M=1)
         g2.init_fields(ph2, mu2)
+        p2_tune = None
+        if args.autotune > 0:  # the P2 kernel choices (p2_* knobs) timed on this block
+            t_p2 = time.time()
+            r2 = g2.autotune(reps=3)
+            p2_tune = {"seconds": round(time.time() - t_p2, 1), "phi": r2["phi"], "mu": r2["mu"],
+                       "best": {k: v for k, v in g2.tuning().items() if k.startswith("p2_")}}
         g2.profile(True)
         g2.step(3)
         torch.cuda.synchronize()
@@ -503,7 +509,7 @@ def main():
         rec["p2"] = {"value": val2, "unit": UNIT, "steps": n2, "ms_per_step": ms2 / n2,
                      "phi_sweep_ms": pr2["phi_sweep"][0] / max(pr2["phi_sweep"][1], 1),
                      "mu_sweep_ms": pr2["mu_sweep"][0] / max(pr2["mu_sweep"][1], 1),
-                     "R_mlups": R2, "frac_of_R": val2 / R2, "F_flop_per_cell": F_STEP_P2,
+                     "R_mlups": R2, "frac_of_R": val2 / R2, "F_flop_per_cell": F_STEP_P2, "autotune": p2_tune,
                      "workload": f"P2: {n}^3 periodic block, 3 phases / 1 mu, anisotropic gamma (reading B6), IC-V",
                      "note": "P2 sweeps (pf_p2.cu k_phi_side / k_mu_side): z-marching tiles (phi 32x8 at 2 CTAs/SM, mu 32x4 at 4), each face flux once with both sides from shared memory, L2 prefetch 2 planes ahead"}
         g2.close()

@@ -313,6 +313,17 @@ typedef struct {
                         of its own cells from the neighbour lanes' carried
                         values (warp shuffles; lanes 0 / 31 load the halo
                         column) instead of two L1 loads; mu_rpt = 2, mu_rpf = 1 */
+  /* P2 parameterisation (pf_p2.cu; tuned by pf_autotune on a P2 context)  */
+  int p2_phi;        /* P2 phi kernel: 0 side-staged (face sides in shared
+                        memory), 1 z-marching with global-memory face operands,
+                        2 one thread per cell (every face twice)               */
+  int p2_mu;         /* P2 mu kernel: the same three                           */
+  int p2_phi_ty;     /* side-staged P2 phi: tile height (4 or 8) and CTAs per  */
+  int p2_phi_minb;   /*   SM: (8, 2) default, (8, 1), (4, 3), (4, 4)           */
+  int p2_mu_ty;      /* side-staged P2 mu: the same, default (4, 4)            */
+  int p2_mu_minb;
+  int p2_phi_pd;     /* side-staged P2 phi / mu: L2 prefetch distance in planes */
+  int p2_mu_pd;      /*   (0 = off, 1..4; default 2)                           */
 } pf_tuning;
 
 /* The built-in defaults (the measured best at 256^3 on one B200,
@@ -349,7 +360,12 @@ int pf_tuning_check(const pf_tuning* t, char* log, int logn);
  * and "split" (PF_VARIANT_SPLIT, which allocates its staggered array) kernel
  * variants are timed the same way and reported ("variants" in the log); the
  * context keeps PF_VARIANT_JIT unless one of them is faster (S§8(f) NEXT-2:
- * full vs split vs fused).                                      */
+ * full vs split vs fused).
+ * P2 context (n_phases = 3): every kernel choice of each sweep in `mask`
+ * (pf_tuning p2_*: side-staged / z-marching / one thread per cell, the
+ * side-staged tile height x CTAs per SM and prefetch distance) is timed the
+ * same way (median of `reps` launches, max over ranks, >= 1 % to replace
+ * the current choice); `passes` and PF_AUTOTUNE_VARIANTS are ignored.      */
 #define PF_AUTOTUNE_VARIANTS 4u
 int pf_autotune(pf_ctx* ctx, unsigned mask, int passes, int reps, char* log, int logn);
 

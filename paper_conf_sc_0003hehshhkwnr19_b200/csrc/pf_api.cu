@@ -1074,6 +1074,11 @@ static int fill_ghost_dims(pf_ctx* ctx, double* f, int ncomp, bool is_mu, int d0
   return PF_OK;
 }
 
+// kernel choice of a P2 sweep from the tuning (pf_tuning p2_*)
+static P2Cfg p2cfg(const pf_tuning& t, bool mu) {
+  return mu ? P2Cfg{t.p2_mu, t.p2_mu_ty, t.p2_mu_minb, t.p2_mu_pd} : P2Cfg{t.p2_phi, t.p2_phi_ty, t.p2_phi_minb, t.p2_phi_pd};
+}
+
 static int fill_ghosts(pf_ctx* ctx, double* f, int ncomp, bool is_mu, bool x_done = false) {
   return fill_ghost_dims(ctx, f, ncomp, is_mu, 0, 3, ctx->stream, x_done);
 }
@@ -1228,7 +1233,7 @@ static int step_impl(pf_ctx* ctx, bool phi_only, bool dry = false) {
     if (int r = join_comm(ctx)) return r;
     cudaEvent_t e0 = nullptr;
     prof_begin(ctx, 0, &e0);
-    p2_launch_phi(ctx->p2par.data(), ctx->dp.Tbase, g, ps, ms, pd, ctx->stream);
+    p2_launch_phi(ctx->p2par.data(), p2cfg(ctx->tune, false), ctx->dp.Tbase, g, ps, ms, pd, ctx->stream);
     ctx->nlaunch[0] += 1;
     prof_end(ctx, 0, e0);
     if (int r = check_launch(ctx, "p2 phi_sweep")) return r;
@@ -1240,7 +1245,7 @@ static int step_impl(pf_ctx* ctx, bool phi_only, bool dry = false) {
       CU(cudaMemcpyAsync(md, ms, ctx->lay.mu_bytes - 256, cudaMemcpyDeviceToDevice, ctx->stream));
     } else {
       prof_begin(ctx, 1, &e0);
-      p2_launch_mu(ctx->p2par.data(), ctx->dp.Tbase, g, ps, pd, ms, md, ctx->stream);
+      p2_launch_mu(ctx->p2par.data(), p2cfg(ctx->tune, true), ctx->dp.Tbase, g, ps, pd, ms, md, ctx->stream);
       ctx->nlaunch[1] += 1;
       prof_end(ctx, 1, e0);
       if (int r2 = check_launch(ctx, "p2 mu_sweep")) return r2;
@@ -1757,6 +1762,15 @@ const std::vector<TuneKnob>& tune_knobs() {
       {"mu_tmem", &pf_tuning::mu_tmem, JIT_MU, {0, 1}},
       {"mu_hcar", &pf_tuning::mu_hcar, JIT_MU, {0, 1}},
       {"mu_xshfl", &pf_tuning::mu_xshfl, JIT_MU, {0, 1}},
+      // P2 (pf_p2.cu): tuned by the P2 branch of pf_autotune
+      {"p2_phi", &pf_tuning::p2_phi, P2_PHI, {0, 1, 2}},
+      {"p2_mu", &pf_tuning::p2_mu, P2_MU, {0, 1, 2}},
+      {"p2_phi_ty", &pf_tuning::p2_phi_ty, P2_PHI, {4, 8}},
+      {"p2_phi_minb", &pf_tuning::p2_phi_minb, P2_PHI, {1, 2, 3, 4}},
+      {"p2_mu_ty", &pf_tuning::p2_mu_ty, P2_MU, {4, 8}},
+      {"p2_mu_minb", &pf_tuning::p2_mu_minb, P2_MU, {1, 2, 3, 4}},
+      {"p2_phi_pd", &pf_tuning::p2_phi_pd, P2_PHI, {0, 1, 2, 3, 4}},
+      {"p2_mu_pd", &pf_tuning::p2_mu_pd, P2_MU, {0, 1, 2, 3, 4}},
   };
   return k;
 }
@@ -1806,6 +1820,119 @@ static int time_sweep(pf_ctx* ctx, JitKernel* k, int which, int reps, double* ou
   for (auto e : ev) cudaEventDestroy(e);
   std::sort(t.begin(), t.end());
   *out = t[reps / 2];
+  return PF_OK;
+}
+
+// P2 (pf_p2.cu): every kernel choice of each sweep (p2_* knobs: kernel,
+// side-staged tile height x CTAs per SM, prefetch distance), each timed as
+// the median of `reps` launches on this context's fields (reads the current
+// level, writes the scratch level: the state is untouched); the times are
+// max-reduced over ranks so that every rank keeps the same choice; a
+// candidate replaces the current choice only if >= 1 % faster
+static int time_p2(pf_ctx* ctx, const pf_tuning& t, bool mu, int reps, double* out) {
+  const double* ps = ctx->phi[ctx->cur];
+  double* pd = ctx->phi[1 - ctx->cur];
+  const double* ms = ctx->mu[ctx->cur];
+  double* md = ctx->mu[1 - ctx->cur];
+  const P2Cfg c = p2cfg(t, mu);
+  auto launch = [&]() {
+    if (mu)
+      p2_launch_mu(ctx->p2par.data(), c, ctx->dp.Tbase, ctx->g, ps, pd, ms, md, ctx->stream);
+    else
+      p2_launch_phi(ctx->p2par.data(), c, ctx->dp.Tbase, ctx->g, ps, ms, pd, ctx->stream);
+    return cudaGetLastError();
+  };
+  for (int i = 0; i < 2; ++i) CU(launch());
+  std::vector<cudaEvent_t> ev(reps + 1);
+  for (auto& e : ev) CU(cudaEventCreate(&e));
+  CU(cudaEventRecord(ev[0], ctx->stream));
+  for (int i = 0; i < reps; ++i) {
+    CU(launch());
+    CU(cudaEventRecord(ev[i + 1], ctx->stream));
+  }
+  CU(cudaEventSynchronize(ev[reps]));
+  std::vector<double> tm(reps);
+  for (int i = 0; i < reps; ++i) {
+    float v = 0;
+    cudaEventElapsedTime(&v, ev[i], ev[i + 1]);
+    tm[i] = v;
+  }
+  for (auto e : ev) cudaEventDestroy(e);
+  std::sort(tm.begin(), tm.end());
+  *out = tm[reps / 2];
+  return PF_OK;
+}
+
+static int autotune_p2(pf_ctx* ctx, unsigned mask, int reps, char* log, int logn) {
+  if (!(mask & (PF_PHI | PF_MU)) || reps < 1 || reps > 1000)
+    return fail(ctx, PF_EINVAL, "pf_autotune: mask PF_PHI|PF_MU, 1 <= reps <= 1000");
+  if (int r = join_comm(ctx)) return r;
+  CU(cudaStreamSynchronize(ctx->stream));
+  const pf_tuning start = ctx->tune;
+  pf_tuning best = start;
+  std::string cl, kj;
+  for (bool mu : {false, true}) {
+    if (!(mask & (mu ? PF_MU : PF_PHI))) continue;
+    if (mu) {  // the mu-sweep reads phi_dst: one phi-sweep of the chosen phi kernel and its ghosts first
+      p2_launch_phi(ctx->p2par.data(), p2cfg(best, false), ctx->dp.Tbase, ctx->g, ctx->phi[ctx->cur],
+                    ctx->mu[ctx->cur], ctx->phi[1 - ctx->cur], ctx->stream);
+      CU(cudaGetLastError());
+      if (int r = fill_ghosts(ctx, ctx->phi[1 - ctx->cur], ctx->nph, false)) return r;
+    }
+    std::vector<pf_tuning> cands{best};
+    for (int k : {0, 1, 2})
+      for (int tm : {0, 1, 2, 3})
+        for (int pdist : {0, 1, 2, 3, 4}) {
+          if (k != 0 && (tm || pdist)) continue;  // tile / prefetch only matter for the side-staged kernels
+          pf_tuning c = best;
+          const int ty = tm < 2 ? 8 : 4, mb = tm == 0 ? 2 : tm == 1 ? 1 : tm == 2 ? 3 : 4;
+          (mu ? c.p2_mu : c.p2_phi) = k;
+          if (k == 0) {
+            (mu ? c.p2_mu_ty : c.p2_phi_ty) = ty;
+            (mu ? c.p2_mu_minb : c.p2_phi_minb) = mb;
+            (mu ? c.p2_mu_pd : c.p2_phi_pd) = pdist;
+          }
+          if (!tuning_check(c) && memcmp(&c, &best, sizeof c)) cands.push_back(c);
+        }
+    std::vector<double> tms(cands.size(), INFINITY);
+    for (size_t i = 0; i < cands.size(); ++i)
+      if (int r = time_p2(ctx, cands[i], mu, reps, &tms[i])) return r;
+    if (ctx->collective()) {
+      double* d = (double*)ctx->red;
+      const int n = (int)cands.size();
+      CU(cudaMemcpyAsync(d, tms.data(), n * sizeof(double), cudaMemcpyHostToDevice, ctx->stream));
+      if (int r = allreduce_max(ctx, d, n)) return r;
+      CU(cudaMemcpyAsync(tms.data(), d, n * sizeof(double), cudaMemcpyDeviceToHost, ctx->stream));
+      CU(cudaStreamSynchronize(ctx->stream));
+    }
+    size_t bi = 0;
+    for (size_t i = 1; i < cands.size(); ++i)
+      if (tms[i] < tms[0] * 0.99 && tms[i] < tms[bi]) bi = i;
+    const char* kname = mu ? "mu" : "phi";
+    for (size_t i = 1; i < cands.size(); ++i) {
+      const pf_tuning& c = cands[i];
+      char b[320];
+      snprintf(b, sizeof b,
+               "%s{\"kernel\": \"p2_%s\", \"pass\": 0, \"knob\": \"kern/ty/minb/pd\", \"value\": %d, \"ms\": %.6f, \"error\": \"\"}",
+               cl.empty() ? "" : ",\n  ", kname,
+               1000 * (mu ? c.p2_mu : c.p2_phi) + 100 * (mu ? c.p2_mu_ty : c.p2_phi_ty) +
+                   10 * (mu ? c.p2_mu_minb : c.p2_phi_minb) + (mu ? c.p2_mu_pd : c.p2_phi_pd),
+               tms[i]);
+      cl += b;
+    }
+    best = cands[bi];
+    char b[256];
+    snprintf(b, sizeof b, "%s\"%s\": {\"start_ms\": %.6f, \"best_ms\": %.6f, \"candidates\": %d}", kj.empty() ? "" : ", ",
+             kname, tms[0], tms[bi], (int)cands.size() - 1);
+    kj += b;
+  }
+  ctx->tune = best;
+  CU(cudaStreamSynchronize(ctx->stream));
+  if (log && logn > 0) {
+    std::string j = "{\"start\": " + tuning_json(start) + ",\n \"best\": " + tuning_json(best) + ",\n " + kj +
+                    ",\n \"reps\": " + std::to_string(reps) + ",\n \"tried\": [\n  " + cl + "]}";
+    snprintf(log, (size_t)logn, "%s", j.c_str());
+  }
   return PF_OK;
 }
 
@@ -1873,7 +2000,8 @@ static int time_candidates(pf_ctx* ctx, const std::vector<pf_tuning>& cands, int
 int pf_autotune(pf_ctx* ctx, unsigned mask, int passes, int reps, char* log, int logn) {
   if (!ctx) return PF_EINVAL;
   if (!ctx->have_params || !ctx->have_fields) return fail(ctx, PF_ESTATE, "pf_autotune before pf_set_params/pf_init_fields");
-  if (ctx->variant != PF_VARIANT_JIT || ctx->p2) return fail(ctx, PF_ESTATE, "pf_autotune tunes the JIT variant of P1 only");
+  if (ctx->p2) return autotune_p2(ctx, mask, reps, log, logn);
+  if (ctx->variant != PF_VARIANT_JIT) return fail(ctx, PF_ESTATE, "pf_autotune tunes the JIT variant (or a P2 context)");
   if (!(mask & (PF_PHI | PF_MU)) || passes < 1 || reps < 1 || reps > 1000)
     return fail(ctx, PF_EINVAL, "pf_autotune: mask PF_PHI|PF_MU, passes >= 1, 1 <= reps <= 1000");
   if (const char* m = tuning_check(ctx->tune)) return fail(ctx, PF_EINVAL, "current tuning invalid: %s", m);

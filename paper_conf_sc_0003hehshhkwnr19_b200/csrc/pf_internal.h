@@ -70,13 +70,19 @@ bool plane_interleaved();  // field layout: [c][z][y][x] (default) or [z][c][y][
 // ---- P2 parameterisation (pf_p2.cu): 3 phases, 1 mu, anisotropic phi ----
 size_t p2_params_size();                                                // bytes of the opaque parameter block
 void p2_fill_params(const pf_params& p, int liquid, void* out);          // host values -> parameter block
-void p2_launch_phi(const void* P, double Tbase, const Geom& g, const double* ps, const double* ms, double* pd,
-                   cudaStream_t s);
-void p2_launch_mu(const void* P, double Tbase, const Geom& g, const double* ps, const double* pd, const double* ms,
-                  double* md, cudaStream_t s);
+// kernel choice of the P2 sweeps (pf_tuning p2_*)
+struct P2Cfg {
+  int kern;    // 0 side-staged, 1 z-marching, 2 one thread per cell
+  int ty, mb;  // side-staged: tile height, CTAs per SM
+  int pd;      // side-staged: L2 prefetch distance (planes)
+};
+void p2_launch_phi(const void* P, const P2Cfg& c, double Tbase, const Geom& g, const double* ps, const double* ms,
+                   double* pd, cudaStream_t s);
+void p2_launch_mu(const void* P, const P2Cfg& c, double Tbase, const Geom& g, const double* ps, const double* pd,
+                  const double* ms, double* md, cudaStream_t s);
 
 // ---- run-time specialisation (NVRTC) -------------------------------------
-enum { JIT_PHI = 0, JIT_MU = 1 };
+enum { JIT_PHI = 0, JIT_MU = 1, P2_PHI = 2, P2_MU = 3 };  // (P2_*: pf_tuning knobs of pf_p2.cu)
 struct JitKernel;  // one specialised sweep compiled for (parameters, geometry, tuning)
 void tuning_default(pf_tuning* t);            // built-in defaults + PF_* environment overrides
 const char* tuning_check(const pf_tuning& t);  // nullptr if valid, else the reason

@@ -9,16 +9,15 @@
 // makes phi the heavy kernel of P2 (Table 1: 3968 normalised FLOPs,
 // P:L1234-1243).  The mu equation (eqs. 8-10) is the P1 one with M = 1.
 //
-// Default: side-staged z-marching sweeps (k_phi_side, k_mu_side: every face
-// flux evaluated once, both sides of a face from shared memory);
-// PF_P2_PHI=march / PF_P2_MU=march: z-marching sweeps that load the face
-// operands from global memory (k_phi_march, k_mu_march); PF_P2_NAIVE=1: one
-// thread per cell, every face evaluated by both of its cells (the paper's
-// "full" kernels).  Written from the paper;
+// Kernels (pf_tuning p2_phi / p2_mu, tuned by pf_autotune): side-staged
+// z-marching sweeps (default; k_phi_side, k_mu_side: every face flux
+// evaluated once, both sides of a face from shared memory), z-marching
+// sweeps that load the face operands from global memory (k_phi_march,
+// k_mu_march), and one thread per cell with every face evaluated by both of
+// its cells (k_phi, k_mu: the paper's "full" kernels).  Written from the paper;
 // parity against the oracle in tests/test_gpu_p2.py.
 // Independent of oracle/ (no shared code).
 #include <math.h>
-#include <string.h>
 
 #include "pf_internal.h"
 
@@ -38,7 +37,7 @@ struct Params {
   double R[N3][N3][9];  // R_ab row-major
   int liquid, aniso;
   int prefetch;  // z-marching sweeps: own column's lines P2_PD planes ahead into L2 (PF_P2_PREFETCH, default 1)
-  int side_pd;   // side-staged mu-sweep: L2 prefetch distance in planes, 0 = off (PF_P2_SIDE_PD, default 2)
+  int side_pd;   // side-staged sweeps: L2 prefetch distance in planes, 0 = off (pf_tuning p2_pd)
   double mu_inf;
 };
 
@@ -936,8 +935,7 @@ void p2_fill_params(const pf_params& p, int liquid, void* out) {
   P.mu_inf = p.mu_inf[0];
   const char* e = getenv("PF_P2_PREFETCH");
   P.prefetch = e ? atoi(e) : 1;
-  const char* e2 = getenv("PF_P2_SIDE_PD");
-  P.side_pd = e2 ? atoi(e2) : 2;
+  P.side_pd = 2;  // (per launch from P2Cfg)
 }
 size_t p2_params_size() { return sizeof(p2::Params); }
 
@@ -949,49 +947,23 @@ static int p2_minb() {
   return e && atoi(e) == 3 ? 3 : 4;
 }
 
-// tile height x CTAs per SM of the side-staged kernels, "8x2", "8x1", "4x3"
-// or "4x4": PF_P2_SIDE (phi, default 8x2: 32 x 8 tiles, 2 CTAs/SM at 128
-// registers) and PF_P2_SIDE_MU (mu, default 4x4: 32 x 4 tiles, 4 CTAs/SM);
+// Kernel choice (pf_tuning p2_*, P2Cfg): kern 0 = side-staged (default),
+// 1 = z-marching with global-memory face operands, 2 = one thread per cell;
+// side-staged tile height x CTAs per SM (8, 2) / (8, 1) / (4, 3) / (4, 4),
 // measured at 256^3 (profiles/r02_ab_p2.json): phi 1.215 / 2.004 / 1.374 /
-// 1.251 ms, mu 0.739 / 1.050 / 0.816 / 0.692 ms
-static const char* p2_side_cfg(bool mu) {
-  const char* e = getenv(mu ? "PF_P2_SIDE_MU" : "PF_P2_SIDE");
-  if (e && (!strcmp(e, "8x2") || !strcmp(e, "8x1") || !strcmp(e, "4x3") || !strcmp(e, "4x4"))) return e;
-  return mu ? "4x4" : "8x2";
-}
-static int p2_side_ty(bool mu) { return p2_side_cfg(mu)[0] - '0'; }
-static int p2_side_mb(bool mu) { return p2_side_cfg(mu)[2] - '0'; }
-
-// PF_P2_PHI=march: the z-marching phi kernel instead of the side-staged one
-// (side 1.215 vs march 1.318 ms at 256^3, profiles/r02_ab_p2.json)
-static bool p2_phi_side() {
-  const char* e = getenv("PF_P2_PHI");
-  return !(e && e[0] == 'm');
-}
-
-// PF_P2_MU=march: the z-marching mu kernel instead of the side-staged one
-static bool p2_mu_march() {
-  const char* e = getenv("PF_P2_MU");
-  return e && e[0] == 'm';
-}
-
-// PF_P2_NAIVE=1: the one-thread-per-cell kernels (every face twice)
-static bool p2_naive() {
-  const char* e = getenv("PF_P2_NAIVE");
-  return e && e[0] == '1';
-}
-
-void p2_launch_phi(const void* Pv, double Tbase, const Geom& g, const double* ps, const double* ms, double* pd,
-                   cudaStream_t s) {
+// 1.251 ms, mu 0.739 / 1.050 / 0.816 / 0.692 ms (defaults phi (8, 2), mu (4, 4))
+void p2_launch_phi(const void* Pv, const P2Cfg& c, double Tbase, const Geom& g, const double* ps, const double* ms,
+                   double* pd, cudaStream_t s) {
   p2::Params P = *reinterpret_cast<const p2::Params*>(Pv);
   P.Tbase = Tbase;
-  if (p2_naive()) {
+  P.side_pd = c.pd;
+  if (c.kern == 2) {
     dim3 b(32, 4, 2), gr((g.nx + 31) / 32, (g.ny + 3) / 4, (g.nz + 1) / 2);
     p2::k_phi<<<gr, b, 0, s>>>(P, g, ps, ms, pd);
     return;
   }
-  if (p2_phi_side()) {
-    const int ty = p2_side_ty(false), mb = p2_side_mb(false);
+  if (c.kern == 0) {
+    const int ty = c.ty, mb = c.mb;
     dim3 b(p2::TXP, ty), gr((g.nx + p2::TXP - 1) / p2::TXP, (g.ny + ty - 1) / ty, (g.nz + p2::ZCS - 1) / p2::ZCS);
     if (ty == 4 && mb == 3)
       p2::k_phi_side<4, 3><<<gr, b, 0, s>>>(P, g, ps, ms, pd);
@@ -1011,11 +983,12 @@ void p2_launch_phi(const void* Pv, double Tbase, const Geom& g, const double* ps
     p2::k_phi_march<3><<<gr, b, 0, s>>>(P, g, ps, ms, pd);
 }
 
-void p2_launch_mu(const void* Pv, double Tbase, const Geom& g, const double* ps, const double* pd, const double* ms,
-                  double* md, cudaStream_t s) {
+void p2_launch_mu(const void* Pv, const P2Cfg& c, double Tbase, const Geom& g, const double* ps, const double* pd,
+                  const double* ms, double* md, cudaStream_t s) {
   p2::Params P = *reinterpret_cast<const p2::Params*>(Pv);
   P.Tbase = Tbase;
-  if (p2_naive()) {
+  P.side_pd = c.pd;
+  if (c.kern == 2) {
     dim3 b(32, 4, 2), gr((g.nx + 31) / 32, (g.ny + 3) / 4, (g.nz + 1) / 2);
     switch (P.liquid) {
       case 0: p2::k_mu<0><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md); break;
@@ -1024,8 +997,8 @@ void p2_launch_mu(const void* Pv, double Tbase, const Geom& g, const double* ps,
     }
     return;
   }
-  if (!p2_mu_march()) {
-    const int ty = p2_side_ty(true), mb = p2_side_mb(true);
+  if (c.kern == 0) {
+    const int ty = c.ty, mb = c.mb;
     dim3 b(p2::TXP, ty), gr((g.nx + p2::TXP - 1) / p2::TXP, (g.ny + ty - 1) / ty, (g.nz + p2::ZCS - 1) / p2::ZCS);
 #define PF_P2_MUS(LL)                                                                         \
   (ty == 4 && mb == 3 ? (p2::k_mu_side<LL, 4, 3><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md))     \

@@ -167,3 +167,37 @@ def test_p2_pure_phase_fields(pfmod, omod, pure):
     res = run_pair(pfmod, omod, shape, P, phi, mu, [3])
     t, ep, em, *_ = res[-1]
     assert ep <= 1e-12 and em <= 1e-12, (ep, em)
+
+
+def test_p2_autotune_and_tuning_knobs(pfmod, omod):
+    """pf_autotune on a P2 context times every kernel choice of both sweeps
+    (p2_* knobs) without touching the state; every choice keeps parity."""
+    P = I.params_p2_stress()
+    shape = (20, 24, 40)
+    phi, mu = I.ic_voronoi(shape, seed=21, N=3, M=1)
+    g = pfmod.PhaseField(shape, P)
+    g.init_fields(phi, mu)
+    rep = g.autotune(reps=3)
+    assert g.state()["step"] == 0
+    p0, m0 = g.download()
+    assert np.array_equal(p0, phi) and np.array_equal(m0, mu)
+    assert rep["phi"]["candidates"] > 10 and rep["mu"]["candidates"] > 10
+    g.step(2)
+    gp, gm = g.download()
+    g.close()
+    o = omod.Oracle(shape, P)
+    o.init(phi, mu)
+    o.step(2)
+    op, om = o.download()
+    assert rel_linf(gp, op) <= 1e-12 and rel_linf(gm, om) <= 1e-12
+    for t in ({"p2_phi": 1, "p2_mu": 1}, {"p2_phi": 2, "p2_mu": 2},
+              {"p2_phi_ty": 4, "p2_phi_minb": 3, "p2_mu_ty": 8, "p2_mu_minb": 1, "p2_phi_pd": 0, "p2_mu_pd": 4}):
+        g = pfmod.PhaseField(shape, P)
+        g.set_tuning(t)
+        g.init_fields(phi, mu)
+        g.step(2)
+        gp, gm = g.download()
+        g.close()
+        assert rel_linf(gp, op) <= 1e-12 and rel_linf(gm, om) <= 1e-12, t
+    with pytest.raises(pfmod.PFError):
+        pfmod.PhaseField(shape, P).set_tuning({"p2_phi_ty": 4, "p2_phi_minb": 2})
