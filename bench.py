@@ -418,6 +418,30 @@ def main():
         "state": {"step": st["step"], "z_off": st["z_off"], "max_sum_err": mon[0], "min_phi": mon[1]},
         "window": window,
     }
+    # ---- the same steps with the anti-trapping skip (tuning mu_atskip): the
+    # mu-sweep skips eq. 10 in warps where it is exactly 0 (bulk phases);
+    # same results, data-dependent time -- reported beside the headline, not
+    # as it (the headline kernel does the full work everywhere)
+    if args.variant == "jit" and not strong and world == 1:
+        tsave = g.tuning()
+        g.set_tuning(dict(tsave, mu_atskip=1))
+        g.step(3)
+        barrier()
+        g.profile(True)
+        a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        na = max(20, min(args.steps, 100))
+        a0.record(stream)
+        g.step(na)
+        a1.record(stream)
+        a1.synchronize()
+        pa = g.profile_read()
+        ams = a0.elapsed_time(a1)
+        rec["atskip"] = {"value": cells_local * na / (ams * 1e-3) / 1e6, "unit": UNIT, "steps": na,
+                         "ms_per_step": ams / na, "mu_sweep_ms": pa["mu_sweep"][0] / max(pa["mu_sweep"][1], 1),
+                         "phi_sweep_ms": pa["phi_sweep"][0] / max(pa["phi_sweep"][1], 1),
+                         "note": "same workload and state continuing after the timed region, tuning mu_atskip = 1 "
+                                 "(bitwise-equal results, tests/test_gpu_autotune.py); data-dependent"}
+        g.set_tuning(tsave)
     # ---- end-to-end through the public API with host buffers ----
     if not args.no_e2e:
         g.profile(False)

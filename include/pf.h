@@ -324,6 +324,12 @@ typedef struct {
   int p2_mu_minb;
   int p2_phi_pd;     /* side-staged P2 phi / mu: L2 prefetch distance in planes */
   int p2_mu_pd;      /*   (0 = off, 1..4; default 2)                           */
+  int mu_atskip;     /* 1: the specialised mu-sweep skips the anti-trapping
+                        current (eq. 10) in a warp whose faces all have it
+                        exactly 0 (pb_l = 0 or every pb_s = 0: bulk phases,
+                        solid-solid boundaries); same results, data-dependent
+                        time; off by default and not searched by pf_autotune
+                        (the benchmark reports it separately)                  */
 } pf_tuning;
 
 /* The built-in defaults (the measured best at 256^3 on one B200,

@@ -1771,6 +1771,8 @@ const std::vector<TuneKnob>& tune_knobs() {
       {"p2_mu_minb", &pf_tuning::p2_mu_minb, P2_MU, {1, 2, 3, 4}},
       {"p2_phi_pd", &pf_tuning::p2_phi_pd, P2_PHI, {0, 1, 2, 3, 4}},
       {"p2_mu_pd", &pf_tuning::p2_mu_pd, P2_MU, {0, 1, 2, 3, 4}},
+      // not searched (data-dependent time; reported separately by bench.py)
+      {"mu_atskip", &pf_tuning::mu_atskip, JIT_MU, {0}},
   };
   return k;
 }

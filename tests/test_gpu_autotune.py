@@ -70,6 +70,9 @@ CORNERS = [
     # own cd_x by warp shuffles, L1 policies
     {"mu_xshfl": 1},
     {"mu_xshfl": 1, "mu_hcar": 1, "mu_ldhint": 3, "mu_ty": 6, "mu_minb": 3, "mu_zc": 5},
+    # warp-uniform skip of the anti-trapping current where it is exactly 0
+    {"mu_atskip": 1},
+    dict(R1, mu_atskip=1),
 ]
 
 
