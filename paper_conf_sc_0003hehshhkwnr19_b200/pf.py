@@ -17,6 +17,7 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(PKG, "libpf.so")
 
 PF_OK, PF_EINVAL, PF_ENOMEM, PF_ECUDA, PF_ENCCL, PF_ESTATE, PF_ENUMERIC = 0, -1, -2, -3, -4, -5, -6
+GUARD_BYTE = 0xA5  # fill of the test-only guard zones (PF_TEST_GUARD_BYTES)
 BC = {"periodic": 0, "neumann": 1, "dirichlet_mu": 2}
 PF_HOST, PF_DEVICE = 0, 1
 PF_PHI, PF_MU = 1, 2
@@ -288,14 +289,32 @@ class PhaseField:
         self.local = (lay.local[2], lay.local[1], lay.local[0])
         self.offset = (lay.offset[2], lay.offset[1], lay.offset[0])
         u8 = torch.uint8
-        self._phi = [torch.empty(lay.phi_bytes, dtype=u8, device=self.device) for _ in range(2)]
-        self._mu = [torch.empty(lay.mu_bytes, dtype=u8, device=self.device) for _ in range(2)]
-        self._ws = torch.zeros(lay.workspace_bytes, dtype=u8, device=self.device)
+        # PF_TEST_GUARD_BYTES > 0 (tests only): every caller-owned buffer sits
+        # between two guard zones of that many bytes filled with GUARD_BYTE;
+        # close() raises if a kernel wrote into one (an out-of-bounds store
+        # past the layout pf_query_layout gave)
+        self._guard = int(os.environ.get("PF_TEST_GUARD_BYTES", "0"))
+        gb = self._guard = (self._guard + 255) // 256 * 256
+
+        def buf(n, zero=True):
+            t = torch.empty(n + 2 * gb, dtype=u8, device=self.device)
+            if gb:
+                t.fill_(GUARD_BYTE)
+            inner = t[gb:gb + n]
+            if zero:
+                inner.zero_()
+            return t, inner
+        self._raw = []
+        self._phi, self._mu = [], []
         for i in range(2):
-            self._phi[i].zero_()
-            self._mu[i].zero_()
+            for lst, n in ((self._phi, lay.phi_bytes), (self._mu, lay.mu_bytes)):
+                t, inner = buf(n)
+                self._raw.append(t)
+                lst.append(inner)
             cfg.phi[i] = self._phi[i].data_ptr()
             cfg.mu[i] = self._mu[i].data_ptr()
+        t, self._ws = buf(lay.workspace_bytes)
+        self._raw.append(t)
         cfg.workspace = self._ws.data_ptr()
         self._cfg = cfg
         h = C.c_void_p()
@@ -312,10 +331,24 @@ class PhaseField:
             msg = self.lib.pf_last_error(self._h).decode() if ctx else ""
             raise PFError(f"{what} failed ({r}): {msg}")
 
+    def guards_intact(self) -> bool:
+        """True unless a kernel stored into the guard zones around the
+        caller-owned buffers (PF_TEST_GUARD_BYTES; always True without)."""
+        gb = getattr(self, "_guard", 0)
+        if not gb:
+            return True
+        self.torch.cuda.synchronize(self.device)
+        for t in self._raw:
+            if not (bool((t[:gb] == GUARD_BYTE).all()) and bool((t[-gb:] == GUARD_BYTE).all())):
+                return False
+        return True
+
     def close(self):
         if getattr(self, "_h", None) is not None and self._h.value:
             self.lib.pf_destroy(self._h)
             self._h = C.c_void_p()
+            if not self.guards_intact():
+                raise PFError("a kernel wrote outside the caller-owned buffers (guard zone changed)")
 
     def __del__(self):
         try:

@@ -107,6 +107,44 @@ def test_compute_sanitizer(tool):
            *variants]
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=2400, cwd=ROOT)
     tail = (r.stdout + r.stderr)[-3000:]
+    if "closed on this pool" in tail:
+        # the GPU pool disabled compute-sanitizer in round 2 (its runs left GPUs
+        # needing a reset); the clean memcheck / racecheck logs of session s23
+        # are in profiles/r02_pytest_sanitizer_s23.log, and test_guard_zones
+        # below checks the same runs for out-of-bounds stores without it
+        pytest.skip("compute-sanitizer closed on this GPU pool: " + tail.strip()[:200])
     assert r.returncode == 0, tail
     assert "sanitize run ok" in r.stdout, tail
     assert "ERROR SUMMARY: 0 errors" in (r.stdout + r.stderr) or "RACECHECK SUMMARY: 0 hazards" in (r.stdout + r.stderr), tail
+
+
+def test_guard_zones():
+    """Out-of-bounds stores without compute-sanitizer: the runs of
+    tools/sanitize_run.py (every kernel family, ragged DS block, tunings,
+    P2, multi-block) with every caller-owned buffer between two 64 KiB guard
+    zones (PF_TEST_GUARD_BYTES, pf.py); close() raises if a kernel wrote into
+    one, and the runs must still agree with each other."""
+    env = dict(os.environ, PF_TEST_GUARD_BYTES="65536")
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "tools", "sanitize_run.py")], capture_output=True,
+                       text=True, timeout=1800, cwd=ROOT, env=env)
+    tail = (r.stdout + r.stderr)[-3000:]
+    assert r.returncode == 0, tail
+    assert "sanitize run ok" in r.stdout, tail
+
+
+def test_guard_zones_detect(monkeypatch):
+    """The guard check itself: a store one byte before / after a buffer is seen."""
+    from paper_conf_sc_0003hehshhkwnr19_b200 import pf
+    monkeypatch.setenv("PF_TEST_GUARD_BYTES", "4096")
+    shape = (8, 8, 32)
+    P = I.params_c4("periodic")
+    g = pf.PhaseField(shape, P)
+    g.init_fields(*I.ic_voronoi(shape, seed=1))
+    g.step(2)
+    assert g.guards_intact()
+    for t, pos in ((g._raw[0], 4095), (g._raw[-1], -4096)):
+        t[pos] = 0
+        assert not g.guards_intact()
+        t[pos] = pf.GUARD_BYTE
+    assert g.guards_intact()
+    g.close()
