@@ -398,6 +398,12 @@ int pf_nccl_unique_id(unsigned char out[128]);
  * log[0..logn).                                                            */
 int pf_jit_compile_only(const pf_params* p, int liquid, int n, const pf_tuning* t, const char* cubin_path, char* log,
                         int logn);
+/* The same for the P2 sweeps (n_phases = 3, n_mu = 1; pf_p2 kernels on the
+ * parameters p as compile-time constants): the phi- and mu-sweep of the
+ * kernel choice in t (p2_* fields; NULL = default) for an n^3 block; cubins to cubin_path
+ * (mu) and cubin_path + ".phi".  Returns the total size or -1 (log).     */
+int pf_jit_compile_only_p2(const pf_params* p, int liquid, int n, const pf_tuning* t, const char* cubin_path, char* log,
+                           int logn);
 
 const char* pf_last_error(const pf_ctx* ctx);
 const char* pf_version(void);

@@ -179,6 +179,8 @@ struct pf_ctx {
   int64_t mu_launches_per_step = 1, ghost_launches_per_step = 0;  // launch accounting of graph replays
   JitKernel* jphi = nullptr;  // specialised sweeps for (dp, g, tune); reset by pf_set_params / pf_set_tuning
   JitKernel* jmu = nullptr;
+  JitKernel* jp2[2] = {nullptr, nullptr};  // P2: specialised phi / mu sweeps and the kernel choices they hold
+  P2Cfg jp2c[2] = {};
   pf_tuning tune;             // tuning of the specialised sweeps (pf_set_tuning, pf_autotune)
   // CUDA-graph steps (S§8(d) D.7): runs of steps between window checks are
   // captured once per (length, buffer parity) and replayed; the per-step
@@ -889,7 +891,7 @@ static int set_params_p2(pf_ctx* ctx, const pf_params* p) {
   p2_fill_params(*p, L, ctx->p2par.data());
   ctx->hp = *p;
   ctx->have_params = true;
-  ctx->jphi = ctx->jmu = nullptr;
+  ctx->jphi = ctx->jmu = ctx->jp2[0] = ctx->jp2[1] = nullptr;
   drop_graphs(ctx);
   return PF_OK;
 }
@@ -978,7 +980,7 @@ int pf_set_params(pf_ctx* ctx, const pf_params* p) {
   pf::fill_dev_params(*p, L, &ctx->dp);
   ctx->hp = *p;
   ctx->have_params = true;
-  ctx->jphi = ctx->jmu = nullptr;
+  ctx->jphi = ctx->jmu = ctx->jp2[0] = ctx->jp2[1] = nullptr;
   drop_graphs(ctx);
   return PF_OK;
 }
@@ -1077,6 +1079,30 @@ static int fill_ghost_dims(pf_ctx* ctx, double* f, int ncomp, bool is_mu, int d0
 // kernel choice of a P2 sweep from the tuning (pf_tuning p2_*)
 static P2Cfg p2cfg(const pf_tuning& t, bool mu) {
   return mu ? P2Cfg{t.p2_mu, t.p2_mu_ty, t.p2_mu_minb, t.p2_mu_pd} : P2Cfg{t.p2_phi, t.p2_phi_ty, t.p2_phi_minb, t.p2_phi_pd};
+}
+
+// one P2 sweep with kernel choice c: the run-time specialised kernel
+// (PF_VARIANT_JIT, the default: pf_p2_dev.cuh on compile-time parameters)
+// or the generic one (PF_VARIANT_TUNED); phi: ps, ms -> pd; mu: ps, pd, ms -> md
+static int p2_sweep(pf_ctx* ctx, const P2Cfg& c, bool mu, const double* ps, double* pd, const double* ms,
+                    double* md) {
+  if (ctx->variant == PF_VARIANT_JIT) {
+    const int w = mu ? 1 : 0;
+    if (!ctx->jp2[w] || memcmp(&ctx->jp2c[w], &c, sizeof c) != 0) {
+      std::string err;
+      ctx->jp2[w] = jit_get_p2(ctx, ctx->p2par.data(), ctx->g, c, mu ? P2_MU : P2_PHI, &err);
+      if (!ctx->jp2[w]) return fail(ctx, PF_ECUDA, "run-time specialisation of the P2 sweeps failed: %s", err.c_str());
+      ctx->jp2c[w] = c;
+    }
+    CU(mu ? jit_launch_p2(ctx->jp2[w], ctx->dp.Tbase, ps, pd, ms, md, ctx->stream)
+          : jit_launch_p2(ctx->jp2[w], ctx->dp.Tbase, ps, ms, nullptr, pd, ctx->stream));
+    return PF_OK;
+  }
+  if (mu)
+    p2_launch_mu(ctx->p2par.data(), c, ctx->dp.Tbase, ctx->g, ps, pd, ms, md, ctx->stream);
+  else
+    p2_launch_phi(ctx->p2par.data(), c, ctx->dp.Tbase, ctx->g, ps, ms, pd, ctx->stream);
+  return PF_OK;
 }
 
 static int fill_ghosts(pf_ctx* ctx, double* f, int ncomp, bool is_mu, bool x_done = false) {
@@ -1233,7 +1259,7 @@ static int step_impl(pf_ctx* ctx, bool phi_only, bool dry = false) {
     if (int r = join_comm(ctx)) return r;
     cudaEvent_t e0 = nullptr;
     prof_begin(ctx, 0, &e0);
-    p2_launch_phi(ctx->p2par.data(), p2cfg(ctx->tune, false), ctx->dp.Tbase, g, ps, ms, pd, ctx->stream);
+    if (int r = p2_sweep(ctx, p2cfg(ctx->tune, false), false, ps, pd, ms, md)) return r;
     ctx->nlaunch[0] += 1;
     prof_end(ctx, 0, e0);
     if (int r = check_launch(ctx, "p2 phi_sweep")) return r;
@@ -1245,7 +1271,7 @@ static int step_impl(pf_ctx* ctx, bool phi_only, bool dry = false) {
       CU(cudaMemcpyAsync(md, ms, ctx->lay.mu_bytes - 256, cudaMemcpyDeviceToDevice, ctx->stream));
     } else {
       prof_begin(ctx, 1, &e0);
-      p2_launch_mu(ctx->p2par.data(), p2cfg(ctx->tune, true), ctx->dp.Tbase, g, ps, pd, ms, md, ctx->stream);
+      if (int r2 = p2_sweep(ctx, p2cfg(ctx->tune, true), true, ps, pd, ms, md)) return r2;
       ctx->nlaunch[1] += 1;
       prof_end(ctx, 1, e0);
       if (int r2 = check_launch(ctx, "p2 mu_sweep")) return r2;
@@ -1711,7 +1737,7 @@ int pf_set_tuning(pf_ctx* ctx, const pf_tuning* t) {
   if (!ctx || !t) return PF_EINVAL;
   if (const char* m = tuning_check(*t)) return fail(ctx, PF_EINVAL, "pf_set_tuning: %s", m);
   ctx->tune = *t;
-  ctx->jphi = ctx->jmu = nullptr;
+  ctx->jphi = ctx->jmu = ctx->jp2[0] = ctx->jp2[1] = nullptr;
   drop_graphs(ctx);
   return PF_OK;
 }
@@ -1837,13 +1863,11 @@ static int time_p2(pf_ctx* ctx, const pf_tuning& t, bool mu, int reps, double* o
   const double* ms = ctx->mu[ctx->cur];
   double* md = ctx->mu[1 - ctx->cur];
   const P2Cfg c = p2cfg(t, mu);
-  auto launch = [&]() {
-    if (mu)
-      p2_launch_mu(ctx->p2par.data(), c, ctx->dp.Tbase, ctx->g, ps, pd, ms, md, ctx->stream);
-    else
-      p2_launch_phi(ctx->p2par.data(), c, ctx->dp.Tbase, ctx->g, ps, ms, pd, ctx->stream);
+  auto launch = [&]() -> cudaError_t {
+    if (p2_sweep(ctx, c, mu, ps, pd, ms, md) != PF_OK) return cudaErrorLaunchFailure;
     return cudaGetLastError();
   };
+  if (int r = p2_sweep(ctx, c, mu, ps, pd, ms, md)) return r;  // (compiles / loads the specialised kernel)
   for (int i = 0; i < 2; ++i) CU(launch());
   std::vector<cudaEvent_t> ev(reps + 1);
   for (auto& e : ev) CU(cudaEventCreate(&e));
@@ -1876,8 +1900,9 @@ static int autotune_p2(pf_ctx* ctx, unsigned mask, int reps, char* log, int logn
   for (bool mu : {false, true}) {
     if (!(mask & (mu ? PF_MU : PF_PHI))) continue;
     if (mu) {  // the mu-sweep reads phi_dst: one phi-sweep of the chosen phi kernel and its ghosts first
-      p2_launch_phi(ctx->p2par.data(), p2cfg(best, false), ctx->dp.Tbase, ctx->g, ctx->phi[ctx->cur],
-                    ctx->mu[ctx->cur], ctx->phi[1 - ctx->cur], ctx->stream);
+      if (int r = p2_sweep(ctx, p2cfg(best, false), false, ctx->phi[ctx->cur], ctx->phi[1 - ctx->cur],
+                           ctx->mu[ctx->cur], ctx->mu[1 - ctx->cur]))
+        return r;
       CU(cudaGetLastError());
       if (int r = fill_ghosts(ctx, ctx->phi[1 - ctx->cur], ctx->nph, false)) return r;
     }
@@ -1896,6 +1921,11 @@ static int autotune_p2(pf_ctx* ctx, unsigned mask, int reps, char* log, int logn
           }
           if (!tuning_check(c) && memcmp(&c, &best, sizeof c)) cands.push_back(c);
         }
+    if (ctx->variant == PF_VARIANT_JIT) {  // every candidate's specialised kernel, on host threads
+      std::vector<std::string> srcs;
+      for (const auto& c : cands) srcs.push_back(p2_specialised_source(ctx->p2par.data(), ctx->g, p2cfg(c, mu), mu ? P2_MU : P2_PHI));
+      jit_precompile_sources(srcs, (int)std::max(1u, std::thread::hardware_concurrency()));
+    }
     std::vector<double> tms(cands.size(), INFINITY);
     for (size_t i = 0; i < cands.size(); ++i)
       if (int r = time_p2(ctx, cands[i], mu, reps, &tms[i])) return r;
@@ -2079,7 +2109,7 @@ int pf_autotune(pf_ctx* ctx, unsigned mask, int passes, int reps, char* log, int
     kj += b;
   }
   ctx->tune = best;
-  ctx->jphi = ctx->jmu = nullptr;
+  ctx->jphi = ctx->jmu = ctx->jp2[0] = ctx->jp2[1] = nullptr;
   drop_graphs(ctx);
   {
     std::string err;

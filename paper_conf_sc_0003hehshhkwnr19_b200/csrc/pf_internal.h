@@ -80,6 +80,10 @@ void p2_launch_phi(const void* P, const P2Cfg& c, double Tbase, const Geom& g, c
                    double* pd, cudaStream_t s);
 void p2_launch_mu(const void* P, const P2Cfg& c, double Tbase, const Geom& g, const double* ps, const double* pd,
                   const double* ms, double* md, cudaStream_t s);
+// launch geometry of a kernel choice (the generic and the specialised kernels)
+void p2_launch_dims(const P2Cfg& c, const Geom& g, dim3* grid, dim3* block);
+// NVRTC source of the specialised P2 sweep `which` (P2_PHI / P2_MU) for kernel choice c
+std::string p2_specialised_source(const void* P, const Geom& g, const P2Cfg& c, int which);
 
 // ---- run-time specialisation (NVRTC) -------------------------------------
 enum { JIT_PHI = 0, JIT_MU = 1, P2_PHI = 2, P2_MU = 3 };  // (P2_*: pf_tuning knobs of pf_p2.cu)
@@ -96,6 +100,8 @@ void jit_release(const void* owner);  // unload every module of `owner` (pf_dest
 // compile the kernels of several tunings into the cubin cache, concurrently
 // on up to nthreads host threads (no device needed)
 void jit_precompile(const DevParams& P, const Geom& g, const std::vector<pf_tuning>& ts, int which, int nthreads);
+// the same for already generated sources (P2: p2_specialised_source)
+void jit_precompile_sources(const std::vector<std::string>& srcs, int nthreads);
 // sv == nullptr: per-step values from P (by value); else a CUDA-graph step:
 // they are copied from device memory sv into the module's constant first
 // [zlo, zhi): a z-slab of planes (the slab schedule); zhi < 0 = all planes
@@ -111,6 +117,12 @@ struct StepBatch {
   int k;
 };
 void launch_set_steps(StepVals* dst, const StepBatch& b, cudaStream_t s);
+// P2 (run-time specialised pf_p2_dev.cuh bodies): the kernel of choice c for
+// parameter block P; launch with the per-step Tbase.  phi: (a, b, c) = (ps,
+// ms, pd); mu: (a, b, c, d) = (ps, pd, ms, md)
+JitKernel* jit_get_p2(const void* owner, const void* P, const Geom& g, const P2Cfg& c, int which, std::string* err);
+cudaError_t jit_launch_p2(JitKernel* m, double Tbase, const double* a, const double* b, const void* c, double* d,
+                          cudaStream_t s);
 int jit_mu_ty_of(const JitKernel* m);
 int jit_mu_tx_of(const JitKernel* m);
 int jit_mu_zc_of(const JitKernel* m);

@@ -74,7 +74,7 @@ ABI_SYMBOLS = ["pf_query_layout", "pf_query_neighbors", "pf_create", "pf_destroy
                "pf_step_phi_only", "pf_halo_exchange", "pf_shift_window", "pf_front_height", "pf_monitor",
                "pf_set_monitors", "pf_download", "pf_get_state", "pf_set_state", "pf_set_variant", "pf_tuning_default", "pf_set_tuning",
                "pf_get_tuning", "pf_tuning_check", "pf_autotune", "pf_profile", "pf_profile_read",
-               "pf_nccl_unique_id", "pf_jit_compile_only", "pf_last_error", "pf_version"]
+               "pf_nccl_unique_id", "pf_jit_compile_only", "pf_jit_compile_only_p2", "pf_last_error", "pf_version"]
 
 _lib = None
 
@@ -115,6 +115,7 @@ def load_library(path: str = LIB_PATH):
     L.pf_profile_read.argtypes = [vp, dp, C.POINTER(C.c_int64)]
     L.pf_nccl_unique_id.argtypes = [C.POINTER(C.c_ubyte)]
     L.pf_jit_compile_only.argtypes = [C.POINTER(PFParams), ip, ip, C.POINTER(PFTuning), C.c_char_p, C.c_char_p, ip]
+    L.pf_jit_compile_only_p2.argtypes = [C.POINTER(PFParams), ip, ip, C.POINTER(PFTuning), C.c_char_p, C.c_char_p, ip]
     L.pf_last_error.argtypes = [vp]
     L.pf_last_error.restype = C.c_char_p
     L.pf_version.restype = C.c_char_p
@@ -194,6 +195,19 @@ def jit_compile_only(params: dict, n: int = 64, cubin_path: str | None = None, t
                                            (cubin_path or "").encode(), log, 8192)
     if r < 0:
         raise PFError(f"specialised compile failed: {log.value.decode()}")
+    return r
+
+
+def jit_compile_only_p2(params: dict, n: int = 64, cubin_path: str | None = None, tuning: dict | None = None) -> int:
+    """As jit_compile_only for the P2 sweeps (3 phases, 1 mu): the specialised
+    phi- and mu-sweep of the kernel choice in `tuning` (p2_* knobs)."""
+    p = make_params(params)
+    log = C.create_string_buffer(8192)
+    t = C.byref(_tuning_struct(tuning)) if tuning is not None else None
+    r = load_library().pf_jit_compile_only_p2(C.byref(p), int(params.get("liquid", 2)), int(n), t,
+                                              (cubin_path or "").encode(), log, 8192)
+    if r < 0:
+        raise PFError(f"specialised P2 compile failed: {log.value.decode()}")
     return r
 
 

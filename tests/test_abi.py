@@ -160,3 +160,26 @@ def test_p2_layout_and_params_struct():
     assert abs(p.aniso_R[0][2][1][0] - P["aniso_R"][0, 2, 1, 0]) == 0.0
     assert p.aniso_delta[1][2] == P["aniso_delta"][1, 2]
     assert p.A0[2][0][0] == P["A0"][2, 0, 0] and p.D[1][0][0] == P["D"][1, 0, 0]
+
+
+@pytest.mark.parametrize("knobs", [{}, {"p2_phi": 1, "p2_mu": 1}, {"p2_phi": 2, "p2_mu": 2},
+                                   {"p2_phi_ty": 4, "p2_phi_minb": 4, "p2_mu_ty": 8, "p2_mu_minb": 1, "p2_phi_pd": 0}])
+def test_p2_specialised_kernels_compile_without_gpu(lib, tmp_path, knobs):
+    """The run-time specialised P2 sweeps (pf_p2_dev.cuh on compile-time
+    parameters) build with NVRTC for every kernel choice; with the P2 set
+    (isotropic unrotated solid-solid pair, one unrotated grain) the phi-sweep
+    issues far fewer fp64 instructions than the generic stress-set build."""
+    from paper_conf_sc_0003hehshhkwnr19_b200 import inputs as I
+    from paper_conf_sc_0003hehshhkwnr19_b200 import pf
+    t = dict(pf.tuning_default(), **knobs)
+    assert pf.tuning_check(t) == "ok"
+    cub = str(tmp_path / "p2.cubin")
+    assert pf.jit_compile_only_p2(I.params_p2(), cubin_path=cub, tuning=t) > 0
+    assert pf.jit_compile_only_p2(dict(I.params_p2_stress(), liquid=0), cubin_path=cub + "s", tuning=t) > 0
+
+    def fp64(path):
+        out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-sass", path], capture_output=True, text=True).stdout
+        assert "pf_p2_jit" in out
+        return len(re.findall(r"\b(DFMA|DADD|DMUL)\b", out))
+    if not knobs:
+        assert fp64(cub + ".phi") < 0.8 * fp64(cub + "s.phi")

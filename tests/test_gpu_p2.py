@@ -125,6 +125,36 @@ def test_p2_invariants_and_monitor(pfmod):
     assert p.shape == (3,) + shape
 
 
+@pytest.mark.parametrize("kern", ["side", "march", "naive"])
+@pytest.mark.parametrize("pset", ["p2", "p2_stress", "p2_iso"])
+def test_p2_specialised_equals_generic(pfmod, omod, pset, kern, monkeypatch):
+    """The run-time specialised P2 sweeps (variant jit, the default: the
+    bodies of pf_p2_dev.cuh on compile-time parameters, isotropic unrotated
+    pairs as 2 q, unrotated pairs without rotation) give the generic
+    kernels' bits (variant tuned), and the generic kernels meet the oracle
+    bar on their own."""
+    monkeypatch.setenv("PF_P2_NAIVE", "1" if kern == "naive" else "0")
+    monkeypatch.setenv("PF_P2_PHI", "march" if kern == "march" else "side")
+    monkeypatch.setenv("PF_P2_MU", "march" if kern == "march" else "side")
+    P = {"p2": I.params_p2(), "p2_stress": I.params_p2_stress(), "p2_iso": I.params_p2(aniso=0)}[pset]
+    shape = (18, 21, 37)
+    phi, mu = I.ic_voronoi(shape, seed=13, N=3, M=1)
+    outs = []
+    for variant in ("jit", "tuned"):
+        g = pfmod.PhaseField(shape, P)
+        g.set_variant(variant)
+        g.init_fields(phi, mu)
+        g.step(3)
+        outs.append(g.download())
+        g.close()
+    assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
+    o = omod.Oracle(shape, P)
+    o.init(phi, mu)
+    o.step(3)
+    op, om = o.download()
+    assert rel_linf(outs[1][0], op) <= 1e-12 and rel_linf(outs[1][1], om) <= 1e-12
+
+
 @pytest.mark.parametrize("cfg", ["8x2", "8x1", "4x3", "4x4"])
 def test_p2_side_tilings_bitwise(pfmod, monkeypatch, cfg):
     """The side-staged kernels' other tile heights / occupancies (PF_P2_SIDE)
