@@ -319,7 +319,7 @@ typedef struct {
                         2 one thread per cell (every face twice)               */
   int p2_mu;         /* P2 mu kernel: the same three                           */
   int p2_phi_ty;     /* side-staged P2 phi: tile height (4 or 8) and CTAs per  */
-  int p2_phi_minb;   /*   SM: (8, 2) default, (8, 1), (4, 3), (4, 4)           */
+  int p2_phi_minb;   /*   SM: (8, 2) default, (8, 1), (4, 3..6)                */
   int p2_mu_ty;      /* side-staged P2 mu: the same, default (4, 4)            */
   int p2_mu_minb;
   int p2_phi_pd;     /* side-staged P2 phi / mu: L2 prefetch distance in planes */

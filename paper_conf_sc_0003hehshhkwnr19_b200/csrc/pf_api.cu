@@ -1908,11 +1908,11 @@ static int autotune_p2(pf_ctx* ctx, unsigned mask, int reps, char* log, int logn
     }
     std::vector<pf_tuning> cands{best};
     for (int k : {0, 1, 2})
-      for (int tm : {0, 1, 2, 3})
+      for (int tm : {0, 1, 2, 3, 4, 5})
         for (int pdist : {0, 1, 2, 3, 4}) {
           if (k != 0 && (tm || pdist)) continue;  // tile / prefetch only matter for the side-staged kernels
           pf_tuning c = best;
-          const int ty = tm < 2 ? 8 : 4, mb = tm == 0 ? 2 : tm == 1 ? 1 : tm == 2 ? 3 : 4;
+          const int ty = tm < 2 ? 8 : 4, mb = tm == 0 ? 2 : tm == 1 ? 1 : tm + 1;  // 8x2 8x1 4x3 4x4 4x5 4x6
           (mu ? c.p2_mu : c.p2_phi) = k;
           if (k == 0) {
             (mu ? c.p2_mu_ty : c.p2_phi_ty) = ty;

@@ -268,6 +268,10 @@ void p2_launch_phi(const void* Pv, const P2Cfg& c, double Tbase, const Geom& g, 
     dim3 b(p2::TXP, ty), gr((g.nx + p2::TXP - 1) / p2::TXP, (g.ny + ty - 1) / ty, (g.nz + p2::ZCS - 1) / p2::ZCS);
     if (ty == 4 && mb == 3)
       p2::k_phi_side<4, 3><<<gr, b, 0, s>>>(P, g, ps, ms, pd);
+    else if (ty == 4 && mb == 5)
+      p2::k_phi_side<4, 5><<<gr, b, 0, s>>>(P, g, ps, ms, pd);
+    else if (ty == 4 && mb == 6)
+      p2::k_phi_side<4, 6><<<gr, b, 0, s>>>(P, g, ps, ms, pd);
     else if (ty == 4)
       p2::k_phi_side<4, 4><<<gr, b, 0, s>>>(P, g, ps, ms, pd);
     else if (mb == 1)
@@ -303,6 +307,8 @@ void p2_launch_mu(const void* Pv, const P2Cfg& c, double Tbase, const Geom& g, c
     dim3 b(p2::TXP, ty), gr((g.nx + p2::TXP - 1) / p2::TXP, (g.ny + ty - 1) / ty, (g.nz + p2::ZCS - 1) / p2::ZCS);
 #define PF_P2_MUS(LL)                                                                         \
   (ty == 4 && mb == 3 ? (p2::k_mu_side<LL, 4, 3><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md))     \
+   : ty == 4 && mb == 5 ? (p2::k_mu_side<LL, 4, 5><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md))   \
+   : ty == 4 && mb == 6 ? (p2::k_mu_side<LL, 4, 6><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md))   \
    : ty == 4          ? (p2::k_mu_side<LL, 4, 4><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md))     \
    : mb == 1          ? (p2::k_mu_side<LL, 8, 1><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md))     \
                       : (p2::k_mu_side<LL, 8, 2><<<gr, b, 0, s>>>(P, g, ps, pd, ms, md)))

@@ -155,7 +155,7 @@ def test_p2_specialised_equals_generic(pfmod, omod, pset, kern, monkeypatch):
     assert rel_linf(outs[1][0], op) <= 1e-12 and rel_linf(outs[1][1], om) <= 1e-12
 
 
-@pytest.mark.parametrize("cfg", ["8x2", "8x1", "4x3", "4x4"])
+@pytest.mark.parametrize("cfg", ["8x2", "8x1", "4x3", "4x4", "4x5", "4x6"])
 def test_p2_side_tilings_bitwise(pfmod, monkeypatch, cfg):
     """The side-staged kernels' other tile heights / occupancies (PF_P2_SIDE)
     give the default's bits: each face flux is computed from the same two

@@ -46,5 +46,5 @@ for a, b in loops:
     st = sum(x["stall"] for x in seg)
     nf = cnt(fp64)
     print(f"loop {ins[a]['addr']:#06x}-{ins[b]['addr']:#06x}: {len(seg)} instr, fp64 {nf}, MUFU {cnt(('MUFU',))}, "
-          f"LDS {cnt(('LDS',))}, STS {cnt(('STS',))}, LDG {cnt(('LDG',))}, STG {cnt(('STG',))}, BAR {cnt(('BAR',))}, "
+          f"LDS {cnt(('LDS',))}, STS {cnt(('STS',))}, LDL {cnt(('LDL',))}, STL {cnt(('STL',))}, LDG {cnt(('LDG',))}, STG {cnt(('STG',))}, BAR {cnt(('BAR',))}, "
           f"stall sum {st} cyc, fp64 pipe {2 * nf} cyc, waits on scoreboards {sum(1 for x in seg if x['wait'])}")
