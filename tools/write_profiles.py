@@ -30,11 +30,16 @@ KEYS = ["gpu__time_duration.sum", "launch__registers_per_thread", "launch__occup
         "lts__t_sector_hit_rate.pct", "smsp__inst_executed.sum", "smsp__sass_inst_executed_op_global_ld.sum",
         "smsp__sass_inst_executed_op_shared_ld.sum", "smsp__sass_inst_executed_op_local_ld.sum"]
 summary = {}
-for kern in ("mu", "phi", "ghost", "p2phi", "p2mu"):
-    rep = os.path.join(src, f"prof_{kern}.ncu-rep")
+# (report, launch in it, name): prof_p2jit holds the specialised P2 phi- and
+# mu-sweep (both named pf_p2_jit), launches 0 and 1
+JOBS = [("mu", 0, "mu"), ("phi", 0, "phi"), ("ghost", 0, "ghost"), ("p2phi", 0, "p2phi"), ("p2mu", 0, "p2mu"),
+        ("p2jit", 0, "p2jitphi"), ("p2jit", 1, "p2jitmu")]
+for rname, li, kern in JOBS:
+    rep = os.path.join(src, f"prof_{rname}.ncu-rep")
     if not os.path.exists(rep):
         continue
-    raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    sel = ["--launch-skip", str(li), "--launch-count", "1"]
+    raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"] + sel, capture_output=True, text=True).stdout
     rows = list(csv.reader(raw.splitlines()))
     h, u, v = rows[0], rows[1], rows[2]
     m = {n: (v[i], u[i]) for i, n in enumerate(h)}
@@ -63,7 +68,7 @@ for kern in ("mu", "phi", "ghost", "p2phi", "p2mu"):
           if n.startswith("smsp__average_warps_issue_stalled") and n.endswith("per_issue_active.ratio")}
     lines += ["", "  warp stall reasons (cycles per issued instruction):"]
     lines += [f"    {k:28s} {x:6.2f}" for k, x in sorted(st.items(), key=lambda kv: -kv[1]) if x > 0.05]
-    srcp = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
+    srcp = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"] + sel,
                           capture_output=True, text=True).stdout
     srows = list(csv.reader(srcp.splitlines()))
     if len(srows) > 2:
