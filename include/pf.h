@@ -268,7 +268,7 @@ typedef struct {
   int mu_prefetch;   /* software prefetch of the own column: 0 off, 1 L2, 2 L1      */
   int mu_pfd;        /* prefetch distance in planes: 2..6                           */
   int mu_rpf;        /* 1: own cell's L1-missing loads one plane ahead in registers */
-  int mu_halo_l1;    /* 1: halo-ring cells' next-plane lines prefetched into L1     */
+  int mu_halo_l1;    /* 1: halo-ring cells' next-plane lines prefetched into L1 (default 0 with mu_hasync, else 1) */
   int mu_fxreg;      /* 1: own -x/-y fluxes taken from registers in the divergence  */
   int mu_qreg;       /* 1: own cell's face-side data kept in registers from the
                         build (no shared-memory re-read; needs registers)        */
@@ -330,6 +330,17 @@ typedef struct {
                         solid-solid boundaries); same results, data-dependent
                         time; off by default and not searched by pf_autotune
                         (the benchmark reports it separately)                  */
+  int mu_hasync;     /* 1: the two-rows mu-sweep stages its halo ring one plane
+                        ahead with asynchronous global -> shared copies
+                        (cp.async: phi_src two planes ahead into a 3-plane
+                        ring, the solids' phi_dst and mu one plane ahead), so
+                        a halo cell builds its side from shared memory with no
+                        global load on the critical path (1: 8-B copies; 2:
+                        the halo rows in 16-B pieces cached in L2 only; 3: as
+                        2, and the tile's edge rows take their outer
+                        y-neighbour from the ring).  Default 1; ignored (0)
+                        unless mu_rpt = 2 and mu_hcar = mu_hpipe = mu_tmem =
+                        0; 3 without mu_rpf acts as 2                          */
 } pf_tuning;
 
 /* The built-in defaults (the measured best at 256^3 on one B200,

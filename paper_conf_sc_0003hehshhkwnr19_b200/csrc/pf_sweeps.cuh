@@ -127,6 +127,9 @@ constexpr int MU_TY = PF_MU_TY;
 #ifndef PF_MU_HCAR  // two-rows mu-sweep: the halo ring's phi_src z column carried in shared memory
 #define PF_MU_HCAR 0
 #endif
+#ifndef PF_MU_HASYNC  // two-rows mu-sweep: halo ring staged one plane ahead by cp.async (global -> shared)
+#define PF_MU_HASYNC 0
+#endif
 #ifndef PF_MU_XSHFL  // two-rows mu-sweep: own cd_x from the lane neighbours' carried phi_src (shuffles)
 #define PF_MU_XSHFL 0
 #endif
@@ -1099,6 +1102,22 @@ __device__ __forceinline__ void tm_ld_side(unsigned ta, FaceSide& s) {
   s.m[1] = v[16];
 }
 #endif
+// asynchronous global -> shared copies (cp.async, sm_80+): 8 B cached in L1
+// (.ca), 16 B cached in L2 only (.cg); completion per thread (wait_all), a
+// CTA barrier after it publishes the data to the other threads
+__device__ __forceinline__ void cp_async8(void* smem, const void* gmem) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"((unsigned)__cvta_generic_to_shared(smem)),
+               "l"(gmem)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"((unsigned)__cvta_generic_to_shared(smem)),
+               "l"(gmem)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
+
 // ===========================================================================
 // mu-sweep with two tile rows per thread (pf_tuning mu_rpt = 2): a CTA of
 // 32 x (MTY/2) threads owns a 32 x MTY tile; thread (lane, w) updates rows
@@ -1144,7 +1163,7 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
   else if (th >= 2 * MTY + MTX && th < 2 * MTY + 2 * MTX) { hx = th - 2 * MTY - MTX + 1; hy = MTY + 1; hwx = true; }
   if (hwx || hwy) hs = hidx<MTX>(hx, hy);
   const int hgx = min(x0 + hx - 1, g.nx), hgy = min(y0 + hy - 1, g.ny);
-#if PF_MU_HCAR
+#if PF_MU_HCAR || PF_MU_HASYNC
   // halo ring with its phi_src z column carried in shared memory (tuning
   // mu_hcar): ring cell ci holds phi_src of planes k-1, k, k+1 in slots
   // (k+2)%3, k%3, (k+1)%3, so a halo cell loads per plane only phi_src(k+1),
@@ -1171,6 +1190,56 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
     ci = ridx(chx, chy);
     cring = g.at(min(x0 + chx - 1, g.nx), min(y0 + chy - 1, g.ny), 0);
   }
+#if PF_MU_HASYNC
+  // tuning mu_hasync: the ring is filled by asynchronous copies (cp.async)
+  // one build ahead -- per plane k, after the barrier that ends the build of
+  // D(k), phi_src(k + 2) into ring slot (k + 2) % 3 (the slot of k - 1, just
+  // read) and the solids' phi_dst / mu of plane k + 1 into dring, completed
+  // before the plane's second barrier -- so a halo cell builds its side with
+  // no global load on the critical path
+  // mu_hasync >= 2: a halo-row cell at odd hx copies itself and its right
+  // neighbour as one 16-B piece (cached in L2 only; rows are 128-B aligned,
+  // the ring's row slots 16-B aligned), the even ones none; column cells
+  // and corners 8 B each.  (Past the ghost cell of a ragged tile the pieces
+  // hold what memory holds there, where the 8-B copies clamp: only inactive
+  // cells read those.)
+  __shared__ __align__(16) double dring[NSOL + M][RC];
+  const bool row16 = PF_MU_HASYNC >= 2 && hwx;
+  const bool cp16 = row16 && (hx & 1);
+  const i64 crow = row16 ? g.at(x0 + hx - 1, hgy, 0) : cring;
+  auto stage = [&](const int kf, const int kd) {
+    if (ci >= 0 && !(row16 && !cp16)) {
+#pragma unroll
+      for (int a = 0; a < N; ++a) {
+        if (cp16)
+          cp_async16(&fring[(kf + 3) % 3][a][ci], ps + a * F + crow + (i64)kf * g.plane);
+        else
+          cp_async8(&fring[(kf + 3) % 3][a][ci], ps + a * F + cring + (i64)kf * g.plane);
+      }
+    }
+    if (kd >= 0 && hs >= 0 && !(row16 && !cp16)) {
+#pragma unroll
+      for (int u = 0; u < NSOL; ++u) {
+        if (cp16)
+          cp_async16(&dring[u][ci], pd + solid_phase(L, u) * F + crow + (i64)kd * g.plane);
+        else
+          cp_async8(&dring[u][ci], pd + solid_phase(L, u) * F + cring + (i64)kd * g.plane);
+      }
+#pragma unroll
+      for (int i = 0; i < M; ++i) {
+        if (cp16)
+          cp_async16(&dring[NSOL + i][ci], ms + i * F + crow + (i64)kd * g.plane);
+        else
+          cp_async8(&dring[NSOL + i][ci], ms + i * F + cring + (i64)kd * g.plane);
+      }
+    }
+    cp_async_commit();
+  };
+  stage(z0 - 1, -1);
+  stage(z0, -1);
+  stage(z0 + 1, z0);
+  cp_async_wait_all();
+#else
   if (ci >= 0) {
     const double* f = ps + cring + (i64)(z0 - 1) * g.plane;
 #pragma unroll
@@ -1179,6 +1248,7 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
       fring[z0 % 3][a][ci] = __ldg(f + a * F + g.plane);
     }
   }
+#endif
   __syncthreads();
 #endif
 
@@ -1300,8 +1370,17 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
         v0[D_CX + a] = __ldg(f0 + 1) - __ldg(f0 - 1);
         v1[D_CX + a] = __ldg(f1 + 1) - __ldg(f1 - 1);
 #endif
+#if PF_MU_HASYNC >= 3
+        // the tile's edge rows take their outer y-neighbour from the staged
+        // ring (the same value: the bottom / top halo row at plane k)
+        const double ym = w == 0 ? fring[k % 3][a][2 * (MTY + 2) + lane] : __ldg(f0 - g.pitch);
+        const double yp = w == TYT - 1 ? fring[k % 3][a][2 * (MTY + 2) + MTX + lane] : __ldg(f1 + g.pitch);
+        v0[D_CY + a] = fcar[1][a] - ym;
+        v1[D_CY + a] = yp - fcar[0][a];
+#else
         v0[D_CY + a] = fcar[1][a] - __ldg(f0 - g.pitch);
         v1[D_CY + a] = __ldg(f1 + g.pitch) - fcar[0][a];
+#endif
 #if PF_MU_TMEM
         v0[D_CZ + a] = !last ? rnf[0][a] - fprev[0][a] : 0.0;
         v1[D_CZ + a] = !last ? rnf[1][a] - fprev[1][a] : 0.0;
@@ -1355,7 +1434,31 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
 #endif
     }
 #endif
-#if PF_MU_HCAR
+#if PF_MU_HASYNC
+    if (!last && hs >= 0) {  // the side from the staged ring (the operands of build_cell: the same bits)
+      const int sm = (k + 2) % 3, s0 = k % 3, sp = (k + 1) % 3;
+      double v[D_NV];
+#pragma unroll
+      for (int a = 0; a < N; ++a) {
+        const double tt = fring[s0][a][tpi] - fring[s0][a][tmi];
+        v[D_F + a] = fring[s0][a][ci];
+        v[D_CX + a] = hwx ? tt : 0.0;
+        v[D_CY + a] = hwx ? 0.0 : tt;
+        v[D_CZ + a] = fring[sp][a][ci] - fring[sm][a][ci];
+        v[D_DP + a] = 0.0;  // the liquid's dphi of a halo cell is never read
+      }
+#pragma unroll
+      for (int u = 0; u < NSOL; ++u) {
+        const int a = solid_phase(L, u);
+        v[D_DP + a] = dring[u][ci] - v[D_F + a];
+      }
+      v[D_MU + 0] = dring[NSOL][ci];
+      v[D_MU + 1] = dring[NSOL + 1][ci];
+      double2* d = reinterpret_cast<double2*>(D + (size_t)hs * D_NV);
+#pragma unroll
+      for (int j = 0; j < D_NV / 2; ++j) d[j] = make_double2(v[2 * j], v[2 * j + 1]);
+    }
+#elif PF_MU_HCAR
     if (!last && ci >= 0) {
       const i64 c = cring + (i64)k * g.plane;
       const int sm = (k + 2) % 3, s0 = k % 3, sp = (k + 1) % 3;
@@ -1391,6 +1494,9 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
     if (!last && hs >= 0) build_cell<NC>(g, ps, pd, ms, hgx, hgy, k, hwx, hwy, true, D, hs);
 #endif
     __syncthreads();
+#if PF_MU_HASYNC
+    if (!last && k + 1 < z1) stage(k + 2, k + 1);  // the next build's ring (overwrites what this build read)
+#endif
     // (b) z-faces k-1/2 and (c) cell updates of plane k-1
 #pragma unroll
     for (int r = 0; r < 2; ++r) {
@@ -1522,6 +1628,9 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
 #pragma unroll
         for (int i = 0; i < M; ++i) fxs[(i * MTY + lane) * (MTX + 1) + MTX] = Fe[i];
       }
+#if PF_MU_HASYNC
+      cp_async_wait_all();  // this thread's staging copies, published by the barrier
+#endif
       __syncthreads();
 #pragma unroll
       for (int i = 0; i < M; ++i) {

@@ -73,6 +73,15 @@ CORNERS = [
     # warp-uniform skip of the anti-trapping current where it is exactly 0
     {"mu_atskip": 1},
     dict(R1, mu_atskip=1),
+    # the halo ring staged one plane ahead by cp.async (alone, ragged chunks /
+    # tiles, without the L1 prefetch, with persistent shares, with shuffles)
+    {"mu_hasync": 1},
+    {"mu_hasync": 1, "mu_zc": 7, "mu_ty": 6, "mu_minb": 3, "mu_rpf": 0, "mu_halo_l1": 0},
+    {"mu_hasync": 1, "mu_pers": 1, "mu_ty": 10, "mu_minb": 2},
+    {"mu_hasync": 1, "mu_xshfl": 1, "mu_zc": 5},
+    {"mu_hasync": 2, "mu_halo_l1": 0},
+    {"mu_hasync": 3, "mu_zc": 7, "mu_ty": 6, "mu_minb": 3, "mu_halo_l1": 0},
+    {"mu_hasync": 3, "mu_pers": 1, "mu_ty": 10, "mu_minb": 2, "mu_xshfl": 1},
 ]
 
 
