@@ -335,12 +335,12 @@ typedef struct {
                         (cp.async: phi_src two planes ahead into a 3-plane
                         ring, the solids' phi_dst and mu one plane ahead), so
                         a halo cell builds its side from shared memory with no
-                        global load on the critical path (1: 8-B copies; 2:
-                        the halo rows in 16-B pieces cached in L2 only; 3: as
-                        2, and the tile's edge rows take their outer
-                        y-neighbour from the ring).  Default 1; ignored (0)
+                        global load on the critical path (1: the ring's
+                        cells, 8-B copies; 2: the whole halo tile's phi_src
+                        planes in 16-B pieces, so the own cells read phi_src
+                        from shared memory too).  Default 1; ignored (0)
                         unless mu_rpt = 2 and mu_hcar = mu_hpipe = mu_tmem =
-                        0; 3 without mu_rpf acts as 2                          */
+                        0; 2 without mu_rpf acts as 1                          */
 } pf_tuning;
 
 /* The built-in defaults (the measured best at 256^3 on one B200,

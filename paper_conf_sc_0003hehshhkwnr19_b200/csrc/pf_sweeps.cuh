@@ -1174,7 +1174,9 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
   // (hx = 1..MTX), top row; the 4 corners are carried by threads 0..3.
   constexpr int RC = 2 * (MTY + 2) + 2 * MTX;
   static_assert(NT - 2 * MTX - 2 * MTY >= 4, "mu_hcar: four free threads carry the ring corners");
+#if PF_MU_HASYNC < 2
   __shared__ __align__(16) double fring[3][N][RC];  // phase-major: a warp's ring reads are contiguous
+#endif
   auto ridx = [](int rx, int ry) {
     return rx == 0 ? ry : rx == MTX + 1 ? MTY + 2 + ry : 2 * (MTY + 2) + (ry == 0 ? 0 : MTX) + rx - 1;
   };
@@ -1197,41 +1199,36 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
   // read) and the solids' phi_dst / mu of plane k + 1 into dring, completed
   // before the plane's second barrier -- so a halo cell builds its side with
   // no global load on the critical path
-  // mu_hasync >= 2: a halo-row cell at odd hx copies itself and its right
-  // neighbour as one 16-B piece (cached in L2 only; rows are 128-B aligned,
-  // the ring's row slots 16-B aligned), the even ones none; column cells
-  // and corners 8 B each.  (Past the ghost cell of a ragged tile the pieces
-  // hold what memory holds there, where the 8-B copies clamp: only inactive
-  // cells read those.)
   __shared__ __align__(16) double dring[NSOL + M][RC];
-  const bool row16 = PF_MU_HASYNC >= 2 && hwx;
-  const bool cp16 = row16 && (hx & 1);
-  const i64 crow = row16 ? g.at(x0 + hx - 1, hgy, 0) : cring;
+#if PF_MU_HASYNC >= 2
+  // mu_hasync 2: the whole halo tile's phi_src planes (rows x0 - 2 .. x0 +
+  // MTX + 1, 16-B pieces cached in L2 only; rows are 128-B aligned) in a
+  // 3-plane ring: the own cells take phi_src(k) and its x / y / z neighbours
+  // from shared memory as well (only phi_dst and mu of the own cells stay
+  // register-prefetched loads).  Past the ghost cell of a ragged tile the
+  // pieces hold what memory holds there (only inactive cells read those).
+  constexpr int TRX = MTX + 4, TRP = TRX / 2;  // ring row length, 16-B pieces per row
+  __shared__ __align__(16) double tring[3][N][MTY + 2][TRX];
+#endif
   auto stage = [&](const int kf, const int kd) {
-    if (ci >= 0 && !(row16 && !cp16)) {
-#pragma unroll
-      for (int a = 0; a < N; ++a) {
-        if (cp16)
-          cp_async16(&fring[(kf + 3) % 3][a][ci], ps + a * F + crow + (i64)kf * g.plane);
-        else
-          cp_async8(&fring[(kf + 3) % 3][a][ci], ps + a * F + cring + (i64)kf * g.plane);
-      }
+#if PF_MU_HASYNC >= 2
+    for (int it = t; it < (MTY + 2) * N * TRP; it += NT) {
+      const int pc = it % TRP, a = (it / TRP) % N, ry = it / (TRP * N);
+      cp_async16(&tring[(kf + 3) % 3][a][ry][2 * pc],
+                 ps + a * F + g.at(x0 - 2 + 2 * pc, min(y0 + ry - 1, g.ny), kf));
     }
-    if (kd >= 0 && hs >= 0 && !(row16 && !cp16)) {
+#else
+    if (ci >= 0) {
 #pragma unroll
-      for (int u = 0; u < NSOL; ++u) {
-        if (cp16)
-          cp_async16(&dring[u][ci], pd + solid_phase(L, u) * F + crow + (i64)kd * g.plane);
-        else
-          cp_async8(&dring[u][ci], pd + solid_phase(L, u) * F + cring + (i64)kd * g.plane);
-      }
+      for (int a = 0; a < N; ++a) cp_async8(&fring[(kf + 3) % 3][a][ci], ps + a * F + cring + (i64)kf * g.plane);
+    }
+#endif
+    if (kd >= 0 && hs >= 0) {
 #pragma unroll
-      for (int i = 0; i < M; ++i) {
-        if (cp16)
-          cp_async16(&dring[NSOL + i][ci], ms + i * F + crow + (i64)kd * g.plane);
-        else
-          cp_async8(&dring[NSOL + i][ci], ms + i * F + cring + (i64)kd * g.plane);
-      }
+      for (int u = 0; u < NSOL; ++u)
+        cp_async8(&dring[u][ci], pd + solid_phase(L, u) * F + cring + (i64)kd * g.plane);
+#pragma unroll
+      for (int i = 0; i < M; ++i) cp_async8(&dring[NSOL + i][ci], ms + i * F + cring + (i64)kd * g.plane);
     }
     cp_async_commit();
   };
@@ -1341,7 +1338,45 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
       asm volatile("prefetch.global.L1 [%0];" ::"l"(ms + F + ch));
     }
     // (a) publish D(k) of the two own cells and of the halo ring
-#if PF_MU_RPF
+#if PF_MU_HASYNC >= 2 && PF_MU_RPF
+    {
+      // mu_hasync 2: phi_src(k) and its neighbours from the staged tile ring
+      // (the operands of the register path below: the same bits); phi_dst
+      // and mu of the own cells register-prefetched one plane ahead
+      const int s0 = k % 3, sp = (k + 1) % 3, sm = (k + 2) % 3;
+      double v0[D_NV], v1[D_NV];
+#pragma unroll
+      for (int r = 0; r < 2; ++r) {
+        double* v = r ? v1 : v0;
+        const int ry = 2 * w + r + 1;
+#pragma unroll
+        for (int a = 0; a < N; ++a) {
+          v[D_F + a] = tring[s0][a][ry][lane + 2];
+          v[D_CX + a] = tring[s0][a][ry][lane + 3] - tring[s0][a][ry][lane + 1];
+          v[D_CY + a] = tring[s0][a][ry + 1][lane + 2] - tring[s0][a][ry - 1][lane + 2];
+          v[D_CZ + a] = !last ? tring[sp][a][ry][lane + 2] - tring[sm][a][ry][lane + 2] : 0.0;
+          v[D_DP + a] = rnd[r][a] - v[D_F + a];
+        }
+        v[D_MU] = rnm[r][0];
+        v[D_MU + 1] = rnm[r][1];
+      }
+      double2* d0 = reinterpret_cast<double2*>(D + (size_t)me[0] * D_NV);
+      double2* d1 = reinterpret_cast<double2*>(D + (size_t)me[1] * D_NV);
+#pragma unroll
+      for (int j = 0; j < D_NV / 2; ++j) {
+        d0[j] = make_double2(v0[2 * j], v0[2 * j + 1]);
+        d1[j] = make_double2(v1[2 * j], v1[2 * j + 1]);
+      }
+#pragma unroll
+      for (int r = 0; r < 2 && !last; ++r) {
+        const i64 c = g.at(xc, yc[r], k);
+#pragma unroll
+        for (int a = 0; a < N; ++a) rnd[r][a] = ldh(pd + a * F + c + g.plane);
+        rnm[r][0] = ldh(ms + c + g.plane);
+        rnm[r][1] = ldh(ms + F + c + g.plane);
+      }
+    }
+#elif PF_MU_RPF
     {
       // as build_own_rpf for both rows; each row's y-neighbour inside the
       // pair is the other row's carried phi_src(k) (for an active row it is
@@ -1370,17 +1405,8 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
         v0[D_CX + a] = __ldg(f0 + 1) - __ldg(f0 - 1);
         v1[D_CX + a] = __ldg(f1 + 1) - __ldg(f1 - 1);
 #endif
-#if PF_MU_HASYNC >= 3
-        // the tile's edge rows take their outer y-neighbour from the staged
-        // ring (the same value: the bottom / top halo row at plane k)
-        const double ym = w == 0 ? fring[k % 3][a][2 * (MTY + 2) + lane] : __ldg(f0 - g.pitch);
-        const double yp = w == TYT - 1 ? fring[k % 3][a][2 * (MTY + 2) + MTX + lane] : __ldg(f1 + g.pitch);
-        v0[D_CY + a] = fcar[1][a] - ym;
-        v1[D_CY + a] = yp - fcar[0][a];
-#else
         v0[D_CY + a] = fcar[1][a] - __ldg(f0 - g.pitch);
         v1[D_CY + a] = __ldg(f1 + g.pitch) - fcar[0][a];
-#endif
 #if PF_MU_TMEM
         v0[D_CZ + a] = !last ? rnf[0][a] - fprev[0][a] : 0.0;
         v1[D_CZ + a] = !last ? rnf[1][a] - fprev[1][a] : 0.0;
@@ -1440,11 +1466,18 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
       double v[D_NV];
 #pragma unroll
       for (int a = 0; a < N; ++a) {
+#if PF_MU_HASYNC >= 2
+        const double tt = hwx ? tring[s0][a][hy][hx + 2] - tring[s0][a][hy][hx]
+                              : tring[s0][a][hy + 1][hx + 1] - tring[s0][a][hy - 1][hx + 1];
+        v[D_F + a] = tring[s0][a][hy][hx + 1];
+        v[D_CZ + a] = tring[sp][a][hy][hx + 1] - tring[sm][a][hy][hx + 1];
+#else
         const double tt = fring[s0][a][tpi] - fring[s0][a][tmi];
         v[D_F + a] = fring[s0][a][ci];
+        v[D_CZ + a] = fring[sp][a][ci] - fring[sm][a][ci];
+#endif
         v[D_CX + a] = hwx ? tt : 0.0;
         v[D_CY + a] = hwx ? 0.0 : tt;
-        v[D_CZ + a] = fring[sp][a][ci] - fring[sm][a][ci];
         v[D_DP + a] = 0.0;  // the liquid's dphi of a halo cell is never read
       }
 #pragma unroll

@@ -80,8 +80,8 @@ CORNERS = [
     {"mu_hasync": 1, "mu_pers": 1, "mu_ty": 10, "mu_minb": 2},
     {"mu_hasync": 1, "mu_xshfl": 1, "mu_zc": 5},
     {"mu_hasync": 2, "mu_halo_l1": 0},
-    {"mu_hasync": 3, "mu_zc": 7, "mu_ty": 6, "mu_minb": 3, "mu_halo_l1": 0},
-    {"mu_hasync": 3, "mu_pers": 1, "mu_ty": 10, "mu_minb": 2, "mu_xshfl": 1},
+    {"mu_hasync": 2, "mu_zc": 7, "mu_ty": 6, "mu_minb": 3},
+    {"mu_hasync": 2, "mu_pers": 1, "mu_ty": 10, "mu_minb": 2, "mu_xshfl": 1},
 ]
 
 
