@@ -341,6 +341,9 @@ typedef struct {
                         from shared memory too).  Default 1; ignored (0)
                         unless mu_rpt = 2 and mu_hcar = mu_hpipe = mu_tmem =
                         0; 2 without mu_rpf acts as 1                          */
+  int p2_mu_hasync;  /* 1: the specialised side-staged P2 mu-sweep (32 x 4 tiles) stages its
+                        halo ring one build ahead with cp.async (as mu_hasync
+                        1; default); same bits                                 */
 } pf_tuning;
 
 /* The built-in defaults (the measured best at 256^3 on one B200,

@@ -1078,7 +1078,8 @@ static int fill_ghost_dims(pf_ctx* ctx, double* f, int ncomp, bool is_mu, int d0
 
 // kernel choice of a P2 sweep from the tuning (pf_tuning p2_*)
 static P2Cfg p2cfg(const pf_tuning& t, bool mu) {
-  return mu ? P2Cfg{t.p2_mu, t.p2_mu_ty, t.p2_mu_minb, t.p2_mu_pd} : P2Cfg{t.p2_phi, t.p2_phi_ty, t.p2_phi_minb, t.p2_phi_pd};
+  return mu ? P2Cfg{t.p2_mu, t.p2_mu_ty, t.p2_mu_minb, t.p2_mu_pd, t.p2_mu_hasync}
+            : P2Cfg{t.p2_phi, t.p2_phi_ty, t.p2_phi_minb, t.p2_phi_pd, 0};
 }
 
 // one P2 sweep with kernel choice c: the run-time specialised kernel
@@ -1798,6 +1799,7 @@ const std::vector<TuneKnob>& tune_knobs() {
       {"p2_mu_minb", &pf_tuning::p2_mu_minb, P2_MU, {1, 2, 3, 4}},
       {"p2_phi_pd", &pf_tuning::p2_phi_pd, P2_PHI, {0, 1, 2, 3, 4}},
       {"p2_mu_pd", &pf_tuning::p2_mu_pd, P2_MU, {0, 1, 2, 3, 4}},
+      {"p2_mu_hasync", &pf_tuning::p2_mu_hasync, P2_MU, {0, 1}},
       // not searched (data-dependent time; reported separately by bench.py)
       {"mu_atskip", &pf_tuning::mu_atskip, JIT_MU, {0}},
   };
@@ -1910,9 +1912,12 @@ static int autotune_p2(pf_ctx* ctx, unsigned mask, int reps, char* log, int logn
     std::vector<pf_tuning> cands{best};
     for (int k : {0, 1, 2})
       for (int tm : {0, 1, 2, 3, 4, 5})
-        for (int pdist : {0, 1, 2, 3, 4}) {
-          if (k != 0 && (tm || pdist)) continue;  // tile / prefetch only matter for the side-staged kernels
+        for (int pdist : {0, 1, 2, 3, 4})
+        for (int ha : {0, 1}) {
+          if (k != 0 && (tm || pdist || ha)) continue;  // tile / prefetch / staging only matter for the side-staged kernels
+          if (ha && (!mu || ctx->variant != PF_VARIANT_JIT || tm < 2)) continue;  // (staging: the specialised mu kernel, 32 x 4 tiles)
           pf_tuning c = best;
+          if (mu) c.p2_mu_hasync = ha;
           const int ty = tm < 2 ? 8 : 4, mb = tm == 0 ? 2 : tm == 1 ? 1 : tm + 1;  // 8x2 8x1 4x3 4x4 4x5 4x6
           (mu ? c.p2_mu : c.p2_phi) = k;
           if (k == 0) {

@@ -75,6 +75,7 @@ struct P2Cfg {
   int kern;    // 0 side-staged, 1 z-marching, 2 one thread per cell
   int ty, mb;  // side-staged: tile height, CTAs per SM
   int pd;      // side-staged: L2 prefetch distance (planes)
+  int hasync;  // side-staged mu, specialised build: halo ring staged by cp.async (p2_mu_hasync)
 };
 void p2_launch_phi(const void* P, const P2Cfg& c, double Tbase, const Geom& g, const double* ps, const double* ms,
                    double* pd, cudaStream_t s);

@@ -176,8 +176,11 @@ void p2_launch_dims(const P2Cfg& c, const Geom& g, dim3* grid, dim3* block) {
 
 std::string p2_specialised_source(const void* Pv, const Geom& g, const P2Cfg& c, int which) {
   const p2::Params& P = *reinterpret_cast<const p2::Params*>(Pv);
-  std::string o = "// generated by pf_p2.cu: P2 parameters as compile-time constants\n#include \"pf_p2_dev.cuh\"\n"
-                  "namespace pf {\nnamespace p2 {\nstruct KP2 {\n  static constexpr bool kSpec = true;\n";
+  std::string o = "// generated by pf_p2.cu: P2 parameters as compile-time constants\n";
+  // (the ring's static shared memory fits the 48-KB static limit beside the
+  // side arrays of 32 x 4 tiles only)
+  if (which == P2_MU && c.kern == 0 && c.hasync && c.ty == 4) o += "#define PF_P2_HASYNC 1\n";
+  o += "#include \"pf_p2_dev.cuh\"\nnamespace pf {\nnamespace p2 {\nstruct KP2 {\n  static constexpr bool kSpec = true;\n";
   put_sd(o, "dx", P.dx);
   put_sd(o, "dt", P.dt);
   put_sd(o, "eps", P.eps);

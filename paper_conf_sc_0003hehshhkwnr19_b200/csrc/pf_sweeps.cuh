@@ -1174,7 +1174,7 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
   // (hx = 1..MTX), top row; the 4 corners are carried by threads 0..3.
   constexpr int RC = 2 * (MTY + 2) + 2 * MTX;
   static_assert(NT - 2 * MTX - 2 * MTY >= 4, "mu_hcar: four free threads carry the ring corners");
-#if PF_MU_HASYNC < 2
+#if PF_MU_HASYNC != 2
   __shared__ __align__(16) double fring[3][N][RC];  // phase-major: a warp's ring reads are contiguous
 #endif
   auto ridx = [](int rx, int ry) {
@@ -1200,7 +1200,7 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
   // before the plane's second barrier -- so a halo cell builds its side with
   // no global load on the critical path
   __shared__ __align__(16) double dring[NSOL + M][RC];
-#if PF_MU_HASYNC >= 2
+#if PF_MU_HASYNC == 2
   // mu_hasync 2: the whole halo tile's phi_src planes (rows x0 - 2 .. x0 +
   // MTX + 1, 16-B pieces cached in L2 only; rows are 128-B aligned) in a
   // 3-plane ring: the own cells take phi_src(k) and its x / y / z neighbours
@@ -1211,7 +1211,7 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
   __shared__ __align__(16) double tring[3][N][MTY + 2][TRX];
 #endif
   auto stage = [&](const int kf, const int kd) {
-#if PF_MU_HASYNC >= 2
+#if PF_MU_HASYNC == 2
     for (int it = t; it < (MTY + 2) * N * TRP; it += NT) {
       const int pc = it % TRP, a = (it / TRP) % N, ry = it / (TRP * N);
       cp_async16(&tring[(kf + 3) % 3][a][ry][2 * pc],
@@ -1338,7 +1338,7 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
       asm volatile("prefetch.global.L1 [%0];" ::"l"(ms + F + ch));
     }
     // (a) publish D(k) of the two own cells and of the halo ring
-#if PF_MU_HASYNC >= 2 && PF_MU_RPF
+#if PF_MU_HASYNC == 2 && PF_MU_RPF
     {
       // mu_hasync 2: phi_src(k) and its neighbours from the staged tile ring
       // (the operands of the register path below: the same bits); phi_dst
@@ -1466,7 +1466,7 @@ __device__ __forceinline__ void mu_r2_body(const PT& P, const RT& R, const GT& g
       double v[D_NV];
 #pragma unroll
       for (int a = 0; a < N; ++a) {
-#if PF_MU_HASYNC >= 2
+#if PF_MU_HASYNC == 2
         const double tt = hwx ? tring[s0][a][hy][hx + 2] - tring[s0][a][hy][hx]
                               : tring[s0][a][hy + 1][hx + 1] - tring[s0][a][hy - 1][hx + 1];
         v[D_F + a] = tring[s0][a][hy][hx + 1];

@@ -125,7 +125,7 @@ def test_p2_invariants_and_monitor(pfmod):
     assert p.shape == (3,) + shape
 
 
-@pytest.mark.parametrize("kern", ["side", "march", "naive"])
+@pytest.mark.parametrize("kern", ["side", "side_hasync", "march", "naive"])
 @pytest.mark.parametrize("pset", ["p2", "p2_stress", "p2_iso"])
 def test_p2_specialised_equals_generic(pfmod, omod, pset, kern, monkeypatch):
     """The run-time specialised P2 sweeps (variant jit, the default: the
@@ -136,6 +136,8 @@ def test_p2_specialised_equals_generic(pfmod, omod, pset, kern, monkeypatch):
     monkeypatch.setenv("PF_P2_NAIVE", "1" if kern == "naive" else "0")
     monkeypatch.setenv("PF_P2_PHI", "march" if kern == "march" else "side")
     monkeypatch.setenv("PF_P2_MU", "march" if kern == "march" else "side")
+    # side_hasync: the specialised mu-sweep stages its halo ring by cp.async
+    monkeypatch.setenv("PF_P2_HASYNC", "1" if kern == "side_hasync" else "0")
     P = {"p2": I.params_p2(), "p2_stress": I.params_p2_stress(), "p2_iso": I.params_p2(aniso=0)}[pset]
     shape = (18, 21, 37)
     phi, mu = I.ic_voronoi(shape, seed=13, N=3, M=1)
