@@ -315,9 +315,9 @@ typedef struct {
                         column) instead of two L1 loads; mu_rpt = 2, mu_rpf = 1 */
   /* P2 parameterisation (pf_p2.cu; tuned by pf_autotune on a P2 context)  */
   int p2_phi;        /* P2 phi kernel: 0 side-staged (face sides in shared
-                        memory), 1 z-marching with global-memory face operands,
-                        2 one thread per cell (every face twice)               */
-  int p2_mu;         /* P2 mu kernel: the same three                           */
+                        memory), 1 z-marching with global-memory face operands
+                        (default), 2 one thread per cell (every face twice)   */
+  int p2_mu;         /* P2 mu kernel: the same three (default 0)              */
   int p2_phi_ty;     /* side-staged P2 phi: tile height (4 or 8) and CTAs per  */
   int p2_phi_minb;   /*   SM: (8, 2) default, (8, 1), (4, 3..6)                */
   int p2_mu_ty;      /* side-staged P2 mu: the same, default (4, 4)            */

@@ -166,6 +166,8 @@ def test_p2_side_tilings_bitwise(pfmod, monkeypatch, cfg):
     shape = (18, 21, 37)
     phi, mu = I.ic_voronoi(shape, seed=11, N=3, M=1)
     outs = []
+    monkeypatch.setenv("PF_P2_PHI", "side")
+    monkeypatch.setenv("PF_P2_MU", "side")
     for c in ("default", cfg):
         monkeypatch.setenv("PF_P2_SIDE", c)
         monkeypatch.setenv("PF_P2_SIDE_MU", c)
