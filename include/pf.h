@@ -297,9 +297,12 @@ typedef struct {
                         mu); 1 = z-slab pipeline: per slab of `slab` mu z-chunks the
                         phi-sweep of the slab (shifted up one plane), its x/y
                         ghosts, then the mu-sweep of the slab while its phi_dst is
-                        still in L2.  Applies to the JIT variant with no exchanged
+                        still in L2; 2 = the same slabs with the mu slabs on a
+                        second stream, each after its phi slab (an event), so
+                        that mu slab s and phi slab s+1 run concurrently and share
+                        the SMs.  Applies to the JIT variant with no exchanged
                         dimension and a non-periodic z (DS); otherwise sched 0     */
-  int slab;          /* mu z-chunks per slab of sched = 1 (1..16)                 */
+  int slab;          /* mu z-chunks per slab of sched = 1, 2 (1..16)              */
   int mu_tmem;       /* 1: the two-rows mu-sweep keeps the carried side of plane
                         k-1 in tensor memory (tcgen05.st / ld, 68 columns per
                         thread) instead of registers, and re-reads the own

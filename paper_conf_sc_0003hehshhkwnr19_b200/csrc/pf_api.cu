@@ -173,6 +173,9 @@ struct pf_ctx {
   // overlap of the halo exchange with interior work
   int first_ex = 3;                 // first exchanged dimension (3 = none)
   cudaStream_t comm_s = nullptr;    // exchange stream
+  cudaStream_t mu_s = nullptr;      // sched = 2: the mu slabs, concurrent with the next phi slab
+  std::vector<cudaEvent_t> ev_slab; // sched = 2: phi slab s (and its ghosts) done
+  cudaEvent_t ev_slab_done = nullptr;
   cudaEvent_t ev_phi = nullptr, ev_phix = nullptr, ev_mu = nullptr, ev_mux = nullptr;
   bool mux_pending = false;         // mu exchange in flight on comm_s
   bool overlap = true;
@@ -798,6 +801,12 @@ int pf_destroy(pf_ctx* ctx) {
     cudaStreamDestroy(ctx->comm_s);
   }
   if (ctx->cap_s) cudaStreamDestroy(ctx->cap_s);
+  if (ctx->mu_s) {
+    cudaStreamSynchronize(ctx->mu_s);
+    cudaStreamDestroy(ctx->mu_s);
+  }
+  for (cudaEvent_t ev : ctx->ev_slab) cudaEventDestroy(ev);
+  if (ctx->ev_slab_done) cudaEventDestroy(ctx->ev_slab_done);
   for (cudaEvent_t ev : {ctx->ev_phi, ctx->ev_phix, ctx->ev_mu, ctx->ev_mux})
     if (ev) cudaEventDestroy(ev);
   if (ctx->pinned) cudaFreeHost(ctx->pinned);
@@ -1131,28 +1140,30 @@ static cudaEvent_t ev_get(pf_ctx* ctx) {
   cudaEventCreate(&e);
   return e;
 }
-static void prof_begin(pf_ctx* ctx, int k, cudaEvent_t* a) {
+static void prof_begin(pf_ctx* ctx, int k, cudaEvent_t* a, cudaStream_t st = nullptr) {
   if (!ctx->prof) return;
   (void)k;
+  if (!st) st = ctx->stream;
   if (ctx->cap_sv) {  // capturing a graph: an event-record node of the graph
     cudaEventCreate(a);
-    cudaEventRecordWithFlags(*a, ctx->stream, cudaEventRecordExternal);
+    cudaEventRecordWithFlags(*a, st, cudaEventRecordExternal);
     return;
   }
   *a = ev_get(ctx);
-  cudaEventRecord(*a, ctx->stream);
+  cudaEventRecord(*a, st);
 }
-static void prof_end(pf_ctx* ctx, int k, cudaEvent_t a) {
+static void prof_end(pf_ctx* ctx, int k, cudaEvent_t a, cudaStream_t st = nullptr) {
   if (!ctx->prof) return;
+  if (!st) st = ctx->stream;
   if (ctx->cap_sv) {
     cudaEvent_t b = nullptr;
     cudaEventCreate(&b);
-    cudaEventRecordWithFlags(b, ctx->stream, cudaEventRecordExternal);
+    cudaEventRecordWithFlags(b, st, cudaEventRecordExternal);
     ctx->cap_prof.push_back({k, {a, b}});
     return;
   }
   cudaEvent_t b = ev_get(ctx);
-  cudaEventRecord(b, ctx->stream);
+  cudaEventRecord(b, st);
   ctx->ev_open.push_back({k, {a, b}});
   if (ctx->ev_open.size() > 4096) {  // drain to bound the pool
     cudaEventSynchronize(b);
@@ -1173,7 +1184,12 @@ static int monitor_check(pf_ctx* ctx, int64_t step_before);
 static int front_height_impl(pf_ctx* ctx, int* H);
 
 static int launch_mu(pf_ctx* ctx, const TileSel* ts, dim3 grid, const double* ps, const double* pd,
-                     const double* ms, double* md) {
+                     const double* ms, double* md, cudaStream_t st = nullptr) {
+  if (st) {  // (the concurrent slab schedule: the specialised sweep on the mu stream)
+    CU(jit_launch_mu(ctx->jmu, ctx->dp, ts, grid, ps, pd, ms, md, st, ctx->cap_sv));
+    ctx->nlaunch[1] += 1;
+    return check_launch(ctx, "mu_sweep");
+  }
   if (ctx->variant == PF_VARIANT_NAIVE)
     launch_mu_naive(ctx->dp, ctx->g, ps, pd, ms, md, ctx->stream);
   else if (ctx->variant == PF_VARIANT_SPLIT)
@@ -1192,6 +1208,22 @@ static int step_slabs(pf_ctx* ctx, const double* ps, double* pd, const double* m
   const int zc = jit_mu_zc_of(ctx->jmu), mty = jit_mu_ty_of(ctx->jmu), mtx = jit_mu_tx_of(ctx->jmu);
   const int H = zc * ctx->tune.slab;
   const int S = (g.nz + H - 1) / H;
+  // sched = 2: the mu slabs on their own stream, each after its phi slab and
+  // ghosts (an event), so that mu slab s runs concurrently with phi slab s + 1
+  // (independent: phi reads phi_src / mu_src, writes other phi_dst planes; mu
+  // slab s reads phi_dst planes <= its top + 1, all written by phi slabs <= s)
+  // and the two kernels share the SMs; the compute stream joins the mu stream
+  // before the mu ghosts
+  const bool conc = ctx->tune.sched == 2;
+  if (conc) {
+    if (!ctx->mu_s) CU(cudaStreamCreateWithFlags(&ctx->mu_s, cudaStreamNonBlocking));
+    if (!ctx->ev_slab_done) CU(cudaEventCreateWithFlags(&ctx->ev_slab_done, cudaEventDisableTiming));
+    while ((int)ctx->ev_slab.size() < S) {
+      cudaEvent_t e = nullptr;
+      CU(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+      ctx->ev_slab.push_back(e);
+    }
+  }
   const dim3 full = tuned_grid_mu(g, mty, zc, mtx);
   BCSpec bxy = ctx->bc_all;  // x / y ghosts of a range of planes: z sides left alone
   bxy.kind_lo[2] = bxy.kind_hi[2] = -1;
@@ -1219,10 +1251,20 @@ static int step_slabs(pf_ctx* ctx, const double* ps, double* pd, const double* m
     if (s == 0)
       if (int r = join_comm(ctx)) return r;  // the previous step's mu ghosts
     const TileSel ts = {{0, 0, zs / zc}, {0, 0, 0}, {0, 0, 0}, 0};
-    prof_begin(ctx, 1, &e0);
-    if (int r = launch_mu(ctx, &ts, dim3(full.x, full.y, (unsigned)((ze - zs + zc - 1) / zc)), ps, pd, ms, md))
+    cudaStream_t mst = nullptr;
+    if (conc) {
+      CU(cudaEventRecord(ctx->ev_slab[s], ctx->stream));
+      CU(cudaStreamWaitEvent(ctx->mu_s, ctx->ev_slab[s], 0));
+      mst = ctx->mu_s;
+    }
+    prof_begin(ctx, 1, &e0, mst);
+    if (int r = launch_mu(ctx, &ts, dim3(full.x, full.y, (unsigned)((ze - zs + zc - 1) / zc)), ps, pd, ms, md, mst))
       return r;
-    prof_end(ctx, 1, e0);
+    prof_end(ctx, 1, e0, mst);
+  }
+  if (conc) {  // join: everything after this waits for the last mu slab
+    CU(cudaEventRecord(ctx->ev_slab_done, ctx->mu_s));
+    CU(cudaStreamWaitEvent(ctx->stream, ctx->ev_slab_done, 0));
   }
   // line 4: mu ghosts on the side stream (overlapping the next step's first phi slab)
   if (ctx->overlap && ctx->comm_s) {
@@ -1308,7 +1350,7 @@ static int step_impl(pf_ctx* ctx, bool phi_only, bool dry = false) {
   // that the slab's top neighbour plane is ready), their x/y ghosts, then the
   // mu-sweep of the slab, which re-reads phi_src / phi_dst while the slab is
   // still in L2.  Same kernels and arithmetic per cell as the two sweeps.
-  if (ctx->variant == PF_VARIANT_JIT && ctx->tune.sched == 1 && ctx->first_ex == 3 && !phi_only && !phi_x_done &&
+  if (ctx->variant == PF_VARIANT_JIT && ctx->tune.sched >= 1 && ctx->first_ex == 3 && !phi_only && !phi_x_done &&
       ctx->cfg.bc_lo[2] != PF_BC_PERIODIC)
     return step_slabs(ctx, ps, pd, ms, md, dry);
   // Algorithm 1, line 1: phi-sweep (reads no mu ghosts: may overlap the previous mu exchange)
@@ -2130,7 +2172,7 @@ int pf_autotune(pf_ctx* ctx, unsigned mask, int passes, int reps, char* log, int
                        ctx->cfg.bc_lo[2] != PF_BC_PERIODIC && !(ctx->g.xwrap && ctx->tune.phi_xghost);
   if (slab_ok) {
     std::vector<pf_tuning> cands;
-    for (int sc : {0, 1})
+    for (int sc : {0, 1, 2})
       for (int sl : {1, 2, 4}) {
         if (sc == 0 && sl != 1) continue;
         pf_tuning c = best;

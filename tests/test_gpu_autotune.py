@@ -245,17 +245,27 @@ def test_slab_schedule_bitwise(pfmod, omod, slab, mu_zc, shape):
     P = I.params_stress(window_check=4, window_frac=0.5)
     phi, mu = I.ic_lamellar(shape, seed=7, z_front=shape[0] // 2 + 2, mu_inf=tuple(P["mu_inf"]))
     outs = []
-    for t in ({"sched": 0, "mu_zc": mu_zc}, {"sched": 1, "slab": slab, "mu_zc": mu_zc}):
-        g = pfmod.PhaseField(shape, P, bc=I.BC_DS)
+    # sched 2: the same slabs with the mu slabs on their own stream, concurrent
+    # with the next phi slab (CUDA-graph steps forced on for one of them)
+    for t in ({"sched": 0, "mu_zc": mu_zc}, {"sched": 1, "slab": slab, "mu_zc": mu_zc},
+              {"sched": 2, "slab": slab, "mu_zc": mu_zc}, {"sched": 2, "slab": slab, "mu_zc": mu_zc, "graph": 1}):
+        t = dict(t)
+        graph = t.pop("graph", 0)
+        if graph:
+            os.environ["PF_GRAPH"] = "1"
+        try:
+            g = pfmod.PhaseField(shape, P, bc=I.BC_DS)
+        finally:
+            os.environ.pop("PF_GRAPH", None)
         g.set_tuning(t)
         g.init_fields(phi, mu)
         g.step(9)
         outs.append((g.download(), g.state()))
         g.close()
     (p0, m0), s0 = outs[0]
-    (p1, m1), s1 = outs[1]
-    assert s0 == s1 and s0["z_off"] > 0
-    assert np.array_equal(p0, p1) and np.array_equal(m0, m1)
+    for (p1, m1), s1 in outs[1:]:
+        assert s0 == s1 and s0["z_off"] > 0
+        assert np.array_equal(p0, p1) and np.array_equal(m0, m1)
     o = omod.Oracle(shape, P, I.BC_DS)
     o.init(phi, mu)
     o.step(9)
