@@ -133,6 +133,12 @@ def test_tuning_defaults_and_range_check(lib):
     {"mu_cly": 2, "mu_ty": 6, "mu_minb": 2, "mu_qreg": 1, "mu_fxreg": 0, "mu_hpipe": 1, "mu_rpt": 1},
     {"mu_rpt": 2, "mu_ty": 6, "mu_minb": 2, "mu_rpf": 0, "mu_prefetch": 2},
     {"phi_rpt": 2, "phi_ty": 16, "phi_minb": 1, "phi_unroll": 2, "phi_xghost": 1},
+    # halo ring staged by cp.async (1), whole-tile staging (2), without the
+    # register prefetch (falls back to 1), the concurrent slab schedule
+    {"mu_hasync": 1, "mu_halo_l1": 0, "mu_zc": 7},
+    {"mu_hasync": 2, "mu_ty": 6, "mu_minb": 3},
+    {"mu_hasync": 2, "mu_rpf": 0},
+    {"sched": 2, "slab": 2, "mu_hasync": 1},
 ])
 def test_tuned_variants_compile_without_gpu(lib, knobs):
     """Extreme corners of the auto-tuning space (pf_autotune's knobs) still
@@ -163,7 +169,8 @@ def test_p2_layout_and_params_struct():
 
 
 @pytest.mark.parametrize("knobs", [{}, {"p2_phi": 1, "p2_mu": 1}, {"p2_phi": 2, "p2_mu": 2},
-                                   {"p2_phi_ty": 4, "p2_phi_minb": 4, "p2_mu_ty": 8, "p2_mu_minb": 1, "p2_phi_pd": 0}])
+                                   {"p2_phi_ty": 4, "p2_phi_minb": 4, "p2_mu_ty": 8, "p2_mu_minb": 1, "p2_phi_pd": 0},
+                                   {"p2_phi": 0, "p2_mu_hasync": 0}, {"p2_mu_ty": 4, "p2_mu_minb": 6, "p2_mu_hasync": 1}])
 def test_p2_specialised_kernels_compile_without_gpu(lib, tmp_path, knobs):
     """The run-time specialised P2 sweeps (pf_p2_dev.cuh on compile-time
     parameters) build with NVRTC for every kernel choice; with the P2 set
