@@ -35,6 +35,18 @@ for ic in ("R", "V", "L"):
     res[ic] = {"mlups": n ** 3 * steps / (ms * 1e-3) / 1e6, "ms_per_step": ms / steps,
                "phi_ms": pr["phi_sweep"][0] / max(pr["phi_sweep"][1], 1),
                "mu_ms": pr["mu_sweep"][0] / max(pr["mu_sweep"][1], 1)}
+    # the data-dependent anti-trapping skip (tuning mu_atskip) on the same state
+    g.set_tuning({"mu_atskip": 1})
+    g.step(3)
+    g.profile(True)
+    e0.record(g.stream)
+    g.step(steps)
+    e1.record(g.stream)
+    e1.synchronize()
+    ms = e0.elapsed_time(e1)
+    pr = g.profile_read()
+    res[ic]["atskip"] = {"mlups": n ** 3 * steps / (ms * 1e-3) / 1e6,
+                         "mu_ms": pr["mu_sweep"][0] / max(pr["mu_sweep"][1], 1)}
     g.close()
     torch.cuda.empty_cache()
 v = [r["mlups"] for r in res.values()]
