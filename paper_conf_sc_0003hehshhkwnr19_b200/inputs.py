@@ -191,6 +191,16 @@ def params_p2(**over) -> dict:
     return P
 
 
+def params_p2_ds(z_front: int, v: float = 0.05, G: float = 0.02, **over) -> dict:
+    """P2 in directional solidification (NEXT-4 "dendritic DS", Fig. 4 right):
+    params_p2 with a frozen gradient G pulled at v, the isotherm placed so
+    that the initial front is undercooled by v tau_sl (as params_ds_growth),
+    moving window; DS boundaries (BC_DS)."""
+    P = params_p2(G=G, v=v, window_check=10, window_frac=0.5, **over)
+    P["T0"] = ds_T0(z_front, G) - v * P["tau"][0, 2]
+    return P
+
+
 def params_p2_stress(seed: int = 20191118, **over) -> dict:
     """P2 stress set (parity only): every pair anisotropic with its own
     strength and a seeded random rotation, unequal gamma / tau, A1 != 0,
@@ -333,6 +343,34 @@ def ic_lamellar(shape, seed: int = 20191117, z_front: int | None = None, ngrains
     for i in range(M):
         mu[i] = mu_inf[i]
     return np.ascontiguousarray(phi), np.ascontiguousarray(mu)
+
+
+def ic_p2_front(shape, seed: int = 20191117, z_front: int | None = None, ngrains: int | None = None,
+                blur: int = 3, noise: float = 0.02):
+    """P2 directional-solidification start: below z_front an x-y Voronoi of
+    the two solid grains (phases 0, 1: the same solid, two orientations),
+    extruded along z, liquid (phase 2) above; blurred, interface noise;
+    mu = 0."""
+    rng = np.random.default_rng(seed)
+    nz, ny, nx = shape
+    if z_front is None:
+        z_front = max(1, nz // 4)
+    if ngrains is None:
+        ngrains = max(2, int(round(nx * ny / 2000.0)))
+    seeds2 = np.stack([np.zeros(ngrains), rng.uniform(0, ny, ngrains), rng.uniform(0, nx, ngrains)], 1)
+    lab2 = _nearest_seed((1, ny, nx), seeds2)[0] % 2
+    phi = np.zeros((3, nz, ny, nx))
+    for a in range(2):
+        phi[a, :z_front][:, lab2 == a] = 1.0
+    phi[2, z_front:] = 1.0
+    for _ in range(blur):
+        for ax in (2, 3):
+            phi = (phi + np.roll(phi, 1, axis=ax) + np.roll(phi, -1, axis=ax)) / 3.0
+        up = np.concatenate([phi[:, :1], phi[:, :-1]], axis=1)
+        dn = np.concatenate([phi[:, 1:], phi[:, -1:]], axis=1)
+        phi = (up + phi + dn) / 3.0
+    phi = _mix_noise(phi, rng, noise)
+    return np.ascontiguousarray(phi), np.zeros((1, nz, ny, nx))
 
 
 def make_ic(kind: str, shape, seed: int = 20191117, **kw):

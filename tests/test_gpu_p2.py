@@ -84,6 +84,22 @@ def test_p2_ds_window_parity(pfmod, omod):
     assert res[-1][3]["z_off"] > 0
 
 
+def test_p2_ds_front_parity(pfmod, omod):
+    """The benchmark's P2 directional-solidification recipe (params_p2_ds,
+    ic_p2_front): grains under liquid, frozen gradient, DS boundaries, the
+    window shifting at the first checks."""
+    shape = (40, 16, 24)
+    zf = 22
+    P = I.params_p2_ds(zf, v=0.1)
+    phi, mu = I.ic_p2_front(shape, seed=3, z_front=zf)
+    res = run_pair(pfmod, omod, shape, P, phi, mu, [1, 60], bc=I.BC_DS)
+    for t, ep, em, gs, os_ in res:
+        assert gs == os_
+        tol = 1e-12 if t == 1 else 1e-10
+        assert ep <= tol and em <= tol, (t, ep, em)
+    assert res[-1][3]["z_off"] > 0
+
+
 def test_p2_1000_steps(pfmod, omod):
     P = I.params_p2_stress()
     shape = (16, 16, 16)
