@@ -347,10 +347,6 @@ typedef struct {
   int p2_mu_hasync;  /* 1: the specialised side-staged P2 mu-sweep (32 x 4 tiles) stages its
                         halo ring one build ahead with cp.async (as mu_hasync
                         1; default); same bits                                 */
-  int phi_muearly;   /* phi-sweep: the cell's mu loaded at the plane's start, before
-                        the face fluxes (1), or one plane ahead into registers
-                        (2), instead of just before the cell update (0); same
-                        bits                                                   */
 } pf_tuning;
 
 /* The built-in defaults (the measured best at 256^3 on one B200,

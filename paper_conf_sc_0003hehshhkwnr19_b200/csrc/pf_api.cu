@@ -1832,7 +1832,6 @@ const std::vector<TuneKnob>& tune_knobs() {
       {"mu_hcar", &pf_tuning::mu_hcar, JIT_MU, {0, 1}},
       {"mu_xshfl", &pf_tuning::mu_xshfl, JIT_MU, {0, 1}},
       {"mu_hasync", &pf_tuning::mu_hasync, JIT_MU, {0, 1, 2}},
-      {"phi_muearly", &pf_tuning::phi_muearly, JIT_PHI, {0, 1, 2}},
       // P2 (pf_p2.cu): tuned by the P2 branch of pf_autotune
       {"p2_phi", &pf_tuning::p2_phi, P2_PHI, {0, 1, 2}},
       {"p2_mu", &pf_tuning::p2_mu, P2_MU, {0, 1, 2}},

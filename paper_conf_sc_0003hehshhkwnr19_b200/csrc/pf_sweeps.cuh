@@ -130,9 +130,6 @@ constexpr int MU_TY = PF_MU_TY;
 #ifndef PF_MU_HASYNC  // two-rows mu-sweep: halo ring staged one plane ahead by cp.async (global -> shared)
 #define PF_MU_HASYNC 0
 #endif
-#ifndef PF_PHI_MUEARLY  // phi-sweep: the cell's mu loaded before the faces (1) or one plane ahead (2)
-#define PF_PHI_MUEARLY 0
-#endif
 #ifndef PF_MU_XSHFL  // two-rows mu-sweep: own cd_x from the lane neighbours' carried phi_src (shuffles)
 #define PF_MU_XSHFL 0
 #endif
@@ -183,9 +180,6 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const RT& R, const G
       p0[a] = __ldg(ps + a * F + c);
     }
     phi_face(P, pm, p0, Fzm);
-#if PF_PHI_MUEARLY == 2
-    double mun0 = __ldg(ms + c), mun1 = __ldg(ms + F + c);
-#endif
 #pragma unroll kPhiUnroll
     for (int z = z0; z < z1; ++z, c += SZ) {
       if (PF_PREFETCH && z + PF_PREFETCH_D <= z1 + 1) {
@@ -194,11 +188,6 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const RT& R, const G
         prefetch_line(ms + c + PF_PREFETCH_D * SZ);
         prefetch_line(ms + F + c + PF_PREFETCH_D * SZ);
       }
-#if PF_PHI_MUEARLY == 1
-      // mu of the cell issued before the face fluxes (its latency then runs
-      // under them instead of stalling the cell update)
-      const double mu0 = __ldg(ms + c), mu1 = __ldg(ms + F + c);
-#endif
       double pp[N], Fzp[N], gd[N][3], divh[N];
       {
         double xm[N], xp[N], ym[N], yp[N], Fa[N], Fb[N];
@@ -234,15 +223,7 @@ __device__ __forceinline__ void phi_tuned_body(const PT& P, const RT& R, const G
 #endif
 #pragma unroll
       for (int a = 0; a < N; ++a) divh[a] += Fzp[a] - Fzm[a];
-#if PF_PHI_MUEARLY == 2
-      const double mu0 = mun0, mu1 = mun1;  // loaded one plane earlier
-      if (z + 1 < z1) {
-        mun0 = __ldg(ms + c + SZ);
-        mun1 = __ldg(ms + F + c + SZ);
-      }
-#elif PF_PHI_MUEARLY == 0
       const double mu0 = __ldg(ms + c), mu1 = __ldg(ms + F + c);
-#endif
       double out[N], xi[N];
       if constexpr (ParamShape<PT>::xi) xi_of(P, R.step, x + g.x0, y + g.y0, z + g.z0, xi);
       phi_cell<TA>(P, plane_T(P, R, (double)z), p0, gd, divh, mu0, mu1, xi, out);

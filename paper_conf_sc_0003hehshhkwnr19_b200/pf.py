@@ -58,7 +58,7 @@ TUNING_KNOBS = ("phi_ty", "phi_minb", "phi_zc", "phi_faces6", "phi_unroll", "phi
                 "mu_ty", "mu_tx", "mu_minb", "mu_zc", "mu_prefetch", "mu_pfd", "mu_rpf", "mu_halo_l1", "mu_fxreg",
                 "mu_qreg", "mu_ldhint", "mu_hpipe", "mu_cly", "mu_rot", "mu_rpt", "phi_rpt", "mu_pers", "phi_pers", "sched", "slab", "mu_tmem",
                "mu_hcar", "mu_xshfl", "p2_phi", "p2_mu", "p2_phi_ty", "p2_phi_minb", "p2_mu_ty", "p2_mu_minb",
-               "p2_phi_pd", "p2_mu_pd", "mu_atskip", "mu_hasync", "p2_mu_hasync", "phi_muearly")
+               "p2_phi_pd", "p2_mu_pd", "mu_atskip", "mu_hasync", "p2_mu_hasync")
 
 
 class PFTuning(C.Structure):

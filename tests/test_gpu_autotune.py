@@ -82,9 +82,6 @@ CORNERS = [
     {"mu_hasync": 2, "mu_halo_l1": 0},
     {"mu_hasync": 2, "mu_zc": 7, "mu_ty": 6, "mu_minb": 3},
     {"mu_hasync": 2, "mu_pers": 1, "mu_ty": 10, "mu_minb": 2, "mu_xshfl": 1},
-    # the phi-sweep's mu loads early / one plane ahead (ragged chunks)
-    {"phi_muearly": 1, "phi_zc": 7},
-    {"phi_muearly": 2, "phi_zc": 7, "phi_ty": 8, "phi_minb": 2},
 ]
 
 
