@@ -152,6 +152,7 @@ def test_p2_fullsize_sampled_cells(pfmod, omod):
     errp = errm = 0.0
     scale_p, scale_m = np.abs(gp).max(), np.abs(gm).max()
     for z, y, x in list(pick) + list(anyc):
+        # (periodic in z as well: wrap the sub-block's planes)
         zr, yr, xr = np.arange(z - 2, z + 3) % n, np.arange(y - 2, y + 3), np.arange(x - 2, x + 3)
         sp = _sub_block(phi, zr, yr, xr).copy()
         sm = _sub_block(mu, zr, yr, xr).copy()
@@ -162,3 +163,51 @@ def test_p2_fullsize_sampled_cells(pfmod, omod):
         errp = max(errp, np.abs(op[:, 2, 2, 2] - gp[:, z, y, x]).max())
         errm = max(errm, np.abs(om[:, 2, 2, 2] - gm[:, z, y, x]).max())
     assert errp / scale_p <= 1e-12 and errm / scale_m <= 1e-12, (errp / scale_p, errm / scale_m)
+
+
+def test_stress_fullsize_sampled_cells(pfmod, omod):
+    """Parameter set S (every general expression: unequal gamma, off-diagonal
+    chi and D, A1 != 0, G v != 0) at the full 256^3 size, IC-V, periodic:
+    one step, sampled cells against oracle sub-blocks (radius 2, z_off at the
+    sub-block origin for the frozen temperature)."""
+    n = NFULL
+    P = I.params_stress()
+    phi, mu = I.ic_voronoi((n, n, n), seed=20191119)
+    g = pfmod.PhaseField((n, n, n), P)
+    g.init_fields(phi, mu)
+    g.step(1)
+    gp, gm = g.download()
+    g.close()
+    rng = np.random.default_rng(7)
+    # z kept 2 planes from the (periodic) z ends: with G v != 0 the frozen
+    # temperature jumps across the periodic z boundary, which a sub-block
+    # placed by z_off cannot reproduce
+    zs, ys, xs = rng.integers(2, n - 2, 80), rng.integers(0, n, 80), rng.integers(0, n, 80)
+    errp = errm = 0.0
+    for z, y, x in zip(zs, ys, xs):
+        zr, yr, xr = np.arange(z - 2, z + 3), np.arange(y - 2, y + 3), np.arange(x - 2, x + 3)
+        o = omod.Oracle((5, 5, 5), dict(P, window_check=0), I.BC_PERIODIC)
+        o.init(_sub_block(phi, zr, yr, xr).copy(), _sub_block(mu, zr, yr, xr).copy())
+        o.set_state(step=0, z_off=int(z) - 2)
+        o.step(1)
+        op, om = o.download()
+        errp = max(errp, np.abs(op[:, 2, 2, 2] - gp[:, z, y, x]).max())
+        errm = max(errm, np.abs(om[:, 2, 2, 2] - gm[:, z, y, x]).max())
+    assert errp / np.abs(gp).max() <= 1e-12 and errm / np.abs(gm).max() <= 1e-12, (errp, errm)
+
+
+def test_fullsize_tunings_bitwise(pfmod, bench_case):
+    """The bench launch configuration against its neighbours at full size:
+    the halo ring loaded instead of cp.async-staged (mu_hasync 0, with the
+    L1 prefetch) and the anti-trapping skip (mu_atskip 1) give the default's
+    bits after one step of the bench workload."""
+    P, phi, mu, gp, gm, _ = bench_case
+    n = NFULL
+    for t in ({"mu_hasync": 0, "mu_halo_l1": 1}, {"mu_atskip": 1}):
+        g = pfmod.PhaseField((n, n, n), P, bc=I.BC_DS)
+        g.set_tuning(t)
+        g.init_fields(phi, mu)
+        g.step(1)
+        p, m = g.download()
+        g.close()
+        assert np.array_equal(p, gp) and np.array_equal(m, gm), t
